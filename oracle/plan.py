@@ -1,0 +1,53 @@
+"""Request plans: which calls each GPU caller issues -- TEST INFRASTRUCTURE ONLY.
+
+A plan is a pure function of (workload, file sizes, grid shape, granularity); the oracle executes
+it with direct host syscalls and the GPU results are compared per request id (reading A18).
+
+  * wordcount / grep (sec. VIII-C, P32.7: "work-group granularity with blocking and
+    weak-ordering"): one pread per work-group chunk; chunk c of a file covers [s, e) =
+    [c*C, min((c+1)*C, size)) and its request is the halo read pread(off=max(s-1,0),
+    len=(e+16)-off) (reading A10) -- the reply is short at end of file (reading A11).
+  * granularity microbenchmark (sec. VII, P26.5-16, Fig. 7): caller c (work-item:
+    global thread id; work-group: block id; kernel: 0) issues R preads of `length` bytes at
+    off = ((c*R + r) * length) mod size, r = 0..R-1.
+"""
+from __future__ import annotations
+
+HALO_BEFORE = 1
+HALO_AFTER = 16     # longest dictionary word / grep pattern (16 B), reading A10
+
+
+def wordcount_chunk_requests(size: int, chunk: int):
+    """[(chunk_index, s, e, off, len)] for one file."""
+    out = []
+    nch = (size + chunk - 1) // chunk
+    for c in range(nch):
+        s = c * chunk
+        e = min(s + chunk, size)
+        off = s - HALO_BEFORE if s else 0
+        out.append((c, s, e, off, e + HALO_AFTER - off))
+    return out
+
+
+def expected_pread_ret(size: int, off: int, length: int, cap: int = 0x7FFFF000) -> int:
+    """POSIX pread on a regular file of stable size: min(len, size-off, per-call cap), >= 0."""
+    return max(0, min(length, size - off, cap))
+
+
+def microbench_requests(granularity: str, n_blocks: int, block_threads: int, R: int, length: int,
+                        size: int):
+    """[(caller, r, off, len)] for the granularity microbenchmark."""
+    if granularity == "wi":
+        callers = n_blocks * block_threads
+    elif granularity == "wg":
+        callers = n_blocks
+    elif granularity == "kernel":
+        callers = 1
+    else:
+        raise ValueError(granularity)
+    out = []
+    for c in range(callers):
+        for r in range(R):
+            off = ((c * R + r) * length) % size
+            out.append((c, r, off, length))
+    return out
