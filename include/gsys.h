@@ -1,0 +1,251 @@
+/*
+ * gsys.h -- C-ABI of libgsys: GPU-issued POSIX system calls on NVIDIA B200 (sm_100a).
+ *
+ * A from-scratch, B200-native take on GENESYS (Vesely et al., "Generic System Calls for GPUs",
+ * ISCA 2018; /root/reference/PAPER.md).  GPU threads claim a slot of a shared "syscall area"
+ * (sec. III step 1), publish the call and ring a doorbell (step 2, the paper's
+ * s_sendmsg interrupt, PAPER.md:24 P24.14), a host service executes the real POSIX call
+ * (steps 3-4, P24.16-21) and returns the result into the slot (step 5, P24.32-36).  The paper's
+ * modified Linux kernel / interrupt path is replaced by a user-space service thread pool,
+ * because the box's kernel cannot be changed (BASELINE.json north_star).
+ *
+ * Every entry point is `extern "C"`, takes plain pointers and sizes, and returns 0 (or a
+ * documented non-negative value) on success and -errno on failure.  One instance exists per CUDA
+ * device per process; it is bound to the device that is current when gsys_init() is called, and
+ * every other entry point acts on the instance of the *current* device.
+ *
+ * Ownership: the library owns the syscall area, claim words, doorbell ring, bounce buffers,
+ * service threads and their CUDA streams.  The caller owns file descriptors (they must stay open
+ * until gsys_wait() returns for every launch that uses them), every buffer it passes (device
+ * memory from cudaMalloc/PyTorch, or pinned host-mapped memory; they must stay alive until the
+ * call completes -- for non-blocking calls until gsys_wait()), and the CUDA streams it passes.
+ */
+#ifndef GSYS_H
+#define GSYS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---------------------------------------------------------------- slot layout (reading A1)
+ * "64 bytes per slot ... the requested system call number, the request state, system call
+ * arguments (as many as 6, in Linux), and padding to avoid false sharing.  The field for
+ * arguments is also re-purposed for the return value" (sec. VI, P24.7-9).
+ * One 64 B, 64 B-aligned line per slot; args[0] carries the i64 result back. */
+typedef struct gsys_slot {
+    uint64_t args[6];   /* bytes  0..47: syscall arguments; args[0] <- return value        */
+    uint32_t nr;        /* bytes 48..51: Linux x86-64 syscall number (pread64 = 17, ...)    */
+    uint32_t flags;     /* bytes 52..55: GSYS_* granularity/blocking/ordering bits (P24.13)  */
+    uint32_t seq;       /* bytes 56..59: per-slot request sequence number                   */
+    uint32_t state;     /* bytes 60..63: gsys_state                                         */
+} gsys_slot;
+
+/* Slot states (PAPER.md:24 P24.10-34, Fig. 6 caption PAPER.md:22; reading A2). */
+enum gsys_state {
+    GSYS_FREE = 0,        /* no request                                        */
+    GSYS_POPULATING = 1,  /* claimed by a GPU thread (cmp-swap, P24.10, P24.46) */
+    GSYS_READY = 2,       /* published, doorbell rung (P24.12-14)               */
+    GSYS_PROCESSING = 3,  /* picked up by a host worker (P24.20)                */
+    GSYS_FINISHED = 4     /* blocking call done, result in args[0] (P24.33)     */
+};
+
+/* ---------------------------------------------------------------- per-call flags
+ * Granularity: exactly one of WI / WG / KERNEL (sec. V-A "work-item, work-group,
+ * or kernel").  Blocking is the default (P20.34-46).  Ordering: strong is the default; relaxed
+ * removes Bar1 for producer calls or Bar2 for consumer calls (PAPER.md:20 P20.24-29, PAPER.md:22
+ * P22.41-42).  WI calls are always strong (P20.31); KERNEL calls must be relaxed (P20.33), so
+ * KERNEL|STRONG returns -EINVAL. */
+#define GSYS_WI          0x01u
+#define GSYS_WG          0x02u
+#define GSYS_KERNEL      0x04u
+#define GSYS_GRAN_MASK   0x07u
+#define GSYS_BLOCKING    0x00u
+#define GSYS_NONBLOCKING 0x08u
+#define GSYS_STRONG      0x00u
+#define GSYS_RELAXED     0x10u
+#define GSYS_WEAK        GSYS_RELAXED
+#define GSYS_SITE(k)     (((uint32_t)(k) & 63u) << 24)   /* kernel-scope call site id 0..63 */
+/* internal bits set by the device library in the slot's flags word */
+#define GSYS_F_PRODUCER  0x100u   /* call class: producer (read-like), P20.24-29            */
+#define GSYS_F_INLINE    0x200u   /* small result goes to the slot's inline payload line    */
+
+/* Syscall numbers served (Linux x86-64). */
+#define GSYS_NR_PREAD64        17
+#define GSYS_NR_PWRITE64       18
+#define GSYS_NR_MADVISE        28
+#define GSYS_NR_SENDTO         44
+#define GSYS_NR_RECVFROM       45
+#define GSYS_NR_GETRUSAGE      98
+#define GSYS_NR_RT_SIGQUEUEINFO 129
+
+#define GSYS_INLINE_BYTES 256u     /* per-slot inline payload (struct rusage = 144 B)  */
+#define GSYS_PREAD_CAP 0x7ffff000ull   /* Linux per-call read cap (reading A11)        */
+
+/* ---------------------------------------------------------------- lifecycle
+ * gsys_init: create the instance for the current CUDA device.
+ *   slots             number of syscall-area slots; 0 = one per resident work-item of the
+ *                     device ("one slot for each active GPU work-item", PAPER.md:24 P24.1),
+ *                     i.e. nsmid x 2048.  Must be <= 2^24.
+ *   coalesce_window_us  coalescing time window in microseconds ("a time window length within
+ *                     which the CPU coalesces system calls", PAPER.md:22 P22.13); 0 = take only
+ *                     requests already present.
+ * Service thread count: env GSYS_THREADS (default min(8, cores-2)); coalescing max count
+ * default 8 (PAPER.md:28 P28.17), see gsys_set_coalesce_max().
+ * Errors: -EINVAL (slots > 2^24), -EALREADY (already initialised on this device), -ENODEV (no
+ * CUDA device), -ENOMEM (pinned/device allocation failed), -ENOTSUP (stream memory operations
+ * unavailable). */
+int gsys_init(uint32_t slots, uint32_t coalesce_window_us);
+
+/* Maximum number of requests one coalesced bundle may hold ("the maximum number of system call
+ * invocations that can be coalesced within the time window", PAPER.md:22 P22.13).  n >= 1;
+ * 1 disables coalescing.  -EINVAL for n == 0 or n > 4096, -ENODEV before gsys_init. */
+int gsys_set_coalesce_max(uint32_t n);
+
+/* Coalescing window in microseconds (same meaning as gsys_init's argument). */
+int gsys_set_coalesce_window(uint32_t us);
+
+/* Merge preads of one regular file whose ranges are adjacent or overlapping into one read of
+ * the union inside a coalesced bundle (north_star extension, reading A8). on = 0/1. */
+int gsys_set_merge(int on);
+
+/* Protocol tracing (debug): on = 1 records every slot transition (GPU and host side) into
+ * trace buffers readable with gsys_trace_read(); capacity = max records per side. */
+int gsys_set_trace(int on, uint32_t capacity);
+
+/* Launch a kernel that may call gsys_* device functions: resets the kernel-scope call sites,
+ * then cudaLaunchKernel(kernel, grid, block, args, smem_bytes, stream).  `kernel` is a
+ * __global__ function pointer, `args` its argument array, `stream` a cudaStream_t (NULL = the
+ * legacy default stream).  CUDA errors map to -EINVAL / -ENOMEM / -EIO. */
+int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz,
+                uint32_t bx, uint32_t by, uint32_t bz, void** args, size_t smem_bytes,
+                void* stream);
+
+/* Drain (sec. IX "a new function call, invoked by the CPU, that ensures all GPU
+ * system calls have completed before the termination of the process", P34.9).  Waits for the
+ * stream (NULL = whole device), then until every request the device has published is processed
+ * and its completion (DMA + state write) has landed.  Returns 0, or the first -errno recorded
+ * for a non-blocking call since the previous gsys_wait (reading A4), which it then clears. */
+int gsys_wait(void* stream);
+
+/* gsys_wait(NULL), stop the service threads, free everything.  Idempotent: 0 if not initialised. */
+int gsys_shutdown(void);
+
+/* Device pointer to the instance's gsys_dev_ctx (see gsys_device.cuh); NULL before init. */
+const void* gsys_device_ctx(void);
+
+/* ---------------------------------------------------------------- statistics */
+typedef struct gsys_stats {
+    uint64_t requests;        /* requests drained from the doorbell ring         */
+    uint64_t completed;       /* requests whose completion was issued            */
+    uint64_t bundles;         /* coalesced bundles handed to workers (P22.9-13)  */
+    uint64_t max_bundle;      /* largest bundle seen                             */
+    uint64_t host_preads;     /* pread(2) calls actually executed on the host    */
+    uint64_t merged;          /* requests served by a merged union read          */
+    uint64_t bytes_read;      /* bytes returned by host preads                   */
+    uint64_t bytes_h2d;       /* bytes DMA'd host -> device                      */
+    uint64_t errors;          /* requests that returned -errno                   */
+    uint64_t per_nr[8];       /* pread, pwrite, madvise, sendto, recvfrom, getrusage, sigq, other */
+    uint32_t threads;         /* service worker threads                          */
+    uint32_t slots;           /* syscall-area slots                              */
+    uint32_t coalesce_max;
+    uint32_t coalesce_window_us;
+} gsys_stats_t;
+
+int gsys_stats(gsys_stats_t* out);
+int gsys_stats_reset(void);
+
+/* Trace record: one slot transition (reading: oracle/protocol.py validates these). */
+typedef struct gsys_trace_rec {
+    uint32_t slot;
+    uint32_t seq;
+    uint8_t from, to;   /* gsys_state values, `from` as observed by the actor */
+    uint8_t actor;      /* 0 = GPU, 1 = host                                   */
+    uint8_t blocking;   /* 1 if the request was blocking                       */
+    uint32_t pad;
+} gsys_trace_rec;
+
+/* Copy up to cap records of each side into gpu_out / host_out (host memory); returns the
+ * counts through n_gpu / n_host and resets the buffers. */
+int gsys_trace_read(gsys_trace_rec* gpu_out, uint32_t gpu_cap, uint32_t* n_gpu,
+                    gsys_trace_rec* host_out, uint32_t host_cap, uint32_t* n_host);
+
+/* Compile-time facts of this build, for tests: slot bytes, inline bytes, state count. */
+int gsys_abi_info(uint32_t* slot_bytes, uint32_t* inline_bytes, uint32_t* nstates);
+
+/* ---------------------------------------------------------------- host-side planning (pure)
+ * The coalescer's merge planner, exported for CPU tests (no device needed).  Given n preads
+ * (fd, off, len) of one bundle, computes the (fd, off) order (reading A8), groups runs on the
+ * same fd whose ranges are adjacent or overlapping (off_{i+1} <= off_i + len_i) while the union
+ * stays <= max_union bytes, and writes for each request its group id and its byte offset inside
+ * the group's union read; group_off/group_len receive each group's union.  Returns the number
+ * of groups.  order[] receives the processing order. */
+int gsys_plan_merge(uint32_t n, const int32_t* fd, const int64_t* off, const uint64_t* len,
+                    uint64_t max_union, uint32_t* order, uint32_t* group, uint64_t* offset_in_group,
+                    int64_t* group_off, uint64_t* group_len);
+
+/* Per-request result of a merged union read that returned r bytes (or -errno):
+ * clamp(r - offset_in_group, 0, len) (reading A8); -errno propagates. */
+int64_t gsys_split_result(int64_t r, uint64_t offset_in_group, uint64_t len);
+
+/* ---------------------------------------------------------------- workloads (the hot path)
+ * Wordcount + grep -F -l over files read with GPU-issued preads (sec. VIII-C,
+ * P32.3-9 wordcount "64 strings", "work-group granularity with blocking and weak-ordering";
+ * PAPER.md:30 P30.27-38 grep -F -l).
+ *   fds, sizes      host arrays [nfiles]: open read-only descriptors and their sizes in bytes.
+ *   chunk           bytes per work-group chunk (multiple of 16, >= 4096); each chunk [s, e) is
+ *                   read with one work-group pread of [max(s-1,0), e+16) (reading A10).
+ *   dict, dlen      host arrays: ndict (<= 64) words, 17-byte stride, lengths 1..16.
+ *   pats, plen      host arrays: npat (<= 8) grep patterns, 17-byte stride, lengths 1..16.
+ *   d_hist          DEVICE uint64[ndict]: whole-token counts are ADDED (reading A9).
+ *   d_file_hits     DEVICE uint32[nfiles] (may be NULL): set to 1 for files containing a pattern.
+ *   gflags          GSYS_WG (the paper's configuration for wordcount) + GSYS_BLOCKING +
+ *                   GSYS_STRONG or GSYS_RELAXED; anything else is -EINVAL.
+ *   blocks          work-groups launched (0 = 4 per SM); threads: threads per work-group
+ *                   (0 = 256; multiple of 32, <= 1024).
+ *   d_req_ret       DEVICE int64[total chunks] (may be NULL): per-chunk pread return value.
+ *   stream          cudaStream_t to launch on.
+ * Asynchronous on `stream`; call gsys_wait(stream) before reading results.  Errors: -EINVAL
+ * for bad sizes/flags, -ENODEV before gsys_init, CUDA errors as in gsys_launch.  Read errors
+ * of individual chunks are visible in d_req_ret (negative) and skip the chunk's scan. */
+int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, uint32_t chunk,
+                   const char* dict, const uint8_t* dlen, uint32_t ndict,
+                   const char* pats, const uint8_t* plen, uint32_t npat,
+                   uint64_t* d_hist, uint32_t* d_file_hits, int64_t* d_req_ret,
+                   uint32_t gflags, uint32_t blocks, uint32_t threads, void* stream);
+
+/* Same scan over text already resident in device memory (no syscalls): the standalone scan
+ * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n]; file boundaries are not
+ * modelled (one file).  Adds into d_hist; d_hit (may be NULL) set to 1 if any pattern occurs. */
+int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
+                     const char* dict, const uint8_t* dlen, uint32_t ndict,
+                     const char* pats, const uint8_t* plen, uint32_t npat,
+                     uint64_t* d_hist, uint32_t* d_hit, uint32_t blocks, uint32_t threads,
+                     void* stream);
+
+/* Syscall microbenchmark (sec. VII, Fig. 7/8/10): every caller of the chosen
+ * granularity (work-item: every thread; work-group: every block; kernel: one per launch) issues
+ * `iters` calls of
+ *   kind 0 = getrusage(RUSAGE_SELF, ru) -- the blocking result lands in the slot's inline line
+ *            and is copied by the caller;
+ *   kind 1 = pread(fd, d_buf + caller*len, len, off), off = ((caller*iters + r) * len) mod size;
+ *            after the call every thread of the calling scope reads the buffer back and the
+ *            scope's byte sum is stored in d_sum[caller*iters + r] (a missing post-call barrier
+ *            or an unordered DMA shows up there);
+ *   kind 2 = pwrite(fd, d_buf + caller*len, len, off) after every thread of the scope wrote its
+ *            share of the buffer (byte i of call idx = (idx*131 + i*7 + 13) & 0xff, written
+ *            with thread-dependent delays, so a missing pre-call barrier shows up in the file).
+ * d_buf: DEVICE or host-mapped, callers*len bytes (NULL allowed for kind 0).  gflags:
+ * granularity + blocking + ordering.  d_ret / d_lat_ns / d_sum (each may be NULL): DEVICE
+ * int64 / uint64 / uint64 [callers*iters]: return value, GPU-observed latency (ns, %globaltimer,
+ * call entry -> return), and the kind-1 byte sum.  Asynchronous; returns the number of callers. */
+int gsys_bench_calls(uint32_t kind, uint32_t gflags, uint32_t blocks, uint32_t threads,
+                     uint32_t iters, int32_t fd, uint64_t len, uint64_t size, void* d_buf,
+                     int64_t* d_ret, uint64_t* d_lat_ns, uint64_t* d_sum, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GSYS_H */

@@ -1,0 +1,395 @@
+/*
+ * gsys_device.cuh -- device side of libgsys (sm_100a): GPU-issued POSIX system calls.
+ *
+ * Implements, per GPU thread, the invocation half of GENESYS (sec. VI):
+ *   a1 caller election + pre-call barrier    P22.39-42, P20.14-33
+ *   a2 slot claim (cmp-swap, "delayed" if not free)                    P24.10-11, P24.46
+ *   a3 marshal nr/flags/seq/args into the 64 B slot (128-bit stores)   P24.8-13
+ *   a4 publish (__threadfence_system) + doorbell (the s_sendmsg analogue, warp-aggregated)
+ *                                                                       P24.12-14, P16.0
+ *   a5 blocking: poll the completion word with backoff; non-blocking: return at once
+ *                                                                       P24.15, P24.32-36
+ *   a6 post-call barrier + result broadcast                             P22.41-42, P28.2-3
+ *
+ * B200 mapping: the syscall area and doorbell ring live in pinned,
+ * host-mapped memory (posted PCIe writes from the GPU, cache-resident for the host); the claim
+ * words, per-slot sequence numbers and completion words live in device memory, so GPU-GPU
+ * arbitration (atomicCAS) and completion polling stay in L2 instead of crossing PCIe (the
+ * paper's Fig. 9 polling-contention problem, PAPER.md:28 P28.7-11).  The host writes a
+ * completion word {seq, ret} with a CUDA stream memory operation ordered after the payload
+ * DMA, so a thread that observes its seq also observes the pread bytes.
+ *
+ * Usage: every device function takes the instance context `const gsys_dev_ctx*` (from
+ * gsys_device_ctx()).  Calls of WG granularity must be reached by every thread of the block,
+ * calls of KERNEL granularity by every thread of every block (reading A16).
+ */
+#ifndef GSYS_DEVICE_CUH
+#define GSYS_DEVICE_CUH
+
+#include <cuda_runtime.h>
+#include <errno.h>
+#include <stdint.h>
+
+#include "gsys.h"
+
+#define GSYS_KSITES 8u          /* kernel-scope call sites per launch          */
+#define GSYS_KROUNDS 4096u      /* kernel-scope calls per site per launch      */
+
+/* Per (site, round) record of a kernel-scope call (reset by gsys_launch). */
+struct gsys_kround {
+    unsigned arrive;   /* blocks that reached this round of the site            */
+    unsigned done;     /* 1 once the caller stored ret (producer calls)          */
+    long long ret;     /* the caller's result, broadcast to the other blocks     */
+};
+
+/* Instance context in device memory (built by gsys_init). */
+struct gsys_dev_ctx {
+    gsys_slot* area;                /* host-mapped [nslots] syscall area                    */
+    unsigned char* inline_buf;      /* host-mapped [nslots * GSYS_INLINE_BYTES]             */
+    unsigned* claim;                /* device [nslots]: 0 free, 1 owned                     */
+    unsigned* seqs;                 /* device [nslots]: last sequence number used           */
+    unsigned long long* mirror;     /* device [nslots]: completion word (seq << 32 | u32 ret) */
+    unsigned long long* ring;       /* host-mapped [ring_mask+1] doorbell entries           */
+    unsigned* ring_tail;            /* device: next doorbell position                       */
+    gsys_kround* krounds;           /* device [GSYS_KSITES * GSYS_KROUNDS]                  */
+    unsigned* kblock;               /* device [kblock_cap * GSYS_KSITES]: rounds per block  */
+    gsys_trace_rec* trace;          /* device trace buffer or nullptr                       */
+    unsigned* trace_n;
+    unsigned trace_cap;
+    unsigned kblock_cap;
+    unsigned nslots;
+    unsigned ring_mask;
+    unsigned poll_ns_max;
+    unsigned pad_;
+};
+
+#ifdef __CUDACC__
+namespace gsys {
+
+/* ------------------------------------------------------------------ PTX helpers */
+__device__ __forceinline__ unsigned smid() { unsigned r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
+__device__ __forceinline__ unsigned warpid() { unsigned r; asm volatile("mov.u32 %0, %%warpid;" : "=r"(r)); return r; }
+__device__ __forceinline__ unsigned laneid() { unsigned r; asm volatile("mov.u32 %0, %%laneid;" : "=r"(r)); return r; }
+__device__ __forceinline__ unsigned lanemask_lt() { unsigned r; asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(r)); return r; }
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); return t;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_sys(const unsigned long long* p) {
+    unsigned long long v; asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory"); return v;
+}
+__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
+    unsigned v; asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
+__device__ __forceinline__ void st_relaxed_sys(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.relaxed.sys.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_gpu(unsigned* p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_v4_sys(void* p, uint4 v) {
+    asm volatile("st.relaxed.sys.global.v4.u32 [%0], {%1, %2, %3, %4};"
+                 :: "l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+__device__ __forceinline__ uint4 ld_v4_sys(const uint4* p) {
+    uint4 v;
+    asm volatile("ld.relaxed.sys.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+
+__device__ __forceinline__ unsigned block_tid() {
+    return threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
+}
+__device__ __forceinline__ unsigned block_threads() { return blockDim.x * blockDim.y * blockDim.z; }
+__device__ __forceinline__ unsigned block_linear() {
+    return blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+}
+
+/* ------------------------------------------------------------------ tracing (debug) */
+__device__ __forceinline__ void trace(const gsys_dev_ctx* c, unsigned s, unsigned seq, unsigned from,
+                                      unsigned to, bool blocking) {
+    if (c->trace == nullptr) return;
+    unsigned i = atomicAdd(c->trace_n, 1u);
+    if (i < c->trace_cap) {
+        gsys_trace_rec r;
+        r.slot = s; r.seq = seq; r.from = (uint8_t)from; r.to = (uint8_t)to; r.actor = 0;
+        r.blocking = blocking ? 1 : 0; r.pad = 0;
+        c->trace[i] = r;
+    }
+}
+
+/* ------------------------------------------------------------------ a2: claim
+ * The slot is chosen by the hardware ID of the calling thread (SM, hardware warp slot, lane),
+ * not the programmer-visible ID (PAPER.md:24 P24.2-6; reading A5).  Exclusivity comes from the
+ * cmp-swap on the device claim word (P24.46), so a stale %warpid can never double-book a slot;
+ * "If the slot is not free, system call invocation is delayed" (P24.11): spin with backoff. */
+__device__ __forceinline__ unsigned hw_slot(const gsys_dev_ctx* c) {
+    return ((smid() * 64u + warpid()) * 32u + laneid()) % c->nslots;
+}
+
+__device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, bool blocking) {
+    unsigned s = hw_slot(c);
+    unsigned ns = 32;
+    while (atomicCAS(&c->claim[s], 0u, 1u) != 0u) {
+        __nanosleep(ns);
+        if (ns < 1024) ns <<= 1;
+    }
+    __threadfence();   /* acquire the slot's previous owner's writes (seqs[s]) */
+    return s;
+}
+
+/* ------------------------------------------------------------------ a3: marshal
+ * args[0..5] as three 128-bit stores, then {nr, flags, seq, state=READY} as the fourth 128-bit
+ * store of the 64 B line (P24.12: "populates the slot ... and changes the state to ready";
+ * P24.13: the blocking bit travels in flags).  Returns the request's sequence number. */
+__device__ __forceinline__ unsigned marshal(const gsys_dev_ctx* c, unsigned s, unsigned nr, unsigned flags,
+                                            const unsigned long long a[6]) {
+    unsigned seq = c->seqs[s] + 1u;
+    if (seq == 0u) seq = 1u;
+    c->seqs[s] = seq;
+    trace(c, s, seq, GSYS_FREE, GSYS_POPULATING, !(flags & GSYS_NONBLOCKING));
+    uint4* line = reinterpret_cast<uint4*>(c->area + s);
+    st_v4_sys(line + 0, make_uint4((unsigned)a[0], (unsigned)(a[0] >> 32), (unsigned)a[1], (unsigned)(a[1] >> 32)));
+    st_v4_sys(line + 1, make_uint4((unsigned)a[2], (unsigned)(a[2] >> 32), (unsigned)a[3], (unsigned)(a[3] >> 32)));
+    st_v4_sys(line + 2, make_uint4((unsigned)a[4], (unsigned)(a[4] >> 32), (unsigned)a[5], (unsigned)(a[5] >> 32)));
+    st_v4_sys(line + 3, make_uint4(nr, flags, seq, (unsigned)GSYS_READY));
+    trace(c, s, seq, GSYS_POPULATING, GSYS_READY, !(flags & GSYS_NONBLOCKING));
+    return seq;
+}
+
+/* ------------------------------------------------------------------ a4: publish + doorbell
+ * __threadfence_system() orders the slot line before the doorbell entry; the entry position is
+ * taken with one warp-aggregated atomicAdd for all lanes of the warp calling together (the
+ * "scalar wavefront instruction" of P24.14).  Entry = (position+1) << 32 | slot, so the host
+ * recognises a fresh entry without the ring ever being cleared. */
+__device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
+    __threadfence_system();
+    unsigned mask = __activemask();
+    unsigned lane = laneid();
+    unsigned leader = __ffs(mask) - 1u;
+    unsigned base = 0;
+    if (lane == leader) base = atomicAdd(c->ring_tail, (unsigned)__popc(mask));
+    base = __shfl_sync(mask, base, leader);
+    unsigned pos = base + (unsigned)__popc(mask & lanemask_lt());
+    st_relaxed_sys(c->ring + (pos & c->ring_mask), ((unsigned long long)(pos + 1u) << 32) | s);
+}
+
+/* ------------------------------------------------------------------ a5: completion */
+__device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
+    const unsigned long long* m = c->mirror + s;
+    unsigned ns = 64;
+    unsigned long long v;
+    for (;;) {
+        v = ld_relaxed_sys(m);
+        if ((unsigned)(v >> 32) == seq) break;
+        __nanosleep(ns);
+        ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
+    }
+    fence_acq_rel_sys();   /* acquire: payload DMA'd before the completion word is visible */
+    return (long long)(int)(unsigned)(v & 0xffffffffull);
+}
+
+__device__ __forceinline__ void release(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
+    trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true);
+    st_release_gpu(&c->claim[s], 0u);      /* "consume the result" then free (reading A3) */
+}
+
+/* One thread, one request: claim -> marshal -> publish -> (poll).  Non-blocking requests keep
+ * the slot until the host frees it (P24.34).  inline_out: for GSYS_F_INLINE calls, where the
+ * host's inline payload is copied after completion (nbytes <= GSYS_INLINE_BYTES). */
+__device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned nr, unsigned flags,
+                                                 const unsigned long long a[6], void* inline_out = nullptr,
+                                                 unsigned inline_bytes = 0) {
+    const bool blocking = !(flags & GSYS_NONBLOCKING);
+    unsigned s = claim(c, blocking);
+    unsigned seq = marshal(c, s, nr, flags, a);
+    doorbell(c, s);
+    if (!blocking) return 0;
+    long long r = wait_done(c, s, seq);
+    if (inline_out != nullptr && r >= 0) {
+        const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
+        uint4* dst = reinterpret_cast<uint4*>(inline_out);
+        for (unsigned i = 0; i < inline_bytes / 16u; i++) dst[i] = ld_v4_sys(src + i);
+    }
+    release(c, s, seq);
+    return r;
+}
+
+/* ------------------------------------------------------------------ a1/a6: granularity + ordering
+ * Work-group (PAPER.md:22 P22.40-42): thread 0 is the designated caller; strong = barrier
+ * before and after; relaxed keeps the barrier before for consumer calls, after for producer
+ * calls.  The result reaches every thread through a shared-memory double buffer whose parity is
+ * broadcast by the Bar2 barrier itself (__syncthreads_or), so back-to-back calls never race.
+ * Relaxed consumer (Bar2 removed): the caller's warp waits with it and gets the result, the
+ * other warps proceed at once and get 0 (reading A17, P28.3). */
+__device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
+                                             const unsigned long long a[6], void* inline_out = nullptr,
+                                             unsigned inline_bytes = 0) {
+    __shared__ long long s_ret[2];
+    __shared__ unsigned s_par;
+    const bool strong = !(flags & GSYS_RELAXED);
+    const bool bar1 = strong || !producer;
+    const bool bar2 = strong || producer;
+    const unsigned tid = block_tid();
+    if (bar1) __syncthreads();
+    long long r = 0;
+    if (tid == 0) r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, inline_out, inline_bytes);
+    if (bar2) {
+        unsigned p = 0;
+        if (tid == 0) { p = (s_par ^ 1u) & 1u; s_par = p; s_ret[p] = r; }
+        p = (unsigned)__syncthreads_or(tid == 0 ? (int)p : 0);
+        return s_ret[p];
+    }
+    if (tid < 32) {
+        unsigned nt = block_threads();
+        unsigned m = nt >= 32 ? 0xffffffffu : ((1u << nt) - 1u);
+        r = __shfl_sync(m, r, 0);
+        return r;
+    }
+    return 0;
+}
+
+/* Work-item (P20.31 "work-item invocations imply strong ordering"): every calling lane issues
+ * its own request; the claim spins diverge, publication and the doorbell are warp-aggregated. */
+__device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
+                                             const unsigned long long a[6], void* inline_out = nullptr,
+                                             unsigned inline_bytes = 0) {
+    return call_thread(c, nr, (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u), a, inline_out,
+                       inline_bytes);
+}
+
+/* Kernel (P20.16-21, P20.33): relaxed only, -EINVAL for strong (reading A13).  Per call site and
+ * per round (the block's n-th call at that site) a record in device memory counts arrivals.
+ * Producer: the FIRST block to arrive calls (it is resident by definition, so nobody can wait
+ * on a block that was never scheduled) and the others wait for its result -- the kernel-scope
+ * "barrier after".  Consumer: the LAST block to arrive calls after every block published its
+ * data (the "barrier before"), and nobody waits.  Both are deadlock-free for grids larger than
+ * the co-resident capacity. */
+__device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
+                                                 const unsigned long long a[6], void* inline_out = nullptr,
+                                                 unsigned inline_bytes = 0) {
+    __shared__ long long s_kret[2];
+    __shared__ unsigned s_kpar;
+    if (!(flags & GSYS_RELAXED)) return -EINVAL;
+    const unsigned tid = block_tid();
+    const unsigned site = (flags >> 24) & (GSYS_KSITES - 1u);
+    const unsigned nb = gridDim.x * gridDim.y * gridDim.z;
+    const unsigned bid = block_linear();
+    if (!producer) __syncthreads();     /* block-level part of the barrier before */
+    long long r = 0;
+    if (tid == 0) {
+        if (bid >= c->kblock_cap) {
+            r = -ENOSPC;
+        } else {
+            unsigned* kb = c->kblock + (size_t)bid * GSYS_KSITES + site;
+            unsigned round = *kb;
+            *kb = round + 1u;
+            if (round >= GSYS_KROUNDS) {
+                r = -ENOSPC;
+            } else {
+                gsys_kround* k = c->krounds + (size_t)site * GSYS_KROUNDS + round;
+                if (producer) {
+                    unsigned t = atomicAdd(&k->arrive, 1u);
+                    if (t == 0u) {
+                        r = call_thread(c, nr, flags | GSYS_F_PRODUCER, a, inline_out, inline_bytes);
+                        k->ret = r;
+                        __threadfence();
+                        st_release_gpu(&k->done, 1u);
+                    } else {
+                        unsigned ns = 64;
+                        while (ld_acquire_gpu(&k->done) == 0u) { __nanosleep(ns); if (ns < 2048) ns <<= 1; }
+                        r = *(volatile long long*)&k->ret;
+                    }
+                } else {
+                    __threadfence();
+                    unsigned t = atomicAdd(&k->arrive, 1u);
+                    if (t == nb - 1u) {
+                        __threadfence();
+                        r = call_thread(c, nr, flags, a, inline_out, inline_bytes);
+                    }
+                }
+            }
+        }
+    }
+    if (producer) {
+        unsigned p = 0;
+        if (tid == 0) { p = (s_kpar ^ 1u) & 1u; s_kpar = p; s_kret[p] = r; }
+        p = (unsigned)__syncthreads_or(tid == 0 ? (int)p : 0);
+        return s_kret[p];
+    }
+    return tid == 0 ? r : 0;
+}
+
+__device__ __forceinline__ bool flags_valid(unsigned flags) {
+    unsigned g = flags & GSYS_GRAN_MASK;
+    return g == GSYS_WI || g == GSYS_WG || g == GSYS_KERNEL;
+}
+
+/* Dispatch on granularity.  Invalid granularity -> -EINVAL (uniform across the scope). */
+__device__ __forceinline__ long long invoke(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
+                                            const unsigned long long a[6], void* inline_out = nullptr,
+                                            unsigned inline_bytes = 0) {
+    switch (flags & GSYS_GRAN_MASK) {
+        case GSYS_WI: return wi_call(c, nr, flags, producer, a, inline_out, inline_bytes);
+        case GSYS_WG: return wg_call(c, nr, flags, producer, a, inline_out, inline_bytes);
+        case GSYS_KERNEL: return kernel_call(c, nr, flags, producer, a, inline_out, inline_bytes);
+        default: return -EINVAL;
+    }
+}
+
+}  // namespace gsys
+
+/* ------------------------------------------------------------------ POSIX-shaped wrappers
+ * Signatures follow POSIX plus the trailing GENESYS flags (P20.31-33).  Blocking calls return the
+ * raw-syscall convention (>= 0, or -errno); non-blocking calls return 0 once published and report
+ * errors at gsys_wait() (reading A4).  Producer (read-like) vs consumer (write-like) class per
+ * P20.24-29; madvise and rt_sigqueueinfo are consumers (reading A7). */
+__device__ __forceinline__ long long gsys_pread(const gsys_dev_ctx* c, int fd, void* buf, size_t n, long long off,
+                                                unsigned gflags) {
+    unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
+                               (unsigned long long)off, 0ull, 0ull};
+    return gsys::invoke(c, GSYS_NR_PREAD64, gflags, true, a);
+}
+__device__ __forceinline__ long long gsys_pwrite(const gsys_dev_ctx* c, int fd, const void* buf, size_t n,
+                                                 long long off, unsigned gflags) {
+    unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
+                               (unsigned long long)off, 0ull, 0ull};
+    return gsys::invoke(c, GSYS_NR_PWRITE64, gflags, false, a);
+}
+/* getrusage: blocking calls land the 144 B struct rusage in the slot's inline line and the
+ * caller copies it to `ru` (any GPU-visible pointer); non-blocking calls hand `ru` to the host. */
+__device__ __forceinline__ long long gsys_getrusage(const gsys_dev_ctx* c, int who, void* ru, unsigned gflags) {
+    bool blocking = !(gflags & GSYS_NONBLOCKING);
+    unsigned long long a[6] = {(unsigned long long)(long long)who, (unsigned long long)ru, 0ull, 0ull, 0ull, 0ull};
+    return gsys::invoke(c, GSYS_NR_GETRUSAGE, gflags | (blocking && ru ? GSYS_F_INLINE : 0u), true, a,
+                        blocking ? ru : nullptr, 144u);
+}
+__device__ __forceinline__ long long gsys_madvise(const gsys_dev_ctx* c, void* addr, size_t len, int advice,
+                                                  unsigned gflags) {
+    unsigned long long a[6] = {(unsigned long long)addr, (unsigned long long)len, (unsigned long long)(long long)advice,
+                               0ull, 0ull, 0ull};
+    return gsys::invoke(c, GSYS_NR_MADVISE, gflags, false, a);
+}
+__device__ __forceinline__ long long gsys_sendto(const gsys_dev_ctx* c, int fd, const void* buf, size_t n, int flags,
+                                                 const void* to, unsigned tolen, unsigned gflags) {
+    unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
+                               (unsigned long long)(long long)flags, (unsigned long long)to, (unsigned long long)tolen};
+    return gsys::invoke(c, GSYS_NR_SENDTO, gflags, false, a);
+}
+__device__ __forceinline__ long long gsys_recvfrom(const gsys_dev_ctx* c, int fd, void* buf, size_t n, int flags,
+                                                   void* from, unsigned* fromlen, unsigned gflags) {
+    unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
+                               (unsigned long long)(long long)flags, (unsigned long long)from,
+                               (unsigned long long)fromlen};
+    return gsys::invoke(c, GSYS_NR_RECVFROM, gflags, true, a);
+}
+__device__ __forceinline__ long long gsys_rt_sigqueueinfo(const gsys_dev_ctx* c, int tgid, int sig, const void* info,
+                                                          unsigned gflags) {
+    unsigned long long a[6] = {(unsigned long long)(long long)tgid, (unsigned long long)(long long)sig,
+                               (unsigned long long)info, 0ull, 0ull, 0ull};
+    return gsys::invoke(c, GSYS_NR_RT_SIGQUEUEINFO, gflags, false, a);
+}
+
+#endif /* __CUDACC__ */
+#endif /* GSYS_DEVICE_CUH */

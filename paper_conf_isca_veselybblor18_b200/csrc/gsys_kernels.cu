@@ -1,0 +1,444 @@
+// gsys_kernels.cu -- sm_100a kernels of the hot path and their C-ABI launchers.
+//
+//   wc_kernel     wordcount + grep -F -l over files read with work-group preads issued from the
+//                 GPU (sec. VIII-C, P32.3-9: "search for occurrences of 64 strings",
+//                 "work-group granularity with blocking and weak-ordering"; PAPER.md:30 P30.27-38
+//                 grep -F -l).  Each work-group loops over 256 KiB chunks: gsys_pread of the
+//                 chunk + halo into its device staging line, then the scan (row a8).
+//   scan_kernel   the same scan over text already in HBM (standalone HBM-roofline measurement).
+//   bench_kernel  granularity x blocking x ordering microbenchmark (sec. VII).
+//
+// Scan (reading A9/A10): a token is a maximal run of [A-Za-z0-9_]; it is owned by the chunk that
+// holds its first byte; a dictionary hit is a whole token byte-equal to one of <= 64 words of
+// <= 16 bytes.  Each thread takes 16 aligned bytes per step plus the next 16 as lookahead
+// (coalesced uint4 loads), classifies all 32 bytes with SWAR into a word-byte bitmask, derives
+// token starts from it, and for each start extracts the <= 16 byte token with a funnel-shift
+// network, filters by length and a perfect hash (smem), verifies with one 128-bit compare and
+// counts into a per-warp shared-memory histogram.  grep tests every owned position whose byte
+// is in the first-byte range of the patterns.  No tensor cores: nothing here is a contraction.
+
+#include <cuda_runtime.h>
+#include <errno.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <mutex>
+#include <vector>
+
+#include "gsys.h"
+#include "gsys_device.cuh"
+#include "gsys_internal.h"
+#include "scan_core.cuh"
+
+namespace {
+
+using namespace gsys_scan;
+
+struct ScanState {
+    const ScanTables* T;   // shared memory
+    unsigned* whist;       // this warp's shared histogram [64]
+    int* hit;              // shared grep-hit flag of the current chunk (nullptr: no grep)
+};
+
+// Scan positions [s, own_end) of a text whose valid bytes end at valid_end; seg0 points at the
+// byte of position s (16-byte aligned); seg0[-1] is the byte before s when s > 0.  Thread t takes
+// the 16-byte steps t, t + blockDim, ... (coalesced uint4 loads; the lookahead B is the next
+// thread's A and is served by L1).
+__device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg0, long long s, long long own_end,
+                                           long long valid_end, const ScanState& S) {
+    const ScanTables& T = *S.T;
+    const bool grep = S.hit != nullptr && T.npat > 0;
+    unsigned* wh = S.whist;
+    for (long long p0 = s + 16ll * threadIdx.x; p0 < own_end; p0 += 16ll * blockDim.x) {
+        const unsigned char* q = seg0 + (p0 - s);
+        const uint4 A = *reinterpret_cast<const uint4*>(q);
+        const uint4 B = (p0 + 16 < valid_end) ? *reinterpret_cast<const uint4*>(q + 16) : make_uint4(0, 0, 0, 0);
+        const unsigned prevb = p0 > 0 ? q[-1] : 0u;
+        const bool g = grep && !*(volatile int*)S.hit;
+        if (scan_step(T, A, B, prevb, p0, own_end, valid_end, g, [wh](unsigned d) { atomicAdd(&wh[d], 1u); }))
+            *S.hit = 1;
+    }
+}
+
+__device__ __forceinline__ void load_tables(ScanTables* sT, const ScanTables* gT) {
+    const unsigned* src = reinterpret_cast<const unsigned*>(gT);
+    unsigned* dst = reinterpret_cast<unsigned*>(sT);
+    for (unsigned i = threadIdx.x; i < sizeof(ScanTables) / 4; i += blockDim.x) dst[i] = src[i];
+}
+
+__device__ __forceinline__ void flush_hist(unsigned* shist, unsigned nwarps, unsigned ndict, unsigned long long* hist) {
+    for (unsigned d = threadIdx.x; d < ndict; d += blockDim.x) {
+        unsigned long long sum = 0;
+        for (unsigned w = 0; w < nwarps; w++) sum += shist[w * MAXD + d];
+        if (sum) atomicAdd(hist + d, sum);
+    }
+}
+
+// ------------------------------------------------------------------ wordcount with GPU-issued preads
+struct WcArgs {
+    const gsys_dev_ctx* ctx;
+    const ScanTables* tables;
+    const int* fds;
+    const unsigned long long* sizes;
+    const unsigned* chunk_base;     // [nfiles + 1] first global chunk of each file
+    unsigned char* staging;         // [gridDim.x * stride]
+    unsigned long long* hist;
+    unsigned* file_hits;
+    long long* req_ret;
+    unsigned nfiles, nchunks, chunk, stride, gflags, pad_;
+};
+
+__global__ void __launch_bounds__(1024) wc_kernel(WcArgs a) {
+    __shared__ ScanTables sT;
+    __shared__ int s_hit;
+    extern __shared__ unsigned shist[];
+    const unsigned nwarps = blockDim.x / 32;
+    load_tables(&sT, a.tables);
+    for (unsigned i = threadIdx.x; i < nwarps * MAXD; i += blockDim.x) shist[i] = 0;
+    __syncthreads();
+    unsigned char* base = a.staging + (size_t)blockIdx.x * a.stride;
+    ScanState S;
+    S.T = &sT;
+    S.whist = shist + (threadIdx.x / 32) * MAXD;
+    for (unsigned k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
+        unsigned lo = 0, hi = a.nfiles;     // largest f with chunk_base[f] <= k
+        while (hi - lo > 1) {
+            unsigned mid = (lo + hi) >> 1;
+            if (a.chunk_base[mid] <= k) lo = mid; else hi = mid;
+        }
+        const unsigned f = lo;
+        const long long size = (long long)a.sizes[f];
+        const long long s = (long long)(k - a.chunk_base[f]) * a.chunk;
+        const long long e = s + a.chunk < size ? s + a.chunk : size;
+        const long long off = s ? s - 1 : 0;
+        const long long len = e + 16 - off;
+        unsigned char* dst = base + 16 - (s - off);
+        const bool grep = a.file_hits != nullptr && sT.npat > 0 && *(volatile unsigned*)&a.file_hits[f] == 0u;
+        if (threadIdx.x == 0) s_hit = 0;
+        // row a1-a6: one work-group pread of the chunk + halo (P32.7)
+        const long long r = gsys_pread(a.ctx, a.fds[f], dst, (size_t)len, off, a.gflags);
+        if (threadIdx.x == 0 && a.req_ret) a.req_ret[k] = r;
+        if (r > 0) {
+            const long long valid_end = off + r;
+            const long long own_end = e < valid_end ? e : valid_end;
+            S.hit = grep ? &s_hit : nullptr;
+            if (own_end > s) scan_range(base + 16, s, own_end, valid_end, S);
+        }
+        __syncthreads();   // the staging line is free again before the next chunk's pread
+        if (threadIdx.x == 0 && grep && s_hit) atomicExch(&a.file_hits[f], 1u);
+    }
+    __syncthreads();
+    flush_hist(shist, nwarps, sT.ndict, a.hist);
+}
+
+// ------------------------------------------------------------------ scan of HBM-resident text
+struct ScanArgs {
+    const ScanTables* tables;
+    const unsigned char* text;
+    unsigned long long n;
+    unsigned long long* hist;
+    unsigned* hit;
+    unsigned long long nchunks;
+    unsigned chunk, pad_;
+};
+
+__global__ void __launch_bounds__(1024) scan_kernel(ScanArgs a) {
+    __shared__ ScanTables sT;
+    __shared__ int s_hit;
+    extern __shared__ unsigned shist[];
+    const unsigned nwarps = blockDim.x / 32;
+    load_tables(&sT, a.tables);
+    for (unsigned i = threadIdx.x; i < nwarps * MAXD; i += blockDim.x) shist[i] = 0;
+    if (threadIdx.x == 0) s_hit = 0;
+    __syncthreads();
+    ScanState S;
+    S.T = &sT;
+    S.whist = shist + (threadIdx.x / 32) * MAXD;
+    S.hit = a.hit ? &s_hit : nullptr;
+    for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
+        const long long s = (long long)k * a.chunk;
+        const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
+        scan_range(a.text + s, s, e, (long long)a.n, S);
+    }
+    __syncthreads();
+    flush_hist(shist, nwarps, sT.ndict, a.hist);
+    if (threadIdx.x == 0 && a.hit && s_hit) atomicExch(a.hit, 1u);
+}
+
+// ------------------------------------------------------------------ granularity microbenchmark
+struct BenchArgs {
+    const gsys_dev_ctx* ctx;
+    unsigned char* buf;
+    long long* ret;
+    unsigned long long* lat;
+    unsigned long long* sum;
+    unsigned long long len, size;
+    int fd;
+    unsigned kind, gflags, iters;
+};
+
+__device__ __forceinline__ unsigned char pw_byte(unsigned long long idx, unsigned long long i) {
+    return (unsigned char)((idx * 131ull + i * 7ull + 13ull) & 0xffull);
+}
+
+// Byte sum of buf[0, n) by the threads of the calling scope (WI: the thread alone; WG: the block;
+// KERNEL: every block sums the whole region).  Returned to thread 0 of the block (WG/KERNEL).
+__device__ unsigned long long scope_sum(const unsigned char* b, unsigned long long n, bool wi) {
+    __shared__ unsigned long long s_acc;
+    if (wi) {
+        unsigned long long acc = 0;
+        for (unsigned long long i = 0; i < n; i++) acc += b[i];
+        return acc;
+    }
+    if (threadIdx.x == 0) s_acc = 0;
+    __syncthreads();
+    unsigned long long acc = 0;
+    for (unsigned long long i = threadIdx.x; i < n; i += blockDim.x) acc += b[i];
+    atomicAdd(&s_acc, acc);
+    __syncthreads();
+    unsigned long long r = s_acc;
+    __syncthreads();
+    return r;
+}
+
+__global__ void bench_kernel(BenchArgs a) {
+    const unsigned gran = a.gflags & GSYS_GRAN_MASK;
+    const unsigned tid = threadIdx.x;
+    const bool wi = gran == GSYS_WI;
+    unsigned long long caller;
+    bool recorder;
+    if (wi) { caller = (unsigned long long)blockIdx.x * blockDim.x + tid; recorder = true; }
+    else if (gran == GSYS_WG) { caller = blockIdx.x; recorder = tid == 0; }
+    else { caller = 0; recorder = blockIdx.x == 0 && tid == 0; }
+    alignas(16) unsigned char ru[160];
+    for (unsigned r = 0; r < a.iters; r++) {
+        const unsigned long long idx = caller * a.iters + r;
+        const unsigned long long off = a.size ? (idx * a.len) % a.size : 0;
+        unsigned char* b = a.buf ? a.buf + caller * a.len : nullptr;
+        if (a.kind == 2) {
+            // produce the payload: every thread of the scope writes its share, late threads first
+            // spin, so a call issued without the pre-call barrier would publish stale bytes
+            unsigned long long t_end = gsys::globaltimer() + (tid % 7) * 3000ull;
+            while (gsys::globaltimer() < t_end) {}
+            if (wi) {
+                for (unsigned long long i = 0; i < a.len; i++) b[i] = pw_byte(idx, i);
+            } else {
+                unsigned long long nthr = blockDim.x, start = tid;
+                if (gran == GSYS_KERNEL) { nthr *= gridDim.x; start += (unsigned long long)blockIdx.x * blockDim.x; }
+                for (unsigned long long i = start; i < a.len; i += nthr) b[i] = pw_byte(idx, i);
+            }
+        }
+        const unsigned long long t0 = gsys::globaltimer();
+        long long rv;
+        if (a.kind == 0) rv = gsys_getrusage(a.ctx, 0 /* RUSAGE_SELF */, ru, a.gflags);
+        else if (a.kind == 1) rv = gsys_pread(a.ctx, a.fd, b, (size_t)a.len, (long long)off, a.gflags);
+        else rv = gsys_pwrite(a.ctx, a.fd, b, (size_t)a.len, (long long)off, a.gflags);
+        const unsigned long long t1 = gsys::globaltimer();
+        unsigned long long sum = 0;
+        if (a.kind == 1 && a.sum && !(a.gflags & GSYS_NONBLOCKING)) {
+            const unsigned long long n = rv > 0 ? (unsigned long long)rv : 0ull;
+            sum = scope_sum(b, n, wi);
+        }
+        if (recorder) {
+            if (a.ret) a.ret[idx] = rv;
+            if (a.lat) a.lat[idx] = t1 - t0;
+            if (a.kind == 1 && a.sum) a.sum[idx] = sum;
+        }
+        if (a.kind == 2 && !wi && !(a.gflags & GSYS_NONBLOCKING) && !(a.gflags & GSYS_RELAXED)) {
+            // strong consumer: Bar2 already separates the call from the next iteration's writes
+        } else if (a.kind == 2) {
+            // relaxed / non-blocking consumer: the buffer may still be read by the host; the
+            // benchmark writes the next payload only after the scope's own call returned
+            __syncthreads();
+        }
+    }
+}
+
+// ------------------------------------------------------------------ host side: tables + workspace
+struct Workspace {
+    unsigned char* up_h = nullptr;   // pinned upload staging
+    unsigned char* up_d = nullptr;
+    size_t up_cap = 0;
+    cudaEvent_t up_ev = nullptr;
+    unsigned char* staging_d = nullptr;
+    size_t staging_cap = 0;
+    int sms = 0;
+};
+Workspace g_ws[64];
+std::mutex g_ws_mu;
+
+Workspace* workspace() {
+    int d = 0;
+    if (cudaGetDevice(&d) != cudaSuccess || d < 0 || d >= 64) return nullptr;
+    Workspace* W = &g_ws[d];
+    if (!W->up_ev) {
+        cudaEventCreateWithFlags(&W->up_ev, cudaEventDisableTiming);
+        cudaDeviceGetAttribute(&W->sms, cudaDevAttrMultiProcessorCount, d);
+    }
+    return W;
+}
+
+int ensure_upload(Workspace* W, size_t bytes) {
+    cudaEventSynchronize(W->up_ev);   // the previous upload has left the pinned staging
+    if (bytes <= W->up_cap) return 0;
+    size_t cap = 1 << 16;
+    while (cap < bytes) cap <<= 1;
+    if (W->up_h) cudaFreeHost(W->up_h);
+    if (W->up_d) { cudaDeviceSynchronize(); cudaFree(W->up_d); }
+    W->up_h = nullptr; W->up_d = nullptr; W->up_cap = 0;
+    if (cudaHostAlloc((void**)&W->up_h, cap, cudaHostAllocDefault) != cudaSuccess) return -ENOMEM;
+    if (cudaMalloc((void**)&W->up_d, cap) != cudaSuccess) return -ENOMEM;
+    W->up_cap = cap;
+    return 0;
+}
+
+int ensure_staging(Workspace* W, size_t bytes) {
+    if (bytes <= W->staging_cap) return 0;
+    if (W->staging_d) { cudaDeviceSynchronize(); cudaFree(W->staging_d); }
+    W->staging_d = nullptr; W->staging_cap = 0;
+    if (cudaMalloc((void**)&W->staging_d, bytes) != cudaSuccess) return -ENOMEM;
+    W->staging_cap = bytes;
+    return 0;
+}
+
+int map_cuda(cudaError_t e) {
+    if (e == cudaSuccess) return 0;
+    if (e == cudaErrorMemoryAllocation) return -ENOMEM;
+    if (e == cudaErrorInvalidValue || e == cudaErrorInvalidConfiguration) return -EINVAL;
+    return -EIO;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+}  // namespace
+
+extern "C" {
+
+int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, uint32_t chunk, const char* dict,
+                   const uint8_t* dlen, uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat,
+                   uint64_t* d_hist, uint32_t* d_file_hits, int64_t* d_req_ret, uint32_t gflags, uint32_t blocks,
+                   uint32_t threads, void* stream) {
+    gsys_dev_ctx* ctx = gsys_internal_ctx_d();
+    if (!ctx) return -ENODEV;
+    if ((gflags & GSYS_GRAN_MASK) != GSYS_WG || (gflags & GSYS_NONBLOCKING)) return -EINVAL;
+    if (nfiles == 0 || !fds || !sizes || !d_hist) return -EINVAL;
+    if (chunk < 4096 || (chunk % 16) || chunk > (1u << 30)) return -EINVAL;
+    if (threads == 0) threads = 256;
+    if (threads % 32 || threads > 1024) return -EINVAL;
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    Workspace* W = workspace();
+    if (!W) return -ENODEV;
+    // chunk table
+    std::vector<unsigned> cbase(nfiles + 1);
+    uint64_t nch = 0;
+    for (uint32_t f = 0; f < nfiles; f++) {
+        cbase[f] = (unsigned)nch;
+        nch += (sizes[f] + chunk - 1) / chunk;
+        if (nch >= (1ull << 32)) return -EINVAL;
+    }
+    cbase[nfiles] = (unsigned)nch;
+    if (blocks == 0) blocks = 4u * (uint32_t)W->sms;
+    if (nch < blocks) blocks = (uint32_t)(nch ? nch : 1);
+    // upload: [tables][fds][sizes][cbase]
+    size_t o_t = 0, o_f = align_up(sizeof(ScanTables), 256), o_s = align_up(o_f + 4ull * nfiles, 256),
+           o_c = align_up(o_s + 8ull * nfiles, 256), total = align_up(o_c + 4ull * (nfiles + 1), 256);
+    int rc = ensure_upload(W, total);
+    if (rc) return rc;
+    rc = build_tables(reinterpret_cast<ScanTables*>(W->up_h + o_t), dict, dlen, ndict, pats, plen, npat);
+    if (rc) return rc;
+    memcpy(W->up_h + o_f, fds, 4ull * nfiles);
+    memcpy(W->up_h + o_s, sizes, 8ull * nfiles);
+    memcpy(W->up_h + o_c, cbase.data(), 4ull * (nfiles + 1));
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
+    cudaEventRecord(W->up_ev, s);
+    size_t stride = align_up((size_t)chunk + 64, 256);
+    rc = ensure_staging(W, stride * blocks);
+    if (rc) return rc;
+    WcArgs a;
+    memset(&a, 0, sizeof a);
+    a.ctx = ctx;
+    a.tables = reinterpret_cast<const ScanTables*>(W->up_d + o_t);
+    a.fds = reinterpret_cast<const int*>(W->up_d + o_f);
+    a.sizes = reinterpret_cast<const unsigned long long*>(W->up_d + o_s);
+    a.chunk_base = reinterpret_cast<const unsigned*>(W->up_d + o_c);
+    a.staging = W->staging_d;
+    a.hist = reinterpret_cast<unsigned long long*>(d_hist);
+    a.file_hits = d_file_hits;
+    a.req_ret = reinterpret_cast<long long*>(d_req_ret);
+    a.nfiles = nfiles;
+    a.nchunks = (unsigned)nch;
+    a.chunk = chunk;
+    a.stride = (unsigned)stride;
+    a.gflags = gflags;
+    if (nch == 0) return 0;
+    void* args[] = {&a};
+    size_t smem = (threads / 32) * MAXD * 4;
+    return gsys_launch((const void*)wc_kernel, blocks, 1, 1, threads, 1, 1, args, smem, stream);
+}
+
+int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const char* dict, const uint8_t* dlen,
+                     uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, uint64_t* d_hist,
+                     uint32_t* d_hit, uint32_t blocks, uint32_t threads, void* stream) {
+    if (!d_hist || (n && !d_text)) return -EINVAL;
+    if (chunk < 16 || chunk % 16) return -EINVAL;
+    if ((uintptr_t)d_text % 16) return -EINVAL;
+    if (threads == 0) threads = 256;
+    if (threads % 32 || threads > 1024) return -EINVAL;
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    Workspace* W = workspace();
+    if (!W) return -ENODEV;
+    size_t total = align_up(sizeof(ScanTables), 256);
+    int rc = ensure_upload(W, total);
+    if (rc) return rc;
+    rc = build_tables(reinterpret_cast<ScanTables*>(W->up_h), dict, dlen, ndict, pats, plen, npat);
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
+    cudaEventRecord(W->up_ev, s);
+    unsigned long long nch = (n + chunk - 1) / chunk;
+    if (nch == 0) return 0;
+    if (blocks == 0) blocks = 4u * (uint32_t)W->sms;
+    if (nch < blocks) blocks = (uint32_t)nch;
+    ScanArgs a;
+    memset(&a, 0, sizeof a);
+    a.tables = reinterpret_cast<const ScanTables*>(W->up_d);
+    a.text = d_text;
+    a.n = n;
+    a.hist = reinterpret_cast<unsigned long long*>(d_hist);
+    a.hit = d_hit;
+    a.nchunks = nch;
+    a.chunk = chunk;
+    size_t smem = (threads / 32) * MAXD * 4;
+    scan_kernel<<<blocks, threads, smem, s>>>(a);
+    return map_cuda(cudaGetLastError());
+}
+
+int gsys_bench_calls(uint32_t kind, uint32_t gflags, uint32_t blocks, uint32_t threads, uint32_t iters, int32_t fd,
+                     uint64_t len, uint64_t size, void* d_buf, int64_t* d_ret, uint64_t* d_lat_ns, uint64_t* d_sum,
+                     void* stream) {
+    gsys_dev_ctx* ctx = gsys_internal_ctx_d();
+    if (!ctx) return -ENODEV;
+    if (kind > 2 || blocks == 0 || threads == 0 || threads > 1024 || iters == 0) return -EINVAL;
+    if (kind >= 1 && (size == 0 || len == 0 || !d_buf)) return -EINVAL;
+    BenchArgs a;
+    memset(&a, 0, sizeof a);
+    a.ctx = ctx;
+    a.buf = (unsigned char*)d_buf;
+    a.ret = reinterpret_cast<long long*>(d_ret);
+    a.lat = reinterpret_cast<unsigned long long*>(d_lat_ns);
+    a.sum = reinterpret_cast<unsigned long long*>(d_sum);
+    a.len = len;
+    a.size = size ? size : 1;
+    a.fd = fd;
+    a.kind = kind;
+    a.gflags = gflags;
+    a.iters = iters;
+    void* args[] = {&a};
+    int rc = gsys_launch((const void*)bench_kernel, blocks, 1, 1, threads, 1, 1, args, 0, stream);
+    if (rc) return rc;
+    unsigned g = gflags & GSYS_GRAN_MASK;
+    return g == GSYS_WI ? (int)(blocks * threads) : g == GSYS_WG ? (int)blocks : 1;
+}
+
+}  // extern "C"

@@ -1,0 +1,250 @@
+"""Thin ctypes binding of libgsys (include/gsys.h).  Argument marshalling only: every step of the
+hot path runs in the library's C++ service and sm_100a kernels.  The library must exist (built by
+``build()``); there is no CPU fallback -- a missing extension raises.
+
+PyTorch is used only for device memory (tensor.data_ptr()) and streams (cuda_stream handles).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from . import build as _build
+
+WI, WG, KERNEL = 0x01, 0x02, 0x04
+BLOCKING, NONBLOCKING = 0x00, 0x08
+STRONG, RELAXED = 0x00, 0x10
+WEAK = RELAXED
+FREE, POPULATING, READY, PROCESSING, FINISHED = 0, 1, 2, 3, 4
+NR_PREAD64, NR_PWRITE64, NR_GETRUSAGE = 17, 18, 98
+
+
+def SITE(k: int) -> int:
+    return (k & 63) << 24
+
+
+class GsysError(OSError):
+    pass
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [("requests", ctypes.c_uint64), ("completed", ctypes.c_uint64), ("bundles", ctypes.c_uint64),
+                ("max_bundle", ctypes.c_uint64), ("host_preads", ctypes.c_uint64), ("merged", ctypes.c_uint64),
+                ("bytes_read", ctypes.c_uint64), ("bytes_h2d", ctypes.c_uint64), ("errors", ctypes.c_uint64),
+                ("per_nr", ctypes.c_uint64 * 8), ("threads", ctypes.c_uint32), ("slots", ctypes.c_uint32),
+                ("coalesce_max", ctypes.c_uint32), ("coalesce_window_us", ctypes.c_uint32)]
+
+    def as_dict(self):
+        d = {k: getattr(self, k) for k, _ in self._fields_ if k != "per_nr"}
+        d["per_nr"] = dict(zip(["pread", "pwrite", "madvise", "sendto", "recvfrom", "getrusage", "sigqueue",
+                                "other"], list(self.per_nr)))
+        return d
+
+
+class TraceRec(ctypes.Structure):
+    _fields_ = [("slot", ctypes.c_uint32), ("seq", ctypes.c_uint32), ("frm", ctypes.c_uint8),
+                ("to", ctypes.c_uint8), ("actor", ctypes.c_uint8), ("blocking", ctypes.c_uint8),
+                ("pad", ctypes.c_uint32)]
+
+
+_P = ctypes.c_void_p
+_U32 = ctypes.c_uint32
+_U64 = ctypes.c_uint64
+_I32 = ctypes.c_int32
+_I64 = ctypes.c_int64
+
+# name -> (restype, argtypes); mirrors include/gsys.h
+SIGNATURES = {
+    "gsys_init": (ctypes.c_int, [_U32, _U32]),
+    "gsys_set_coalesce_max": (ctypes.c_int, [_U32]),
+    "gsys_set_coalesce_window": (ctypes.c_int, [_U32]),
+    "gsys_set_merge": (ctypes.c_int, [ctypes.c_int]),
+    "gsys_set_trace": (ctypes.c_int, [ctypes.c_int, _U32]),
+    "gsys_launch": (ctypes.c_int, [_P, _U32, _U32, _U32, _U32, _U32, _U32, _P, ctypes.c_size_t, _P]),
+    "gsys_wait": (ctypes.c_int, [_P]),
+    "gsys_shutdown": (ctypes.c_int, []),
+    "gsys_device_ctx": (_P, []),
+    "gsys_stats": (ctypes.c_int, [_P]),
+    "gsys_stats_reset": (ctypes.c_int, []),
+    "gsys_trace_read": (ctypes.c_int, [_P, _U32, _P, _P, _U32, _P]),
+    "gsys_abi_info": (ctypes.c_int, [_P, _P, _P]),
+    "gsys_plan_merge": (ctypes.c_int, [_U32, _P, _P, _P, _U64, _P, _P, _P, _P, _P]),
+    "gsys_split_result": (_I64, [_I64, _U64, _U64]),
+    "gsys_wordcount": (ctypes.c_int, [_P, _P, _U32, _U32, ctypes.c_char_p, _P, _U32, ctypes.c_char_p, _P, _U32,
+                                      _P, _P, _P, _U32, _U32, _U32, _P]),
+    "gsys_scan_device": (ctypes.c_int, [_P, _U64, _U32, ctypes.c_char_p, _P, _U32, ctypes.c_char_p, _P, _U32,
+                                        _P, _P, _U32, _U32, _P]),
+    "gsys_bench_calls": (ctypes.c_int, [_U32, _U32, _U32, _U32, _U32, _I32, _U64, _U64, _P, _P, _P, _P, _P]),
+}
+
+_lib = None
+
+
+def lib():
+    """Load libgsys.so (building it in-tree if stale).  Raises if it cannot be built/loaded."""
+    global _lib
+    if _lib is None:
+        path = _build.LIB
+        if not os.path.exists(path) or os.environ.get("GSYS_REBUILD"):
+            _build.build()
+        L = ctypes.CDLL(path)
+        for name, (res, args) in SIGNATURES.items():
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    return _lib
+
+
+def _check(rc: int, what: str) -> int:
+    if rc < 0:
+        raise GsysError(-rc, f"{what}: {os.strerror(-rc)}")
+    return rc
+
+
+def _stream(stream) -> int | None:
+    if stream is None:
+        return None
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def gsys_init(slots: int = 0, coalesce_window_us: int = 0) -> int:
+    return _check(lib().gsys_init(slots, coalesce_window_us), "gsys_init")
+
+
+def gsys_set_coalesce_max(n: int) -> int:
+    return _check(lib().gsys_set_coalesce_max(n), "gsys_set_coalesce_max")
+
+
+def gsys_set_coalesce_window(us: int) -> int:
+    return _check(lib().gsys_set_coalesce_window(us), "gsys_set_coalesce_window")
+
+
+def gsys_set_merge(on: bool) -> int:
+    return _check(lib().gsys_set_merge(int(bool(on))), "gsys_set_merge")
+
+
+def gsys_set_trace(on: bool, capacity: int = 0) -> int:
+    return _check(lib().gsys_set_trace(int(bool(on)), capacity), "gsys_set_trace")
+
+
+def gsys_wait(stream=None) -> int:
+    """Drain: returns the first non-blocking -errno (or 0); raises only on CUDA errors."""
+    rc = lib().gsys_wait(_stream(stream))
+    if rc < 0 and -rc in (5,):   # EIO from CUDA
+        raise GsysError(-rc, "gsys_wait")
+    return rc
+
+
+def gsys_shutdown() -> int:
+    return lib().gsys_shutdown()
+
+
+def gsys_device_ctx() -> int:
+    return lib().gsys_device_ctx() or 0
+
+
+def gsys_stats() -> dict:
+    s = Stats()
+    _check(lib().gsys_stats(ctypes.byref(s)), "gsys_stats")
+    return s.as_dict()
+
+
+def gsys_stats_reset() -> int:
+    return _check(lib().gsys_stats_reset(), "gsys_stats_reset")
+
+
+def gsys_trace_read(cap: int = 1 << 20):
+    g = (TraceRec * cap)()
+    h = (TraceRec * cap)()
+    ng = ctypes.c_uint32(0)
+    nh = ctypes.c_uint32(0)
+    _check(lib().gsys_trace_read(g, cap, ctypes.byref(ng), h, cap, ctypes.byref(nh)), "gsys_trace_read")
+    conv = lambda arr, n: [(r.slot, r.seq, r.frm, r.to, "gpu" if r.actor == 0 else "cpu", bool(r.blocking))  # noqa: E731
+                           for r in arr[: min(n, cap)]]
+    return conv(g, ng.value), conv(h, nh.value)
+
+
+def gsys_abi_info():
+    a, b, c = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
+    lib().gsys_abi_info(ctypes.byref(a), ctypes.byref(b), ctypes.byref(c))
+    return a.value, b.value, c.value
+
+
+def gsys_plan_merge(fds, offs, lens, max_union: int):
+    import numpy as np
+    n = len(fds)
+    fd = np.asarray(fds, dtype=np.int32)
+    off = np.asarray(offs, dtype=np.int64)
+    ln = np.asarray(lens, dtype=np.uint64)
+    order = np.zeros(n, dtype=np.uint32)
+    group = np.zeros(n, dtype=np.uint32)
+    oig = np.zeros(n, dtype=np.uint64)
+    goff = np.zeros(max(n, 1), dtype=np.int64)
+    glen = np.zeros(max(n, 1), dtype=np.uint64)
+    ng = _check(lib().gsys_plan_merge(n, fd.ctypes.data, off.ctypes.data, ln.ctypes.data, max_union,
+                                      order.ctypes.data, group.ctypes.data, oig.ctypes.data, goff.ctypes.data,
+                                      glen.ctypes.data), "gsys_plan_merge")
+    return order, group, oig, goff[:ng], glen[:ng]
+
+
+def gsys_split_result(r: int, offset_in_group: int, length: int) -> int:
+    return lib().gsys_split_result(r, offset_in_group, length)
+
+
+def pack_words(words):
+    buf = bytearray(17 * len(words))
+    lens = (ctypes.c_uint8 * max(len(words), 1))()
+    for i, w in enumerate(words):
+        if not 1 <= len(w) <= 16:
+            raise ValueError("words must be 1..16 bytes")
+        buf[17 * i: 17 * i + len(w)] = w
+        lens[i] = len(w)
+    return bytes(buf), lens
+
+
+def gsys_wordcount(fds, sizes, chunk: int, dict_words, patterns, d_hist, d_file_hits=None, d_req_ret=None,
+                   gflags: int = WG | BLOCKING | STRONG, blocks: int = 0, threads: int = 0, stream=None) -> int:
+    """Launch the GPU-syscall wordcount/grep (asynchronous; gsys_wait(stream) before reading).
+    d_hist: device uint64 tensor [ndict] (added into); d_file_hits: device int32 [nfiles] or None;
+    d_req_ret: device int64 [chunks] or None."""
+    n = len(fds)
+    fd_arr = (ctypes.c_int32 * n)(*fds)
+    sz_arr = (ctypes.c_uint64 * n)(*sizes)
+    d, dl = pack_words(dict_words)
+    p, pl = pack_words(patterns)
+    rc = lib().gsys_wordcount(fd_arr, sz_arr, n, chunk, d, dl, len(dict_words), p, pl, len(patterns),
+                              d_hist.data_ptr(), d_file_hits.data_ptr() if d_file_hits is not None else None,
+                              d_req_ret.data_ptr() if d_req_ret is not None else None, gflags, blocks, threads,
+                              _stream(stream))
+    return _check(rc, "gsys_wordcount")
+
+
+def gsys_scan_device(d_text, n: int, chunk: int, dict_words, patterns, d_hist, d_hit=None, blocks: int = 0,
+                     threads: int = 0, stream=None) -> int:
+    d, dl = pack_words(dict_words)
+    p, pl = pack_words(patterns)
+    rc = lib().gsys_scan_device(d_text.data_ptr(), n, chunk, d, dl, len(dict_words), p, pl, len(patterns),
+                                d_hist.data_ptr(), d_hit.data_ptr() if d_hit is not None else None, blocks, threads,
+                                _stream(stream))
+    return _check(rc, "gsys_scan_device")
+
+
+def gsys_bench_calls(kind: str, gflags: int, blocks: int, threads: int, iters: int, fd: int = -1, length: int = 0,
+                     size: int = 0, d_buf=None, d_ret=None, d_lat=None, d_sum=None, stream=None) -> int:
+    k = {"getrusage": 0, "pread": 1, "pwrite": 2}[kind]
+    ptr = lambda t: t.data_ptr() if t is not None else None  # noqa: E731
+    rc = lib().gsys_bench_calls(k, gflags, blocks, threads, iters, fd, length, size, ptr(d_buf), ptr(d_ret),
+                                ptr(d_lat), ptr(d_sum), _stream(stream))
+    return _check(rc, "gsys_bench_calls")
+
+
+def header_functions(path: str | None = None) -> list[str]:
+    """Names of the functions declared in include/gsys.h (for the export test)."""
+    import re
+    path = path or os.path.join(_build.INCLUDE, "gsys.h")
+    src = open(path).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:const\s+)?[\w\s\*]+?\b(gsys_\w+)\s*\(", src, flags=re.M)))

@@ -1,0 +1,305 @@
+"""GPU parity tests (B200, via gpurun): the CUDA path through the C-ABI vs the CPU oracle.
+
+All data is integer: histograms, pread return values, byte sums and file contents must match the
+oracle bit-exactly.  Inputs are the seeded generator's files on tmpfs."""
+import errno
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import inputs
+import oracle
+from oracle import plan, protocol
+from paper_conf_isca_veselybblor18_b200 import gsys as G
+from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+WORDS = None
+PATS = None
+
+
+@pytest.fixture(scope="module", autouse=True)
+def gsys_instance():
+    global WORDS, PATS
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    W.ensure_init()
+    WORDS, PATS = inputs.dictionary(), inputs.patterns()
+    yield
+
+
+@pytest.fixture(scope="module")
+def file16m(tmpdir_shm):
+    p = os.path.join(tmpdir_shm, "config1_16MiB.txt")
+    census, _ = inputs.write_file(p, inputs.SEED_FILE16M, 0, 16 << 20)
+    return p, census
+
+
+@pytest.fixture(scope="module")
+def ragged_corpus(tmpdir_shm):
+    sizes = [0, 1, 15, 4095, 4096 + 17, (256 << 10) - 1, 256 << 10, (256 << 10) + 1, (1 << 20) + 333, 777777,
+             65536, 3 * 4096]
+    return inputs.make_corpus(len(sizes), sizes, seed=inputs.SEED_CORPUS, root=tmpdir_shm, tag="ragged")
+
+
+def oracle_hist_hits(paths):
+    h, hits, _, _ = oracle.corpus(paths, WORDS, PATS, nthreads=4)
+    return h, hits
+
+
+def as_u64(t):
+    return t.cpu().numpy().astype(np.uint64)
+
+
+# ---------------------------------------------------------------------------- wordcount (rows a1-a8)
+@pytest.mark.parametrize("order", [G.STRONG, G.RELAXED])
+def test_wordcount_config1_parity(file16m, order):
+    """Config 1: 16 MiB file, 64 work-groups, WG + blocking (+ strong / relaxed)."""
+    p, census = file16m
+    res = W.wordcount_files([p], WORDS, PATS, chunk=256 << 10, gflags=G.WG | G.BLOCKING | order)
+    assert res.wait_rc == 0
+    data = open(p, "rb").read()
+    want = oracle.count_tokens(data, WORDS)
+    assert np.array_equal(as_u64(res.hist), want)
+    assert np.array_equal(want, census)
+    reqs = plan.wordcount_chunk_requests(len(data), 256 << 10)
+    assert len(reqs) == 64
+    _, rets = oracle.read_file_plan(p, 256 << 10)
+    assert res.req_ret.tolist() == rets.tolist()
+    assert res.req_ret.tolist() == [plan.expected_pread_ret(len(data), r[3], r[4]) for r in reqs]
+    assert bool(res.file_hits[0]) == oracle.grep(data, PATS)
+
+
+@pytest.mark.parametrize("chunk,blocks,threads", [(4096, 7, 64), (256 << 10, 0, 256), (64 << 10, 3, 1024),
+                                                  (1 << 20, 1, 128)])
+def test_wordcount_ragged_corpus(ragged_corpus, chunk, blocks, threads):
+    c = ragged_corpus
+    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, blocks=blocks, threads=threads,
+                            gflags=G.WG | G.BLOCKING | G.RELAXED)
+    h, hits = oracle_hist_hits(c.paths)
+    assert res.wait_rc == 0
+    assert np.array_equal(as_u64(res.hist), h)
+    assert np.array_equal(h, c.census)
+    assert res.file_hits.tolist() == hits.tolist()
+    want = []
+    for s in c.sizes:
+        want += [plan.expected_pread_ret(s, r[3], r[4]) for r in plan.wordcount_chunk_requests(s, chunk)]
+    assert res.req_ret.tolist() == want
+
+
+def test_wordcount_grep_corpus(tmpdir_shm):
+    c = inputs.make_corpus(48, 128 << 10, seed=inputs.SEED_CORPUS, root=tmpdir_shm, tag="grep48")
+    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=32 << 10)
+    assert res.file_hits.tolist() == [1 if m else 0 for m in c.pmasks]
+    assert np.array_equal(as_u64(res.hist), c.census)
+
+
+@pytest.mark.parametrize("window,cmax,merge", [(0, 1, 0), (0, 8, 1), (5, 8, 1), (50, 64, 1), (50, 64, 0)])
+def test_wordcount_coalescing_invariance(ragged_corpus, window, cmax, merge):
+    """Results are identical with and without coalescing / merging (reading A8), bundles <= max."""
+    c = ragged_corpus
+    G.gsys_set_coalesce_window(window)
+    G.gsys_set_coalesce_max(cmax)
+    G.gsys_set_merge(merge)
+    G.gsys_stats_reset()
+    try:
+        res = W.wordcount_files(c.paths, WORDS, PATS, chunk=16 << 10)
+        st = G.gsys_stats()
+    finally:
+        G.gsys_set_coalesce_window(0)
+        G.gsys_set_coalesce_max(8)
+        G.gsys_set_merge(1)
+    h, hits = oracle_hist_hits(c.paths)
+    assert np.array_equal(as_u64(res.hist), h)
+    assert res.file_hits.tolist() == hits.tolist()
+    want = []
+    for s in c.sizes:
+        want += [plan.expected_pread_ret(s, r[3], r[4]) for r in plan.wordcount_chunk_requests(s, 16 << 10)]
+    assert res.req_ret.tolist() == want
+    assert st["max_bundle"] <= cmax
+    if not merge:
+        assert st["merged"] == 0
+
+
+def test_scan_device_parity():
+    """Scan of HBM-resident text (no syscalls), ragged size, several chunk sizes."""
+    for fid, size in [(0, (8 << 20) + 13), (1, 4097), (2, 100)]:
+        buf, census, _ = inputs.gen_bytes(inputs.SEED_CORPUS, fid, size, grep_plants=True)
+        d_text = torch.zeros(size + 64, dtype=torch.uint8, device="cuda")
+        d_text[:size].copy_(torch.from_numpy(buf))
+        for chunk in (16, 4096, 1 << 20):
+            hist = torch.zeros(64, dtype=torch.int64, device="cuda")
+            hit = torch.zeros(1, dtype=torch.int32, device="cuda")
+            G.gsys_scan_device(d_text, size, chunk, WORDS, PATS, hist, hit)
+            torch.cuda.synchronize()
+            assert np.array_equal(as_u64(hist), oracle.count_tokens(buf, WORDS))
+            assert bool(hit.item()) == oracle.grep(buf, PATS)
+
+
+# ---------------------------------------------------------------------------- microbenchmark matrix
+VALID_CELLS = [(G.WI, G.BLOCKING, G.STRONG), (G.WI, G.NONBLOCKING, G.STRONG),
+               (G.WG, G.BLOCKING, G.STRONG), (G.WG, G.BLOCKING, G.RELAXED),
+               (G.WG, G.NONBLOCKING, G.STRONG), (G.WG, G.NONBLOCKING, G.RELAXED),
+               (G.KERNEL, G.BLOCKING, G.RELAXED), (G.KERNEL, G.NONBLOCKING, G.RELAXED)]
+
+
+@pytest.fixture(scope="module")
+def file1m(tmpdir_shm):
+    p = os.path.join(tmpdir_shm, "mb_1MiB.txt")
+    inputs.write_file(p, 7, 0, (1 << 20) + 100)
+    return p
+
+
+@pytest.mark.parametrize("gran,blk,order", VALID_CELLS)
+def test_bench_pread_matrix(file1m, gran, blk, order):
+    size = os.path.getsize(file1m)
+    data = open(file1m, "rb").read()
+    blocks, threads, iters, length = 6, 64, 3, 1000
+    callers = {G.WI: blocks * threads, G.WG: blocks, G.KERNEL: 1}[gran]
+    d_buf = torch.zeros(callers * length + 64, dtype=torch.uint8, device="cuda")
+    fd = os.open(file1m, os.O_RDONLY)
+    G.gsys_stats_reset()
+    try:
+        ncall, ret, lat, sm, rc = W.bench_calls("pread", gran | blk | order, blocks, threads, iters, fd, length,
+                                                size, d_buf, want_sum=True)
+    finally:
+        os.close(fd)
+    st = G.gsys_stats()
+    assert rc == 0 and ncall == callers
+    assert st["per_nr"]["pread"] == callers * iters == protocol.requests_per_call(
+        {G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}[gran], blocks * threads, blocks) * iters
+    reqs = plan.microbench_requests({G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}[gran], blocks, threads, iters,
+                                    length, size)
+    if blk == G.BLOCKING:
+        assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs]
+        assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs]
+    else:
+        assert ret.tolist() == [0] * len(reqs)
+    # after the drain the buffers hold the last iteration's bytes
+    host = d_buf.cpu().numpy()
+    for c in range(callers):
+        off = ((c * iters + iters - 1) * length) % size
+        want = data[off: off + length]
+        assert bytes(host[c * length: c * length + len(want)]) == want
+
+
+@pytest.mark.parametrize("gran,blk,order", VALID_CELLS)
+def test_bench_getrusage_matrix(gran, blk, order):
+    G.gsys_stats_reset()
+    ncall, ret, lat, _, rc = W.bench_calls("getrusage", gran | blk | order, 5, 96, 2)
+    st = G.gsys_stats()
+    assert rc == 0
+    assert st["per_nr"]["getrusage"] == ncall * 2
+    assert ret.tolist() == [0] * (ncall * 2)
+    if blk == G.BLOCKING:
+        assert int(lat.min()) > 0
+
+
+def test_kernel_strong_is_einval(file1m):
+    G.gsys_stats_reset()
+    _, ret, _, _, rc = W.bench_calls("getrusage", G.KERNEL | G.BLOCKING | G.STRONG, 4, 64, 2)
+    assert ret.tolist() == [-errno.EINVAL] * 2
+    assert G.gsys_stats()["per_nr"]["getrusage"] == 0
+
+
+def test_kernel_granularity_larger_than_residency(file1m):
+    """Kernel-scope producer calls must not deadlock when the grid exceeds co-residency."""
+    size = os.path.getsize(file1m)
+    fd = os.open(file1m, os.O_RDONLY)
+    d_buf = torch.zeros(4096, dtype=torch.uint8, device="cuda")
+    try:
+        _, ret, _, _, rc = W.bench_calls("pread", G.KERNEL | G.BLOCKING | G.RELAXED, 148 * 40, 256, 3, fd, 4000,
+                                         size, d_buf)
+    finally:
+        os.close(fd)
+    assert rc == 0
+    assert ret.tolist() == [plan.expected_pread_ret(size, (r * 4000) % size, 4000) for r in range(3)]
+
+
+def test_errors_surface(file1m):
+    d_buf = torch.zeros(1 << 16, dtype=torch.uint8, device="cuda")
+    _, ret, _, _, rc = W.bench_calls("pread", G.WG | G.BLOCKING, 2, 32, 1, -1, 100, 1000, d_buf)
+    assert ret.tolist() == [-errno.EBADF] * 2 and rc == 0
+    _, ret, _, _, rc = W.bench_calls("pread", G.WG | G.NONBLOCKING, 2, 32, 1, -1, 100, 1000, d_buf)
+    assert ret.tolist() == [0, 0] and rc == -errno.EBADF        # reading A4
+    assert G.gsys_wait() == 0                                     # cleared
+
+
+# ---------------------------------------------------------------------------- ordering semantics
+@pytest.mark.parametrize("gran,blk,order", [(G.WG, G.BLOCKING, G.STRONG), (G.WG, G.BLOCKING, G.RELAXED),
+                                            (G.WG, G.NONBLOCKING, G.RELAXED), (G.WI, G.BLOCKING, G.STRONG),
+                                            (G.KERNEL, G.BLOCKING, G.RELAXED)])
+def test_pwrite_consumer_barrier(tmpdir_shm, gran, blk, order):
+    """Consumer calls keep Bar1 (P22.42): every thread's share of the buffer must reach the file."""
+    blocks, threads, length = 4, 256, 8192
+    callers = {G.WI: blocks * threads, G.WG: blocks, G.KERNEL: 1}[gran]
+    if gran == G.WI:
+        length = 64
+    size = callers * length
+    p = os.path.join(tmpdir_shm, f"pw_{gran}_{blk}_{order}.bin")
+    open(p, "wb").write(b"\0" * size)
+    fd = os.open(p, os.O_RDWR)
+    d_buf = torch.zeros(size, dtype=torch.uint8, device="cuda")
+    try:
+        _, ret, _, _, rc = W.bench_calls("pwrite", gran | blk | order, blocks, threads, 1, fd, length, size, d_buf)
+    finally:
+        os.close(fd)
+    assert rc == 0
+    got = open(p, "rb").read()
+    for c in range(callers):
+        want = bytes(((c * 131 + i * 7 + 13) & 0xFF) for i in range(length))
+        assert got[c * length: (c + 1) * length] == want, c
+
+
+# ---------------------------------------------------------------------------- protocol trace (rows a2-a5, a7)
+def test_protocol_trace_validates(file1m):
+    size = os.path.getsize(file1m)
+    G.gsys_set_trace(True, 1 << 16)
+    try:
+        fd = os.open(file1m, os.O_RDONLY)
+        d_buf = torch.zeros(8 * 2000, dtype=torch.uint8, device="cuda")
+        try:
+            W.bench_calls("pread", G.WG | G.BLOCKING, 8, 64, 3, fd, 2000, size, d_buf)
+            W.bench_calls("getrusage", G.WG | G.NONBLOCKING | G.RELAXED, 8, 64, 2)
+            W.bench_calls("getrusage", G.WI | G.BLOCKING, 2, 64, 1)
+        finally:
+            os.close(fd)
+        gtr, htr = G.gsys_trace_read()
+    finally:
+        G.gsys_set_trace(False)
+    by_req = {}
+    for rec in gtr + htr:
+        by_req.setdefault((rec[0], rec[1]), []).append(rec)
+    assert len(by_req) == 8 * 3 + 8 * 2 + 2 * 64
+    records, blocking = [], {}
+    for req, recs in by_req.items():
+        pre = [r for r in recs if r[4] == "gpu" and r[2] in (protocol.FREE, protocol.POPULATING)]
+        host = [r for r in recs if r[4] == "cpu"]
+        post = [r for r in recs if r[4] == "gpu" and r[2] == protocol.FINISHED]
+        for r in pre + host + post:
+            records.append((req, r[0], r[2], r[3], r[4]))
+        blocking[req] = recs[0][5]
+    assert protocol.check_trace(records, lambda r: blocking[r]) == len(by_req)
+
+
+# ---------------------------------------------------------------------------- full size (config 3 shape)
+@pytest.mark.slow
+def test_full_size_corpus_census(tmpdir_shm):
+    """8 GiB, 512 x 16 MiB files, the bench launch configuration: whole-corpus histogram equals
+    the generator's census and grep hits equal the planted set; 4 sampled files through the oracle."""
+    import shutil
+    free = shutil.disk_usage(tmpdir_shm).free
+    if free < (10 << 30):
+        pytest.skip("tmpfs too small for the 8 GiB corpus")
+    c = inputs.make_corpus(512, 16 << 20, seed=inputs.SEED_CORPUS, root=tmpdir_shm, tag="full8g")
+    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=256 << 10, gflags=G.WG | G.BLOCKING | G.RELAXED)
+    assert np.array_equal(as_u64(res.hist), c.census)
+    assert res.file_hits.tolist() == [1 if m else 0 for m in c.pmasks]
+    assert (res.req_ret > 0).all()
+    for f in (0, 101, 255, 511):
+        h, hits = oracle_hist_hits([c.paths[f]])
+        r1 = W.wordcount_files([c.paths[f]], WORDS, PATS, chunk=256 << 10)
+        assert np.array_equal(as_u64(r1.hist), h) and r1.file_hits.tolist() == hits.tolist()
