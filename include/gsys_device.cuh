@@ -358,11 +358,14 @@ __device__ __forceinline__ long long gsys_pwrite(const gsys_dev_ctx* c, int fd, 
     return gsys::invoke(c, GSYS_NR_PWRITE64, gflags, false, a);
 }
 /* getrusage: blocking calls land the 144 B struct rusage in the slot's inline line and the
- * caller copies it to `ru` (any GPU-visible pointer); non-blocking calls hand `ru` to the host. */
+ * caller copies it to `ru` (any pointer the thread can write, including local memory);
+ * non-blocking calls hand a global `ru` to the host, which writes it asynchronously -- for a
+ * thread-local `ru` the non-blocking result is discarded, as for every non-blocking call (P24.34). */
 __device__ __forceinline__ long long gsys_getrusage(const gsys_dev_ctx* c, int who, void* ru, unsigned gflags) {
-    bool blocking = !(gflags & GSYS_NONBLOCKING);
+    const bool blocking = !(gflags & GSYS_NONBLOCKING);
+    const bool inl = ru != nullptr && (blocking || !__isGlobal(ru));
     unsigned long long a[6] = {(unsigned long long)(long long)who, (unsigned long long)ru, 0ull, 0ull, 0ull, 0ull};
-    return gsys::invoke(c, GSYS_NR_GETRUSAGE, gflags | (blocking && ru ? GSYS_F_INLINE : 0u), true, a,
+    return gsys::invoke(c, GSYS_NR_GETRUSAGE, gflags | (inl ? GSYS_F_INLINE : 0u), true, a,
                         blocking ? ru : nullptr, 144u);
 }
 __device__ __forceinline__ long long gsys_madvise(const gsys_dev_ctx* c, void* addr, size_t len, int advice,
