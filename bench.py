@@ -1,0 +1,413 @@
+#!/usr/bin/env python
+"""bench.py -- headline benchmark of the GENESYS hot path on B200.
+
+Metric (BASELINE.json): "GPU-issued syscalls/sec (WG granularity) and pread-wordcount GB/s at
+1/2/4/8 B200".  One step = one pass of the whole hot path over the config-3 workload: every
+work-group of the wordcount/grep kernel issues GPU-side preads of its 256 KiB chunks (rows
+a1-a6), the host service drains/coalesces/executes them and DMAs the bytes (a7), the kernel scans
+them (a8), the per-rank histogram + grep hits are all-reduced over NCCL (a9, N > 1 only) and the
+service is drained (a10).  The workload is 512 synthetic 16 MiB text files (8 GiB) on tmpfs,
+sharded by whole files across ranks (fixed total: strong scaling).  `value` = corpus GB/s
+(device-timed, CUDA events on the launch stream, max over ranks); `e2e` = the same through the
+public Python API (files in -> host histogram out, wall clock); the WG syscall rate is reported
+in `secondary`.  `--impl reference` times the CPU oracle on a bounded sample.
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GPU-issued syscalls/sec (WG granularity) and pread-wordcount GB/s at 1/2/4/8 B200"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gsys", choices=["gsys", "reference"])
+    ap.add_argument("--files", type=int, default=512)
+    ap.add_argument("--file-mib", type=int, default=16)
+    ap.add_argument("--chunk-kib", type=int, default=256)
+    ap.add_argument("--order", default="relaxed", choices=["strong", "relaxed"])
+    ap.add_argument("--blocks", type=int, default=296, help="work-groups (2 per SM)")
+    ap.add_argument("--threads", type=int, default=256)
+    ap.add_argument("--staging", default="host", choices=["device", "host"])
+    ap.add_argument("--cmax", type=int, default=8, help="coalescing max bundle (P22.13)")
+    ap.add_argument("--window", type=int, default=0, help="coalescing window us (P22.13)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip scan roofline / syscall-rate extras")
+    ap.add_argument("--root", default=None, help="corpus directory (default /dev/shm/gsys_corpus)")
+    return ap.parse_args()
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() in ("active", "0x1", "yes"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def host_cores() -> int:
+    return len(os.sched_getaffinity(0))
+
+
+def cpu_model() -> str:
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def workload_config(a, nbytes, world):
+    return {
+        "workload": f"config3: pread-driven grep + wordcount, {a.files} x {a.file_mib} MiB synthetic text files "
+                    f"({nbytes / 2**30:.2f} GiB) on tmpfs, WG granularity, blocking + {a.order}, "
+                    f"{a.chunk_kib} KiB chunks, {a.staging} staging, files sharded across {world} GPU(s), "
+                    f"NCCL histogram all-reduce",
+        "files": a.files, "bytes": nbytes, "chunk": a.chunk_kib << 10, "blocks": a.blocks or "2/SM",
+        "staging": a.staging, "coalesce_max": a.cmax, "coalesce_window_us": a.window,
+        "threads_per_wg": a.threads, "dictionary_words": 64, "grep_patterns": 8,
+        "l2": "inputs larger than L2 (8 GiB corpus streamed from the host every step)",
+        "input_residency": "host page cache (tmpfs); the GPU-issued preads move it to HBM inside the timed region",
+        "parallelism": f"files/{world}",
+    }
+
+
+def run_reference(a):
+    """--impl reference: the CPU oracle (plain C, all host cores) on a bounded sample per step."""
+    rank, world, local = dist_env()
+    if rank != 0:
+        return 0
+    import inputs
+    import oracle
+    corpus = inputs.make_corpus(a.files, a.file_mib << 20, root=a.root)
+    words, pats = inputs.dictionary(), inputs.patterns()
+    sample = corpus.paths[: max(1, min(len(corpus.paths), 32))]
+    sbytes = sum(os.path.getsize(p) for p in sample)
+    nthr = host_cores()
+    for _ in range(a.warmup):
+        oracle.corpus(sample[:2], words, pats, chunk=a.chunk_kib << 10, nthreads=nthr)
+    times = []
+    for _ in range(a.steps):
+        _, _, secs, _ = oracle.corpus(sample, words, pats, chunk=a.chunk_kib << 10, nthreads=nthr)
+        times.append(secs)
+    t = sum(times)
+    value = sbytes * a.steps / t / 1e9
+    out = {"impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world,
+           "steps": a.steps, "warmup": a.warmup, "ms_per_step": t / a.steps * 1e3, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+           "config": workload_config(a, corpus.total_bytes, world),
+           "cpu_baseline": {"value": value, "unit": "GB/s", "cores": nthr, "kind": "oracle",
+                            "sample": f"{len(sample)} of {a.files} files ({sbytes / 2**20:.0f} MiB) per step, "
+                                      f"pread + scalar wordcount + grep, {nthr} pthreads, {cpu_model()}"},
+           "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        return run_reference(a)
+    import torch
+    import torch.distributed as dist
+
+    import inputs
+    from paper_conf_isca_veselybblor18_b200 import gsys as G
+    from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # corpus: local rank 0 writes it once per node; everyone shards by whole files
+    if local == 0:
+        corpus = inputs.make_corpus(a.files, a.file_mib << 20, root=a.root)
+    barrier()
+    corpus = inputs.make_corpus(a.files, a.file_mib << 20, root=a.root)
+    words, pats = inputs.dictionary(), inputs.patterns()
+    lo, hi = rank * a.files // world, (rank + 1) * a.files // world
+    mine = corpus.paths[lo:hi]
+    chunk = a.chunk_kib << 10
+    gflags = G.WG | G.BLOCKING | (G.RELAXED if a.order == "relaxed" else G.STRONG)
+
+    W.ensure_init()
+    G.gsys_set_coalesce_max(a.cmax)
+    G.gsys_set_coalesce_window(a.window)
+    staging = G.STAGE_HOST if a.staging == "host" else G.STAGE_DEVICE
+    stream = torch.cuda.Stream(device=dev)
+    of = W.OpenFiles(mine).__enter__()
+    my_bytes = sum(of.sizes)
+    nf = len(mine)
+    d_hist = torch.zeros(64, dtype=torch.int64, device=dev)
+    d_hits = torch.zeros(max(nf, 1), dtype=torch.int32, device=dev)
+    d_all = torch.zeros(64 + a.files, dtype=torch.int64, device=dev)
+
+    def step():
+        d_hist.zero_()
+        d_hits.zero_()
+        G.gsys_wordcount(of.fds, of.sizes, chunk, words, pats, d_hist, d_hits, None, gflags, a.blocks, a.threads,
+                         stream, staging)
+        G.gsys_wait(stream)
+        if world > 1:
+            d_all.zero_()
+            d_all[:64].copy_(d_hist)
+            d_all[64 + lo: 64 + hi].copy_(d_hits.to(torch.int64)[:nf])
+            dist.all_reduce(d_all)
+
+    with torch.cuda.stream(stream):
+        for _ in range(a.warmup):
+            step()
+        barrier()
+        clk = Clocks(local)
+        clk.start()
+        ev0 = torch.cuda.Event(enable_timing=True)
+        ev1 = torch.cuda.Event(enable_timing=True)
+        G.gsys_stats_reset()
+        barrier()
+        ev0.record(stream)
+        for _ in range(a.steps):
+            step()
+        ev1.record(stream)
+        ev1.synchronize()
+        barrier()
+        clocks = clk.stop()
+        st = G.gsys_stats()
+    dev_s = max_over_ranks(ev0.elapsed_time(ev1) / 1e3)
+    value = corpus.total_bytes * a.steps / dev_s / 1e9
+    # parity of the last step against the generator census (cheap, exact)
+    if world > 1:
+        hist_ok = bool((d_all[:64].cpu().numpy().astype("uint64") == corpus.census).all())
+    else:
+        hist_ok = bool((d_hist.cpu().numpy().astype("uint64") == corpus.census).all())
+
+    # ---- e2e through the public API (files in -> host histogram out), wall clock
+    barrier()
+    e2e_t = []
+    for _ in range(max(1, min(a.steps, 3))):
+        barrier()
+        t0 = time.perf_counter()
+        res = W.wordcount_files(mine, words, pats, chunk=chunk, gflags=gflags, blocks=a.blocks, threads=a.threads,
+                                stream=stream, staging=staging)
+        if world > 1:
+            v = torch.zeros(64 + a.files, dtype=torch.int64)
+            v[:64] = res.hist
+            v[64 + lo: 64 + hi] = res.file_hits.to(torch.int64)[:nf]
+            vd = v.to(dev)
+            dist.all_reduce(vd)
+            vd.cpu()
+        e2e_t.append(max_over_ranks(time.perf_counter() - t0))
+    e2e_s = statistics.median(e2e_t)
+    e2e_value = corpus.total_bytes / e2e_s / 1e9
+
+    # ---- roofline of the dominant kernel (wc_kernel): host-link bound
+    extras = {}
+    h2d_peak = None
+    if not a.no_extras:
+        h2d_peak = measure_h2d(dev)
+        extras["scan"] = scan_roofline(G, dev, corpus, words, pats, chunk)
+        extras["syscalls"] = wg_syscall_rate(G, W, dev)
+    kernel_s = dev_s / a.steps
+    algo_bytes = my_bytes + sum(((s + chunk - 1) // chunk) * 17 for s in of.sizes)   # chunk + halo
+    rank_achieved = algo_bytes / kernel_s / 1e9
+    roofline = {"bound": "host-link", "achieved": rank_achieved, "peak": h2d_peak, "unit": "GB/s",
+                "frac": (rank_achieved / h2d_peak) if h2d_peak else None, "traffic": None,
+                "kernel": "wc_kernel (GPU-issued WG preads + scan), one launch per step per rank",
+                "peak_source": "measured live: pinned cudaMemcpyAsync H2D, 256 MiB x 8, this box's PCIe link "
+                               "(MEASURED_PEAKS.json has no host-link figure)"}
+    of.__exit__()
+
+    cpu_baseline = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        cpu_baseline = cpu_baseline_leg(a, corpus, words, pats, chunk)
+    if world > 1:
+        dist.barrier()
+    if rank == 0:
+        syscalls_per_step = st["requests"] / a.steps
+        out = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": a.steps,
+               "warmup": a.warmup, "ms_per_step": dev_s / a.steps * 1e3, "higher_is_better": True,
+               "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+               "config": workload_config(a, corpus.total_bytes, world),
+               "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": my_bytes * world,
+                       "d2h_bytes_per_step": (64 + a.files) * 8, "api": "workloads.wordcount_files"},
+               "gpu_launches": a.steps,
+               "roofline": roofline,
+               "cpu_baseline": cpu_baseline,
+               "clocks": clocks,
+               "parity": {"hist_equals_generator_census": hist_ok},
+               "secondary": {"wg_syscalls_per_s_in_wordcount": syscalls_per_step * world / (dev_s / a.steps),
+                             **({"getrusage_wg": extras["syscalls"]} if "syscalls" in extras else {}),
+                             **({"scan_hbm": extras["scan"]} if "scan" in extras else {})},
+               "service": {"threads": st["threads"], "coalesce_max": st["coalesce_max"],
+                           "window_us": st["coalesce_window_us"], "bundles_per_step": st["bundles"] / a.steps,
+                           "merged_per_step": st["merged"] / a.steps,
+                           "host_preads_per_step": st["host_preads"] / a.steps},
+               "host": {"cores": host_cores(), "cpu": cpu_model()}}
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def measure_h2d(dev):
+    import torch
+    n = 256 << 20
+    h = torch.empty(n, dtype=torch.uint8).pin_memory()
+    d = torch.empty(n, dtype=torch.uint8, device=dev)
+    s = torch.cuda.Stream(device=dev)
+    with torch.cuda.stream(s):
+        for _ in range(2):
+            d.copy_(h, non_blocking=True)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(8):
+            d.copy_(h, non_blocking=True)
+        e1.record(s)
+        e1.synchronize()
+    return n * 8 / (e0.elapsed_time(e1) / 1e3) / 1e9
+
+
+def scan_roofline(G, dev, corpus, words, pats, chunk):
+    """Standalone scan (row a8) over 1 GiB of corpus text resident in HBM: GB/s vs measured HBM."""
+    import torch
+    nb = min(len(corpus.paths), 64)
+    parts = [torch.from_file(p, dtype=torch.uint8, size=os.path.getsize(p)) for p in corpus.paths[:nb]]
+    text = torch.cat(parts).to(dev)
+    n = text.numel()
+    hist = torch.zeros(64, dtype=torch.int64, device=dev)
+    hit = torch.zeros(1, dtype=torch.int32, device=dev)
+    s = torch.cuda.Stream(device=dev)
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 256, s)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 10
+        e0.record(s)
+        for _ in range(reps):
+            G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 256, s)
+        e1.record(s)
+        e1.synchronize()
+    t = e0.elapsed_time(e1) / 1e3 / reps
+    peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
+    ach = n / t / 1e9
+    del text
+    return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "bytes": n,
+            "ms": t * 1e3, "kernel": "scan_kernel (HBM-resident text, 4 blocks/SM x 256 threads)",
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
+
+
+def wg_syscall_rate(G, W, dev):
+    """getrusage(RUSAGE_SELF) at WG granularity, blocking: 4 WGs/SM x 256 threads x 20 calls."""
+    import torch
+    blocks, threads, iters = 592, 256, 20
+    W.bench_calls("getrusage", G.WG | G.BLOCKING | G.RELAXED, blocks, threads, 2)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    _, ret, lat, _, rc = W.bench_calls("getrusage", G.WG | G.BLOCKING | G.RELAXED, blocks, threads, iters)
+    dt = time.perf_counter() - t0
+    lat_us = (lat.double() / 1e3).cpu()
+    return {"calls_per_s": blocks * iters / dt, "callers": blocks, "iters": iters,
+            "lat_p50_us": float(lat_us.median()), "lat_p99_us": float(lat_us.quantile(0.99)),
+            "all_ok": bool((ret == 0).all())}
+
+
+def cpu_baseline_leg(a, corpus, words, pats, chunk):
+    import oracle
+    nthr = host_cores()
+    sample = corpus.paths[:32]
+    sbytes = sum(os.path.getsize(p) for p in sample)
+    oracle.corpus(sample[:1], words, pats, chunk=chunk, nthreads=nthr)
+    _, _, secs, _ = oracle.corpus(sample, words, pats, chunk=chunk, nthreads=nthr)
+    rate = oracle.syscall_rate("getrusage", nthr, 200000)
+    pread_ceiling = {str(t): oracle.pread_only(corpus.paths[:64], t, chunk) / 1e9 for t in (1, 4, 8, nthr)}
+    return {"value": sbytes / secs / 1e9, "unit": "GB/s", "cores": nthr, "kind": "oracle",
+            "host_pread_only_GBps_by_threads": pread_ceiling,
+            "sample": f"{len(sample)} of {a.files} files ({sbytes / 2**20:.0f} MiB): pread + scalar wordcount + grep, "
+                      f"{nthr} pthreads, {cpu_model()}",
+            "getrusage_direct_calls_per_s": rate}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

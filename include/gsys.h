@@ -68,6 +68,14 @@ enum gsys_state {
 #define GSYS_RELAXED     0x10u
 #define GSYS_WEAK        GSYS_RELAXED
 #define GSYS_SITE(k)     (((uint32_t)(k) & 63u) << 24)   /* kernel-scope call site id 0..63 */
+/* Completion through system memory: the caller's buffer is pinned host-mapped memory, so the
+ * host service performs the call in place and signals completion with a plain store into the
+ * slot's host-mapped completion word, which the GPU polls over PCIe (the paper's "CPU-GPU
+ * communication ... via atomic reads/writes in system memory", PAPER.md:16 P16.8).  Without
+ * the flag the GPU polls a device-memory completion word written by a CUDA stream memory
+ * operation ordered after the payload DMA.  Either way the result is correct for any buffer;
+ * the flag picks the fast path. */
+#define GSYS_HOSTBUF     0x20u
 /* internal bits set by the device library in the slot's flags word */
 #define GSYS_F_PRODUCER  0x100u   /* call class: producer (read-like), P20.24-29            */
 #define GSYS_F_INLINE    0x200u   /* small result goes to the slot's inline payload line    */
@@ -92,7 +100,7 @@ enum gsys_state {
  *   coalesce_window_us  coalescing time window in microseconds ("a time window length within
  *                     which the CPU coalesces system calls", PAPER.md:22 P22.13); 0 = take only
  *                     requests already present.
- * Service thread count: env GSYS_THREADS (default min(8, cores-2)); coalescing max count
+ * Service thread count: env GSYS_THREADS (default min(16, cores-2)); coalescing max count
  * default 8 (PAPER.md:28 P28.17), see gsys_set_coalesce_max().
  * Errors: -EINVAL (slots > 2^24), -EALREADY (already initialised on this device), -ENODEV (no
  * CUDA device), -ENOMEM (pinned/device allocation failed), -ENOTSUP (stream memory operations
@@ -148,6 +156,10 @@ typedef struct gsys_stats {
     uint64_t bytes_h2d;       /* bytes DMA'd host -> device                      */
     uint64_t errors;          /* requests that returned -errno                   */
     uint64_t per_nr[8];       /* pread, pwrite, madvise, sendto, recvfrom, getrusage, sigq, other */
+    uint64_t ns_busy;         /* worker time spent processing bundles (sum over workers)   */
+    uint64_t ns_syscall;      /* ... of which inside the POSIX calls themselves             */
+    uint64_t ns_cuda;         /* ... of which in CUDA API calls (copies, memops, events)    */
+    uint64_t ns_bounce_wait;  /* ... of which waiting for bounce-ring DMA to drain          */
     uint32_t threads;         /* service worker threads                          */
     uint32_t slots;           /* syscall-area slots                              */
     uint32_t coalesce_max;
@@ -190,7 +202,15 @@ int gsys_plan_merge(uint32_t n, const int32_t* fd, const int64_t* off, const uin
  * clamp(r - offset_in_group, 0, len) (reading A8); -errno propagates. */
 int64_t gsys_split_result(int64_t r, uint64_t offset_in_group, uint64_t len);
 
-/* ---------------------------------------------------------------- workloads (the hot path)
+/* Self-test of a worker's pinned bounce-ring allocator (host logic, no device): `iters` random
+ * allocations of up to `cap` bytes with random commit points against a fake completion model;
+ * checks that no allocation overlaps a region whose DMA may still be in flight.  0 or -EPROTO. */
+int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap);
+
+/* ---------------------------------------------------------------- workloads (the hot path) */
+#define GSYS_STAGE_DEVICE 0u
+#define GSYS_STAGE_HOST   1u
+/*
  * Wordcount + grep -F -l over files read with GPU-issued preads (sec. VIII-C,
  * P32.3-9 wordcount "64 strings", "work-group granularity with blocking and weak-ordering";
  * PAPER.md:30 P30.27-38 grep -F -l).
@@ -203,8 +223,12 @@ int64_t gsys_split_result(int64_t r, uint64_t offset_in_group, uint64_t len);
  *   d_file_hits     DEVICE uint32[nfiles] (may be NULL): set to 1 for files containing a pattern.
  *   gflags          GSYS_WG (the paper's configuration for wordcount) + GSYS_BLOCKING +
  *                   GSYS_STRONG or GSYS_RELAXED; anything else is -EINVAL.
- *   blocks          work-groups launched (0 = 4 per SM); threads: threads per work-group
- *                   (0 = 256; multiple of 32, <= 1024).
+ *   staging         GSYS_STAGE_DEVICE: each work-group's pread lands in a device (HBM) line,
+ *                   the host service DMAs it from its pinned bounce ring;  GSYS_STAGE_HOST: the
+ *                   pread lands in a pinned host-mapped line ("syscall buffers" in system memory,
+ *                   PAPER.md:24 P24.37-51) and the scan reads it over PCIe (zero-copy).
+ *   blocks          work-groups launched (0 = 2 per SM); threads: threads per work-group
+ *                   (0 = 256; multiple of 32, <= 256).
  *   d_req_ret       DEVICE int64[total chunks] (may be NULL): per-chunk pread return value.
  *   stream          cudaStream_t to launch on.
  * Asynchronous on `stream`; call gsys_wait(stream) before reading results.  Errors: -EINVAL
@@ -214,7 +238,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
                    const char* dict, const uint8_t* dlen, uint32_t ndict,
                    const char* pats, const uint8_t* plen, uint32_t npat,
                    uint64_t* d_hist, uint32_t* d_file_hits, int64_t* d_req_ret,
-                   uint32_t gflags, uint32_t blocks, uint32_t threads, void* stream);
+                   uint32_t gflags, uint32_t staging, uint32_t blocks, uint32_t threads, void* stream);
 
 /* Same scan over text already resident in device memory (no syscalls): the standalone scan
  * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n]; file boundaries are not
@@ -224,6 +248,12 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
                      const char* pats, const uint8_t* plen, uint32_t npat,
                      uint64_t* d_hist, uint32_t* d_hit, uint32_t blocks, uint32_t threads,
                      void* stream);
+
+/* Diagnostics: when on, gsys_wordcount's work-groups accumulate (thread 0, %globaltimer) the
+ * time spent inside their gsys_pread calls, the time spent scanning, and the chunk count;
+ * gsys_read_profile copies {wait_ns, scan_ns, chunks} to host memory (optionally resetting). */
+int gsys_set_profile(int on);
+int gsys_read_profile(uint64_t* out3, int reset);
 
 /* Syscall microbenchmark (sec. VII, Fig. 7/8/10): every caller of the chosen
  * granularity (work-item: every thread; work-group: every block; kernel: one per launch) issues

@@ -49,6 +49,8 @@ struct gsys_dev_ctx {
     unsigned* claim;                /* device [nslots]: 0 free, 1 owned                     */
     unsigned* seqs;                 /* device [nslots]: last sequence number used           */
     unsigned long long* mirror;     /* device [nslots]: completion word (seq << 32 | u32 ret) */
+    unsigned long long* hdone;      /* host-mapped [nslots]: completion word for host-store completions */
+    unsigned* lat_hint;             /* device [nslots]: EWMA of the slot's round-trip latency (ns)  */
     unsigned long long* ring;       /* host-mapped [ring_mask+1] doorbell entries           */
     unsigned* ring_tail;            /* device: next doorbell position                       */
     gsys_kround* krounds;           /* device [GSYS_KSITES * GSYS_KROUNDS]                  */
@@ -59,8 +61,8 @@ struct gsys_dev_ctx {
     unsigned kblock_cap;
     unsigned nslots;
     unsigned ring_mask;
-    unsigned poll_ns_max;
-    unsigned pad_;
+    unsigned poll_ns_max;           /* backoff cap for device-memory polls                      */
+    unsigned poll_ns_host;          /* poll interval for host-memory (PCIe) polls               */
 };
 
 #ifdef __CUDACC__
@@ -175,18 +177,44 @@ __device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
     st_relaxed_sys(c->ring + (pos & c->ring_mask), ((unsigned long long)(pos + 1u) << 32) | s);
 }
 
-/* ------------------------------------------------------------------ a5: completion */
-__device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
-    const unsigned long long* m = c->mirror + s;
-    unsigned ns = 64;
+/* ------------------------------------------------------------------ a5: completion
+ * Blocking callers poll the slot's completion word until it carries their sequence number:
+ * the device-memory word (L2-resident; written by a stream memory operation after the DMA) or,
+ * for GSYS_HOSTBUF / inline calls, the host-mapped word the service stores directly (each poll
+ * is one PCIe read, so the backoff starts longer and caps at poll_ns_max). */
+__device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq, bool host) {
     unsigned long long v;
-    for (;;) {
-        v = ld_relaxed_sys(m);
-        if ((unsigned)(v >> 32) == seq) break;
-        __nanosleep(ns);
-        ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
+    if (!host) {
+        const unsigned long long* m = c->mirror + s;
+        unsigned ns = 64;
+        for (;;) {
+            v = ld_relaxed_sys(m);
+            if ((unsigned)(v >> 32) == seq) break;
+            __nanosleep(ns);
+            ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
+        }
+    } else {
+        // every poll is a PCIe round trip: sleep ~3/4 of this slot's recent latency first, then
+        // poll at a fixed interval, so hundreds of waiting work-groups do not flood the link
+        const unsigned long long* m = c->hdone + s;
+        const unsigned long long t0 = globaltimer();
+        unsigned first = (c->lat_hint[s] >> 2) * 3u;
+        while (first > 0) {
+            unsigned d = first > 500000u ? 500000u : first;
+            __nanosleep(d);
+            first -= d;
+        }
+        for (;;) {
+            v = ld_relaxed_sys(m);
+            if ((unsigned)(v >> 32) == seq) break;
+            __nanosleep(c->poll_ns_host);
+        }
+        const unsigned long long dt = globaltimer() - t0;
+        const unsigned h = c->lat_hint[s];
+        const unsigned d32 = dt > 4000000ull ? 4000000u : (unsigned)dt;
+        c->lat_hint[s] = h ? (h - (h >> 3) + (d32 >> 3)) : d32;
     }
-    fence_acq_rel_sys();   /* acquire: payload DMA'd before the completion word is visible */
+    fence_acq_rel_sys();   /* acquire: the payload is visible before the completion word */
     return (long long)(int)(unsigned)(v & 0xffffffffull);
 }
 
@@ -206,7 +234,7 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     unsigned seq = marshal(c, s, nr, flags, a);
     doorbell(c, s);
     if (!blocking) return 0;
-    long long r = wait_done(c, s, seq);
+    long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) != 0u);
     if (inline_out != nullptr && r >= 0) {
         const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
         uint4* dst = reinterpret_cast<uint4*>(inline_out);

@@ -60,6 +60,8 @@ def lib():
             L.oracle_syscall_rate.restype = ctypes.c_double
             L.oracle_syscall_rate.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_uint64, ctypes.c_int,
                                               ctypes.c_uint64, ctypes.c_uint64]
+            L.oracle_pread_only.restype = ctypes.c_double
+            L.oracle_pread_only.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_uint64]
             _lib = L
     return _lib
 
@@ -153,4 +155,13 @@ def syscall_rate(kind: str, nthreads: int, iters: int, fd: int = -1, length: int
     r = lib().oracle_syscall_rate(k, nthreads, iters, fd, length, size)
     if r < 0:
         raise OSError(int(-r), "oracle_syscall_rate")
+    return r
+
+
+def pread_only(paths, nthreads: int, chunk: int = 256 << 10) -> float:
+    """Host pread ceiling in bytes/s: nthreads threads pread the files in chunk-byte calls."""
+    arr = (ctypes.c_char_p * len(paths))(*[p.encode() for p in paths])
+    r = lib().oracle_pread_only(ctypes.cast(arr, ctypes.c_void_p), len(paths), nthreads, chunk)
+    if r < 0:
+        raise OSError(int(-r), "oracle_pread_only")
     return r

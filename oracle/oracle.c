@@ -194,6 +194,57 @@ int oracle_corpus(const char* const* paths, int nfiles, int nthreads, uint64_t c
     return J.err;
 }
 
+typedef struct {
+    const char* const* paths; int nfiles; uint64_t chunk; int next; pthread_mutex_t mu; uint64_t bytes; int err;
+} pread_job_t;
+
+static void* pread_only_worker(void* arg) {
+    pread_job_t* J = (pread_job_t*)arg;
+    uint8_t* buf = (uint8_t*)malloc(J->chunk + 64);
+    uint64_t bytes = 0;
+    int err = 0;
+    for (;;) {
+        pthread_mutex_lock(&J->mu);
+        int f = J->next++;
+        pthread_mutex_unlock(&J->mu);
+        if (f >= J->nfiles) break;
+        int fd = open(J->paths[f], O_RDONLY);
+        if (fd < 0) { err = -errno; continue; }
+        for (uint64_t off = 0;; off += J->chunk) {
+            ssize_t r = pread(fd, buf, J->chunk, (off_t)off);
+            if (r < 0) { err = -errno; break; }
+            bytes += (uint64_t)r;
+            if ((uint64_t)r < J->chunk) break;
+        }
+        close(fd);
+    }
+    free(buf);
+    pthread_mutex_lock(&J->mu);
+    J->bytes += bytes;
+    if (err && !J->err) J->err = err;
+    pthread_mutex_unlock(&J->mu);
+    return NULL;
+}
+
+/* Host pread ceiling: nthreads threads pread every file in `chunk`-byte calls into private
+ * buffers, no scan (the host-side co-roofline of the GPU-syscall wordcount).  Returns bytes/s
+ * (or a negative errno). */
+double oracle_pread_only(const char* const* paths, int nfiles, int nthreads, uint64_t chunk) {
+    pread_job_t J;
+    memset(&J, 0, sizeof J);
+    J.paths = paths; J.nfiles = nfiles; J.chunk = chunk;
+    pthread_mutex_init(&J.mu, NULL);
+    pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * nthreads);
+    double t0 = now_s();
+    for (int t = 0; t < nthreads; t++) pthread_create(&th[t], NULL, pread_only_worker, &J);
+    for (int t = 0; t < nthreads; t++) pthread_join(th[t], NULL);
+    double dt = now_s() - t0;
+    free(th);
+    pthread_mutex_destroy(&J.mu);
+    if (J.err) return (double)J.err;
+    return (double)J.bytes / dt;
+}
+
 typedef struct { uint64_t iters; int fd; uint64_t len; uint64_t size; int kind; int tid; int err; } rate_job_t;
 
 static void* rate_worker(void* arg) {

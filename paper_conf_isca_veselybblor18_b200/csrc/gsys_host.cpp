@@ -3,16 +3,18 @@
 // Replaces GENESYS's kernel-side processing (sec. VI "CPU-side system call
 // processing", P24.16-35) with a user-space service, because the box's kernel cannot be changed
 // (BASELINE.json north_star):
-//   * the paper's interrupt handler, which "creates a new kernel task and adds it to Linux's
-//     work-queue" after "waiting for a predetermined amount of time" to coalesce (P24.17-18,
-//     P24.29-30), becomes ONE dispatcher thread per GPU that polls the doorbell ring the GPU
-//     writes (the s_sendmsg analogue, P24.14) and cuts the entries into bundles of at most
-//     coalesce_max requests or coalesce_window microseconds (P22.9-13);
-//   * the "OS worker thread" that "atomically switches any ready system call requests to the
-//     processing state" and "carries out the system call work" (P24.19-21) becomes a pool of
-//     worker threads that execute a bundle in (fd, offset) order (reading A8), merge preads of
-//     adjacent/overlapping ranges into one read of the union (north_star extension), DMA payloads
-//     into device buffers and publish results (P24.32-35);
+//   * the paper's interrupt handler ("creates a new kernel task and adds it to Linux's
+//     work-queue" after "waiting for a predetermined amount of time" to coalesce, P24.17-18,
+//     P24.29-30) and its OS worker thread ("atomically switches any ready system call requests to
+//     the processing state" and "carries out the system call work", P24.19-21) become a pool of
+//     worker threads that poll the doorbell ring the GPU writes (the s_sendmsg analogue, P24.14).
+//     A free worker claims the run of ready entries at the ring head -- at most coalesce_max, and
+//     it keeps extending the run for up to coalesce_window microseconds (P22.9-13) -- so bundles
+//     grow by themselves when the service is the bottleneck;
+//   * a bundle executes in (fd, offset) order (reading A8), preads of adjacent/overlapping ranges
+//     of one regular file are merged into one read of the union (north_star extension), payloads
+//     for device buffers go through a pinned bounce ring and one cudaMemcpyBatchAsync per bundle,
+//     payloads for host-mapped buffers are read in place (P24.32-35);
 //   * results are returned with CUDA stream memory operations ordered after the payload DMA:
 //     blocking -> completion word {seq, ret} (state "finished"), non-blocking -> claim word
 //     cleared (state "free"), P24.33-34;
@@ -79,61 +81,68 @@ int cuda_err(cudaError_t e) {
     return -EIO;
 }
 
-// ------------------------------------------------------------------ bounded MPMC queue (Vyukov)
-class MPMC {
+// ------------------------------------------------------------------ bounce ring allocator
+// Ring allocator over [0, cap) of a worker's pinned bounce buffer.  Regions are handed out in
+// order; a region stays "in flight" until the completion token recorded after its DMA has fired.
+// alloc() waits for exactly the in-flight regions that overlap the new range: the previous lap's
+// tail when it wraps, then the oldest regions of the current lap.  Ops supplies
+// make_token() (flush queued copies + record an event), wait(token) and recycle(token); the
+// self-test below drives it with a fake Ops.
+template <class Token, class Ops>
+class BounceRing {
    public:
-    explicit MPMC(size_t cap_pow2) : mask_(cap_pow2 - 1), cells_(cap_pow2) {
-        for (size_t i = 0; i < cap_pow2; i++) cells_[i].seq.store(i, std::memory_order_relaxed);
-        enq_.store(0); deq_.store(0);
-    }
-    bool push(uint64_t v) {
-        size_t pos = enq_.load(std::memory_order_relaxed);
-        for (;;) {
-            Cell& c = cells_[pos & mask_];
-            size_t seq = c.seq.load(std::memory_order_acquire);
-            intptr_t d = (intptr_t)seq - (intptr_t)pos;
-            if (d == 0) {
-                if (enq_.compare_exchange_weak(pos, pos + 1, std::memory_order_relaxed)) {
-                    c.val = v;
-                    c.seq.store(pos + 1, std::memory_order_release);
-                    return true;
-                }
-            } else if (d < 0) {
-                return false;
-            } else {
-                pos = enq_.load(std::memory_order_relaxed);
-            }
+    static constexpr size_t NONE = ~(size_t)0;
+    BounceRing(size_t cap, Ops* ops) : cap_(cap), ops_(ops) {}
+    size_t alloc(size_t n) {
+        n = (n + 255) & ~(size_t)255;
+        if (n == 0) n = 256;
+        if (n > cap_) return NONE;
+        if (head_ + n > cap_) {                 // wrap: retire what is left of the previous lap
+            while (!q_.empty() && q_.front().lo >= head_) retire_front();
+            head_ = 0;
         }
+        const size_t lo = head_, hi = head_ + n;
+        while (!q_.empty() && q_.front().lo < hi && lo < q_.front().hi) retire_front();
+        q_.push_back(Region{lo, hi, Token{}, false, false});
+        npending_++;
+        head_ = hi;
+        return lo;
     }
-    bool pop(uint64_t* v) {
-        size_t pos = deq_.load(std::memory_order_relaxed);
-        for (;;) {
-            Cell& c = cells_[pos & mask_];
-            size_t seq = c.seq.load(std::memory_order_acquire);
-            intptr_t d = (intptr_t)seq - (intptr_t)(pos + 1);
-            if (d == 0) {
-                if (deq_.compare_exchange_weak(pos, pos + 1, std::memory_order_relaxed)) {
-                    *v = c.val;
-                    c.seq.store(pos + mask_ + 1, std::memory_order_release);
-                    return true;
-                }
-            } else if (d < 0) {
-                return false;
-            } else {
-                pos = deq_.load(std::memory_order_relaxed);
-            }
+    // attach one completion token to every region allocated since the previous commit
+    void commit() {
+        if (!npending_) return;
+        Token t = ops_->make_token();
+        size_t first = q_.size() - npending_;
+        for (size_t i = first; i < q_.size(); i++) {
+            q_[i].tok = t;
+            q_[i].committed = true;
+            q_[i].last = (i + 1 == q_.size());
         }
+        npending_ = 0;
     }
+    // invariant for tests: no in-flight region other than the newest overlaps [lo, hi)
+    bool disjoint_from_inflight(size_t lo, size_t hi) const {
+        for (size_t i = 0; i + 1 < q_.size(); i++)
+            if (q_[i].lo < hi && lo < q_[i].hi) return false;
+        return true;
+    }
+    void drain() {
+        while (!q_.empty()) retire_front();
+    }
+    size_t inflight() const { return q_.size(); }
 
    private:
-    struct alignas(64) Cell {
-        std::atomic<size_t> seq;
-        uint64_t val;
-    };
-    size_t mask_;
-    std::vector<Cell> cells_;
-    alignas(64) std::atomic<size_t> enq_;
-    alignas(64) std::atomic<size_t> deq_;
+    struct Region { size_t lo, hi; Token tok; bool committed, last; };
+    void retire_front() {
+        if (!q_.front().committed) commit();
+        Region f = q_.front();
+        ops_->wait(f.tok);
+        if (f.last) ops_->recycle(f.tok);
+        q_.pop_front();
+    }
+    size_t cap_, head_ = 0, npending_ = 0;
+    Ops* ops_;
+    std::deque<Region> q_;
 };
 
 enum PtrKind { PK_INVALID = 0, PK_DEVICE = 1, PK_HOST = 2 };
@@ -145,6 +154,7 @@ struct Req {
     uint64_t a[6];
     int64_t ret;
     bool ok;
+    bool dma;      // a host->device copy was queued for this request
 };
 
 // ------------------------------------------------------------------ worker
@@ -154,11 +164,32 @@ struct Worker {
     std::thread th;
     cudaStream_t stream = nullptr;
     uint8_t* bounce = nullptr;       // pinned
-    size_t bcap = 0, bhead = 0;
-    struct Region { size_t lo, hi; cudaEvent_t ev; bool last; };
-    std::deque<Region> inflight;
-    std::vector<size_t> pending;      // indices into `inflight` awaiting an event (uncommitted)
+    size_t bcap = 0;
+    // BounceRing ops: a token is a CUDA event recorded after the queued copies were issued
+    struct RingOps {
+        Worker* w;
+        cudaEvent_t make_token() {
+            w->flush_copies();
+            Timer t(w->t_cuda);
+            cudaEvent_t e = w->get_event();
+            cudaEventRecord(e, w->stream);
+            return e;
+        }
+        void wait(cudaEvent_t e) { Timer t(w->t_wait); cudaEventSynchronize(e); }
+        void recycle(cudaEvent_t e) { w->evpool.push_back(e); }
+    };
+    RingOps ring_ops{this};
+    uint64_t t_sys = 0, t_cuda = 0, t_wait = 0;   // per-bundle timers (ns)
+    struct Timer {
+        uint64_t& acc; uint64_t t0;
+        explicit Timer(uint64_t& a) : acc(a), t0(now_ns()) {}
+        ~Timer() { acc += now_ns() - t0; }
+    };
+    BounceRing<cudaEvent_t, RingOps>* ring = nullptr;
     std::vector<cudaEvent_t> evpool;
+    // copies queued for one cudaMemcpyBatchAsync per bundle
+    std::vector<void*> cp_dst, cp_src;
+    std::vector<size_t> cp_len;
     std::vector<Req> reqs;
     std::vector<CUstreamBatchMemOpParams> ops;
     struct Cache { uintptr_t lo, hi; PtrKind kind; intptr_t host_delta; uint64_t gen; };
@@ -174,43 +205,13 @@ struct Worker {
         cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
         return e;
     }
-    // allocate n bytes of pinned bounce, waiting for in-flight DMA that still reads the range
+    // n bytes of pinned bounce; waits for in-flight DMA still reading the range
     uint8_t* alloc(size_t n) {
-        n = (n + 255) & ~(size_t)255;
-        if (n > bcap) return nullptr;
-        if (bhead + n > bcap) bhead = 0;
-        size_t lo = bhead, hi = bhead + n;
-        while (!inflight.empty()) {
-            Region& f = inflight.front();
-            bool overlap = f.lo < hi && lo < f.hi;
-            if (!overlap) break;
-            if (f.ev) {
-                cudaEventSynchronize(f.ev);
-                if (f.last) evpool.push_back(f.ev);
-            } else {
-                // uncommitted region of the current bundle: commit first, then wait
-                commit();
-                continue;
-            }
-            inflight.pop_front();
-            for (auto& p : pending) p--;   // indices shift
-        }
-        inflight.push_back(Region{lo, hi, nullptr, false});
-        pending.push_back(inflight.size() - 1);
-        bhead = hi;
-        return bounce + lo;
+        size_t o = ring->alloc(n);
+        return o == ring->NONE ? nullptr : bounce + o;
     }
-    // record one event after the copies issued so far and attach it to uncommitted regions
-    void commit() {
-        if (pending.empty()) return;
-        cudaEvent_t e = get_event();
-        cudaEventRecord(e, stream);
-        for (size_t i = 0; i < pending.size(); i++) {
-            inflight[pending[i]].ev = e;
-            inflight[pending[i]].last = (i + 1 == pending.size());
-        }
-        pending.clear();
-    }
+    void commit() { ring->commit(); }
+    void flush_copies();
     PtrKind resolve(uintptr_t p, size_t n, uint8_t** host);
     void run();
     void process(uint64_t h0, uint32_t n);
@@ -220,8 +221,13 @@ struct Worker {
     int64_t do_generic(Req& r);
     int read_small(uintptr_t p, void* out, size_t n);
     int write_small(uintptr_t p, const void* in, size_t n);
+    // queue a host->device copy; issued with the bundle's other copies by flush_copies()
+    bool dma_flag = false;
     void h2d(void* dst, const void* src, size_t n) {
-        cudaMemcpyAsync(dst, src, n, cudaMemcpyHostToDevice, stream);
+        dma_flag = true;
+        cp_dst.push_back(dst);
+        cp_src.push_back(const_cast<void*>(src));
+        cp_len.push_back(n);
     }
 };
 
@@ -239,7 +245,10 @@ struct Instance {
     uint32_t* claim_d = nullptr;
     uint32_t* seqs_d = nullptr;
     unsigned long long* mirror_d = nullptr;
+    uint64_t* hdone_h = nullptr;        // pinned, mapped: host-store completion words
+    uint64_t* hdone_d = nullptr;
     uint32_t* tail_d = nullptr;
+    uint32_t* lat_hint_d = nullptr;
     gsys_kround* krounds_d = nullptr;
     uint32_t* kblock_d = nullptr;
     uint32_t kblock_cap = 0;
@@ -253,11 +262,9 @@ struct Instance {
     bool mem64 = true;
 
     // service
-    std::thread dispatcher;
     std::vector<Worker*> workers;
-    MPMC* queue = nullptr;
     std::atomic<bool> stop{false};
-    std::atomic<uint64_t> head{0};         // doorbell entries consumed (dispatcher)
+    alignas(64) std::atomic<uint64_t> head{0};   // doorbell entries claimed by workers
     std::atomic<uint64_t> completed{0};    // requests whose completion was issued
     std::atomic<int> first_err{0};
     std::atomic<uint32_t> coalesce_max{8};
@@ -271,6 +278,7 @@ struct Instance {
     uint32_t nthreads = 0;
 
     // stats
+    std::atomic<uint64_t> st_ns_busy{0}, st_ns_syscall{0}, st_ns_cuda{0}, st_ns_wait{0};
     std::atomic<uint64_t> st_bundles{0}, st_max_bundle{0}, st_host_preads{0}, st_merged{0},
         st_bytes_read{0}, st_bytes_h2d{0}, st_errors{0};
     std::atomic<uint64_t> st_nr[8];
@@ -291,7 +299,10 @@ struct Instance {
             htrace.push_back(r);
         }
     }
-    void dispatch_loop();
+    bool ready(uint64_t pos) const {
+        uint64_t v = __atomic_load_n(&ring_h[pos & (ring_cap - 1)], __ATOMIC_ACQUIRE);
+        return (uint32_t)(v >> 32) == (uint32_t)(pos + 1);
+    }
 };
 
 Instance* g_inst[64] = {nullptr};
@@ -316,76 +327,71 @@ inline int nr_index(uint32_t nr) {
     }
 }
 
-// ------------------------------------------------------------------ dispatcher (interrupt-handler analogue)
-void Instance::dispatch_loop() {
-    cudaSetDevice(dev);
-    const uint32_t mask = ring_cap - 1;
-    uint64_t h = head.load();
+// ------------------------------------------------------------------ worker (interrupt handler + OS worker)
+void Worker::run() {
+    cudaSetDevice(inst->dev);
+    Instance* I = inst;
     uint64_t idle_since = now_ns();
-    uint64_t last_kick = kick.load();
-    auto ready = [&](uint64_t pos) -> bool {
-        uint64_t v = __atomic_load_n(&ring_h[pos & mask], __ATOMIC_ACQUIRE);
-        return (uint32_t)(v >> 32) == (uint32_t)(pos + 1);
-    };
-    while (!stop.load(std::memory_order_relaxed)) {
-        if (!ready(h)) {
-            uint64_t k = kick.load(std::memory_order_relaxed);
+    uint64_t last_kick = I->kick.load();
+    while (!I->stop.load(std::memory_order_relaxed)) {
+        uint64_t h = I->head.load(std::memory_order_acquire);
+        if (!I->ready(h)) {
+            uint64_t k = I->kick.load(std::memory_order_relaxed);
             if (k != last_kick) { last_kick = k; idle_since = now_ns(); }
-            if (now_ns() - idle_since > 5000000ull) {
-                struct timespec ts = {0, 20000};
-                nanosleep(&ts, nullptr);
+            if (now_ns() - idle_since > 2000000ull) {
+                std::unique_lock<std::mutex> lk(I->sleep_mu);
+                I->sleepers.fetch_add(1);
+                I->sleep_cv.wait_for(lk, std::chrono::microseconds(50));
+                I->sleepers.fetch_sub(1);
             } else {
                 _mm_pause();
             }
             continue;
         }
-        // first entry of a bundle: the coalescing window starts now (reading A19)
-        uint64_t h0 = h;
-        uint32_t cmax = coalesce_max.load(std::memory_order_relaxed);
-        uint64_t win = (uint64_t)window_us.load(std::memory_order_relaxed) * 1000ull;
-        uint64_t t0 = win ? now_ns() : 0;
-        h++;
-        while (h - h0 < cmax) {
-            if (ready(h)) { h++; continue; }
-            if (!win || now_ns() - t0 >= win) break;
-            _mm_pause();
+        // claim the run of ready entries at the head (a coalesced bundle, P22.9-13)
+        const uint32_t cmax = I->coalesce_max.load(std::memory_order_relaxed);
+        uint32_t n = 1;
+        while (n < cmax && I->ready(h + n)) n++;
+        if (!I->head.compare_exchange_strong(h, h + n, std::memory_order_acq_rel)) continue;
+        // coalescing window: keep extending the run for up to window microseconds (reading A19)
+        const uint64_t win = (uint64_t)I->window_us.load(std::memory_order_relaxed) * 1000ull;
+        if (win && n < cmax) {
+            const uint64_t t0 = now_ns();
+            while (n < cmax && now_ns() - t0 < win) {
+                uint64_t e = h + n;
+                if (!I->ready(e)) { _mm_pause(); continue; }
+                if (!I->head.compare_exchange_strong(e, e + 1, std::memory_order_acq_rel)) break;
+                n++;
+            }
         }
-        uint32_t n = (uint32_t)(h - h0);
-        while (!queue->push((h0 << 16) | (uint64_t)(n - 1))) _mm_pause();
-        head.store(h, std::memory_order_release);
-        st_bundles.fetch_add(1, std::memory_order_relaxed);
-        uint64_t mb = st_max_bundle.load(std::memory_order_relaxed);
-        while (n > mb && !st_max_bundle.compare_exchange_weak(mb, n)) {}
-        if (sleepers.load(std::memory_order_relaxed) > 0) {
-            std::lock_guard<std::mutex> g(sleep_mu);
-            sleep_cv.notify_one();
-        }
+        I->st_bundles.fetch_add(1, std::memory_order_relaxed);
+        uint64_t mb = I->st_max_bundle.load(std::memory_order_relaxed);
+        while (n > mb && !I->st_max_bundle.compare_exchange_weak(mb, n)) {}
+        process(h, n);
         idle_since = now_ns();
     }
 }
 
-// ------------------------------------------------------------------ worker (OS worker-thread analogue)
-void Worker::run() {
-    cudaSetDevice(inst->dev);
-    uint64_t idle_since = now_ns();
-    uint64_t item;
-    while (!inst->stop.load(std::memory_order_relaxed)) {
-        if (inst->queue->pop(&item)) {
-            uint64_t h0 = item >> 16;
-            uint32_t n = (uint32_t)(item & 0xffff) + 1;
-            process(h0, n);
-            idle_since = now_ns();
-            continue;
-        }
-        if (now_ns() - idle_since > 2000000ull) {
-            std::unique_lock<std::mutex> lk(inst->sleep_mu);
-            inst->sleepers.fetch_add(1);
-            inst->sleep_cv.wait_for(lk, std::chrono::microseconds(500));
-            inst->sleepers.fetch_sub(1);
-        } else {
-            _mm_pause();
+void Worker::flush_copies() {
+    size_t n = cp_dst.size();
+    if (!n) return;
+    Timer tm(t_cuda);
+    if (n == 1) {
+        cudaMemcpyAsync(cp_dst[0], cp_src[0], cp_len[0], cudaMemcpyHostToDevice, stream);
+    } else {
+        cudaMemcpyAttributes attr;
+        memset(&attr, 0, sizeof attr);
+        attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+        size_t idx0 = 0, fail = 0;
+        if (cudaMemcpyBatchAsync(cp_dst.data(), cp_src.data(), cp_len.data(), n, &attr, &idx0, 1, &fail, stream) !=
+            cudaSuccess) {
+            cudaGetLastError();
+            for (size_t i = 0; i < n; i++) cudaMemcpyAsync(cp_dst[i], cp_src[i], cp_len[i], cudaMemcpyHostToDevice, stream);
         }
     }
+    cp_dst.clear();
+    cp_src.clear();
+    cp_len.clear();
 }
 
 PtrKind Worker::resolve(uintptr_t p, size_t n, uint8_t** host) {
@@ -465,7 +471,8 @@ int64_t Worker::do_pread(Req& r) {
     if (k == PK_INVALID) return -EFAULT;
     inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
     if (k == PK_HOST) {
-        ssize_t z = pread(fd, hp, n, off);
+        ssize_t z;
+        { Timer tm(t_sys); z = pread(fd, hp, n, off); }
         if (z < 0) return -(int64_t)errno;
         inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
         return z;
@@ -477,7 +484,8 @@ int64_t Worker::do_pread(Req& r) {
         uint64_t piece = std::min<uint64_t>(want - total, piece_max);
         uint8_t* b = alloc(piece);
         if (!b) return total ? (int64_t)total : -ENOMEM;
-        ssize_t z = pread(fd, b, piece, off + (int64_t)total);
+        ssize_t z;
+        { Timer tm(t_sys); z = pread(fd, b, piece, off + (int64_t)total); }
         if (z < 0) return total ? (int64_t)total : -(int64_t)errno;
         if (z > 0) {
             h2d((void*)(buf + total), b, (size_t)z);
@@ -529,7 +537,9 @@ int64_t Worker::do_getrusage(Req& r) {
     int who = (int)(int64_t)r.a[0];
     uintptr_t dst = (uintptr_t)r.a[1];
     if (r.flags & GSYS_F_INLINE) {
-        if (getrusage(who, &ru) != 0) return -(int64_t)errno;
+        int z;
+        { Timer tm(t_sys); z = getrusage(who, &ru); }
+        if (z != 0) return -(int64_t)errno;
         memcpy(inst->inline_h + (size_t)r.slot * GSYS_INLINE_BYTES, &ru, sizeof ru);
         return 0;
     }
@@ -605,6 +615,8 @@ int64_t Worker::do_generic(Req& r) {
 
 void Worker::process(uint64_t h0, uint32_t n) {
     Instance* I = inst;
+    const uint64_t t_begin = now_ns();
+    t_sys = t_cuda = t_wait = 0;
     const uint32_t mask = I->ring_cap - 1;
     reqs.resize(n);
     for (uint32_t i = 0; i < n; i++) {
@@ -617,6 +629,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         r.seq = sl->seq;
         for (int k = 0; k < 6; k++) r.a[k] = sl->args[k];
         r.ret = 0;
+        r.dma = false;
         // "atomically switches any ready system call requests to the processing state" (P24.20)
         uint32_t expect = GSYS_READY;
         r.ok = __atomic_compare_exchange_n((uint32_t*)&I->area_h[r.slot].state, &expect, (uint32_t)GSYS_PROCESSING,
@@ -658,7 +671,8 @@ void Worker::process(uint64_t h0, uint32_t n) {
             if (!okd) continue;
             uint8_t* b = alloc(mg_len[g]);
             if (!b) continue;
-            ssize_t z = pread(fd, b, mg_len[g], mg_off[g]);
+            ssize_t z;
+            { Timer tm(t_sys); z = pread(fd, b, mg_len[g], mg_off[g]); }
             I->st_host_preads.fetch_add(1, std::memory_order_relaxed);
             int64_t zr = z < 0 ? -(int64_t)errno : (int64_t)z;
             if (zr > 0) I->st_bytes_read.fetch_add((uint64_t)zr, std::memory_order_relaxed);
@@ -667,6 +681,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
                 int64_t ri = gsys_split_result(zr, mgoff_in[j], r.a[2]);
                 r.ret = ri;
                 done[midx[j]] = true;
+                dma_flag = false;
                 if (ri > 0) {
                     uint8_t* hp = nullptr;
                     PtrKind k = resolve((uintptr_t)r.a[1], r.a[2], &hp);
@@ -677,6 +692,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
                         I->st_bytes_h2d.fetch_add((uint64_t)ri, std::memory_order_relaxed);
                     }
                 }
+                r.dma = dma_flag;
             }
             I->st_merged.fetch_add(mem.size(), std::memory_order_relaxed);
         }
@@ -684,24 +700,32 @@ void Worker::process(uint64_t h0, uint32_t n) {
         for (uint32_t t = 0; t < m; t++) {
             uint32_t i = midx[morder[t]];
             if (done[i]) continue;
+            dma_flag = false;
             reqs[i].ret = do_pread(reqs[i]);
+            reqs[i].dma = dma_flag;
             done[i] = true;
         }
     }
     for (uint32_t i = 0; i < n; i++) {
         Req& r = reqs[i];
         if (!r.ok || done[i]) continue;
+        dma_flag = false;
         switch (r.nr) {
             case GSYS_NR_PREAD64: r.ret = do_pread(r); break;
             case GSYS_NR_PWRITE64: r.ret = do_pwrite(r); break;
             case GSYS_NR_GETRUSAGE: r.ret = do_getrusage(r); break;
             default: r.ret = do_generic(r); break;
         }
+        r.dma = dma_flag;
     }
 
+    flush_copies();
     // ---- completion (P24.32-35): result into args[0]; blocking -> finished + completion word,
-    // non-blocking -> free + claim word cleared.  Stream memops are ordered after the DMA above.
+    // non-blocking -> free + claim word cleared.  GSYS_HOSTBUF / inline requests complete with a
+    // host store into the host-mapped word (after their DMA, if any, has drained); the others
+    // with a stream memory operation ordered after the DMA above.
     ops.clear();
+    bool need_sync = false;
     for (uint32_t i = 0; i < n; i++) {
         Req& r = reqs[i];
         const bool blocking = !(r.flags & GSYS_NONBLOCKING);
@@ -717,11 +741,20 @@ void Worker::process(uint64_t h0, uint32_t n) {
         CUstreamBatchMemOpParams op;
         memset(&op, 0, sizeof op);
         if (blocking) {
+            const uint64_t word = ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret;
+            if (r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) {
+                if (r.dma) { need_sync = true; continue; }
+                if (r.ok) {
+                    __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
+                    I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true);
+                }
+                __atomic_store_n(&I->hdone_h[r.slot], word, __ATOMIC_RELEASE);
+                continue;
+            }
             if (r.ok) {
                 __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
                 I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true);
             }
-            uint64_t word = ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret;
             if (I->mem64) {
                 op.writeValue.operation = CU_STREAM_MEM_OP_WRITE_VALUE_64;
                 op.writeValue.address = (CUdeviceptr)(I->mirror_d + r.slot);
@@ -750,9 +783,31 @@ void Worker::process(uint64_t h0, uint32_t n) {
             ops.push_back(op);
         }
     }
+    if (need_sync) {
+        // host-store completions whose payload went through the DMA: wait for it to land first
+        cudaEvent_t e = get_event();
+        {
+            Timer tm(t_wait);
+            cudaEventRecord(e, stream);
+            cudaEventSynchronize(e);
+        }
+        evpool.push_back(e);
+        for (uint32_t i = 0; i < n; i++) {
+            Req& r = reqs[i];
+            if ((r.flags & GSYS_NONBLOCKING) || !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) || !r.dma) continue;
+            gsys_slot* sl = I->area_h + r.slot;
+            if (r.ok) {
+                __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
+                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true);
+            }
+            __atomic_store_n(&I->hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret,
+                             __ATOMIC_RELEASE);
+        }
+    }
     for (size_t i = 0; i < ops.size(); i += 128) {
         unsigned cnt = (unsigned)std::min<size_t>(128, ops.size() - i);
-        CUresult cr = p_batch((CUstream)stream, cnt, ops.data() + i, 0);
+        CUresult cr;
+        { Timer tm(t_cuda); cr = p_batch((CUstream)stream, cnt, ops.data() + i, 0); }
         if (cr != CUDA_SUCCESS) {
             fprintf(stderr, "gsys: cuStreamBatchMemOp failed (%d)\n", (int)cr);
             int z = 0;
@@ -761,6 +816,10 @@ void Worker::process(uint64_t h0, uint32_t n) {
     }
     commit();
     I->completed.fetch_add(n, std::memory_order_release);
+    I->st_ns_busy.fetch_add(now_ns() - t_begin, std::memory_order_relaxed);
+    I->st_ns_syscall.fetch_add(t_sys, std::memory_order_relaxed);
+    I->st_ns_cuda.fetch_add(t_cuda, std::memory_order_relaxed);
+    I->st_ns_wait.fetch_add(t_wait, std::memory_order_relaxed);
 }
 
 int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
@@ -822,10 +881,16 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
         return fail(-ENOMEM);
     memset(I->ring_h, 0, (size_t)rc * 8);
     cudaHostGetDevicePointer((void**)&I->ring_d, I->ring_h, 0);
+    if (cudaHostAlloc((void**)&I->hdone_h, (size_t)slots * 8, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
+        return fail(-ENOMEM);
+    memset(I->hdone_h, 0, (size_t)slots * 8);
+    cudaHostGetDevicePointer((void**)&I->hdone_d, I->hdone_h, 0);
     if (cudaMalloc(&I->claim_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     if (cudaMalloc(&I->seqs_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     if (cudaMalloc(&I->mirror_d, (size_t)slots * 8) != cudaSuccess) return fail(-ENOMEM);
     if (cudaMalloc(&I->tail_d, 64) != cudaSuccess) return fail(-ENOMEM);
+    if (cudaMalloc(&I->lat_hint_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
+    cudaMemset(I->lat_hint_d, 0, (size_t)slots * 4);
     if (cudaMalloc(&I->krounds_d, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS) != cudaSuccess) return fail(-ENOMEM);
     I->kblock_cap = 4096;
     if (cudaMalloc(&I->kblock_d, (size_t)I->kblock_cap * GSYS_KSITES * 4) != cudaSuccess) return fail(-ENOMEM);
@@ -843,6 +908,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.claim = I->claim_d;
     c.seqs = I->seqs_d;
     c.mirror = I->mirror_d;
+    c.hdone = (unsigned long long*)I->hdone_d;
+    c.lat_hint = I->lat_hint_d;
     c.ring = (unsigned long long*)I->ring_d;
     c.ring_tail = I->tail_d;
     c.krounds = I->krounds_d;
@@ -855,6 +922,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.ring_mask = rc - 1;
     ev = getenv("GSYS_POLL_NS_MAX");
     c.poll_ns_max = (ev && atoi(ev) > 0) ? (unsigned)atoi(ev) : 1024u;
+    ev = getenv("GSYS_POLL_NS_HOST");
+    c.poll_ns_host = (ev && atoi(ev) > 0) ? (unsigned)atoi(ev) : 4096u;
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);
     if (cudaDeviceSynchronize() != cudaSuccess) return fail(-EIO);
 
@@ -862,13 +931,10 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     long cores = (long)std::thread::hardware_concurrency();
     cpu_set_t cs;
     if (sched_getaffinity(0, sizeof cs, &cs) == 0) cores = CPU_COUNT(&cs);
-    uint32_t nthr = (uint32_t)std::max<long>(1, std::min<long>(12, cores / 2));
+    uint32_t nthr = (uint32_t)std::max<long>(1, std::min<long>(16, cores - 2));
     ev = getenv("GSYS_THREADS");
     if (ev && atoi(ev) > 0) nthr = (uint32_t)atoi(ev);
     I->nthreads = nthr;
-    size_t qcap = 1;
-    while (qcap < (size_t)rc) qcap <<= 1;
-    I->queue = new MPMC(qcap);
     size_t bcap = 32ull << 20;
     ev = getenv("GSYS_BOUNCE_MB");
     if (ev && atoi(ev) > 0) bcap = (size_t)atoi(ev) << 20;
@@ -879,12 +945,12 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
         cudaStreamCreateWithFlags(&w->stream, cudaStreamNonBlocking);
         if (cudaHostAlloc((void**)&w->bounce, bcap, cudaHostAllocDefault) != cudaSuccess) return fail(-ENOMEM);
         w->bcap = bcap;
+        w->ring = new BounceRing<cudaEvent_t, Worker::RingOps>(bcap, &w->ring_ops);
         w->reqs.reserve(4096);
         w->ops.reserve(8192);
         I->workers.push_back(w);
     }
     for (Worker* w : I->workers) w->th = std::thread([w] { w->run(); });
-    I->dispatcher = std::thread([I] { I->dispatch_loop(); });
     *out = I;
     return 0;
 }
@@ -1018,6 +1084,10 @@ int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint3
     cudaMemsetAsync(I->krounds_d, 0, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS, s);
     I->gen.fetch_add(1);
     I->kick.fetch_add(1);
+    if (I->sleepers.load(std::memory_order_relaxed) > 0) {
+        std::lock_guard<std::mutex> lk(I->sleep_mu);
+        I->sleep_cv.notify_all();
+    }
     cudaError_t e = cudaLaunchKernel(kernel, dim3(gx, gy, gz), dim3(bx, by, bz), args, smem_bytes, s);
     return cuda_err(e);
 }
@@ -1050,24 +1120,25 @@ int gsys_shutdown(void) {
         std::lock_guard<std::mutex> lk(I->sleep_mu);
         I->sleep_cv.notify_all();
     }
-    if (I->dispatcher.joinable()) I->dispatcher.join();
     for (Worker* w : I->workers) {
         if (w->th.joinable()) w->th.join();
         cudaStreamSynchronize(w->stream);
-        for (auto& rg : w->inflight) if (rg.ev && rg.last) cudaEventDestroy(rg.ev);
+        w->ring->drain();
+        delete w->ring;
         for (auto e : w->evpool) cudaEventDestroy(e);
         cudaStreamDestroy(w->stream);
         cudaFreeHost(w->bounce);
         delete w;
     }
-    delete I->queue;
     cudaFreeHost(I->area_h);
     cudaFreeHost(I->inline_h);
     cudaFreeHost(I->ring_h);
+    cudaFreeHost(I->hdone_h);
     cudaFree(I->claim_d);
     cudaFree(I->seqs_d);
     cudaFree(I->mirror_d);
     cudaFree(I->tail_d);
+    cudaFree(I->lat_hint_d);
     cudaFree(I->krounds_d);
     cudaFree(I->kblock_d);
     cudaFree(I->ctx_d);
@@ -1100,6 +1171,10 @@ int gsys_stats(gsys_stats_t* out) {
     out->bytes_h2d = I->st_bytes_h2d.load();
     out->errors = I->st_errors.load();
     for (int k = 0; k < 8; k++) out->per_nr[k] = I->st_nr[k].load();
+    out->ns_busy = I->st_ns_busy.load();
+    out->ns_syscall = I->st_ns_syscall.load();
+    out->ns_cuda = I->st_ns_cuda.load();
+    out->ns_bounce_wait = I->st_ns_wait.load();
     out->threads = I->nthreads;
     out->slots = I->nslots;
     out->coalesce_max = I->coalesce_max.load();
@@ -1112,6 +1187,10 @@ int gsys_stats_reset(void) {
     if (!I) return -ENODEV;
     I->st_bundles.store(0);
     I->st_max_bundle.store(0);
+    I->st_ns_busy.store(0);
+    I->st_ns_syscall.store(0);
+    I->st_ns_cuda.store(0);
+    I->st_ns_wait.store(0);
     I->st_host_preads.store(0);
     I->st_merged.store(0);
     I->st_bytes_read.store(0);
@@ -1163,6 +1242,42 @@ int gsys_plan_merge(uint32_t n, const int32_t* fd, const int64_t* off, const uin
         group_len[g] = (uint64_t)(u1 - u0);
     }
     return g + 1;
+}
+
+// Self-test of the bounce ring allocator with a fake completion model: random allocation sizes
+// and commit points; after every allocation no other in-flight region may overlap the new one,
+// and every waited token must have been issued.  Returns 0 or -EPROTO.
+namespace {
+struct FakeOps {
+    uint64_t issued = 0, waited_max = 0, waits = 0;
+    bool bad = false;
+    uint64_t make_token() { return ++issued; }
+    void wait(uint64_t t) {
+        if (t == 0 || t > issued) bad = true;
+        waits++;
+        if (t > waited_max) waited_max = t;
+    }
+    void recycle(uint64_t) {}
+};
+}  // namespace
+
+int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap) {
+    if (cap < 4096) return -EINVAL;
+    FakeOps ops;
+    BounceRing<uint64_t, FakeOps> ring(cap, &ops);
+    uint64_t x = seed | 1;
+    for (uint32_t i = 0; i < iters; i++) {
+        x ^= x << 13; x ^= x >> 7; x ^= x << 17;
+        size_t n = 1 + (size_t)(x % (cap / ((x >> 20) % 4 == 0 ? 1 : 8)));
+        size_t lo = ring.alloc(n);
+        if (n > cap) { if (lo != ring.NONE) return -EPROTO; continue; }
+        if (lo == ring.NONE) return -EPROTO;
+        size_t hi = lo + ((n + 255) & ~(size_t)255);
+        if (hi > cap || !ring.disjoint_from_inflight(lo, hi)) return -EPROTO;
+        if ((x >> 33) % 3 == 0) ring.commit();
+    }
+    ring.drain();
+    return ops.bad ? -EPROTO : 0;
 }
 
 int64_t gsys_split_result(int64_t r, uint64_t offset_in_group, uint64_t len) {

@@ -20,6 +20,7 @@
 #include <cuda_runtime.h>
 #include <errno.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <mutex>
@@ -40,23 +41,85 @@ struct ScanState {
     int* hit;              // shared grep-hit flag of the current chunk (nullptr: no grep)
 };
 
+// Load policies: LD_NC for text that is immutable during the kernel (HBM scan), LD_CG for device
+// staging lines refilled by the copy engine between chunks (L2 is the point of coherence; skip
+// L1), LD_SYS for host-mapped staging lines refilled by host preads (ld.cv: cached system-memory
+// lines are considered stale and fetched again; unlike strong .sys loads these still coalesce
+// into full PCIe read requests -- the strong form ran at ~35 MB/s per work-group).
+enum LoadPolicy { LD_NC = 0, LD_CG = 1, LD_SYS = 2, LD_CA = 3 };
+
+template <int P>
+__device__ __forceinline__ uint4 ld16(const unsigned char* p) {
+    uint4 v;
+    if (P == LD_NC)
+        asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    else if (P == LD_CG)
+        asm volatile("ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    else if (P == LD_CA)
+        asm volatile("ld.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    else
+        asm volatile("ld.global.cv.v4.u32 {%0, %1, %2, %3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    return v;
+}
+template <int P>
+__device__ __forceinline__ unsigned ld1(const unsigned char* p) {
+    unsigned v;
+    if (P == LD_NC) asm volatile("ld.global.nc.u8 %0, [%1];" : "=r"(v) : "l"(p));
+    else if (P == LD_CG) asm volatile("ld.global.cg.u8 %0, [%1];" : "=r"(v) : "l"(p));
+    else if (P == LD_CA) asm volatile("ld.global.u8 %0, [%1];" : "=r"(v) : "l"(p));
+    else asm volatile("ld.global.cv.u8 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v & 0xffu;
+}
+
 // Scan positions [s, own_end) of a text whose valid bytes end at valid_end; seg0 points at the
-// byte of position s (16-byte aligned); seg0[-1] is the byte before s when s > 0.  Thread t takes
-// the 16-byte steps t, t + blockDim, ... (coalesced uint4 loads; the lookahead B is the next
-// thread's A and is served by L1).
+// byte of position s (16-byte aligned); seg0[-1] is the byte before s when s > 0.  Each warp
+// takes 512 consecutive bytes per step, lane l the 16 bytes at +16*l (one coalesced uint4 load);
+// the 16-byte lookahead B is lane l+1's A and the byte before is lane l-1's last byte (warp
+// shuffles), so every byte crosses the memory system once; lanes 31 / 0 fetch the edges.  A warp
+// issues the loads of SCAN_U steps before it processes them (memory-level parallelism for the
+// PCIe-latency-bound host-mapped case and for HBM).
+constexpr int SCAN_U = 4;
+
+template <int P>
 __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                            long long valid_end, const ScanState& S) {
     const ScanTables& T = *S.T;
     const bool grep = S.hit != nullptr && T.npat > 0;
     unsigned* wh = S.whist;
-    for (long long p0 = s + 16ll * threadIdx.x; p0 < own_end; p0 += 16ll * blockDim.x) {
-        const unsigned char* q = seg0 + (p0 - s);
-        const uint4 A = *reinterpret_cast<const uint4*>(q);
-        const uint4 B = (p0 + 16 < valid_end) ? *reinterpret_cast<const uint4*>(q + 16) : make_uint4(0, 0, 0, 0);
-        const unsigned prevb = p0 > 0 ? q[-1] : 0u;
-        const bool g = grep && !*(volatile int*)S.hit;
-        if (scan_step(T, A, B, prevb, p0, own_end, valid_end, g, [wh](unsigned d) { atomicAdd(&wh[d], 1u); }))
-            *S.hit = 1;
+    const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const long long wstride = 512ll * nwarps;
+    for (long long base0 = s + 512ll * warp; base0 < own_end; base0 += wstride * SCAN_U) {
+        uint4 Av[SCAN_U], Be[SCAN_U];
+        unsigned pe[SCAN_U];
+#pragma unroll
+        for (int u = 0; u < SCAN_U; u++) {
+            const long long p0 = base0 + wstride * u + 16ll * lane;
+            const unsigned char* q = seg0 + (p0 - s);
+            Av[u] = p0 < valid_end ? ld16<P>(q) : make_uint4(0, 0, 0, 0);
+            Be[u] = (lane == 31u && p0 + 16 < valid_end) ? ld16<P>(q + 16) : make_uint4(0, 0, 0, 0);
+            pe[u] = (lane == 0u && p0 > 0 && p0 - 1 < valid_end) ? ld1<P>(q - 1) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < SCAN_U; u++) {
+            const long long base = base0 + wstride * u;
+            if (base >= own_end) break;   // warp-uniform
+            const long long p0 = base + 16ll * lane;
+            const uint4 A = Av[u];
+            uint4 B;
+            B.x = __shfl_down_sync(0xffffffffu, A.x, 1);
+            B.y = __shfl_down_sync(0xffffffffu, A.y, 1);
+            B.z = __shfl_down_sync(0xffffffffu, A.z, 1);
+            B.w = __shfl_down_sync(0xffffffffu, A.w, 1);
+            unsigned prevb = __shfl_up_sync(0xffffffffu, A.w >> 24, 1);
+            if (lane == 31u) B = Be[u];
+            if (lane == 0u) prevb = pe[u];
+            if (p0 < own_end) {
+                const bool g = grep && !*(volatile int*)S.hit;
+                if (scan_step(T, A, B, prevb, p0, own_end, valid_end, g, [wh](unsigned d) { atomicAdd(&wh[d], 1u); }))
+                    *S.hit = 1;
+            }
+        }
     }
 }
 
@@ -85,10 +148,11 @@ struct WcArgs {
     unsigned long long* hist;
     unsigned* file_hits;
     long long* req_ret;
-    unsigned nfiles, nchunks, chunk, stride, gflags, pad_;
+    unsigned long long* prof;       // optional: [0] ns waiting in the call, [1] ns scanning, [2] chunks
+    unsigned nfiles, nchunks, chunk, stride, gflags, host_staging, ld_policy, pad_;
 };
 
-__global__ void __launch_bounds__(1024) wc_kernel(WcArgs a) {
+__global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
     __shared__ ScanTables sT;
     __shared__ int s_hit;
     extern __shared__ unsigned shist[];
@@ -116,16 +180,32 @@ __global__ void __launch_bounds__(1024) wc_kernel(WcArgs a) {
         const bool grep = a.file_hits != nullptr && sT.npat > 0 && *(volatile unsigned*)&a.file_hits[f] == 0u;
         if (threadIdx.x == 0) s_hit = 0;
         // row a1-a6: one work-group pread of the chunk + halo (P32.7)
-        const long long r = gsys_pread(a.ctx, a.fds[f], dst, (size_t)len, off, a.gflags);
+        const unsigned long long t0 = a.prof ? gsys::globaltimer() : 0ull;
+        const long long r = gsys_pread(a.ctx, a.fds[f], dst, (size_t)len, off,
+                                       a.gflags | (a.host_staging == 1u ? GSYS_HOSTBUF : 0u));
+        const unsigned long long t1 = a.prof ? gsys::globaltimer() : 0ull;
         if (threadIdx.x == 0 && a.req_ret) a.req_ret[k] = r;
         if (r > 0) {
             const long long valid_end = off + r;
             const long long own_end = e < valid_end ? e : valid_end;
             S.hit = grep ? &s_hit : nullptr;
-            if (own_end > s) scan_range(base + 16, s, own_end, valid_end, S);
+            if (own_end > s) {
+                switch (a.ld_policy) {
+                    case LD_SYS: scan_range<LD_SYS>(base + 16, s, own_end, valid_end, S); break;
+                    case LD_CA: scan_range<LD_CA>(base + 16, s, own_end, valid_end, S); break;
+                    case LD_NC: scan_range<LD_NC>(base + 16, s, own_end, valid_end, S); break;
+                    default: scan_range<LD_CG>(base + 16, s, own_end, valid_end, S); break;
+                }
+            }
         }
         __syncthreads();   // the staging line is free again before the next chunk's pread
         if (threadIdx.x == 0 && grep && s_hit) atomicExch(&a.file_hits[f], 1u);
+        if (a.prof && threadIdx.x == 0) {
+            const unsigned long long t2 = gsys::globaltimer();
+            atomicAdd(&a.prof[0], t1 - t0);
+            atomicAdd(&a.prof[1], t2 - t1);
+            atomicAdd(&a.prof[2], 1ull);
+        }
     }
     __syncthreads();
     flush_hist(shist, nwarps, sT.ndict, a.hist);
@@ -142,7 +222,7 @@ struct ScanArgs {
     unsigned chunk, pad_;
 };
 
-__global__ void __launch_bounds__(1024) scan_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(256, 4) scan_kernel(ScanArgs a) {
     __shared__ ScanTables sT;
     __shared__ int s_hit;
     extern __shared__ unsigned shist[];
@@ -158,7 +238,7 @@ __global__ void __launch_bounds__(1024) scan_kernel(ScanArgs a) {
     for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         const long long s = (long long)k * a.chunk;
         const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
-        scan_range(a.text + s, s, e, (long long)a.n, S);
+        scan_range<LD_NC>(a.text + s, s, e, (long long)a.n, S);
     }
     __syncthreads();
     flush_hist(shist, nwarps, sT.ndict, a.hist);
@@ -262,6 +342,10 @@ struct Workspace {
     cudaEvent_t up_ev = nullptr;
     unsigned char* staging_d = nullptr;
     size_t staging_cap = 0;
+    unsigned long long* prof_d = nullptr;  // wc_kernel profile counters (gsys_set_profile)
+    bool prof_on = false;
+    unsigned char* hstaging = nullptr;    // pinned, host-mapped (zero-copy staging)
+    size_t hstaging_cap = 0;
     int sms = 0;
 };
 Workspace g_ws[64];
@@ -301,6 +385,16 @@ int ensure_staging(Workspace* W, size_t bytes) {
     return 0;
 }
 
+int ensure_hstaging(Workspace* W, size_t bytes) {
+    if (bytes <= W->hstaging_cap) return 0;
+    if (W->hstaging) { cudaDeviceSynchronize(); cudaFreeHost(W->hstaging); }
+    W->hstaging = nullptr; W->hstaging_cap = 0;
+    if (cudaHostAlloc((void**)&W->hstaging, bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
+        return -ENOMEM;
+    W->hstaging_cap = bytes;
+    return 0;
+}
+
 int map_cuda(cudaError_t e) {
     if (e == cudaSuccess) return 0;
     if (e == cudaErrorMemoryAllocation) return -ENOMEM;
@@ -316,15 +410,16 @@ extern "C" {
 
 int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, uint32_t chunk, const char* dict,
                    const uint8_t* dlen, uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat,
-                   uint64_t* d_hist, uint32_t* d_file_hits, int64_t* d_req_ret, uint32_t gflags, uint32_t blocks,
-                   uint32_t threads, void* stream) {
+                   uint64_t* d_hist, uint32_t* d_file_hits, int64_t* d_req_ret, uint32_t gflags, uint32_t staging,
+                   uint32_t blocks, uint32_t threads, void* stream) {
     gsys_dev_ctx* ctx = gsys_internal_ctx_d();
     if (!ctx) return -ENODEV;
     if ((gflags & GSYS_GRAN_MASK) != GSYS_WG || (gflags & GSYS_NONBLOCKING)) return -EINVAL;
+    if (staging > GSYS_STAGE_HOST) return -EINVAL;
     if (nfiles == 0 || !fds || !sizes || !d_hist) return -EINVAL;
     if (chunk < 4096 || (chunk % 16) || chunk > (1u << 30)) return -EINVAL;
     if (threads == 0) threads = 256;
-    if (threads % 32 || threads > 1024) return -EINVAL;
+    if (threads % 32 || threads > 256) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
@@ -337,7 +432,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
         if (nch >= (1ull << 32)) return -EINVAL;
     }
     cbase[nfiles] = (unsigned)nch;
-    if (blocks == 0) blocks = 4u * (uint32_t)W->sms;
+    if (blocks == 0) blocks = 2u * (uint32_t)W->sms;
     if (nch < blocks) blocks = (uint32_t)(nch ? nch : 1);
     // upload: [tables][fds][sizes][cbase]
     size_t o_t = 0, o_f = align_up(sizeof(ScanTables), 256), o_s = align_up(o_f + 4ull * nfiles, 256),
@@ -353,8 +448,16 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
     cudaEventRecord(W->up_ev, s);
     size_t stride = align_up((size_t)chunk + 64, 256);
-    rc = ensure_staging(W, stride * blocks);
-    if (rc) return rc;
+    unsigned char* stage = nullptr;
+    if (staging == GSYS_STAGE_HOST) {
+        rc = ensure_hstaging(W, stride * blocks);
+        if (rc) return rc;
+        cudaHostGetDevicePointer((void**)&stage, W->hstaging, 0);
+    } else {
+        rc = ensure_staging(W, stride * blocks);
+        if (rc) return rc;
+        stage = W->staging_d;
+    }
     WcArgs a;
     memset(&a, 0, sizeof a);
     a.ctx = ctx;
@@ -362,7 +465,12 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.fds = reinterpret_cast<const int*>(W->up_d + o_f);
     a.sizes = reinterpret_cast<const unsigned long long*>(W->up_d + o_s);
     a.chunk_base = reinterpret_cast<const unsigned*>(W->up_d + o_c);
-    a.staging = W->staging_d;
+    a.staging = stage;
+    if (W->prof_on) {
+        if (!W->prof_d && cudaMalloc((void**)&W->prof_d, 64) != cudaSuccess) return -ENOMEM;
+        a.prof = W->prof_d;
+    }
+    a.host_staging = staging == GSYS_STAGE_HOST ? 1u : 0u;
     a.hist = reinterpret_cast<unsigned long long*>(d_hist);
     a.file_hits = d_file_hits;
     a.req_ret = reinterpret_cast<long long*>(d_req_ret);
@@ -377,6 +485,27 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     return gsys_launch((const void*)wc_kernel, blocks, 1, 1, threads, 1, 1, args, smem, stream);
 }
 
+int gsys_set_profile(int on) {
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    Workspace* W = workspace();
+    if (!W) return -ENODEV;
+    W->prof_on = on != 0;
+    if (W->prof_on && !W->prof_d) {
+        if (cudaMalloc((void**)&W->prof_d, 64) != cudaSuccess) return -ENOMEM;
+        cudaMemset(W->prof_d, 0, 64);
+    }
+    return 0;
+}
+
+int gsys_read_profile(uint64_t* out3, int reset) {
+    std::lock_guard<std::mutex> g(g_ws_mu);
+    Workspace* W = workspace();
+    if (!W || !W->prof_d) return -ENODEV;
+    if (cudaMemcpy(out3, W->prof_d, 24, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    if (reset) cudaMemset(W->prof_d, 0, 64);
+    return 0;
+}
+
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const char* dict, const uint8_t* dlen,
                      uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, uint64_t* d_hist,
                      uint32_t* d_hit, uint32_t blocks, uint32_t threads, void* stream) {
@@ -384,7 +513,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
     if (threads == 0) threads = 256;
-    if (threads % 32 || threads > 1024) return -EINVAL;
+    if (threads % 32 || threads > 256) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;

@@ -14,6 +14,7 @@ from . import build as _build
 WI, WG, KERNEL = 0x01, 0x02, 0x04
 BLOCKING, NONBLOCKING = 0x00, 0x08
 STRONG, RELAXED = 0x00, 0x10
+HOSTBUF = 0x20
 WEAK = RELAXED
 FREE, POPULATING, READY, PROCESSING, FINISHED = 0, 1, 2, 3, 4
 NR_PREAD64, NR_PWRITE64, NR_GETRUSAGE = 17, 18, 98
@@ -31,7 +32,9 @@ class Stats(ctypes.Structure):
     _fields_ = [("requests", ctypes.c_uint64), ("completed", ctypes.c_uint64), ("bundles", ctypes.c_uint64),
                 ("max_bundle", ctypes.c_uint64), ("host_preads", ctypes.c_uint64), ("merged", ctypes.c_uint64),
                 ("bytes_read", ctypes.c_uint64), ("bytes_h2d", ctypes.c_uint64), ("errors", ctypes.c_uint64),
-                ("per_nr", ctypes.c_uint64 * 8), ("threads", ctypes.c_uint32), ("slots", ctypes.c_uint32),
+                ("per_nr", ctypes.c_uint64 * 8), ("ns_busy", ctypes.c_uint64), ("ns_syscall", ctypes.c_uint64),
+                ("ns_cuda", ctypes.c_uint64), ("ns_bounce_wait", ctypes.c_uint64),
+                ("threads", ctypes.c_uint32), ("slots", ctypes.c_uint32),
                 ("coalesce_max", ctypes.c_uint32), ("coalesce_window_us", ctypes.c_uint32)]
 
     def as_dict(self):
@@ -70,8 +73,11 @@ SIGNATURES = {
     "gsys_abi_info": (ctypes.c_int, [_P, _P, _P]),
     "gsys_plan_merge": (ctypes.c_int, [_U32, _P, _P, _P, _U64, _P, _P, _P, _P, _P]),
     "gsys_split_result": (_I64, [_I64, _U64, _U64]),
+    "gsys_selftest_bounce": (ctypes.c_int, [_U64, _U32, _U64]),
+    "gsys_set_profile": (ctypes.c_int, [ctypes.c_int]),
+    "gsys_read_profile": (ctypes.c_int, [_P, ctypes.c_int]),
     "gsys_wordcount": (ctypes.c_int, [_P, _P, _U32, _U32, ctypes.c_char_p, _P, _U32, ctypes.c_char_p, _P, _U32,
-                                      _P, _P, _P, _U32, _U32, _U32, _P]),
+                                      _P, _P, _P, _U32, _U32, _U32, _U32, _P]),
     "gsys_scan_device": (ctypes.c_int, [_P, _U64, _U32, ctypes.c_char_p, _P, _U32, ctypes.c_char_p, _P, _U32,
                                         _P, _P, _U32, _U32, _P]),
     "gsys_bench_calls": (ctypes.c_int, [_U32, _U32, _U32, _U32, _U32, _I32, _U64, _U64, _P, _P, _P, _P, _P]),
@@ -167,6 +173,16 @@ def gsys_trace_read(cap: int = 1 << 20):
     return conv(g, ng.value), conv(h, nh.value)
 
 
+def gsys_set_profile(on: bool) -> int:
+    return _check(lib().gsys_set_profile(int(bool(on))), "gsys_set_profile")
+
+
+def gsys_read_profile(reset: bool = True) -> dict:
+    out = (ctypes.c_uint64 * 3)()
+    _check(lib().gsys_read_profile(out, int(bool(reset))), "gsys_read_profile")
+    return {"wait_ns": out[0], "scan_ns": out[1], "chunks": out[2]}
+
+
 def gsys_abi_info():
     a, b, c = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
     lib().gsys_abi_info(ctypes.byref(a), ctypes.byref(b), ctypes.byref(c))
@@ -205,8 +221,12 @@ def pack_words(words):
     return bytes(buf), lens
 
 
+STAGE_DEVICE, STAGE_HOST = 0, 1
+
+
 def gsys_wordcount(fds, sizes, chunk: int, dict_words, patterns, d_hist, d_file_hits=None, d_req_ret=None,
-                   gflags: int = WG | BLOCKING | STRONG, blocks: int = 0, threads: int = 0, stream=None) -> int:
+                   gflags: int = WG | BLOCKING | STRONG, blocks: int = 0, threads: int = 0, stream=None,
+                   staging: int = STAGE_DEVICE) -> int:
     """Launch the GPU-syscall wordcount/grep (asynchronous; gsys_wait(stream) before reading).
     d_hist: device uint64 tensor [ndict] (added into); d_file_hits: device int32 [nfiles] or None;
     d_req_ret: device int64 [chunks] or None."""
@@ -217,8 +237,8 @@ def gsys_wordcount(fds, sizes, chunk: int, dict_words, patterns, d_hist, d_file_
     p, pl = pack_words(patterns)
     rc = lib().gsys_wordcount(fd_arr, sz_arr, n, chunk, d, dl, len(dict_words), p, pl, len(patterns),
                               d_hist.data_ptr(), d_file_hits.data_ptr() if d_file_hits is not None else None,
-                              d_req_ret.data_ptr() if d_req_ret is not None else None, gflags, blocks, threads,
-                              _stream(stream))
+                              d_req_ret.data_ptr() if d_req_ret is not None else None, gflags, staging, blocks,
+                              threads, _stream(stream))
     return _check(rc, "gsys_wordcount")
 
 

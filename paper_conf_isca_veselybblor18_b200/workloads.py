@@ -78,7 +78,7 @@ def nchunks(sizes, chunk: int) -> int:
 
 def wordcount_fds(fds, sizes, dict_words, patterns, chunk: int = 256 << 10, gflags: int = G.WG | G.BLOCKING | G.STRONG,
                   blocks: int = 0, threads: int = 0, stream=None, want_ret: bool = True,
-                  d_hist=None, d_hits=None, d_ret=None):
+                  d_hist=None, d_hits=None, d_ret=None, staging: int = G.STAGE_DEVICE):
     """Launch + drain on device tensors (no host copies).  Returns (d_hist, d_hits, d_ret, rc)."""
     ensure_init()
     dev = torch.device("cuda", torch.cuda.current_device())
@@ -89,17 +89,18 @@ def wordcount_fds(fds, sizes, dict_words, patterns, chunk: int = 256 << 10, gfla
     if d_ret is None and want_ret:
         d_ret = torch.full((max(nchunks(sizes, chunk), 1),), -(1 << 40), dtype=torch.int64, device=dev)
     stream = stream or torch.cuda.current_stream()
-    G.gsys_wordcount(fds, sizes, chunk, dict_words, patterns, d_hist, d_hits, d_ret, gflags, blocks, threads, stream)
+    G.gsys_wordcount(fds, sizes, chunk, dict_words, patterns, d_hist, d_hits, d_ret, gflags, blocks, threads, stream,
+                     staging)
     rc = G.gsys_wait(stream)
     return d_hist, d_hits, d_ret, rc
 
 
 def wordcount_files(paths, dict_words, patterns, chunk: int = 256 << 10, gflags: int = G.WG | G.BLOCKING | G.STRONG,
-                    blocks: int = 0, threads: int = 0, stream=None) -> WordcountResult:
+                    blocks: int = 0, threads: int = 0, stream=None, staging: int = G.STAGE_DEVICE) -> WordcountResult:
     """The public end-to-end call: files in, host histogram / grep hits / pread returns out."""
     with OpenFiles(paths) as of:
         h, hits, ret, rc = wordcount_fds(of.fds, of.sizes, dict_words, patterns, chunk, gflags, blocks, threads,
-                                         stream)
+                                         stream, staging=staging)
         out = WordcountResult(h.cpu(), hits.cpu() if hits is not None else None,
                               ret.cpu() if ret is not None else None, rc)
     return out

@@ -104,3 +104,11 @@ def test_split_result_equals_individual_pread(tmpdir_shm):
     finally:
         os.close(fd)
     assert G.gsys_split_result(-errno.EIO, 5, 10) == -errno.EIO
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 12345])
+@pytest.mark.parametrize("cap", [4096, 1 << 20, 32 << 20])
+def test_bounce_ring_never_overlaps_inflight(seed, cap):
+    """Regression for the wrap bug: a wrapped allocation must wait for the previous lap's tail
+    and for the current lap's oldest regions before reusing bounce memory."""
+    assert G.lib().gsys_selftest_bounce(seed, 20000, cap) == 0

@@ -55,11 +55,13 @@ def as_u64(t):
 
 
 # ---------------------------------------------------------------------------- wordcount (rows a1-a8)
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
 @pytest.mark.parametrize("order", [G.STRONG, G.RELAXED])
-def test_wordcount_config1_parity(file16m, order):
-    """Config 1: 16 MiB file, 64 work-groups, WG + blocking (+ strong / relaxed)."""
+def test_wordcount_config1_parity(file16m, order, staging):
+    """Config 1: 16 MiB file, 64 work-groups, WG + blocking (+ strong / relaxed), device or
+    host-mapped (zero-copy) staging."""
     p, census = file16m
-    res = W.wordcount_files([p], WORDS, PATS, chunk=256 << 10, gflags=G.WG | G.BLOCKING | order)
+    res = W.wordcount_files([p], WORDS, PATS, chunk=256 << 10, gflags=G.WG | G.BLOCKING | order, staging=staging)
     assert res.wait_rc == 0
     data = open(p, "rb").read()
     want = oracle.count_tokens(data, WORDS)
@@ -73,12 +75,13 @@ def test_wordcount_config1_parity(file16m, order):
     assert bool(res.file_hits[0]) == oracle.grep(data, PATS)
 
 
-@pytest.mark.parametrize("chunk,blocks,threads", [(4096, 7, 64), (256 << 10, 0, 256), (64 << 10, 3, 1024),
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
+@pytest.mark.parametrize("chunk,blocks,threads", [(4096, 7, 64), (256 << 10, 0, 256), (64 << 10, 3, 256),
                                                   (1 << 20, 1, 128)])
-def test_wordcount_ragged_corpus(ragged_corpus, chunk, blocks, threads):
+def test_wordcount_ragged_corpus(ragged_corpus, chunk, blocks, threads, staging):
     c = ragged_corpus
     res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, blocks=blocks, threads=threads,
-                            gflags=G.WG | G.BLOCKING | G.RELAXED)
+                            gflags=G.WG | G.BLOCKING | G.RELAXED, staging=staging)
     h, hits = oracle_hist_hits(c.paths)
     assert res.wait_rc == 0
     assert np.array_equal(as_u64(res.hist), h)
@@ -287,7 +290,8 @@ def test_protocol_trace_validates(file1m):
 
 # ---------------------------------------------------------------------------- full size (config 3 shape)
 @pytest.mark.slow
-def test_full_size_corpus_census(tmpdir_shm):
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
+def test_full_size_corpus_census(tmpdir_shm, staging):
     """8 GiB, 512 x 16 MiB files, the bench launch configuration: whole-corpus histogram equals
     the generator's census and grep hits equal the planted set; 4 sampled files through the oracle."""
     import shutil
@@ -295,11 +299,13 @@ def test_full_size_corpus_census(tmpdir_shm):
     if free < (10 << 30):
         pytest.skip("tmpfs too small for the 8 GiB corpus")
     c = inputs.make_corpus(512, 16 << 20, seed=inputs.SEED_CORPUS, root=tmpdir_shm, tag="full8g")
-    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=256 << 10, gflags=G.WG | G.BLOCKING | G.RELAXED)
-    assert np.array_equal(as_u64(res.hist), c.census)
+    for chunk in (256 << 10, 1 << 20):
+        res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, gflags=G.WG | G.BLOCKING | G.RELAXED,
+                                staging=staging)
+        assert np.array_equal(as_u64(res.hist), c.census)
     assert res.file_hits.tolist() == [1 if m else 0 for m in c.pmasks]
     assert (res.req_ret > 0).all()
     for f in (0, 101, 255, 511):
         h, hits = oracle_hist_hits([c.paths[f]])
-        r1 = W.wordcount_files([c.paths[f]], WORDS, PATS, chunk=256 << 10)
+        r1 = W.wordcount_files([c.paths[f]], WORDS, PATS, chunk=256 << 10, staging=staging)
         assert np.array_equal(as_u64(r1.hist), h) and r1.file_hits.tolist() == hits.tolist()
