@@ -1,0 +1,13 @@
+"""scan_kernel over 1 GiB HBM-resident corpus text (for ncu kernel replay)."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import inputs
+from paper_conf_isca_veselybblor18_b200 import gsys as G
+c = inputs.make_corpus(512, 16 << 20)
+text = torch.cat([torch.from_file(p, dtype=torch.uint8, size=os.path.getsize(p)) for p in c.paths[:64]]).cuda()
+hist = torch.zeros(64, dtype=torch.int64, device="cuda")
+for _ in range(3):
+    G.gsys_scan_device(text, text.numel(), 256 << 10, inputs.dictionary(), inputs.patterns(), hist, None, 0, 256)
+torch.cuda.synchronize()
+print("ok")

@@ -1,0 +1,13 @@
+"""Single wordcount launch for ncu (application replay): 64 x 16 MiB files, host staging."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import inputs
+from paper_conf_isca_veselybblor18_b200 import gsys as G
+from paper_conf_isca_veselybblor18_b200 import workloads as W
+staging = G.STAGE_DEVICE if (len(sys.argv) > 1 and sys.argv[1] == "device") else G.STAGE_HOST
+c = inputs.make_corpus(512, 16 << 20)
+paths = c.paths[:64]
+res = W.wordcount_files(paths, inputs.dictionary(), inputs.patterns(), chunk=256 << 10,
+                        gflags=G.WG | G.BLOCKING | G.RELAXED, blocks=296, staging=staging)
+print("ok", int(res.hist.sum()))
