@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip scan roofline / syscall-rate extras")
     ap.add_argument("--root", default=None, help="corpus directory (default /dev/shm/gsys_corpus)")
+    ap.add_argument("--mode", default="wordcount", choices=["wordcount", "syscalls"],
+                    help="syscalls: config-2 granularity x blocking x ordering sweep (one JSON line)")
     return ap.parse_args()
 
 
@@ -176,6 +178,8 @@ def main():
     a = parse()
     if a.impl == "reference":
         return run_reference(a)
+    if a.mode == "syscalls":
+        return run_syscalls(a)
     import torch
     import torch.distributed as dist
 
@@ -207,7 +211,8 @@ def main():
     barrier()
     corpus = inputs.make_corpus(a.files, a.file_mib << 20, root=a.root)
     words, pats = inputs.dictionary(), inputs.patterns()
-    lo, hi = rank * a.files // world, (rank + 1) * a.files // world
+    from paper_conf_isca_veselybblor18_b200 import dist as D
+    lo, hi = D.shard_range(a.files, rank, world)
     mine = corpus.paths[lo:hi]
     chunk = a.chunk_kib << 10
     gflags = G.WG | G.BLOCKING | (G.RELAXED if a.order == "relaxed" else G.STRONG)
@@ -222,7 +227,7 @@ def main():
     nf = len(mine)
     d_hist = torch.zeros(64, dtype=torch.int64, device=dev)
     d_hits = torch.zeros(max(nf, 1), dtype=torch.int32, device=dev)
-    d_all = torch.zeros(64 + a.files, dtype=torch.int64, device=dev)
+    d_all = [None]
 
     def step():
         d_hist.zero_()
@@ -230,11 +235,8 @@ def main():
         G.gsys_wordcount(of.fds, of.sizes, chunk, words, pats, d_hist, d_hits, None, gflags, a.blocks, a.threads,
                          stream, staging)
         G.gsys_wait(stream)
-        if world > 1:
-            d_all.zero_()
-            d_all[:64].copy_(d_hist)
-            d_all[64 + lo: 64 + hi].copy_(d_hits.to(torch.int64)[:nf])
-            dist.all_reduce(d_all)
+        if world > 1:   # row a9: the path's only collective
+            d_all[0] = D.reduce_result(D.pack_result(d_hist, d_hits[:nf], lo, hi, a.files))
 
     with torch.cuda.stream(stream):
         for _ in range(a.warmup):
@@ -258,7 +260,7 @@ def main():
     value = corpus.total_bytes * a.steps / dev_s / 1e9
     # parity of the last step against the generator census (cheap, exact)
     if world > 1:
-        hist_ok = bool((d_all[:64].cpu().numpy().astype("uint64") == corpus.census).all())
+        hist_ok = bool((d_all[0][:64].cpu().numpy().astype("uint64") == corpus.census).all())
     else:
         hist_ok = bool((d_hist.cpu().numpy().astype("uint64") == corpus.census).all())
 
@@ -271,12 +273,7 @@ def main():
         res = W.wordcount_files(mine, words, pats, chunk=chunk, gflags=gflags, blocks=a.blocks, threads=a.threads,
                                 stream=stream, staging=staging)
         if world > 1:
-            v = torch.zeros(64 + a.files, dtype=torch.int64)
-            v[:64] = res.hist
-            v[64 + lo: 64 + hi] = res.file_hits.to(torch.int64)[:nf]
-            vd = v.to(dev)
-            dist.all_reduce(vd)
-            vd.cpu()
+            D.reduce_result(D.pack_result(res.hist.to(dev), res.file_hits.to(dev), lo, hi, a.files)).cpu()
         e2e_t.append(max_over_ranks(time.perf_counter() - t0))
     e2e_s = statistics.median(e2e_t)
     e2e_value = corpus.total_bytes / e2e_s / 1e9
@@ -407,6 +404,113 @@ def cpu_baseline_leg(a, corpus, words, pats, chunk):
             "sample": f"{len(sample)} of {a.files} files ({sbytes / 2**20:.0f} MiB): pread + scalar wordcount + grep, "
                       f"{nthr} pthreads, {cpu_model()}",
             "getrusage_direct_calls_per_s": rate}
+
+
+def run_syscalls(a):
+    """Config 2 (BASELINE.json configs[1]): getrusage / pread microbenchmark over work-item,
+    work-group and kernel granularity x blocking x ordering (sec. VII, Fig. 7/8/10),
+    plus the unloaded ping-pong, a Fig-7 file-size sweep and a Fig-10 coalescing sweep.  Rates
+    are calls / wall time of launch..gsys_wait; latency is GPU-observed (%globaltimer) per call."""
+    import torch
+
+    import oracle
+    from paper_conf_isca_veselybblor18_b200 import gsys as G
+    from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+    torch.cuda.set_device(0)
+    W.ensure_init()
+    gname = {G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}
+    cells = [(G.WI, G.BLOCKING, G.STRONG), (G.WI, G.NONBLOCKING, G.STRONG),
+             (G.WG, G.BLOCKING, G.STRONG), (G.WG, G.BLOCKING, G.RELAXED),
+             (G.WG, G.NONBLOCKING, G.STRONG), (G.WG, G.NONBLOCKING, G.RELAXED),
+             (G.KERNEL, G.BLOCKING, G.RELAXED), (G.KERNEL, G.NONBLOCKING, G.RELAXED)]
+    root = a.root or "/dev/shm"
+    path = os.path.join(root, "gsys_mb_1GiB.bin")
+    if not os.path.exists(path) or os.path.getsize(path) != (1 << 30):
+        with open(path, "wb") as f:
+            for _ in range(16):
+                f.write(os.urandom(64 << 20))
+    fd = os.open(path, os.O_RDONLY)
+    size = 1 << 30
+    blocks, threads = 592, 256
+    out = {"mode": "syscalls", "metric": "GPU-issued syscalls/sec and GPU-observed round-trip latency",
+           "grid": f"{blocks} blocks x {threads} threads", "cells": []}
+    hbuf = torch.empty(blocks * threads * 4096, dtype=torch.uint8).pin_memory()
+    dbuf = torch.empty(blocks * threads * 4096, dtype=torch.uint8, device="cuda")
+
+    def run(kind, flags, bl, th, iters, length=0, sz=0, buf=None):
+        W.bench_calls(kind, flags, bl, th, 1, fd, length, sz or 1, buf)
+        G.gsys_stats_reset()
+        r0 = G.gsys_stats()["requests"]
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        n, ret, lat, _, rc = W.bench_calls(kind, flags, bl, th, iters, fd, length, sz or 1, buf)
+        dt = time.perf_counter() - t0
+        st = G.gsys_stats()
+        calls = st["requests"] - r0
+        lat_us = lat.double().cpu() / 1e3
+        blocking = not (flags & G.NONBLOCKING)
+        return {"calls": calls, "seconds": dt, "calls_per_s": calls / dt, "callers": n,
+                "lat_p50_us": float(lat_us.median()) if blocking else None,
+                "lat_p99_us": float(lat_us.quantile(0.99)) if blocking else None,
+                "issue_p50_us": None if blocking else float(lat_us.median()),
+                "ok": bool((ret >= 0).all()) and rc == 0,
+                "service_busy_frac": st["ns_busy"] / 1e9 / dt / st["threads"]}
+
+    for kind, iters_by in (("getrusage", {G.WI: 5, G.WG: 50, G.KERNEL: 200}),
+                           ("pread", {G.WI: 2, G.WG: 20, G.KERNEL: 100})):
+        for gran, blk, order in cells:
+            flags = gran | blk | order
+            for bufkind in (("device", "host") if kind == "pread" else ("-",)):
+                buf = None
+                if kind == "pread":
+                    buf = dbuf if bufkind == "device" else hbuf
+                    if bufkind == "host":
+                        flags |= G.HOSTBUF
+                r = run(kind, flags, blocks, threads, iters_by[gran], 4096 if kind == "pread" else 0, size, buf)
+                r.update({"kind": kind, "granularity": gname[gran], "blocking": not (blk & G.NONBLOCKING),
+                          "ordering": "relaxed" if order else "strong", "buffer": bufkind,
+                          "bytes_per_call": 4096 if kind == "pread" else 144})
+                out["cells"].append(r)
+    # unloaded ping-pong (1 caller, sequential blocking calls): the intrinsic round trip
+    out["pingpong_getrusage"] = run("getrusage", G.WG | G.BLOCKING, 1, 32, 2000)
+    out["pingpong_pread4k_host"] = run("pread", G.WG | G.BLOCKING | G.HOSTBUF, 1, 32, 2000, 4096, size, hbuf)
+    out["pingpong_pread4k_device"] = run("pread", G.WG | G.BLOCKING, 1, 32, 2000, 4096, size, dbuf)
+    # Fig. 7 (left): fixed number of work-items, whole file read at each granularity
+    fig7 = []
+    for fsz in (16 << 20, 256 << 20, 1 << 30):
+        for gran in (G.WI, G.WG, G.KERNEL):
+            callers = blocks * threads if gran == G.WI else blocks if gran == G.WG else 1
+            length = max(16, fsz // callers // 16 * 16)
+            flags = gran | G.BLOCKING | (G.RELAXED if gran == G.KERNEL else G.STRONG) | G.HOSTBUF
+            big = torch.empty(callers * length, dtype=torch.uint8).pin_memory()
+            r = run("pread", flags, blocks, threads, 1, length, fsz, big)
+            r.update({"file_bytes": fsz, "granularity": gname[gran], "bytes_per_call": length,
+                      "GBps": callers * length / r["seconds"] / 1e9})
+            fig7.append(r)
+            del big
+    out["fig7_granularity"] = fig7
+    # Fig. 10: coalescing on/off for small preads (WG, blocking), device buffers
+    fig10 = []
+    for length in (64, 1024, 16384):
+        for cmax, win in ((1, 0), (8, 0), (8, 20)):
+            G.gsys_set_coalesce_max(cmax)
+            G.gsys_set_coalesce_window(win)
+            r = run("pread", G.WG | G.BLOCKING, blocks, threads, 20, length, size, dbuf)
+            r.update({"bytes_per_call": length, "coalesce_max": cmax, "window_us": win,
+                      "ns_per_byte": r["seconds"] * 1e9 / (r["calls"] * length)})
+            fig10.append(r)
+    G.gsys_set_coalesce_max(8)
+    G.gsys_set_coalesce_window(0)
+    out["fig10_coalescing"] = fig10
+    nthr = host_cores()
+    out["oracle_direct"] = {"cores": nthr, "getrusage_calls_per_s": oracle.syscall_rate("getrusage", nthr, 200000),
+                            "pread4k_calls_per_s": oracle.syscall_rate("pread", nthr, 100000, fd, 4096, size),
+                            "getrusage_1thread": oracle.syscall_rate("getrusage", 1, 200000)}
+    out["service_threads"] = G.gsys_stats()["threads"]
+    os.close(fd)
+    print(json.dumps(out), flush=True)
+    return 0
 
 
 if __name__ == "__main__":

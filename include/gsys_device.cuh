@@ -50,7 +50,8 @@ struct gsys_dev_ctx {
     unsigned* seqs;                 /* device [nslots]: last sequence number used           */
     unsigned long long* mirror;     /* device [nslots]: completion word (seq << 32 | u32 ret) */
     unsigned long long* hdone;      /* host-mapped [nslots]: completion word for host-store completions */
-    unsigned* lat_hint;             /* device [nslots]: EWMA of the slot's round-trip latency (ns)  */
+    unsigned* lat_hint;             /* device [nslots]: learned sleep before the first host poll (ns) */
+    unsigned* nbpend;               /* device [nslots]: seq of a non-blocking request still in service */
     unsigned long long* ring;       /* host-mapped [ring_mask+1] doorbell entries           */
     unsigned* ring_tail;            /* device: next doorbell position                       */
     gsys_kround* krounds;           /* device [GSYS_KSITES * GSYS_KROUNDS]                  */
@@ -137,7 +138,15 @@ __device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, bool blocking) 
         __nanosleep(ns);
         if (ns < 1024) ns <<= 1;
     }
-    __threadfence();   /* acquire the slot's previous owner's writes (seqs[s]) */
+    __threadfence();   /* acquire the slot's previous owner's writes (seqs[s], nbpend[s]) */
+    // A non-blocking caller hands the claim back at once but the host may still be serving its
+    // request (P24.34: the CPU sets the slot free): reuse waits for that completion word.
+    const unsigned pend = c->nbpend[s];
+    if (pend) {
+        while ((unsigned)(ld_relaxed_sys(c->hdone + s) >> 32) != pend) __nanosleep(c->poll_ns_host);
+        fence_acq_rel_sys();
+        c->nbpend[s] = 0u;
+    }
     return s;
 }
 
@@ -194,25 +203,30 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
         }
     } else {
-        // every poll is a PCIe round trip: sleep ~3/4 of this slot's recent latency first, then
-        // poll at a fixed interval, so hundreds of waiting work-groups do not flood the link
+        // every poll is a PCIe round trip, so a waiting caller first sleeps for the slot's learned
+        // "sleep hint" and then polls at a fixed interval.  The hint adapts multiplicatively on
+        // the number of polls the wait took: 1 poll means it may have overslept (shrink by 1/4),
+        // more than 2 means it woke too early (grow by the extra polling time / 2), so the
+        // sleep converges just below the service latency without feeding on its own length.
         const unsigned long long* m = c->hdone + s;
-        const unsigned long long t0 = globaltimer();
-        unsigned first = (c->lat_hint[s] >> 2) * 3u;
-        while (first > 0) {
-            unsigned d = first > 500000u ? 500000u : first;
+        const unsigned hint = c->lat_hint[s];
+        unsigned left = hint;
+        while (left > 0) {
+            const unsigned d = left > 100000u ? 100000u : left;
             __nanosleep(d);
-            first -= d;
+            left -= d;
         }
+        unsigned polls = 0;
         for (;;) {
             v = ld_relaxed_sys(m);
+            polls++;
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(c->poll_ns_host);
         }
-        const unsigned long long dt = globaltimer() - t0;
-        const unsigned h = c->lat_hint[s];
-        const unsigned d32 = dt > 4000000ull ? 4000000u : (unsigned)dt;
-        c->lat_hint[s] = h ? (h - (h >> 3) + (d32 >> 3)) : d32;
+        unsigned nh = hint;
+        if (polls <= 1) nh = hint - (hint >> 2);
+        else if (polls > 2) nh = hint + (polls - 2) * (c->poll_ns_host >> 1);
+        c->lat_hint[s] = nh > 200000u ? 200000u : nh;
     }
     fence_acq_rel_sys();   /* acquire: the payload is visible before the completion word */
     return (long long)(int)(unsigned)(v & 0xffffffffull);
@@ -233,7 +247,11 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     unsigned s = claim(c, blocking);
     unsigned seq = marshal(c, s, nr, flags, a);
     doorbell(c, s);
-    if (!blocking) return 0;
+    if (!blocking) {
+        c->nbpend[s] = seq;
+        st_release_gpu(&c->claim[s], 0u);
+        return 0;
+    }
     long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) != 0u);
     if (inline_out != nullptr && r >= 0) {
         const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);

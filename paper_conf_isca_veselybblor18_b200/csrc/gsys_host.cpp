@@ -15,9 +15,10 @@
 //     of one regular file are merged into one read of the union (north_star extension), payloads
 //     for device buffers go through a pinned bounce ring and one cudaMemcpyBatchAsync per bundle,
 //     payloads for host-mapped buffers are read in place (P24.32-35);
-//   * results are returned with CUDA stream memory operations ordered after the payload DMA:
-//     blocking -> completion word {seq, ret} (state "finished"), non-blocking -> claim word
-//     cleared (state "free"), P24.33-34;
+//   * results go back as a completion word {seq, ret} (P24.32-34): a plain host store into pinned
+//     host-mapped memory that the GPU polls (system-memory buffers, inline results and every
+//     non-blocking call), or a CUDA stream memory operation ordered after the payload DMA into
+//     device memory (blocking calls on device buffers);
 //   * gsys_wait() is the paper's drain function (sec. IX, P34.9).
 // Context fix-ups (P24.22-28) are unnecessary: the service runs inside the invoking process.
 
@@ -249,6 +250,7 @@ struct Instance {
     uint64_t* hdone_d = nullptr;
     uint32_t* tail_d = nullptr;
     uint32_t* lat_hint_d = nullptr;
+    uint32_t* nbpend_d = nullptr;
     gsys_kround* krounds_d = nullptr;
     uint32_t* kblock_d = nullptr;
     uint32_t kblock_cap = 0;
@@ -394,7 +396,23 @@ void Worker::flush_copies() {
     cp_len.clear();
 }
 
+// Pinned host ranges allocated by the library itself (e.g. the wordcount's zero-copy staging):
+// recognised without a driver call, so the service never touches the CUDA API while serving
+// system-memory buffers (which also keeps it out of a profiler's serialisation lock).
+struct HostRange { std::atomic<uintptr_t> lo{0}, hi{0}; };
+HostRange g_host_ranges[32];
+std::atomic<int> g_nhost_ranges{0};
+
 PtrKind Worker::resolve(uintptr_t p, size_t n, uint8_t** host) {
+    const int nr = g_nhost_ranges.load(std::memory_order_acquire);
+    for (int i = 0; i < nr; i++) {
+        const uintptr_t lo = g_host_ranges[i].lo.load(std::memory_order_relaxed);
+        const uintptr_t hi = g_host_ranges[i].hi.load(std::memory_order_relaxed);
+        if (p >= lo && p + n <= hi) {
+            if (host) *host = (uint8_t*)p;
+            return PK_HOST;
+        }
+    }
     uint64_t g = inst->gen.load(std::memory_order_relaxed);
     for (auto& c : cache) {
         if (c.gen == g && p >= c.lo && p + n <= c.hi) {
@@ -663,10 +681,13 @@ void Worker::process(uint64_t h0, uint32_t n) {
             int fd = mfd[mem[0]];
             struct stat st;
             if (fstat(fd, &st) != 0 || !S_ISREG(st.st_mode)) continue;
+            // merge only where it saves work: device destinations go through the bounce anyway;
+            // for large reads into host memory the union read would add a second memcpy
             bool okd = true;
             for (uint32_t j : mem) {
                 Req& r = reqs[midx[j]];
-                if (r.a[2] == 0 || resolve((uintptr_t)r.a[1], r.a[2], nullptr) == PK_INVALID) { okd = false; break; }
+                PtrKind k = r.a[2] ? resolve((uintptr_t)r.a[1], r.a[2], nullptr) : PK_INVALID;
+                if (k == PK_INVALID || (k == PK_HOST && r.a[2] > (64u << 10))) { okd = false; break; }
             }
             if (!okd) continue;
             uint8_t* b = alloc(mg_len[g]);
@@ -720,10 +741,11 @@ void Worker::process(uint64_t h0, uint32_t n) {
     }
 
     flush_copies();
-    // ---- completion (P24.32-35): result into args[0]; blocking -> finished + completion word,
-    // non-blocking -> free + claim word cleared.  GSYS_HOSTBUF / inline requests complete with a
-    // host store into the host-mapped word (after their DMA, if any, has drained); the others
-    // with a stream memory operation ordered after the DMA above.
+    // ---- completion (P24.32-35): result into args[0]; blocking -> "finished" + completion word,
+    // non-blocking -> "free" + completion word (which the slot's next GPU claimer waits for).
+    // Non-blocking, GSYS_HOSTBUF and inline requests complete with a host store into the
+    // host-mapped word (after their DMA, if any, has drained); blocking requests for device
+    // buffers complete with a stream memory operation ordered after the DMA above.
     ops.clear();
     bool need_sync = false;
     for (uint32_t i = 0; i < n; i++) {
@@ -772,15 +794,15 @@ void Worker::process(uint64_t h0, uint32_t n) {
                 ops.push_back(op);
             }
         } else {
+            // non-blocking: "the state is changed to free" (P24.34); the GPU's next claimer of this
+            // slot waits for the host-mapped completion word (after any DMA has drained)
+            if (r.dma) { need_sync = true; continue; }
             if (r.ok) {
                 __atomic_store_n(&sl->state, (uint32_t)GSYS_FREE, __ATOMIC_RELEASE);
                 I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FREE, false);
             }
-            op.writeValue.operation = CU_STREAM_MEM_OP_WRITE_VALUE_32;
-            op.writeValue.address = (CUdeviceptr)(I->claim_d + r.slot);
-            op.writeValue.value = 0;
-            op.writeValue.flags = CU_STREAM_WRITE_VALUE_DEFAULT;
-            ops.push_back(op);
+            __atomic_store_n(&I->hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret,
+                             __ATOMIC_RELEASE);
         }
     }
     if (need_sync) {
@@ -794,11 +816,12 @@ void Worker::process(uint64_t h0, uint32_t n) {
         evpool.push_back(e);
         for (uint32_t i = 0; i < n; i++) {
             Req& r = reqs[i];
-            if ((r.flags & GSYS_NONBLOCKING) || !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) || !r.dma) continue;
+            const bool nb = (r.flags & GSYS_NONBLOCKING) != 0;
+            if (!r.dma || (!nb && !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)))) continue;
             gsys_slot* sl = I->area_h + r.slot;
             if (r.ok) {
-                __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
-                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true);
+                __atomic_store_n(&sl->state, nb ? (uint32_t)GSYS_FREE : (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
+                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, nb ? GSYS_FREE : GSYS_FINISHED, !nb);
             }
             __atomic_store_n(&I->hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret,
                              __ATOMIC_RELEASE);
@@ -891,6 +914,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     if (cudaMalloc(&I->tail_d, 64) != cudaSuccess) return fail(-ENOMEM);
     if (cudaMalloc(&I->lat_hint_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     cudaMemset(I->lat_hint_d, 0, (size_t)slots * 4);
+    if (cudaMalloc(&I->nbpend_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
+    cudaMemset(I->nbpend_d, 0, (size_t)slots * 4);
     if (cudaMalloc(&I->krounds_d, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS) != cudaSuccess) return fail(-ENOMEM);
     I->kblock_cap = 4096;
     if (cudaMalloc(&I->kblock_d, (size_t)I->kblock_cap * GSYS_KSITES * 4) != cudaSuccess) return fail(-ENOMEM);
@@ -910,6 +935,7 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.mirror = I->mirror_d;
     c.hdone = (unsigned long long*)I->hdone_d;
     c.lat_hint = I->lat_hint_d;
+    c.nbpend = I->nbpend_d;
     c.ring = (unsigned long long*)I->ring_d;
     c.ring_tail = I->tail_d;
     c.krounds = I->krounds_d;
@@ -962,6 +988,22 @@ gsys_dev_ctx* gsys_internal_ctx_d() {
     Instance* I = current();
     return I ? I->ctx_d : nullptr;
 }
+void gsys_internal_register_host_range(const void* p, size_t n, int add) {
+    const uintptr_t lo = (uintptr_t)p, hi = lo + n;
+    if (add) {
+        int i = g_nhost_ranges.load();
+        if (i >= 32) return;
+        g_host_ranges[i].lo.store(lo);
+        g_host_ranges[i].hi.store(hi);
+        g_nhost_ranges.store(i + 1, std::memory_order_release);
+    } else {
+        // ranges are only removed when the library frees them, i.e. while no call can use them
+        int nr = g_nhost_ranges.load();
+        for (int i = 0; i < nr; i++)
+            if (g_host_ranges[i].lo.load() == lo) { g_host_ranges[i].lo.store(1); g_host_ranges[i].hi.store(0); }
+    }
+}
+
 int gsys_internal_nslots() {
     Instance* I = current();
     return I ? (int)I->nslots : 0;
@@ -1139,6 +1181,7 @@ int gsys_shutdown(void) {
     cudaFree(I->mirror_d);
     cudaFree(I->tail_d);
     cudaFree(I->lat_hint_d);
+    cudaFree(I->nbpend_d);
     cudaFree(I->krounds_d);
     cudaFree(I->kblock_d);
     cudaFree(I->ctx_d);

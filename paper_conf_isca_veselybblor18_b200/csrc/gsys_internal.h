@@ -1,9 +1,13 @@
 // gsys_internal.h -- private glue between the host service (gsys_host.cpp) and the workload
 // launchers (gsys_kernels.cu) built into the same libgsys.so.  Not part of the C-ABI.
 #pragma once
+#include <stddef.h>
 
 struct gsys_dev_ctx;
 
 // device pointer of the current device's instance context, or nullptr before gsys_init()
 gsys_dev_ctx* gsys_internal_ctx_d();
 int gsys_internal_nslots();
+
+// pinned host ranges owned by the library (staging): the service resolves them without the driver
+void gsys_internal_register_host_range(const void* p, size_t n, int add);

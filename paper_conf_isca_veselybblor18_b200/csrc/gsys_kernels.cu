@@ -387,11 +387,16 @@ int ensure_staging(Workspace* W, size_t bytes) {
 
 int ensure_hstaging(Workspace* W, size_t bytes) {
     if (bytes <= W->hstaging_cap) return 0;
-    if (W->hstaging) { cudaDeviceSynchronize(); cudaFreeHost(W->hstaging); }
+    if (W->hstaging) {
+        cudaDeviceSynchronize();
+        gsys_internal_register_host_range(W->hstaging, W->hstaging_cap, 0);
+        cudaFreeHost(W->hstaging);
+    }
     W->hstaging = nullptr; W->hstaging_cap = 0;
     if (cudaHostAlloc((void**)&W->hstaging, bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return -ENOMEM;
     W->hstaging_cap = bytes;
+    gsys_internal_register_host_range(W->hstaging, bytes, 1);
     return 0;
 }
 
