@@ -8,14 +8,14 @@
 //   scan_kernel   the same scan over text already in HBM (standalone HBM-roofline measurement).
 //   bench_kernel  granularity x blocking x ordering microbenchmark (sec. VII).
 //
-// Scan (reading A9/A10): a token is a maximal run of [A-Za-z0-9_]; it is owned by the chunk that
-// holds its first byte; a dictionary hit is a whole token byte-equal to one of <= 64 words of
-// <= 16 bytes.  Each thread takes 16 aligned bytes per step plus the next 16 as lookahead
-// (coalesced uint4 loads), classifies all 32 bytes with SWAR into a word-byte bitmask, derives
-// token starts from it, and for each start extracts the <= 16 byte token with a funnel-shift
-// network, filters by length and a perfect hash (smem), verifies with one 128-bit compare and
-// counts into a per-warp shared-memory histogram.  grep tests every owned position whose byte
-// is in the first-byte range of the patterns.  No tensor cores: nothing here is a contraction.
+// Scan (reading A9/A10, csrc/scan_core.cuh): a token is a maximal run of [A-Za-z0-9_]; it is owned
+// by the chunk that holds its first byte; a dictionary hit is a whole token byte-equal to one of
+// <= 64 words of <= 16 bytes.  Each lane takes 16 aligned bytes per step (one coalesced uint4 load;
+// the 16-byte lookahead and the byte before come from the neighbouring lanes by warp shuffle) and
+// runs them through a byte DFA built from a trie of the dictionary, held in shared memory (one
+// LDS per byte, no per-token divergence); hits go to a per-warp shared histogram.  grep tests
+// every owned position whose byte is in the first-byte range of the patterns.  No tensor cores:
+// nothing here is a contraction.
 
 #include <cuda_runtime.h>
 #include <errno.h>
@@ -36,9 +36,11 @@ namespace {
 using namespace gsys_scan;
 
 struct ScanState {
-    const ScanTables* T;   // shared memory
-    unsigned* whist;       // this warp's shared histogram [64]
-    int* hit;              // shared grep-hit flag of the current chunk (nullptr: no grep)
+    const ScanTables* T;        // shared memory
+    const unsigned short* dfa;  // shared memory, T->nstates x NCOL
+    unsigned* whist;            // this warp's shared histogram [64]
+    unsigned char* stage;       // shared memory, WARP_STAGE bytes per warp
+    int* hit;                   // shared grep-hit flag of the current chunk (nullptr: no grep)
 };
 
 // Load policies: LD_NC for text that is immutable during the kernel (HBM scan), LD_CG for device
@@ -72,61 +74,112 @@ __device__ __forceinline__ unsigned ld1(const unsigned char* p) {
     return v & 0xffu;
 }
 
+
+
+// count a DFA emission (h = word + 1, 0 = none) without a branch: predicated shared reduction
+__device__ __forceinline__ void red_hit(unsigned* wh, unsigned h) {
+    const unsigned addr = (unsigned)__cvta_generic_to_shared(wh) + (h - 1u) * 4u;
+    asm volatile("{ .reg .pred p; setp.ne.u32 p, %1, 0; @p red.shared.add.u32 [%0], 1; }" :: "r"(addr), "r"(h)
+                 : "memory");
+}
+
 // Scan positions [s, own_end) of a text whose valid bytes end at valid_end; seg0 points at the
-// byte of position s (16-byte aligned); seg0[-1] is the byte before s when s > 0.  Each warp
-// takes 512 consecutive bytes per step, lane l the 16 bytes at +16*l (one coalesced uint4 load);
-// the 16-byte lookahead B is lane l+1's A and the byte before is lane l-1's last byte (warp
-// shuffles), so every byte crosses the memory system once; lanes 31 / 0 fetch the edges.  A warp
-// issues the loads of SCAN_U steps before it processes them (memory-level parallelism for the
-// PCIe-latency-bound host-mapped case and for HBM).
-constexpr int SCAN_U = 4;
+// byte of position s (16-byte aligned); seg0[-1] is the byte before s when s > 0.  A warp takes
+// 2 KiB tiles.  Each tile arrives by cp.async (LDGSTS: global -> shared without registers, bytes
+// past valid_end zero-filled): four coalesced 16 B pieces per lane into a warp-private buffer
+// laid out as 33 lane slots of 64 + 16 B (the padding spreads the banks), plus the 16 B after the
+// tile and the 4 B word ending at the byte before it.  Two buffers per warp: the copy of tile i+1
+// is in flight while the DFA runs over tile i (the PCIe / HBM latency is hidden behind the DFA).
+// Lane l then runs the DFA over its contiguous 64 B span with the next slot's first 16 B as
+// lookahead.  Every byte crosses the memory system once.
+constexpr unsigned SLOT = 80;
+constexpr unsigned STAGE_BYTES = 33 * SLOT + 16;       // slots + the 4-byte "previous" word (padded)
+constexpr unsigned WARP_STAGE = 2 * STAGE_BYTES;       // double buffer
+
+__device__ __forceinline__ void cp_async16(unsigned dst, const void* src, unsigned src_bytes) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async4(unsigned dst, const void* src, unsigned src_bytes) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" :: "r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
+
+// issue the copies of the tile starting at `base` into buffer `buf` (shared address)
+__device__ __forceinline__ void stage_tile(unsigned buf, const unsigned char* seg0, long long s, long long base,
+                                           long long valid_end, unsigned lane) {
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+        const long long p = base + 512 * k + 16 * lane;
+        const long long left = valid_end - p;
+        const unsigned n = left >= 16 ? 16u : (left > 0 ? (unsigned)left : 0u);
+        const unsigned slot = 8u * k + (lane >> 2);
+        cp_async16(buf + slot * SLOT + 16u * (lane & 3u), seg0 + (n ? p - s : 0), n);
+    }
+    if (lane == 0u) {
+        const long long p = base + 2048;
+        const long long left = valid_end - p;
+        const unsigned n = left >= 16 ? 16u : (left > 0 ? (unsigned)left : 0u);
+        cp_async16(buf + 32u * SLOT, seg0 + (n ? p - s : 0), n);
+        cp_async4(buf + 33u * SLOT, seg0 + (base > 0 ? base - 4 - s : 0), base > 0 ? 4u : 0u);
+    }
+}
 
 template <int P>
 __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                            long long valid_end, const ScanState& S) {
     const ScanTables& T = *S.T;
+    const unsigned short* dfa = S.dfa;
     const bool grep = S.hit != nullptr && T.npat > 0;
     unsigned* wh = S.whist;
+    auto on_hit = [wh](unsigned h) { red_hit(wh, h); };
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    const long long wstride = 512ll * nwarps;
-    for (long long base0 = s + 512ll * warp; base0 < own_end; base0 += wstride * SCAN_U) {
-        uint4 Av[SCAN_U], Be[SCAN_U];
-        unsigned pe[SCAN_U];
-#pragma unroll
-        for (int u = 0; u < SCAN_U; u++) {
-            const long long p0 = base0 + wstride * u + 16ll * lane;
-            const unsigned char* q = seg0 + (p0 - s);
-            Av[u] = p0 < valid_end ? ld16<P>(q) : make_uint4(0, 0, 0, 0);
-            Be[u] = (lane == 31u && p0 + 16 < valid_end) ? ld16<P>(q + 16) : make_uint4(0, 0, 0, 0);
-            pe[u] = (lane == 0u && p0 > 0 && p0 - 1 < valid_end) ? ld1<P>(q - 1) : 0u;
+    unsigned char* stage = S.stage + warp * WARP_STAGE;
+    const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
+    const long long step = 2048ll * nwarps;
+    long long base = s + 2048ll * warp;
+    if (base < own_end) stage_tile(stage_s, seg0, s, base, valid_end, lane);
+    cp_async_commit();
+    for (unsigned it = 0; base < own_end; base += step, it ^= 1u) {
+        const long long nxt = base + step;
+        if (nxt < own_end) stage_tile(stage_s + (it ^ 1u) * STAGE_BYTES, seg0, s, nxt, valid_end, lane);
+        cp_async_commit();
+        cp_async_wait<1>();          // this tile's copies (issued one iteration earlier) have landed
+        __syncwarp();
+        const unsigned char* buf = stage + it * STAGE_BYTES;
+        Win W;
+        W.w0 = *reinterpret_cast<const uint4*>(buf + lane * SLOT);
+        W.w1 = *reinterpret_cast<const uint4*>(buf + lane * SLOT + 16u);
+        W.w2 = *reinterpret_cast<const uint4*>(buf + lane * SLOT + 32u);
+        W.w3 = *reinterpret_cast<const uint4*>(buf + lane * SLOT + 48u);
+        W.w4 = *reinterpret_cast<const uint4*>(buf + (lane + 1u) * SLOT);
+        const unsigned prevb = lane ? (unsigned)buf[(lane - 1u) * SLOT + 63u] : (unsigned)buf[33u * SLOT + 3u];
+        const long long p0 = base + 64ll * lane;
+        if (p0 < own_end) {
+            dfa_lane64(dfa, W, prevb, p0, own_end, valid_end, on_hit);
+            if (grep && !*(volatile int*)S.hit && grep_lane64(T, W, p0, own_end, valid_end)) *S.hit = 1;
         }
-#pragma unroll
-        for (int u = 0; u < SCAN_U; u++) {
-            const long long base = base0 + wstride * u;
-            if (base >= own_end) break;   // warp-uniform
-            const long long p0 = base + 16ll * lane;
-            const uint4 A = Av[u];
-            uint4 B;
-            B.x = __shfl_down_sync(0xffffffffu, A.x, 1);
-            B.y = __shfl_down_sync(0xffffffffu, A.y, 1);
-            B.z = __shfl_down_sync(0xffffffffu, A.z, 1);
-            B.w = __shfl_down_sync(0xffffffffu, A.w, 1);
-            unsigned prevb = __shfl_up_sync(0xffffffffu, A.w >> 24, 1);
-            if (lane == 31u) B = Be[u];
-            if (lane == 0u) prevb = pe[u];
-            if (p0 < own_end) {
-                const bool g = grep && !*(volatile int*)S.hit;
-                if (scan_step(T, A, B, prevb, p0, own_end, valid_end, g, [wh](unsigned d) { atomicAdd(&wh[d], 1u); }))
-                    *S.hit = 1;
-            }
-        }
+        __syncwarp();                // every lane is done with this buffer before it is refilled
     }
+    cp_async_wait<0>();
 }
 
-__device__ __forceinline__ void load_tables(ScanTables* sT, const ScanTables* gT) {
-    const unsigned* src = reinterpret_cast<const unsigned*>(gT);
-    unsigned* dst = reinterpret_cast<unsigned*>(sT);
-    for (unsigned i = threadIdx.x; i < sizeof(ScanTables) / 4; i += blockDim.x) dst[i] = src[i];
+// Dynamic shared memory: [ScanTables + DFA (tables_bytes)] [per-warp histograms] [warp stages].
+__device__ __forceinline__ unsigned* load_tables(unsigned char* smem, const ScanTables* gT, unsigned nwarps,
+                                                 ScanState& S) {
+    const unsigned nst = gT->nstates;
+    const size_t tb = (tables_bytes(nst) + 15) & ~(size_t)15;
+    const uint4* src = reinterpret_cast<const uint4*>(gT);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (unsigned i = threadIdx.x; i < tb / 16; i += blockDim.x) dst[i] = src[i];
+    unsigned* shist = reinterpret_cast<unsigned*>(smem + tb);
+    for (unsigned i = threadIdx.x; i < nwarps * MAXD; i += blockDim.x) shist[i] = 0;
+    S.stage = smem + tb + nwarps * MAXD * 4;
+    S.T = reinterpret_cast<const ScanTables*>(smem);
+    S.dfa = reinterpret_cast<const unsigned short*>(smem + sizeof(ScanTables));
+    S.whist = shist + (threadIdx.x / 32) * MAXD;
+    return shist;
 }
 
 __device__ __forceinline__ void flush_hist(unsigned* shist, unsigned nwarps, unsigned ndict, unsigned long long* hist) {
@@ -153,17 +206,14 @@ struct WcArgs {
 };
 
 __global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
-    __shared__ ScanTables sT;
     __shared__ int s_hit;
-    extern __shared__ unsigned shist[];
+    extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
-    load_tables(&sT, a.tables);
-    for (unsigned i = threadIdx.x; i < nwarps * MAXD; i += blockDim.x) shist[i] = 0;
+    ScanState S;
+    unsigned* shist = load_tables(smem, a.tables, nwarps, S);
+    const ScanTables& sT = *S.T;
     __syncthreads();
     unsigned char* base = a.staging + (size_t)blockIdx.x * a.stride;
-    ScanState S;
-    S.T = &sT;
-    S.whist = shist + (threadIdx.x / 32) * MAXD;
     for (unsigned k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         unsigned lo = 0, hi = a.nfiles;     // largest f with chunk_base[f] <= k
         while (hi - lo > 1) {
@@ -219,26 +269,25 @@ struct ScanArgs {
     unsigned long long* hist;
     unsigned* hit;
     unsigned long long nchunks;
-    unsigned chunk, pad_;
+    unsigned chunk, ld_policy;
 };
 
-__global__ void __launch_bounds__(256, 4) scan_kernel(ScanArgs a) {
-    __shared__ ScanTables sT;
+__global__ void __launch_bounds__(512, 2) scan_kernel(ScanArgs a) {
     __shared__ int s_hit;
-    extern __shared__ unsigned shist[];
+    extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
-    load_tables(&sT, a.tables);
-    for (unsigned i = threadIdx.x; i < nwarps * MAXD; i += blockDim.x) shist[i] = 0;
+    ScanState S;
+    unsigned* shist = load_tables(smem, a.tables, nwarps, S);
+    const ScanTables& sT = *S.T;
     if (threadIdx.x == 0) s_hit = 0;
     __syncthreads();
-    ScanState S;
-    S.T = &sT;
-    S.whist = shist + (threadIdx.x / 32) * MAXD;
     S.hit = a.hit ? &s_hit : nullptr;
     for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         const long long s = (long long)k * a.chunk;
         const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
-        scan_range<LD_NC>(a.text + s, s, e, (long long)a.n, S);
+        if (a.ld_policy == LD_CG) scan_range<LD_CG>(a.text + s, s, e, (long long)a.n, S);
+        else if (a.ld_policy == LD_CA) scan_range<LD_CA>(a.text + s, s, e, (long long)a.n, S);
+        else scan_range<LD_NC>(a.text + s, s, e, (long long)a.n, S);
     }
     __syncthreads();
     flush_hist(shist, nwarps, sT.ndict, a.hist);
@@ -400,6 +449,12 @@ int ensure_hstaging(Workspace* W, size_t bytes) {
     return 0;
 }
 
+int ensure_smem_attr(const void* fn, size_t bytes) {
+    if (bytes <= 48 * 1024) return 0;
+    if (bytes > 227 * 1024) return -E2BIG;
+    return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) == cudaSuccess ? 0 : -EINVAL;
+}
+
 int map_cuda(cudaError_t e) {
     if (e == cudaSuccess) return 0;
     if (e == cudaErrorMemoryAllocation) return -ENOMEM;
@@ -440,11 +495,14 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     if (blocks == 0) blocks = 2u * (uint32_t)W->sms;
     if (nch < blocks) blocks = (uint32_t)(nch ? nch : 1);
     // upload: [tables][fds][sizes][cbase]
-    size_t o_t = 0, o_f = align_up(sizeof(ScanTables), 256), o_s = align_up(o_f + 4ull * nfiles, 256),
+    size_t tb = 0;
+    int rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb);
+    if (rc && rc != -ENOSPC) return rc;
+    size_t o_t = 0, o_f = align_up(tb, 256), o_s = align_up(o_f + 4ull * nfiles, 256),
            o_c = align_up(o_s + 8ull * nfiles, 256), total = align_up(o_c + 4ull * (nfiles + 1), 256);
-    int rc = ensure_upload(W, total);
+    rc = ensure_upload(W, total);
     if (rc) return rc;
-    rc = build_tables(reinterpret_cast<ScanTables*>(W->up_h + o_t), dict, dlen, ndict, pats, plen, npat);
+    rc = build_tables(W->up_h + o_t, tb, dict, dlen, ndict, pats, plen, npat, nullptr);
     if (rc) return rc;
     memcpy(W->up_h + o_f, fds, 4ull * nfiles);
     memcpy(W->up_h + o_s, sizes, 8ull * nfiles);
@@ -486,7 +544,9 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.gflags = gflags;
     if (nch == 0) return 0;
     void* args[] = {&a};
-    size_t smem = (threads / 32) * MAXD * 4;
+    size_t smem = align_up(tb, 16) + (threads / 32) * (MAXD * 4 + WARP_STAGE);
+    rc = ensure_smem_attr((const void*)wc_kernel, smem);
+    if (rc) return rc;
     return gsys_launch((const void*)wc_kernel, blocks, 1, 1, threads, 1, 1, args, smem, stream);
 }
 
@@ -517,22 +577,25 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (!d_hist || (n && !d_text)) return -EINVAL;
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
-    if (threads == 0) threads = 256;
-    if (threads % 32 || threads > 256) return -EINVAL;
+    if (threads == 0) threads = 512;
+    if (threads % 32 || threads > 512) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
-    size_t total = align_up(sizeof(ScanTables), 256);
-    int rc = ensure_upload(W, total);
+    size_t tb = 0;
+    int rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb);
+    if (rc && rc != -ENOSPC) return rc;
+    size_t total = align_up(tb, 256);
+    rc = ensure_upload(W, total);
     if (rc) return rc;
-    rc = build_tables(reinterpret_cast<ScanTables*>(W->up_h), dict, dlen, ndict, pats, plen, npat);
+    rc = build_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr);
     if (rc) return rc;
     cudaStream_t s = (cudaStream_t)stream;
     cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
     cudaEventRecord(W->up_ev, s);
     unsigned long long nch = (n + chunk - 1) / chunk;
     if (nch == 0) return 0;
-    if (blocks == 0) blocks = 4u * (uint32_t)W->sms;
+    if (blocks == 0) blocks = 2u * (uint32_t)W->sms;
     if (nch < blocks) blocks = (uint32_t)nch;
     ScanArgs a;
     memset(&a, 0, sizeof a);
@@ -543,7 +606,13 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     a.hit = d_hit;
     a.nchunks = nch;
     a.chunk = chunk;
-    size_t smem = (threads / 32) * MAXD * 4;
+    {
+        const char* ev = getenv("GSYS_SCAN_LD");   // diagnostics: 1 = ld.cg, 3 = ld.ca instead of ld.nc
+        a.ld_policy = ev ? (unsigned)atoi(ev) : (unsigned)LD_NC;
+    }
+    size_t smem = align_up(tb, 16) + (threads / 32) * (MAXD * 4 + WARP_STAGE);
+    rc = ensure_smem_attr((const void*)scan_kernel, smem);
+    if (rc) return rc;
     scan_kernel<<<blocks, threads, smem, s>>>(a);
     return map_cuda(cudaGetLastError());
 }

@@ -5,11 +5,25 @@
 // Definitions (reading A9/A10): a token is a maximal run of [A-Za-z0-9_]; it is owned
 // by the chunk holding its first byte; a dictionary hit is a whole token byte-equal to one of <= 64
 // words of <= 16 bytes; grep -F reports whether any pattern occurs as a substring.
+//
+// Wordcount runs a byte-level DFA built from a trie of the dictionary ("search for occurrences of
+// 64 strings", PAPER.md:32 P32.6): state ROOT (at a token start), DEAD (inside a token that can no
+// longer match) and one state per dictionary prefix.  A byte b selects column clamp(b-47, 0, 76):
+// column 0 holds every byte <= '/', 76 every byte >= '{', 1..75 the bytes '0'..'z' one by one, so
+// the table needs 77 columns and no class lookup.  A non-word byte leaves any state for ROOT and,
+// from a state that spells a whole dictionary word, emits that word.  Entry (u16) = next state in
+// bits 0..8 (<= 512 states) | (word+1) in bits 9..15 (terminating entries only; their next state
+// is ROOT = 0), so one shared-memory load, one AND and one shift per byte, no per-token branch.
+// Hits are counted with a predicated shared-memory reduction on the device (no divergence).  Two
+// segments run interleaved per lane (two independent state chains) to hide the load latency.
+// grep keeps a SWAR first-byte range filter plus a 128-bit verify per candidate.
 #pragma once
 #include <cuda_runtime.h>
 #include <errno.h>
 #include <stdint.h>
 #include <string.h>
+
+#include <vector>
 
 #ifdef __CUDACC__
 #define GSYS_HD __host__ __device__ __forceinline__
@@ -32,40 +46,28 @@ inline unsigned host_funnelshift_r(unsigned lo, unsigned hi, unsigned sh) {
 #define GSYS_FSHR __funnelshift_r
 #endif
 
-constexpr int HBITS = 10;
-constexpr int HB = 1 << HBITS;
 constexpr int MAXD = 64;
 constexpr int MAXP = 8;
+constexpr int NCOL = 77;                 // DFA columns (see header)
+constexpr unsigned ROOT = 0u, DEAD = 1u;
+constexpr unsigned MAX_STATES = 512;    // 9-bit next-state field
 
 struct ScanTables {
-    uint4 words[MAXD];          // zero-padded dictionary words
     uint4 pats[MAXP];           // zero-padded grep patterns
-    unsigned hmul[5];
-    unsigned lenmask;           // bit L: some word has length L
     unsigned ndict, npat;
+    unsigned nstates;           // DFA states; the table (nstates x NCOL u16) follows the struct
     unsigned fb_lo, fb_hi;      // first-byte range of patterns (SWAR candidate filter)
     unsigned fbmap[8];          // exact first-byte bitmap
-    unsigned char dlen[MAXD];
     unsigned char plen[MAXP];
-    unsigned short bucket[HB];  // 0 = empty, else dictionary index + 1
+    unsigned pad_[2];
 };
+static_assert(sizeof(ScanTables) % 16 == 0, "ScanTables must keep the DFA 16-byte aligned");
 
-// ------------------------------------------------------------------ device helpers
+GSYS_HD size_t tables_bytes(unsigned nstates) { return sizeof(ScanTables) + (size_t)nstates * NCOL * 2; }
+
+// ------------------------------------------------------------------ helpers
 GSYS_HD unsigned compress4(unsigned m80) { return ((m80 >> 7) * 0x10204080u) >> 28; }
 
-// 4-bit mask of bytes of x in [A-Za-z0-9_]
-GSYS_HD unsigned class4(unsigned x) {
-    unsigned lo7 = x & 0x7f7f7f7fu;
-    unsigned y = lo7 | 0x20202020u;                 // ASCII case fold
-    unsigned letter = (y + 0x1f1f1f1fu) & ~(y + 0x05050505u);      // 'a'..'z'
-    unsigned digit = (lo7 + 0x50505050u) & ~(lo7 + 0x46464646u);   // '0'..'9'
-    unsigned t = lo7 ^ 0x5f5f5f5fu;
-    unsigned us = ~((t + 0x7f7f7f7fu) | t);                        // '_'
-    return compress4((letter | digit | us) & ~x & 0x80808080u);
-}
-GSYS_HD unsigned class16(uint4 v) {
-    return class4(v.x) | (class4(v.y) << 4) | (class4(v.z) << 8) | (class4(v.w) << 12);
-}
 // 4-bit mask of bytes of x in [lo, hi] (lo <= hi < 0x80)
 GSYS_HD unsigned range4(unsigned x, unsigned add_lo, unsigned add_hi) {
     unsigned lo7 = x & 0x7f7f7f7fu;
@@ -73,6 +75,11 @@ GSYS_HD unsigned range4(unsigned x, unsigned add_lo, unsigned add_hi) {
 }
 GSYS_HD bool is_word_byte(unsigned c) {
     return (c - 'a' < 26u) || (c - 'A' < 26u) || (c - '0' < 10u) || c == '_';
+}
+GSYS_HD unsigned dfa_col(unsigned b) {
+    int c = (int)b - 47;
+    c = c < 0 ? 0 : c;
+    return (unsigned)(c > NCOL - 1 ? NCOL - 1 : c);
 }
 
 // 16 bytes of the 32-byte window (A, B) starting at byte j (0..15), little-endian
@@ -88,7 +95,6 @@ GSYS_HD void extract16(const uint4& A, const uint4& B, unsigned j, unsigned t[4]
     t[3] = GSYS_FSHR(v3, v4, sh);
 }
 GSYS_HD void mask_len(unsigned t[4], unsigned len) {
-#pragma unroll
     for (int k = 0; k < 4; k++) {
         int kept = (int)len - 4 * k;
         kept = kept < 0 ? 0 : (kept > 4 ? 4 : kept);
@@ -96,58 +102,94 @@ GSYS_HD void mask_len(unsigned t[4], unsigned len) {
         t[k] &= m;
     }
 }
+// byte i (0..31) of the window (A, B)
+GSYS_HD unsigned window_byte(const uint4& A, const uint4& B, unsigned i) {
+    const unsigned q = i >> 2;
+    const unsigned w = q < 4 ? (q < 2 ? (q == 0 ? A.x : A.y) : (q == 2 ? A.z : A.w))
+                             : (q < 6 ? (q == 4 ? B.x : B.y) : (q == 6 ? B.z : B.w));
+    return (w >> (8 * (i & 3u))) & 0xffu;
+}
 
+// One DFA transition; returns the word id + 1 emitted (0 = none).
+GSYS_HD unsigned dfa_step(const unsigned short* __restrict__ dfa, unsigned& st, unsigned b) {
+    const unsigned e = dfa[st * NCOL + dfa_col(b)];
+    st = e & 0x1ffu;
+    return e >> 9;
+}
 
-// One 16-byte step of the scan at text position p0 (16-byte aligned relative to the chunk):
-//   A = bytes [p0, p0+16), B = bytes [p0+16, p0+32) (zeros past valid_end), prevb = byte p0-1
-//   (only meaningful when p0 > 0).  Owned token starts are positions in [p0, min(p0+16, own_end));
-//   bytes at or beyond valid_end do not exist (end of file / short read).
-// on_word(d) is called once per whole-token hit of dictionary word d; the return value is true
-// if a grep pattern starts at an owned position (only evaluated when grep is true).
-template <class OnWord>
-GSYS_HD bool scan_step(const ScanTables& T, const uint4& A, const uint4& B, unsigned prevb, long long p0,
-                       long long own_end, long long valid_end, bool grep, OnWord&& on_word) {
-    unsigned M = class16(A) | (class16(B) << 16);
-    const long long nvalid = valid_end - p0;
-    if (nvalid < 32) M &= (1u << nvalid) - 1u;
-    const unsigned prevw = (p0 > 0 && is_word_byte(prevb)) ? 1u : 0u;
-    const long long nown = own_end - p0;
-    const unsigned ownm = nown >= 16 ? 0xffffu : ((1u << nown) - 1u);
-    unsigned starts = M & ~((M << 1) | prevw) & ownm;
-    while (starts) {
-        const unsigned j = GSYS_FFS(starts) - 1u;
-        starts &= starts - 1u;
-        const unsigned len = (unsigned)GSYS_FFS(~(M >> j)) - 1u;
-        if (len > 16u || !((T.lenmask >> len) & 1u)) continue;
-        unsigned t[4];
-        extract16(A, B, j, t);
-        mask_len(t, len);
-        const unsigned h = (t[0] * T.hmul[0] + t[1] * T.hmul[1] + t[2] * T.hmul[2] + t[3] * T.hmul[3] +
-                            len * T.hmul[4]) >> (32 - HBITS);
-        const unsigned b = T.bucket[h];
-        if (b) {
-            const unsigned d = b - 1u;
-            const uint4 w = T.words[d];
-            if (T.dlen[d] == len && w.x == t[0] && w.y == t[1] && w.z == t[2] && w.w == t[3]) on_word(d);
-        }
+// Start state of a step at p0: inside a token owned by the left neighbour -> DEAD.
+GSYS_HD unsigned start_state(unsigned prevb, long long p0) {
+    return (p0 > 0 && is_word_byte(prevb)) ? DEAD : ROOT;
+}
+
+// Follow the token still open after owned byte index `from` of window (A, B) to its end.
+template <class OnHit>
+GSYS_HD void dfa_finish(const unsigned short* __restrict__ dfa, unsigned st, const uint4& A, const uint4& B,
+                        unsigned from, unsigned nvalid, OnHit&& on_hit) {
+    for (unsigned i = from; st > DEAD; i++) {
+        const unsigned b = i < nvalid ? window_byte(A, B, i) : 0u;   // past the data: terminator
+        on_hit(dfa_step(dfa, st, b));
+        if (i >= nvalid) break;
     }
-    if (!grep) return false;
+}
+
+// Two full 16-byte steps (both owned and valid for all 16 bytes) run interleaved.
+template <class OnHit>
+GSYS_HD void dfa_pair(const unsigned short* __restrict__ dfa, unsigned& s0, unsigned& s1, const uint4& A0,
+                      const uint4& A1, OnHit&& on_hit) {
+    const unsigned w0[4] = {A0.x, A0.y, A0.z, A0.w};
+    const unsigned w1[4] = {A1.x, A1.y, A1.z, A1.w};
+#pragma unroll
+    for (int i = 0; i < 16; i++) {
+        const unsigned h0 = dfa_step(dfa, s0, (w0[i >> 2] >> (8 * (i & 3))) & 0xffu);
+        const unsigned h1 = dfa_step(dfa, s1, (w1[i >> 2] >> (8 * (i & 3))) & 0xffu);
+        on_hit(h0);
+        on_hit(h1);
+    }
+}
+
+// One 16-byte step of the scan at text position p0:
+//   A = bytes [p0, p0+16), B = bytes [p0+16, p0+32) (zeros past valid_end), prevb = byte p0-1
+//   (meaningful when p0 > 0).  Owned token starts are the positions [p0, min(p0+16, own_end));
+//   a token owned here is followed into B until it ends (at most 16 + 1 bytes); bytes at or past
+//   valid_end do not exist (end of file / short read) and terminate the token.
+// on_hit(h) receives every DFA emission value (h = word id + 1, or 0 for none) -- the device
+// counts with a predicated reduction, the host emulation with a branch.
+template <class OnHit>
+GSYS_HD void dfa_segment(const unsigned short* __restrict__ dfa, const uint4& A, const uint4& B, unsigned prevb,
+                         long long p0, long long own_end, long long valid_end, OnHit&& on_hit) {
+    const long long nvalid_ll = valid_end - p0;
+    const unsigned nvalid = nvalid_ll >= 32 ? 32u : (unsigned)nvalid_ll;
+    const long long nown_ll = own_end - p0;
+    const unsigned nown = nown_ll >= 16 ? 16u : (unsigned)nown_ll;
+    unsigned st = start_state(prevb, p0);
+    for (unsigned i = 0; i < nown && i < nvalid; i++) on_hit(dfa_step(dfa, st, window_byte(A, B, i)));
+    dfa_finish(dfa, st, A, B, nown, nvalid, on_hit);
+}
+
+// grep part of a step: true if a pattern starts at an owned position of [p0, p0+16).
+GSYS_HD bool grep_step(const ScanTables& T, const uint4& A, const uint4& B, long long p0, long long own_end,
+                       long long valid_end) {
+    const long long nvalid_ll = valid_end - p0;
+    const unsigned nvalid = nvalid_ll >= 32 ? 32u : (unsigned)nvalid_ll;
+    const long long nown_ll = own_end - p0;
+    const unsigned nown = nown_ll >= 16 ? 16u : (unsigned)nown_ll;
     const bool fb_swar = T.fb_hi < 0x80u;
     const unsigned add_lo = (0x80u - T.fb_lo) * 0x01010101u, add_hi = (0x7fu - T.fb_hi) * 0x01010101u;
     unsigned cand = fb_swar ? (range4(A.x, add_lo, add_hi) | (range4(A.y, add_lo, add_hi) << 4) |
                                (range4(A.z, add_lo, add_hi) << 8) | (range4(A.w, add_lo, add_hi) << 12))
                             : 0xffffu;
-    cand &= ownm;
+    cand &= nown >= 16u ? 0xffffu : ((1u << nown) - 1u);
     while (cand) {
         const unsigned j = GSYS_FFS(cand) - 1u;
         cand &= cand - 1u;
-        const unsigned c0 = ((j < 4 ? A.x : j < 8 ? A.y : j < 12 ? A.z : A.w) >> (8 * (j & 3))) & 0xffu;
+        const unsigned c0 = window_byte(A, B, j);
         if (!((T.fbmap[c0 >> 5] >> (c0 & 31)) & 1u)) continue;
         unsigned t[4];
         extract16(A, B, j, t);
         for (unsigned p = 0; p < T.npat; p++) {
             const unsigned L = T.plen[p];
-            if ((long long)(j + L) > nvalid) continue;
+            if (j + L > nvalid) continue;
             unsigned u[4] = {t[0], t[1], t[2], t[3]};
             mask_len(u, L);
             const uint4 w = T.pats[p];
@@ -157,46 +199,133 @@ GSYS_HD bool scan_step(const ScanTables& T, const uint4& A, const uint4& B, unsi
     return false;
 }
 
+// A lane's 80-byte window as five named vectors (never an indexed array, so it stays in registers)
+struct Win {
+    uint4 w0, w1, w2, w3, w4;
+    GSYS_HD uint4 get(unsigned k) const {   // by value: component-wise selects, no addressable array
+        uint4 r = w4;
+        if (k == 3) r = w3;
+        if (k == 2) r = w2;
+        if (k == 1) r = w1;
+        if (k == 0) r = w0;
+        return r;
+    }
+};
+
+// byte i (0..79) of the window
+GSYS_HD unsigned lane_byte(const Win& W, unsigned i) {
+    const uint4 a = W.get(i >> 4);
+    return window_byte(a, a, i & 15u);
+}
+
+// A lane's 64-byte span at p0: W[0..3] = bytes [p0, p0+64), W[4] = [p0+64, p0+80) (zeros past
+// valid_end).  Owned token starts: [p0, min(p0+64, own_end)); the token open at the end of the
+// owned range is followed to its end (<= 17 more bytes, all inside W[4] for a full span).
+template <class OnHit>
+GSYS_HD void dfa_lane64(const unsigned short* __restrict__ dfa, const Win& W, unsigned prevb, long long p0,
+                        long long own_end, long long valid_end, OnHit&& on_hit) {
+    const long long nvalid_ll = valid_end - p0;
+    const unsigned nvalid = nvalid_ll >= 80 ? 80u : (unsigned)nvalid_ll;
+    const long long nown_ll = own_end - p0;
+    const unsigned nown = nown_ll >= 64 ? 64u : (unsigned)nown_ll;
+    unsigned st = start_state(prevb, p0);
+    if (nown == 64u && nvalid >= 64u) {
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint4 q = W.get((unsigned)k);
+            const unsigned wv[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+            for (int i = 0; i < 16; i++) on_hit(dfa_step(dfa, st, (wv[i >> 2] >> (8 * (i & 3))) & 0xffu));
+        }
+        for (unsigned i = 64; st > DEAD; i++) {
+            const unsigned b = i < nvalid ? window_byte(W.w4, W.w4, i - 64u) : 0u;
+            on_hit(dfa_step(dfa, st, b));
+            if (i >= nvalid) break;
+        }
+        return;
+    }
+    for (unsigned i = 0; i < nown && i < nvalid; i++) on_hit(dfa_step(dfa, st, lane_byte(W, i)));
+    for (unsigned i = nown; st > DEAD; i++) {
+        const unsigned b = i < nvalid ? lane_byte(W, i) : 0u;
+        on_hit(dfa_step(dfa, st, b));
+        if (i >= nvalid) break;
+    }
+}
+
+// grep over a lane's span: the four 16-byte steps with their 32-byte windows.
+GSYS_HD bool grep_lane64(const ScanTables& T, const Win& W, long long p0, long long own_end, long long valid_end) {
+    for (unsigned k = 0; k < 4; k++) {
+        const long long q = p0 + 16 * k;
+        if (q >= own_end) break;
+        const uint4 a = W.get(k), b = W.get(k + 1);
+        if (grep_step(T, a, b, q, own_end, valid_end)) return true;
+    }
+    return false;
+}
+
+// Whole step (wordcount + grep) for one segment -- the reference composition used by the host
+// emulation; the kernels run the 64-byte lane spans above (checked equal by the CPU tests).
+template <class OnHit>
+GSYS_HD bool scan_step(const ScanTables& T, const unsigned short* __restrict__ dfa, const uint4& A, const uint4& B,
+                       unsigned prevb, long long p0, long long own_end, long long valid_end, bool grep,
+                       OnHit&& on_hit) {
+    dfa_segment(dfa, A, B, prevb, p0, own_end, valid_end, on_hit);
+    return grep && grep_step(T, A, B, p0, own_end, valid_end);
+}
+
 // ------------------------------------------------------------------ host: table builder
-inline uint32_t lcg_next(uint64_t* s) {
-    *s = *s * 6364136223846793005ull + 1442695040888963407ull;
-    return (uint32_t)(*s >> 32);
-}
-
-inline unsigned hash_host(const uint32_t t[4], unsigned len, const unsigned m[5]) {
-    return (t[0] * m[0] + t[1] * m[1] + t[2] * m[2] + t[3] * m[3] + len * m[4]) >> (32 - HBITS);
-}
-
-inline int build_tables(ScanTables* T, const char* dict, const uint8_t* dlen, uint32_t ndict, const char* pats,
-                 const uint8_t* plen, uint32_t npat) {
+// Writes ScanTables followed by the DFA (nstates x NCOL u16) into `out` (tables_bytes(nstates)
+// bytes, capacity `cap`).  Dictionary words must be 1..16 bytes; a word containing a non-word
+// byte can never equal a token and gets no trie path; duplicate words count once (first wins).
+// -E2BIG when the trie needs more than 512 states (distinct prefixes + 2).
+inline int build_tables(void* out, size_t cap, const char* dict, const uint8_t* dlen, uint32_t ndict,
+                        const char* pats, const uint8_t* plen, uint32_t npat, size_t* used) {
     if (ndict > (uint32_t)MAXD || npat > (uint32_t)MAXP) return -EINVAL;
     if (ndict && (!dict || !dlen)) return -EINVAL;
     if (npat && (!pats || !plen)) return -EINVAL;
+    // trie over the DFA columns
+    std::vector<short> child;            // [state][NCOL]
+    std::vector<unsigned char> acc;      // word id + 1 per state
+    child.assign(2 * NCOL, -1);
+    acc.assign(2, 0);
+    for (uint32_t d = 0; d < ndict; d++) {
+        if (dlen[d] < 1 || dlen[d] > 16) return -EINVAL;
+        const unsigned char* w = (const unsigned char*)dict + 17 * d;
+        bool ok = true;
+        for (unsigned k = 0; k < dlen[d]; k++) ok = ok && is_word_byte(w[k]);
+        if (!ok) continue;
+        unsigned s = ROOT;
+        for (unsigned k = 0; k < dlen[d]; k++) {
+            const unsigned c = dfa_col(w[k]);
+            if (child[s * NCOL + c] < 0) {
+                child[s * NCOL + c] = (short)acc.size();
+                acc.push_back(0);
+                child.resize(acc.size() * NCOL, -1);
+            }
+            s = (unsigned)child[s * NCOL + c];
+        }
+        if (!acc[s]) acc[s] = (unsigned char)(d + 1);
+    }
+    const unsigned nstates = (unsigned)acc.size();
+    if (nstates > MAX_STATES) return -E2BIG;     // dictionary trie too large for the 9-bit state field
+    const size_t need = tables_bytes(nstates);
+    if (used) *used = need;
+    if (!out || need > cap) return -ENOSPC;
+    ScanTables* T = (ScanTables*)out;
     memset(T, 0, sizeof *T);
     T->ndict = ndict;
     T->npat = npat;
-    uint32_t w[MAXD][4];
-    for (uint32_t d = 0; d < ndict; d++) {
-        if (dlen[d] < 1 || dlen[d] > 16) return -EINVAL;
-        uint8_t b[16] = {0};
-        memcpy(b, dict + 17 * d, dlen[d]);
-        memcpy(w[d], b, 16);
-        memcpy(&T->words[d], b, 16);
-        T->dlen[d] = dlen[d];
-        T->lenmask |= 1u << dlen[d];
-    }
-    uint64_t seed = 0x9E3779B97F4A7C15ull;
-    for (int attempt = 0;; attempt++) {
-        if (attempt > 100000) return -EINVAL;   // duplicate dictionary words
-        for (int k = 0; k < 5; k++) T->hmul[k] = lcg_next(&seed) | 1u;
-        memset(T->bucket, 0, sizeof T->bucket);
-        bool ok = true;
-        for (uint32_t d = 0; d < ndict && ok; d++) {
-            unsigned h = hash_host(w[d], dlen[d], T->hmul);
-            if (T->bucket[h]) ok = false;
-            else T->bucket[h] = (unsigned short)(d + 1);
+    T->nstates = nstates;
+    unsigned short* dfa = (unsigned short*)((unsigned char*)out + sizeof(ScanTables));
+    for (unsigned s = 0; s < nstates; s++) {
+        for (unsigned c = 0; c < (unsigned)NCOL; c++) {
+            const unsigned b = c == 0 ? 0u : (c == NCOL - 1 ? 255u : c + 47u);   // a byte of the column
+            unsigned short e;
+            if (!is_word_byte(b)) e = (unsigned short)((s >= 2 ? acc[s] : 0u) << 9);
+            else if (s == DEAD) e = (unsigned short)DEAD;
+            else e = child[s * NCOL + c] >= 0 ? (unsigned short)child[s * NCOL + c] : (unsigned short)DEAD;
+            dfa[s * NCOL + c] = e;
         }
-        if (ok) break;
     }
     T->fb_lo = 0xff;
     T->fb_hi = 0;

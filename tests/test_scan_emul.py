@@ -28,17 +28,25 @@ def emul():
                                "-o", LIB, SRC])
     L = ctypes.CDLL(LIB)
     P = ctypes.c_void_p
-    L.scan_emul.argtypes = [P, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_char_p, P, ctypes.c_uint32,
-                            ctypes.c_char_p, P, ctypes.c_uint32, P, P]
+    L.scan_emul2.argtypes = [P, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_char_p, P, ctypes.c_uint32,
+                             ctypes.c_char_p, P, ctypes.c_uint32, P, P, ctypes.c_int]
 
     def run(text, words, pats, chunk):
+        h0, g0 = run2(text, words, pats, chunk, 0)
+        h1, g1 = run2(text, words, pats, chunk, 1)
+        h2, g2 = run2(text, words, pats, chunk, 2)
+        assert np.array_equal(h0, h1) and g0 == g1     # paired 16-byte steps == reference composition
+        assert np.array_equal(h0, h2) and g0 == g2     # the kernels' 64-byte lane spans == reference
+        return h0, g0
+
+    def run2(text, words, pats, chunk, pairs):
         arr = np.frombuffer(text, dtype=np.uint8) if isinstance(text, (bytes, bytearray)) else text
         d, dl = pack_words(words)
         p, pl = pack_words(pats) if pats else (b"", None)
         hist = np.zeros(len(words), dtype=np.uint64)
         hit = ctypes.c_uint32(0)
-        rc = L.scan_emul(arr.ctypes.data, arr.size, chunk, d, dl, len(words), p, pl, len(pats), hist.ctypes.data,
-                         ctypes.byref(hit))
+        rc = L.scan_emul2(arr.ctypes.data, arr.size, chunk, d, dl, len(words), p, pl, len(pats), hist.ctypes.data,
+                          ctypes.byref(hit), pairs)
         assert rc == 0
         return hist, bool(hit.value)
     return run
@@ -90,3 +98,12 @@ def test_scan_emul_long_tokens_and_high_bytes(emul):
     for chunk in (16, 32, 4096):
         hist, _ = emul(text, words, [], chunk)
         assert np.array_equal(hist, oracle.count_tokens(text, words))
+
+
+def test_scan_emul_duplicate_and_nonword_dictionary_entries(emul):
+    words = [b"ab", b"ab", b"a-b", b"x", b"x_y", b"Q"]
+    text = b"ab a-b ab, x x_y xQ Q ab_ a b " * 20
+    for chunk in (16, 64):
+        hist, _ = emul(text, words, [], chunk)
+        assert np.array_equal(hist, oracle.count_tokens(text, words))
+        assert hist[1] == 0 and hist[2] == 0
