@@ -272,7 +272,7 @@ struct ScanArgs {
     unsigned chunk, ld_policy;
 };
 
-__global__ void __launch_bounds__(512, 2) scan_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(512, 1) scan_kernel(ScanArgs a) {
     __shared__ int s_hit;
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;

@@ -15,12 +15,12 @@ dev = host.to("cuda")
 hist = torch.zeros(64, dtype=torch.int64, device="cuda")
 for name, t in [("hbm", dev), ("host_mapped", host)]:
     for blocks in (592, 1184):
-        G.gsys_scan_device(t, n, 256 << 10, words, pats, hist, None, blocks, 256)
+        G.gsys_scan_device(t, n, 256 << 10, words, pats, hist, None, blocks, int(os.environ.get("ZC_THREADS", "512")))
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         for _ in range(3):
-            G.gsys_scan_device(t, n, 256 << 10, words, pats, hist, None, blocks, 256)
+            G.gsys_scan_device(t, n, 256 << 10, words, pats, hist, None, blocks, int(os.environ.get("ZC_THREADS", "512")))
         e1.record(); e1.synchronize()
         print(json.dumps({"scan": name, "blocks": blocks, "GBps": 3 * n / (e0.elapsed_time(e1) / 1e3) / 1e9}), flush=True)
 # plain torch copy host->device via SM reads? use a reduction that reads host memory directly
