@@ -79,6 +79,7 @@ enum gsys_state {
 /* internal bits set by the device library in the slot's flags word */
 #define GSYS_F_PRODUCER  0x100u   /* call class: producer (read-like), P20.24-29            */
 #define GSYS_F_INLINE    0x200u   /* small result goes to the slot's inline payload line    */
+#define GSYS_F_INLINE_IN 0x400u   /* small input (siginfo, sockaddr) is in the inline line   */
 
 /* Syscall numbers served (Linux x86-64). */
 #define GSYS_NR_PREAD64        17
@@ -274,6 +275,42 @@ int gsys_read_profile(uint64_t* out3, int reset);
 int gsys_bench_calls(uint32_t kind, uint32_t gflags, uint32_t blocks, uint32_t threads,
                      uint32_t iters, int32_t fd, uint64_t len, uint64_t size, void* d_buf,
                      int64_t* d_ret, uint64_t* d_lat_ns, uint64_t* d_sum, void* stream);
+
+/* ---------------------------------------------------------------- next rows
+ * Config 5a -- memory management (sec. VIII-A, miniamr): one work-group per mesh
+ * block, `iters` iterations.  Each iteration a work-group smooths its slice of d_field ([2][nblocks]
+ * [field_words] floats, ping-pong), reads the resident set size with a GPU-issued pread of
+ * statm_fd (= open("/proc/self/statm"); statm_buf: pinned host-mapped [nblocks][128] bytes) and
+ * getrusage(RUSAGE_SELF), and, when d_levels[t][b] == 0 (block coarsened) and RSS >=
+ * watermark_bytes, releases the host mirror [host_mesh + b*block_bytes, +block_bytes) with
+ * madvise(MADV_DONTNEED) at work-group granularity with `gflags` (paper: GSYS_WG |
+ * GSYS_NONBLOCKING | GSYS_RELAXED), once per block.  Outputs (DEVICE): d_released[b] = t+1 of
+ * the release (0 = kept), d_rss[t] = resident bytes and d_maxrss[t] = ru_maxrss (KiB) seen by
+ * work-group 0.  host_mesh must be private anonymous, page-aligned, pageable (not pinned)
+ * memory.  Asynchronous; gsys_wait() surfaces madvise errors.  -EINVAL on bad arguments. */
+int gsys_amr_release(uint64_t host_mesh, uint32_t nblocks, uint64_t block_bytes, const uint8_t* d_levels,
+                     uint32_t iters, int32_t statm_fd, uint64_t watermark_bytes, uint64_t page_bytes,
+                     float* d_field, uint32_t field_words, uint8_t* statm_buf, uint32_t* d_released,
+                     int64_t* d_rss, int64_t* d_maxrss, uint32_t gflags, void* stream);
+
+/* Config 5b -- signals (sec. VIII-B, signal-search): work-group b counts the
+ * (overlapping) occurrences of key[0..keylen) (keylen 1..16) in block b of d_data ([nblocks]
+ * [block_bytes], DEVICE), stores the count in counts[b] (host-mapped or device), then calls
+ * rt_sigqueueinfo(tgid, sig, {si_signo = sig, si_code = SI_QUEUE, si_pid = tgid, si_uid = uid,
+ * si_value.sival_int = b}) with `gflags` (paper: GSYS_WG | GSYS_NONBLOCKING).  The caller must
+ * block `sig` in every thread and consume it with sigwaitinfo (libgsys's own service threads
+ * block all asynchronous signals).  Asynchronous; -EINVAL on bad arguments. */
+int gsys_signal_search(const uint8_t* d_data, uint32_t nblocks, uint64_t block_bytes, const uint8_t* key,
+                       uint32_t keylen, int32_t tgid, int32_t sig, int32_t uid, uint32_t* counts,
+                       uint32_t gflags, void* stream);
+
+/* Host-side consumer for GPU-issued signals: installs an async-signal-safe SA_SIGINFO handler
+ * for `sig` (SIGRTMIN..SIGRTMAX) that appends si_value.sival_int to a ring of `capacity` entries
+ * (any thread of the process may take the signal); gsys_sigsink_read drains up to cap values
+ * (and CLOCK_MONOTONIC arrival times, t_ns may be NULL) and returns how many it copied.
+ * -EINVAL for a non-real-time signal, -ENODEV before install. */
+int gsys_sigsink_install(int32_t sig, uint32_t capacity);
+int gsys_sigsink_read(int32_t* values, uint64_t* t_ns, uint32_t cap);
 
 #ifdef __cplusplus
 }

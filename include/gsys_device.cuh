@@ -69,6 +69,16 @@ struct gsys_dev_ctx {
 #ifdef __CUDACC__
 namespace gsys {
 
+/* Small per-call payloads carried in the slot's host-mapped inline line (GSYS_INLINE_BYTES):
+ * `in` is copied there by the caller before the request is published (siginfo, sockaddr), `out`
+ * receives the host's result after a blocking call completes (struct rusage). */
+struct InlineIO {
+    void* out = nullptr;
+    unsigned out_bytes = 0;
+    const void* in = nullptr;
+    unsigned in_bytes = 0;
+};
+
 /* ------------------------------------------------------------------ PTX helpers */
 __device__ __forceinline__ unsigned smid() { unsigned r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r; }
 __device__ __forceinline__ unsigned warpid() { unsigned r; asm volatile("mov.u32 %0, %%warpid;" : "=r"(r)); return r; }
@@ -237,14 +247,24 @@ __device__ __forceinline__ void release(const gsys_dev_ctx* c, unsigned s, unsig
     st_release_gpu(&c->claim[s], 0u);      /* "consume the result" then free (reading A3) */
 }
 
-/* One thread, one request: claim -> marshal -> publish -> (poll).  Non-blocking requests keep
- * the slot until the host frees it (P24.34).  inline_out: for GSYS_F_INLINE calls, where the
- * host's inline payload is copied after completion (nbytes <= GSYS_INLINE_BYTES). */
+/* One thread, one request: claim -> (inline input) -> marshal -> publish -> (poll).  A non-blocking
+ * request's slot is reused only after the host has served it (P24.34, A15).  io.out: for
+ * GSYS_F_INLINE calls, where the host's inline result is copied after completion. */
 __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned nr, unsigned flags,
-                                                 const unsigned long long a[6], void* inline_out = nullptr,
-                                                 unsigned inline_bytes = 0) {
+                                                 const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     const bool blocking = !(flags & GSYS_NONBLOCKING);
     unsigned s = claim(c, blocking);
+    if (io.in != nullptr) {   /* input payload into the inline line; published by marshal's fence */
+        uint4* dst = reinterpret_cast<uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
+        const unsigned char* src = reinterpret_cast<const unsigned char*>(io.in);
+        for (unsigned i = 0; i < (io.in_bytes + 15u) / 16u; i++) {
+            uint4 v;
+            unsigned char* vb = reinterpret_cast<unsigned char*>(&v);
+            for (unsigned k = 0; k < 16u; k++) vb[k] = 16u * i + k < io.in_bytes ? src[16u * i + k] : 0u;
+            st_v4_sys(dst + i, v);
+        }
+        flags |= GSYS_F_INLINE_IN;
+    }
     unsigned seq = marshal(c, s, nr, flags, a);
     doorbell(c, s);
     if (!blocking) {
@@ -253,10 +273,10 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         return 0;
     }
     long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) != 0u);
-    if (inline_out != nullptr && r >= 0) {
+    if (io.out != nullptr && r >= 0) {
         const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
-        uint4* dst = reinterpret_cast<uint4*>(inline_out);
-        for (unsigned i = 0; i < inline_bytes / 16u; i++) dst[i] = ld_v4_sys(src + i);
+        uint4* dst = reinterpret_cast<uint4*>(io.out);
+        for (unsigned i = 0; i < io.out_bytes / 16u; i++) dst[i] = ld_v4_sys(src + i);
     }
     release(c, s, seq);
     return r;
@@ -270,8 +290,7 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
  * Relaxed consumer (Bar2 removed): the caller's warp waits with it and gets the result, the
  * other warps proceed at once and get 0 (reading A17, P28.3). */
 __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                             const unsigned long long a[6], void* inline_out = nullptr,
-                                             unsigned inline_bytes = 0) {
+                                             const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     __shared__ long long s_ret[2];
     __shared__ unsigned s_par;
     const bool strong = !(flags & GSYS_RELAXED);
@@ -280,7 +299,7 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
     const unsigned tid = block_tid();
     if (bar1) __syncthreads();
     long long r = 0;
-    if (tid == 0) r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, inline_out, inline_bytes);
+    if (tid == 0) r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, io);
     if (bar2) {
         unsigned p = 0;
         if (tid == 0) { p = (s_par ^ 1u) & 1u; s_par = p; s_ret[p] = r; }
@@ -299,10 +318,8 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
 /* Work-item (P20.31 "work-item invocations imply strong ordering"): every calling lane issues
  * its own request; the claim spins diverge, publication and the doorbell are warp-aggregated. */
 __device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                             const unsigned long long a[6], void* inline_out = nullptr,
-                                             unsigned inline_bytes = 0) {
-    return call_thread(c, nr, (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u), a, inline_out,
-                       inline_bytes);
+                                             const unsigned long long a[6], const InlineIO& io = InlineIO()) {
+    return call_thread(c, nr, (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u), a, io);
 }
 
 /* Kernel (P20.16-21, P20.33): relaxed only, -EINVAL for strong (reading A13).  Per call site and
@@ -313,8 +330,7 @@ __device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr,
  * data (the "barrier before"), and nobody waits.  Both are deadlock-free for grids larger than
  * the co-resident capacity. */
 __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                                 const unsigned long long a[6], void* inline_out = nullptr,
-                                                 unsigned inline_bytes = 0) {
+                                                 const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     __shared__ long long s_kret[2];
     __shared__ unsigned s_kpar;
     if (!(flags & GSYS_RELAXED)) return -EINVAL;
@@ -338,7 +354,7 @@ __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned
                 if (producer) {
                     unsigned t = atomicAdd(&k->arrive, 1u);
                     if (t == 0u) {
-                        r = call_thread(c, nr, flags | GSYS_F_PRODUCER, a, inline_out, inline_bytes);
+                        r = call_thread(c, nr, flags | GSYS_F_PRODUCER, a, io);
                         k->ret = r;
                         __threadfence();
                         st_release_gpu(&k->done, 1u);
@@ -352,7 +368,7 @@ __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned
                     unsigned t = atomicAdd(&k->arrive, 1u);
                     if (t == nb - 1u) {
                         __threadfence();
-                        r = call_thread(c, nr, flags, a, inline_out, inline_bytes);
+                        r = call_thread(c, nr, flags, a, io);
                     }
                 }
             }
@@ -374,12 +390,11 @@ __device__ __forceinline__ bool flags_valid(unsigned flags) {
 
 /* Dispatch on granularity.  Invalid granularity -> -EINVAL (uniform across the scope). */
 __device__ __forceinline__ long long invoke(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                            const unsigned long long a[6], void* inline_out = nullptr,
-                                            unsigned inline_bytes = 0) {
+                                            const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     switch (flags & GSYS_GRAN_MASK) {
-        case GSYS_WI: return wi_call(c, nr, flags, producer, a, inline_out, inline_bytes);
-        case GSYS_WG: return wg_call(c, nr, flags, producer, a, inline_out, inline_bytes);
-        case GSYS_KERNEL: return kernel_call(c, nr, flags, producer, a, inline_out, inline_bytes);
+        case GSYS_WI: return wi_call(c, nr, flags, producer, a, io);
+        case GSYS_WG: return wg_call(c, nr, flags, producer, a, io);
+        case GSYS_KERNEL: return kernel_call(c, nr, flags, producer, a, io);
         default: return -EINVAL;
     }
 }
@@ -411,8 +426,10 @@ __device__ __forceinline__ long long gsys_getrusage(const gsys_dev_ctx* c, int w
     const bool blocking = !(gflags & GSYS_NONBLOCKING);
     const bool inl = ru != nullptr && (blocking || !__isGlobal(ru));
     unsigned long long a[6] = {(unsigned long long)(long long)who, (unsigned long long)ru, 0ull, 0ull, 0ull, 0ull};
-    return gsys::invoke(c, GSYS_NR_GETRUSAGE, gflags | (inl ? GSYS_F_INLINE : 0u), true, a,
-                        blocking ? ru : nullptr, 144u);
+    gsys::InlineIO io;
+    io.out = blocking ? ru : nullptr;
+    io.out_bytes = 144u;
+    return gsys::invoke(c, GSYS_NR_GETRUSAGE, gflags | (inl ? GSYS_F_INLINE : 0u), true, a, io);
 }
 __device__ __forceinline__ long long gsys_madvise(const gsys_dev_ctx* c, void* addr, size_t len, int advice,
                                                   unsigned gflags) {
@@ -433,11 +450,17 @@ __device__ __forceinline__ long long gsys_recvfrom(const gsys_dev_ctx* c, int fd
                                (unsigned long long)fromlen};
     return gsys::invoke(c, GSYS_NR_RECVFROM, gflags, true, a);
 }
+/* rt_sigqueueinfo: the 128 B siginfo travels in the slot's inline line (copied by the caller before
+ * publishing), so `info` may live anywhere the caller can read -- registers/local memory included --
+ * and a non-blocking call does not have to keep it alive. */
 __device__ __forceinline__ long long gsys_rt_sigqueueinfo(const gsys_dev_ctx* c, int tgid, int sig, const void* info,
                                                           unsigned gflags) {
     unsigned long long a[6] = {(unsigned long long)(long long)tgid, (unsigned long long)(long long)sig,
                                (unsigned long long)info, 0ull, 0ull, 0ull};
-    return gsys::invoke(c, GSYS_NR_RT_SIGQUEUEINFO, gflags, false, a);
+    gsys::InlineIO io;
+    io.in = info;
+    io.in_bytes = info ? 128u : 0u;
+    return gsys::invoke(c, GSYS_NR_RT_SIGQUEUEINFO, gflags, false, a, io);
 }
 
 #endif /* __CUDACC__ */

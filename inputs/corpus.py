@@ -182,3 +182,24 @@ def make_corpus(nfiles: int, file_size, seed: int = SEED_CORPUS, grep_plants: bo
     with open(manifest, "w") as f:
         json.dump(m, f)
     return Corpus(d, paths, sizes, tot, pmasks, seed, m)
+
+
+# ---------------------------------------------------------------------------- config 5 inputs
+SEED_AMR = 6
+SEED_SIGNAL = 7
+
+
+def amr_levels(iters: int, nblocks: int, seed: int = SEED_AMR, p_coarsen: float = 0.04):
+    """Refinement level per (iteration, block) for the AMR-style mesh (config 5a, PAPER.md:28
+    sec. VIII-A: "when lower resolution is possible ... miniamr reduces memory"): level 1..3, and 0
+    (block coarsened, its host mirror may be released) with probability p_coarsen."""
+    rng = np.random.default_rng(seed)
+    lv = rng.integers(1, 4, size=(iters, nblocks), dtype=np.uint8)
+    lv[rng.random((iters, nblocks)) < p_coarsen] = 0
+    return lv
+
+
+def signal_blocks(nblocks: int, block_bytes: int, seed: int = SEED_SIGNAL):
+    """Data array for signal-search (config 5b, sec. VIII-B): synthetic text blocks."""
+    buf, _, _ = gen_bytes(seed, 0, nblocks * block_bytes)
+    return buf

@@ -60,6 +60,8 @@ def lib():
             L.oracle_syscall_rate.restype = ctypes.c_double
             L.oracle_syscall_rate.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_uint64, ctypes.c_int,
                                               ctypes.c_uint64, ctypes.c_uint64]
+            L.oracle_count_key.restype = ctypes.c_uint64
+            L.oracle_count_key.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_char_p, ctypes.c_uint64]
             L.oracle_pread_only.restype = ctypes.c_double
             L.oracle_pread_only.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_uint64]
             _lib = L
@@ -165,3 +167,9 @@ def pread_only(paths, nthreads: int, chunk: int = 256 << 10) -> float:
     if r < 0:
         raise OSError(int(-r), "oracle_pread_only")
     return r
+
+
+def count_key(data, key: bytes) -> int:
+    """Overlapping occurrences of key in data (signal-search lookup, sec. VIII-B)."""
+    arr = np.frombuffer(data, dtype=np.uint8) if isinstance(data, (bytes, bytearray)) else data
+    return int(lib().oracle_count_key(arr.ctypes.data, arr.size, key, len(key)))

@@ -194,6 +194,16 @@ int oracle_corpus(const char* const* paths, int nfiles, int nthreads, uint64_t c
     return J.err;
 }
 
+/* Occurrences (overlapping) of key[0..k) in data[0..n): the signal-search lookup of PAPER.md:30
+ * sec. VIII-B ("parallel lookup in a data array"), written as the definition. */
+uint64_t oracle_count_key(const uint8_t* data, uint64_t n, const uint8_t* key, uint64_t k) {
+    uint64_t c = 0;
+    if (k == 0 || k > n) return 0;
+    for (uint64_t i = 0; i + k <= n; i++)
+        if (memcmp(data + i, key, k) == 0) c++;
+    return c;
+}
+
 typedef struct {
     const char* const* paths; int nfiles; uint64_t chunk; int next; pthread_mutex_t mu; uint64_t bytes; int err;
 } pread_job_t;

@@ -51,3 +51,19 @@ def microbench_requests(granularity: str, n_blocks: int, block_threads: int, R: 
             off = ((c * R + r) * length) % size
             out.append((c, r, off, length))
     return out
+
+
+def amr_released(levels, rss_ok=None):
+    """Config 5a rule (sec. VIII-A: "When the RSS exceeds a watermark, madvise
+    relinquishes memory"; a block is released when it is coarsened): block b is released at the
+    first iteration t with levels[t][b] == 0 and RSS >= watermark (rss_ok[t], default always),
+    once.  Returns released[b] = t+1, or 0 if never."""
+    iters, nblocks = len(levels), len(levels[0]) if len(levels) else 0
+    out = [0] * nblocks
+    for t in range(iters):
+        if rss_ok is not None and not rss_ok[t]:
+            continue
+        for b in range(nblocks):
+            if out[b] == 0 and levels[t][b] == 0:
+                out[b] = t + 1
+    return out

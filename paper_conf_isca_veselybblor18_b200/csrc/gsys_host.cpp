@@ -331,6 +331,16 @@ inline int nr_index(uint32_t nr) {
 
 // ------------------------------------------------------------------ worker (interrupt handler + OS worker)
 void Worker::run() {
+    // service threads take no asynchronous signals: a GPU-issued rt_sigqueueinfo to this process
+    // must reach the application's sigwaitinfo consumer, never a worker
+    sigset_t ss;
+    sigfillset(&ss);
+    sigdelset(&ss, SIGSEGV);
+    sigdelset(&ss, SIGBUS);
+    sigdelset(&ss, SIGFPE);
+    sigdelset(&ss, SIGILL);
+    sigdelset(&ss, SIGABRT);
+    pthread_sigmask(SIG_BLOCK, &ss, nullptr);
     cudaSetDevice(inst->dev);
     Instance* I = inst;
     uint64_t idle_since = now_ns();
@@ -580,7 +590,10 @@ int64_t Worker::do_generic(Req& r) {
         case GSYS_NR_RT_SIGQUEUEINFO: {
             siginfo_t si;
             memset(&si, 0, sizeof si);
-            if (r.a[2] && read_small((uintptr_t)r.a[2], &si, sizeof si) != 0) return -EFAULT;
+            if (r.flags & GSYS_F_INLINE_IN)
+                memcpy(&si, inst->inline_h + (size_t)r.slot * GSYS_INLINE_BYTES, sizeof si);
+            else if (r.a[2] && read_small((uintptr_t)r.a[2], &si, sizeof si) != 0)
+                return -EFAULT;
             long z = syscall(SYS_rt_sigqueueinfo, (pid_t)r.a[0], (int)r.a[1], r.a[2] ? &si : nullptr);
             return z < 0 ? -(int64_t)errno : z;
         }
@@ -1285,6 +1298,62 @@ int gsys_plan_merge(uint32_t n, const int32_t* fd, const int64_t* off, const uin
         group_len[g] = (uint64_t)(u1 - u0);
     }
     return g + 1;
+}
+
+// ---------------------------------------------------------------- signal sink (config 5b)
+// A process-directed signal may land on any thread of the process (PyTorch owns several), so the
+// consumer side is an async-signal-safe SA_SIGINFO handler that appends si_value to a ring; the
+// application drains it with gsys_sigsink_read().
+namespace {
+std::atomic<uint64_t> g_sig_head{0}, g_sig_tail{0};
+int32_t* g_sig_ring = nullptr;
+uint64_t* g_sig_ts = nullptr;
+uint32_t g_sig_cap = 0;
+std::atomic<uint64_t> g_sig_dropped{0};
+
+void sigsink_handler(int, siginfo_t* si, void*) {
+    const uint64_t i = g_sig_tail.fetch_add(1, std::memory_order_relaxed);
+    if (i - g_sig_head.load(std::memory_order_relaxed) >= g_sig_cap) { g_sig_dropped.fetch_add(1); return; }
+    struct timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    g_sig_ts[i % g_sig_cap] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+    __atomic_store_n(&g_sig_ring[i % g_sig_cap], si->si_value.sival_int, __ATOMIC_RELEASE);
+}
+}  // namespace
+
+int gsys_sigsink_install(int32_t sig, uint32_t capacity) {
+    if (sig < SIGRTMIN || sig > SIGRTMAX || capacity == 0) return -EINVAL;
+    if (!g_sig_ring) {
+        g_sig_ring = (int32_t*)calloc(capacity, sizeof(int32_t));
+        g_sig_ts = (uint64_t*)calloc(capacity, sizeof(uint64_t));
+        if (!g_sig_ring || !g_sig_ts) return -ENOMEM;
+        for (uint32_t i = 0; i < capacity; i++) g_sig_ring[i] = INT32_MIN;
+        g_sig_cap = capacity;
+    }
+    struct sigaction sa;
+    memset(&sa, 0, sizeof sa);
+    sa.sa_sigaction = sigsink_handler;
+    sa.sa_flags = SA_SIGINFO | SA_RESTART;
+    sigemptyset(&sa.sa_mask);
+    return sigaction(sig, &sa, nullptr) == 0 ? 0 : -errno;
+}
+
+int gsys_sigsink_read(int32_t* values, uint64_t* t_ns, uint32_t cap) {
+    if (!g_sig_ring) return -ENODEV;
+    uint32_t n = 0;
+    uint64_t h = g_sig_head.load(std::memory_order_relaxed);
+    const uint64_t t = g_sig_tail.load(std::memory_order_acquire);
+    while (h < t && n < cap) {
+        int32_t v = __atomic_load_n(&g_sig_ring[h % g_sig_cap], __ATOMIC_ACQUIRE);
+        if (v == INT32_MIN) break;   // slot claimed by a handler that has not stored yet
+        values[n] = v;
+        if (t_ns) t_ns[n] = g_sig_ts[h % g_sig_cap];
+        g_sig_ring[h % g_sig_cap] = INT32_MIN;
+        n++;
+        h++;
+    }
+    g_sig_head.store(h, std::memory_order_release);
+    return (int)n;
 }
 
 // Self-test of the bounce ring allocator with a fake completion model: random allocation sizes

@@ -30,6 +30,11 @@
 #else
 #define GSYS_HD inline
 #endif
+#ifdef __CUDA_ARCH__
+#define GSYS_UNROLL _Pragma("unroll")
+#else
+#define GSYS_UNROLL
+#endif
 
 namespace gsys_scan {
 
@@ -139,7 +144,7 @@ GSYS_HD void dfa_pair(const unsigned short* __restrict__ dfa, unsigned& s0, unsi
                       const uint4& A1, OnHit&& on_hit) {
     const unsigned w0[4] = {A0.x, A0.y, A0.z, A0.w};
     const unsigned w1[4] = {A1.x, A1.y, A1.z, A1.w};
-#pragma unroll
+GSYS_UNROLL
     for (int i = 0; i < 16; i++) {
         const unsigned h0 = dfa_step(dfa, s0, (w0[i >> 2] >> (8 * (i & 3))) & 0xffu);
         const unsigned h1 = dfa_step(dfa, s1, (w1[i >> 2] >> (8 * (i & 3))) & 0xffu);
@@ -230,11 +235,11 @@ GSYS_HD void dfa_lane64(const unsigned short* __restrict__ dfa, const Win& W, un
     const unsigned nown = nown_ll >= 64 ? 64u : (unsigned)nown_ll;
     unsigned st = start_state(prevb, p0);
     if (nown == 64u && nvalid >= 64u) {
-#pragma unroll
+GSYS_UNROLL
         for (int k = 0; k < 4; k++) {
             const uint4 q = W.get((unsigned)k);
             const unsigned wv[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
+GSYS_UNROLL
             for (int i = 0; i < 16; i++) on_hit(dfa_step(dfa, st, (wv[i >> 2] >> (8 * (i & 3))) & 0xffu));
         }
         for (unsigned i = 64; st > DEAD; i++) {

@@ -75,6 +75,11 @@ SIGNATURES = {
     "gsys_split_result": (_I64, [_I64, _U64, _U64]),
     "gsys_selftest_bounce": (ctypes.c_int, [_U64, _U32, _U64]),
     "gsys_set_profile": (ctypes.c_int, [ctypes.c_int]),
+    "gsys_amr_release": (ctypes.c_int, [_U64, _U32, _U64, _P, _U32, _I32, _U64, _U64, _P, _U32, _P, _P, _P, _P, _U32,
+                                        _P]),
+    "gsys_signal_search": (ctypes.c_int, [_P, _U32, _U64, ctypes.c_char_p, _U32, _I32, _I32, _I32, _P, _U32, _P]),
+    "gsys_sigsink_install": (ctypes.c_int, [_I32, _U32]),
+    "gsys_sigsink_read": (ctypes.c_int, [_P, _P, _U32]),
     "gsys_read_profile": (ctypes.c_int, [_P, ctypes.c_int]),
     "gsys_wordcount": (ctypes.c_int, [_P, _P, _U32, _U32, ctypes.c_char_p, _P, _U32, ctypes.c_char_p, _P, _U32,
                                       _P, _P, _P, _U32, _U32, _U32, _U32, _P]),
@@ -259,6 +264,22 @@ def gsys_bench_calls(kind: str, gflags: int, blocks: int, threads: int, iters: i
     rc = lib().gsys_bench_calls(k, gflags, blocks, threads, iters, fd, length, size, ptr(d_buf), ptr(d_ret),
                                 ptr(d_lat), ptr(d_sum), _stream(stream))
     return _check(rc, "gsys_bench_calls")
+
+
+def gsys_amr_release(host_mesh: int, nblocks: int, block_bytes: int, d_levels, iters: int, statm_fd: int,
+                     watermark_bytes: int, page_bytes: int, d_field, field_words: int, statm_buf, d_released, d_rss,
+                     d_maxrss, gflags: int = WG | NONBLOCKING | RELAXED, stream=None) -> int:
+    rc = lib().gsys_amr_release(host_mesh, nblocks, block_bytes, d_levels.data_ptr(), iters, statm_fd,
+                                watermark_bytes, page_bytes, d_field.data_ptr(), field_words, statm_buf.data_ptr(),
+                                d_released.data_ptr(), d_rss.data_ptr(), d_maxrss.data_ptr(), gflags, _stream(stream))
+    return _check(rc, "gsys_amr_release")
+
+
+def gsys_signal_search(d_data, nblocks: int, block_bytes: int, key: bytes, tgid: int, sig: int, uid: int, counts,
+                       gflags: int = WG | NONBLOCKING, stream=None) -> int:
+    rc = lib().gsys_signal_search(d_data.data_ptr(), nblocks, block_bytes, key, len(key), tgid, sig, uid,
+                                  counts.data_ptr(), gflags, _stream(stream))
+    return _check(rc, "gsys_signal_search")
 
 
 def header_functions(path: str | None = None) -> list[str]:

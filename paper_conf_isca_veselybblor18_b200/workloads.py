@@ -121,3 +121,84 @@ def bench_calls(kind: str, gflags: int, blocks: int, threads: int, iters: int, f
     G.gsys_bench_calls(kind, gflags, blocks, threads, iters, fd, length, size, d_buf, d_ret, d_lat, d_sum, stream)
     rc = G.gsys_wait(stream)
     return callers, d_ret, d_lat, d_sum, rc
+
+
+# ---------------------------------------------------------------------------- config 5 (next rows)
+class HostMesh:
+    """Private anonymous, page-aligned, pageable host memory (mmap) for the AMR mirror."""
+
+    def __init__(self, nbytes: int):
+        import mmap
+        self.mm = mmap.mmap(-1, nbytes, flags=mmap.MAP_PRIVATE | mmap.MAP_ANONYMOUS)
+        import ctypes
+        self._c = ctypes.c_char.from_buffer(self.mm)
+        self.addr = ctypes.addressof(self._c)
+        self.nbytes = nbytes
+
+    def view(self):
+        import numpy as np
+        return np.frombuffer(self.mm, dtype=np.uint8)
+
+
+def amr_run(levels, block_bytes: int = 64 << 10, watermark_bytes: int = 0, field_words: int = 4096,
+            gflags: int = G.WG | G.NONBLOCKING | G.RELAXED, fill: int = 0xA5, stream=None):
+    """Config 5a: GPU-issued madvise/getrusage/pread(/proc/self/statm) over an AMR-style mesh.
+    Returns (released[b] host array, rss[t], maxrss_kib[t], mesh, wait_rc)."""
+    import numpy as np
+    ensure_init()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    lv = np.ascontiguousarray(levels, dtype=np.uint8)
+    iters, nblocks = lv.shape
+    mesh = HostMesh(nblocks * block_bytes)
+    mesh.view()[:] = fill
+    d_levels = torch.from_numpy(lv).to(dev)
+    d_field = torch.rand(2 * nblocks * field_words, device=dev)
+    statm = torch.zeros(nblocks * 128, dtype=torch.uint8).pin_memory()
+    d_rel = torch.zeros(nblocks, dtype=torch.int32, device=dev)
+    d_rss = torch.zeros(iters, dtype=torch.int64, device=dev)
+    d_max = torch.zeros(iters, dtype=torch.int64, device=dev)
+    fd = os.open("/proc/self/statm", os.O_RDONLY)
+    try:
+        stream = stream or torch.cuda.current_stream()
+        G.gsys_amr_release(mesh.addr, nblocks, block_bytes, d_levels, iters, fd, watermark_bytes,
+                           os.sysconf("SC_PAGE_SIZE"), d_field, field_words, statm, d_rel, d_rss, d_max, gflags,
+                           stream)
+        rc = G.gsys_wait(stream)
+    finally:
+        os.close(fd)
+    return d_rel.cpu().numpy(), d_rss.cpu().numpy(), d_max.cpu().numpy(), mesh, rc
+
+
+def signal_search_run(data_dev, nblocks: int, block_bytes: int, key: bytes, sig: int | None = None,
+                      consumer=None, gflags: int = G.WG | G.NONBLOCKING, stream=None, timeout_s: float = 60.0):
+    """Config 5b: GPU work-groups search their block and signal the host with rt_sigqueueinfo;
+    `consumer(block_id)` runs on the host for each signal as it arrives.
+    Returns (counts[b], received ids in arrival order, arrival times ns, wait_rc)."""
+    import ctypes
+    import signal as _signal
+    import time
+    import numpy as np
+    ensure_init()
+    sig = sig or (_signal.SIGRTMIN + 3)
+    L = G.lib()
+    rc = L.gsys_sigsink_install(sig, max(1024, 2 * nblocks))
+    if rc:
+        raise G.GsysError(-rc, "gsys_sigsink_install")
+    counts = torch.zeros(nblocks, dtype=torch.int32).pin_memory()
+    stream = stream or torch.cuda.current_stream()
+    G.gsys_signal_search(data_dev, nblocks, block_bytes, key, os.getpid(), sig, os.getuid(), counts, gflags, stream)
+    got, ts = [], []
+    vals = (ctypes.c_int32 * 4096)()
+    tns = (ctypes.c_uint64 * 4096)()
+    t_end = time.time() + timeout_s
+    while len(got) < nblocks and time.time() < t_end:
+        n = L.gsys_sigsink_read(vals, tns, 4096)
+        for i in range(max(n, 0)):
+            got.append(int(vals[i]))
+            ts.append(int(tns[i]))
+            if consumer is not None:
+                consumer(int(vals[i]))
+        if n <= 0:
+            time.sleep(0.0002)
+    rc = G.gsys_wait(stream)
+    return counts.numpy().copy(), got, ts, rc

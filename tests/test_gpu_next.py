@@ -1,0 +1,61 @@
+"""GPU parity for the §8(f) next rows (config 5): GPU-issued madvise + getrusage + pread of
+/proc/self/statm on an AMR-style mesh, and rt_sigqueueinfo from a signal-search kernel."""
+import numpy as np
+import pytest
+import torch
+
+import inputs
+import oracle
+from oracle import plan
+from paper_conf_isca_veselybblor18_b200 import gsys as G
+from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def gsys_instance():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    W.ensure_init()
+    yield
+
+
+@pytest.mark.parametrize("gflags", [G.WG | G.NONBLOCKING | G.RELAXED, G.WG | G.BLOCKING | G.RELAXED,
+                                    G.WG | G.BLOCKING | G.STRONG])
+def test_amr_madvise_releases_exactly_the_coarsened_blocks(gflags):
+    lv = inputs.amr_levels(6, 96)
+    bs = 64 << 10
+    released, rss, maxrss, mesh, rc = W.amr_run(lv, block_bytes=bs, watermark_bytes=0, gflags=gflags)
+    assert rc == 0
+    want = plan.amr_released(lv)
+    assert released.tolist() == want
+    assert any(want) and not all(want)
+    view = mesh.view().reshape(lv.shape[1], bs)
+    for b, t in enumerate(want):
+        if t:
+            assert not view[b].any(), b          # MADV_DONTNEED on private anonymous memory -> zero pages
+        else:
+            assert (view[b] == 0xA5).all(), b
+    assert (rss > 0).all() and (maxrss > 0).all()
+
+
+def test_amr_watermark_gates_release():
+    lv = inputs.amr_levels(4, 64, seed=11)
+    released, rss, maxrss, mesh, rc = W.amr_run(lv, watermark_bytes=1 << 50)
+    assert rc == 0 and not released.any()
+    assert (mesh.view() == 0xA5).all()
+
+
+@pytest.mark.parametrize("gflags", [G.WG | G.NONBLOCKING, G.WG | G.BLOCKING | G.RELAXED])
+def test_signal_search_counts_and_ids(gflags):
+    nb, bs = 512, 32 << 10
+    data = inputs.signal_blocks(nb, bs)
+    d = torch.from_numpy(data).cuda()
+    key = inputs.dictionary()[0]
+    counts, got, ts, rc = W.signal_search_run(d, nb, bs, key, gflags=gflags)
+    assert rc == 0
+    assert sorted(got) == list(range(nb))                  # every work-group signalled exactly once
+    want = [oracle.count_key(data[b * bs:(b + 1) * bs], key) for b in range(nb)]
+    assert counts.tolist() == want
+    assert sum(want) > 0

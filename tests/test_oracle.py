@@ -239,3 +239,18 @@ def test_request_count_closed_forms():
     assert protocol.requests_per_call("kernel", 151552, 592) == 1
     assert len(plan.microbench_requests("wi", 3, 64, 2, 4096, 1 << 20)) == 3 * 64 * 2
     assert len(plan.microbench_requests("kernel", 3, 64, 5, 4096, 1 << 20)) == 5
+
+
+def test_count_key_brute_force():
+    rng = np.random.default_rng(4)
+    for _ in range(500):
+        n = int(rng.integers(0, 60))
+        d = bytes(rng.choice(list(b"ab"), size=n).tolist())
+        k = bytes(rng.choice(list(b"ab"), size=int(rng.integers(1, 4))).tolist())
+        assert oracle.count_key(d, k) == sum(1 for i in range(len(d) - len(k) + 1) if d[i:i + len(k)] == k)
+
+
+def test_amr_release_rule():
+    lv = [[1, 0, 2, 3], [0, 0, 1, 3], [2, 2, 0, 3]]
+    assert plan.amr_released(lv) == [2, 1, 3, 0]
+    assert plan.amr_released(lv, rss_ok=[False, True, True]) == [2, 2, 3, 0]
