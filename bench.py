@@ -49,8 +49,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip scan roofline / syscall-rate extras")
     ap.add_argument("--root", default=None, help="corpus directory (default /dev/shm/gsys_corpus)")
-    ap.add_argument("--mode", default="wordcount", choices=["wordcount", "syscalls"],
-                    help="syscalls: config-2 granularity x blocking x ordering sweep (one JSON line)")
+    ap.add_argument("--mode", default="wordcount", choices=["wordcount", "syscalls", "memcached", "mm"],
+                    help="syscalls: config-2 sweep; memcached: config 4; mm: config 5 (one JSON line each)")
     return ap.parse_args()
 
 
@@ -180,6 +180,10 @@ def main():
         return run_reference(a)
     if a.mode == "syscalls":
         return run_syscalls(a)
+    if a.mode == "memcached":
+        return run_memcached(a)
+    if a.mode == "mm":
+        return run_mm(a)
     import torch
     import torch.distributed as dist
 
@@ -509,6 +513,127 @@ def run_syscalls(a):
                             "getrusage_1thread": oracle.syscall_rate("getrusage", 1, 200000)}
     out["service_threads"] = G.gsys_stats()["threads"]
     os.close(fd)
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def run_memcached(a):
+    """Config 4 (BASELINE.json configs[3]): memcached-style binary-UDP GET server.  GPU server =
+    work-groups issuing recvfrom/sendto (WG, blocking, weak -- P32.29-30); CPU server = the
+    oracle's threaded C server over the same store; same load generator, same request stream.
+    Reported: requests/s and client-side latency for 16 and 1024 elements per bucket (the paper's
+    large-bucket case, P32.33) with 1 KiB values."""
+    import ctypes
+    import threading
+
+    import numpy as np
+    import torch
+
+    import oracle
+    from inputs import mc as MC
+    from oracle import mc as OM
+    from paper_conf_isca_veselybblor18_b200 import gsys as G
+    from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+    torch.cuda.set_device(0)
+    W.ensure_init()
+    out = {"mode": "memcached", "metric": "GET requests/s (binary memcached over UDP loopback)", "cases": []}
+    nthr = host_cores()
+    for per_bucket in (16, 1024):
+        nbuckets = 64
+        nkeys = nbuckets * per_bucket * 3 // 4
+        keys, vals = MC.dataset(nkeys, vlen=1024)
+        reqs = MC.requests(keys, 20000)
+        pkts = [MC.encode_get(i, k) for i, k in enumerate(reqs)]
+        table = dict(zip(keys, vals))
+        for nwg in (4, 8, 12):
+            resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=nwg, nbuckets=nbuckets,
+                                                    bucket_cap=per_bucket * 2, client_threads=4, window=8)
+            ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
+            lat_us = np.array(lat, dtype=np.float64) / 1e3
+            out["cases"].append({"server": "gpu", "elements_per_bucket": per_bucket, "work_groups": nwg,
+                                 "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
+                                 "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
+                                 "requests": len(pkts)})
+        kb, ko, kl, vb, vo, vl = MC.pack(keys, vals)
+        for st in (1, 4):
+            sock = MC.udp_server_socket()
+            stop = ctypes.c_int(0)
+            th = threading.Thread(target=lambda: oracle.lib().oracle_mc_serve(
+                sock.fileno(), st, kb.ctypes.data, ko.ctypes.data, kl.ctypes.data, vb.ctypes.data, vo.ctypes.data,
+                vl.ctypes.data, len(keys), nbuckets, ctypes.addressof(stop)))
+            th.start()
+            try:
+                resp, lat, secs = MC.run_client(sock.getsockname()[1], pkts, nthreads=4, window=8)
+            finally:
+                stop.value = 1
+                th.join()
+                sock.close()
+            lat_us = np.array(lat, dtype=np.float64) / 1e3
+            ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
+            out["cases"].append({"server": "cpu-oracle", "threads": st, "elements_per_bucket": per_bucket,
+                                 "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
+                                 "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
+                                 "requests": len(pkts)})
+    out["host_cores"] = nthr
+    out["service_threads"] = G.gsys_stats()["threads"]
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def run_mm(a):
+    """Config 5 (BASELINE.json configs[4]): (a) AMR-style mesh whose coarsened blocks are released
+    with GPU-issued madvise(MADV_DONTNEED) once RSS (GPU-issued pread of /proc/self/statm) passes a
+    watermark; (b) signal-search: GPU work-groups notify the host with rt_sigqueueinfo and the host
+    hashes each block (SHA-512, as in the paper, P30.14) as its signal arrives vs after the kernel."""
+    import hashlib
+
+    import numpy as np
+    import torch
+
+    import inputs
+    from oracle import plan
+    from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+    torch.cuda.set_device(0)
+    W.ensure_init()
+    out = {"mode": "mm"}
+    # (a) AMR: 1024 blocks x 256 KiB mirror (256 MiB), 12 iterations
+    nb, bs, iters = 1024, 256 << 10, 12
+    lv = inputs.amr_levels(iters, nb, p_coarsen=0.03)
+    t0 = time.perf_counter()
+    released, rss, maxrss, mesh, rc = W.amr_run(lv, block_bytes=bs, watermark_bytes=0)
+    dt = time.perf_counter() - t0
+    want = plan.amr_released(lv)
+    view = mesh.view().reshape(nb, bs)
+    zero_ok = all((not view[b].any()) == bool(want[b]) for b in range(nb))
+    out["amr"] = {"blocks": nb, "block_bytes": bs, "iters": iters, "seconds": dt, "wait_rc": rc,
+                  "released_blocks": int((released > 0).sum()), "released_equals_rule": released.tolist() == want,
+                  "released_read_back_zero": zero_ok, "rss_first_MiB": float(rss[0]) / 2**20,
+                  "rss_last_MiB": float(rss[-1]) / 2**20, "maxrss_last_MiB": float(maxrss[-1]) / 1024,
+                  "madvise_calls": int((released > 0).sum()), "statm_preads": nb * iters, "getrusage_calls": nb * iters}
+    del mesh
+    # (b) signal-search: 2048 blocks x 64 KiB
+    nb, bs = 2048, 64 << 10
+    data = inputs.signal_blocks(nb, bs)
+    d = torch.from_numpy(data).cuda()
+    key = inputs.dictionary()[0]
+    digests = {}
+
+    def consume(b):
+        digests[b] = hashlib.sha512(data[b * bs:(b + 1) * bs].tobytes()).hexdigest()
+    t0 = time.perf_counter()
+    counts, got, ts, rc = W.signal_search_run(d, nb, bs, key, consumer=consume)
+    overlapped = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    counts2, got2, _, _ = W.signal_search_run(d, nb, bs, key)
+    for b in range(nb):
+        hashlib.sha512(data[b * bs:(b + 1) * bs].tobytes()).hexdigest()
+    serial = time.perf_counter() - t0
+    out["signal_search"] = {"blocks": nb, "block_bytes": bs, "signals_received": len(got),
+                            "ids_exact_once": sorted(got) == list(range(nb)), "digests": len(digests),
+                            "overlapped_s": overlapped, "search_then_hash_s": serial,
+                            "speedup": serial / overlapped if overlapped > 0 else None}
     print(json.dumps(out), flush=True)
     return 0
 

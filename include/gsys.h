@@ -304,6 +304,27 @@ int gsys_signal_search(const uint8_t* d_data, uint32_t nblocks, uint64_t block_b
                        uint32_t keylen, int32_t tgid, int32_t sig, int32_t uid, uint32_t* counts,
                        uint32_t gflags, void* stream);
 
+/* Config 4 -- memcached-style UDP GET server (sec. VIII-D).  gsys_mc_build lays the
+ * key/value set out for the GPU: n keys (1..32 B, key_len[i] bytes at keys+key_off[i]) and values
+ * (<= 4096 B at vals+val_off[i]) go to FNV-1a buckets of bucket_cap entries: d_entries (DEVICE,
+ * gsys_mc_entries_bytes(nbuckets, bucket_cap) bytes), d_bucket_n (DEVICE u32[nbuckets]) and
+ * d_heap (DEVICE, heap_bytes >= max(val_off+val_len)).  -E2BIG when a bucket overflows.
+ * gsys_mc_serve launches nwg work-groups that loop recvfrom(fd) -> lookup -> sendto with the
+ * memcached binary protocol over UDP (8-byte frame header; GET hit: status 0, 4-byte flags +
+ * value; miss: status 1 + "Not found"), both calls WG-granularity, blocking, `gflags` ordering
+ * (paper: weak).  io: pinned host-mapped [nwg][8192] request/reply buffers; stop: host-mapped
+ * u32 the host sets to 1 to end the server (checked whenever recvfrom times out -- set
+ * SO_RCVTIMEO on fd); d_stats (DEVICE u64[4]): served, misses, malformed, receive timeouts.
+ * Keep nwg below the service thread count: each waiting recvfrom occupies a service thread. */
+uint64_t gsys_mc_entries_bytes(uint32_t nbuckets, uint32_t bucket_cap);
+int gsys_mc_build(const uint8_t* keys, const uint32_t* key_off, const uint8_t* key_len, const uint8_t* vals,
+                  const uint64_t* val_off, const uint32_t* val_len, uint32_t n, uint32_t nbuckets,
+                  uint32_t bucket_cap, void* d_entries, uint32_t* d_bucket_n, uint8_t* d_heap,
+                  uint64_t heap_bytes);
+int gsys_mc_serve(int32_t fd, const void* d_entries, const uint32_t* d_bucket_n, const uint8_t* d_heap,
+                  uint32_t nbuckets, uint32_t bucket_cap, uint32_t nwg, uint8_t* io, const uint32_t* stop,
+                  uint64_t* d_stats, uint32_t gflags, void* stream);
+
 /* Host-side consumer for GPU-issued signals: installs an async-signal-safe SA_SIGINFO handler
  * for `sig` (SIGRTMIN..SIGRTMAX) that appends si_value.sival_int to a ring of `capacity` entries
  * (any thread of the process may take the signal); gsys_sigsink_read drains up to cap values

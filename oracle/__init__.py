@@ -60,6 +60,9 @@ def lib():
             L.oracle_syscall_rate.restype = ctypes.c_double
             L.oracle_syscall_rate.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_uint64, ctypes.c_int,
                                               ctypes.c_uint64, ctypes.c_uint64]
+            L.oracle_mc_serve.restype = ctypes.c_int64
+            L.oracle_mc_serve.argtypes = [ctypes.c_int, ctypes.c_int] + [ctypes.c_void_p] * 6 + [
+                ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p]
             L.oracle_count_key.restype = ctypes.c_uint64
             L.oracle_count_key.argtypes = [ctypes.c_void_p, ctypes.c_uint64, ctypes.c_char_p, ctypes.c_uint64]
             L.oracle_pread_only.restype = ctypes.c_double

@@ -29,6 +29,7 @@
 #include <stdlib.h>
 #include <string.h>
 #include <sys/resource.h>
+#include <sys/socket.h>
 #include <sys/stat.h>
 #include <sys/types.h>
 #include <time.h>
@@ -294,4 +295,81 @@ double oracle_syscall_rate(int kind, int nthreads, uint64_t iters_per_thread, in
     free(th); free(R);
     if (err) return (double)err;
     return (double)iters_per_thread * nthreads / dt;
+}
+
+/*
+ * CPU memcached-style GET server (config 4 baseline, sec. VIII-D "a CPU version of this
+ * workload"): nthreads threads loop recvfrom(fd) -> look the key up -> sendto, until *stop.  The
+ * store is the plain list of n (key, value) pairs grouped into nbuckets buckets by a djb2 hash of
+ * the key (the CPU version's own table; nothing is shared with the GPU path), scanned linearly.
+ * Replies follow the definition in oracle/mc.py.  Returns requests served.
+ */
+typedef struct {
+    int fd; volatile int* stop;
+    const uint8_t* keys; const uint32_t* koff; const uint8_t* klen;
+    const uint8_t* vals; const uint64_t* voff; const uint32_t* vlen;
+    const uint32_t* order; const uint32_t* bstart; uint32_t nbuckets;
+    uint64_t served;
+} mc_job_t;
+
+static uint32_t djb2(const uint8_t* k, uint32_t n) {
+    uint32_t h = 5381;
+    for (uint32_t i = 0; i < n; i++) h = h * 33u + k[i];
+    return h;
+}
+
+static void* mc_worker(void* arg) {
+    mc_job_t* J = (mc_job_t*)arg;
+    uint8_t rx[2048], tx[8192];
+    uint64_t served = 0;
+    while (!*J->stop) {
+        struct sockaddr_storage from;
+        socklen_t fl = sizeof from;
+        ssize_t r = recvfrom(J->fd, rx, sizeof rx, 0, (struct sockaddr*)&from, &fl);
+        if (r < 32 || rx[8] != 0x80 || rx[9] != 0x00) continue;
+        uint32_t klen = ((uint32_t)rx[10] << 8) | rx[11], ext = rx[12];
+        if (klen < 1 || klen > 32 || 32 + ext + klen > (uint32_t)r) continue;
+        const uint8_t* key = rx + 32 + ext;
+        uint32_t b = djb2(key, klen) % J->nbuckets;
+        int64_t hit = -1;
+        for (uint32_t j = J->bstart[b]; j < J->bstart[b + 1]; j++) {
+            uint32_t i = J->order[j];
+            if (J->klen[i] == klen && memcmp(J->keys + J->koff[i], key, klen) == 0) { hit = i; break; }
+        }
+        memset(tx, 0, 36);
+        tx[0] = rx[0]; tx[1] = rx[1]; tx[5] = 1;
+        tx[8] = 0x81; tx[9] = rx[9];
+        uint32_t body = hit >= 0 ? 4 + J->vlen[hit] : 9;
+        tx[12] = hit >= 0 ? 4 : 0;
+        tx[15] = hit >= 0 ? 0 : 1;
+        tx[16] = (uint8_t)(body >> 24); tx[17] = (uint8_t)(body >> 16); tx[18] = (uint8_t)(body >> 8); tx[19] = (uint8_t)body;
+        memcpy(tx + 20, rx + 20, 4);
+        size_t len;
+        if (hit >= 0) { memcpy(tx + 36, J->vals + J->voff[hit], J->vlen[hit]); len = 36 + J->vlen[hit]; }
+        else { memcpy(tx + 32, "Not found", 9); len = 41; }
+        sendto(J->fd, tx, len, 0, (struct sockaddr*)&from, fl);
+        served++;
+    }
+    __atomic_add_fetch(&J->served, served, __ATOMIC_RELAXED);
+    return NULL;
+}
+
+int64_t oracle_mc_serve(int fd, int nthreads, const uint8_t* keys, const uint32_t* koff, const uint8_t* klen,
+                        const uint8_t* vals, const uint64_t* voff, const uint32_t* vlen, uint32_t n,
+                        uint32_t nbuckets, volatile int* stop) {
+    uint32_t* bstart = (uint32_t*)calloc(nbuckets + 1, sizeof(uint32_t));
+    uint32_t* order = (uint32_t*)malloc(sizeof(uint32_t) * (n ? n : 1));
+    uint32_t* fill = (uint32_t*)calloc(nbuckets, sizeof(uint32_t));
+    for (uint32_t i = 0; i < n; i++) bstart[djb2(keys + koff[i], klen[i]) % nbuckets + 1]++;
+    for (uint32_t b = 0; b < nbuckets; b++) bstart[b + 1] += bstart[b];
+    for (uint32_t i = 0; i < n; i++) {
+        uint32_t b = djb2(keys + koff[i], klen[i]) % nbuckets;
+        order[bstart[b] + fill[b]++] = i;
+    }
+    mc_job_t J = {fd, stop, keys, koff, klen, vals, voff, vlen, order, bstart, nbuckets, 0};
+    pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * nthreads);
+    for (int t = 0; t < nthreads; t++) pthread_create(&th[t], NULL, mc_worker, &J);
+    for (int t = 0; t < nthreads; t++) pthread_join(th[t], NULL);
+    free(th); free(bstart); free(order); free(fill);
+    return (int64_t)J.served;
 }

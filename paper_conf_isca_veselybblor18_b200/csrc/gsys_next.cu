@@ -20,6 +20,8 @@
 #include <string.h>
 #include <sys/mman.h>
 
+#include <vector>
+
 #include "gsys.h"
 #include "gsys_device.cuh"
 #include "gsys_internal.h"
@@ -140,9 +142,200 @@ __global__ void __launch_bounds__(256) sig_kernel(SigArgs a) {
     gsys_rt_sigqueueinfo(a.ctx, a.tgid, a.sig, si, a.gflags);
 }
 
+// ------------------------------------------------------------------ config 4: memcached-style UDP GETs
+// Layout (device): McEntry[nbuckets][bucket_cap] (keys zero-padded to 32 B), bucket fill counts,
+// and a value heap.  One work-group per in-flight request: recvfrom -> parse -> FNV-1a bucket ->
+// all threads compare the bucket's entries (up to 1024, the paper's large-bucket case, P32.33) ->
+// reply assembled in the work-group's host-mapped buffer -> sendto (both WG, blocking, weak --
+// the paper's choice, P32.29-30).
+struct McEntry {
+    uint4 k0, k1;
+    unsigned klen, vlen;
+    unsigned long long voff;
+};
+static_assert(sizeof(McEntry) == 48, "McEntry layout");
+
+constexpr unsigned MC_IO_BYTES = 8192;       // per work-group: rx | tx | from | fromlen
+constexpr unsigned MC_RX = 0, MC_TX = 2048, MC_FROM = 7168, MC_FROMLEN = 7296;
+constexpr unsigned MC_MAXKEY = 32, MC_MAXVAL = 4096;
+
+__host__ __device__ __forceinline__ unsigned mc_hash(const unsigned char* k, unsigned n) {
+    unsigned h = 2166136261u;
+    for (unsigned i = 0; i < n; i++) { h ^= k[i]; h *= 16777619u; }
+    return h;
+}
+
+struct McArgs {
+    const gsys_dev_ctx* ctx;
+    const McEntry* entries;
+    const unsigned* bucket_n;
+    const unsigned char* heap;
+    unsigned char* io;              // host-mapped [nwg][MC_IO_BYTES]
+    const volatile unsigned* stop;  // host-mapped stop flag
+    unsigned long long* stats;      // device [4]: served, misses, malformed, recv timeouts
+    unsigned nbuckets, cap, gflags;
+    int fd;
+};
+
+__device__ __forceinline__ unsigned be16(const unsigned char* p) { return ((unsigned)p[0] << 8) | p[1]; }
+__device__ __forceinline__ unsigned be32(const unsigned char* p) {
+    return ((unsigned)p[0] << 24) | ((unsigned)p[1] << 16) | ((unsigned)p[2] << 8) | p[3];
+}
+__device__ __forceinline__ void put_be16(unsigned char* p, unsigned v) { p[0] = (unsigned char)(v >> 8); p[1] = (unsigned char)v; }
+__device__ __forceinline__ void put_be32(unsigned char* p, unsigned v) {
+    p[0] = (unsigned char)(v >> 24); p[1] = (unsigned char)(v >> 16); p[2] = (unsigned char)(v >> 8); p[3] = (unsigned char)v;
+}
+
+__global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
+    __shared__ unsigned s_found, s_len, s_keylen, s_bucket, s_ok, s_done;
+    __shared__ __align__(16) unsigned char s_key[MC_MAXKEY];
+    unsigned char* io = a.io + (size_t)blockIdx.x * MC_IO_BYTES;
+    unsigned char* rx = io + MC_RX;
+    unsigned char* tx = io + MC_TX;
+    void* from = io + MC_FROM;
+    unsigned* fromlen = reinterpret_cast<unsigned*>(io + MC_FROMLEN);
+    const unsigned gf = a.gflags | GSYS_HOSTBUF;
+    for (;;) {
+        if (threadIdx.x == 0) *(volatile unsigned*)fromlen = 128u;
+        const long long r = gsys_recvfrom(a.ctx, a.fd, rx, 2048, 0, from, fromlen, gf);   // producer: Bar2
+        if (r < 0) {
+            if (threadIdx.x == 0) {
+                s_done = *a.stop;
+                if (r == -EAGAIN || r == -EWOULDBLOCK) atomicAdd(&a.stats[3], 1ull);
+            }
+            __syncthreads();
+            if (s_done) break;
+            continue;
+        }
+        if (threadIdx.x == 0) {
+            const volatile unsigned char* v = rx;
+            unsigned ok = r >= 32 && v[8] == 0x80 && v[9] == 0x00;
+            unsigned char hdr[32];
+            for (int i = 0; i < 32; i++) hdr[i] = v[i];
+            const unsigned klen = be16(hdr + 10), ext = hdr[12];
+            ok = ok && klen >= 1 && klen <= MC_MAXKEY && (long long)(32 + ext + klen) <= r;
+            s_keylen = ok ? klen : 0u;
+            for (unsigned i = 0; i < MC_MAXKEY; i++) s_key[i] = (ok && i < klen) ? v[32 + ext + i] : 0u;
+            s_bucket = ok ? mc_hash(s_key, klen) % a.nbuckets : 0u;
+            s_ok = ok;
+            s_found = 0xffffffffu;
+            if (!ok) atomicAdd(&a.stats[2], 1ull);
+        }
+        __syncthreads();
+        if (!s_ok) continue;
+        // parallel bucket scan
+        const uint4 K0 = *reinterpret_cast<const uint4*>(s_key), K1 = *reinterpret_cast<const uint4*>(s_key + 16);
+        const unsigned n = a.bucket_n[s_bucket];
+        const McEntry* B = a.entries + (size_t)s_bucket * a.cap;
+        for (unsigned i = threadIdx.x; i < n; i += blockDim.x) {
+            const McEntry e = B[i];
+            if (e.klen == s_keylen && e.k0.x == K0.x && e.k0.y == K0.y && e.k0.z == K0.z && e.k0.w == K0.w &&
+                e.k1.x == K1.x && e.k1.y == K1.y && e.k1.z == K1.z && e.k1.w == K1.w)
+                atomicMin(&s_found, i);
+        }
+        __syncthreads();
+        const bool hit = s_found != 0xffffffffu;
+        const McEntry* e = hit ? B + s_found : nullptr;
+        const unsigned vlen = hit ? e->vlen : 0u;
+        // reply: UDP frame header + binary response header (+ flags + value | "Not found")
+        if (threadIdx.x == 0) {
+            const volatile unsigned char* v = rx;
+            unsigned char h[36];
+            for (int i = 0; i < 36; i++) h[i] = 0;
+            h[0] = v[0]; h[1] = v[1];                 // request id
+            put_be16(h + 4, 1u);                      // total datagrams
+            h[8] = 0x81;                              // magic: response
+            h[9] = 0x00;                              // opcode: GET
+            h[12] = hit ? 4 : 0;                      // extras length (flags)
+            put_be16(h + 14, hit ? 0u : 1u);          // status: 0 ok, 1 key not found
+            put_be32(h + 16, hit ? 4u + vlen : 9u);   // total body
+            for (int i = 0; i < 4; i++) h[20 + i] = v[20 + i];   // opaque
+            for (int i = 0; i < 36; i++) tx[i] = h[i];            // flags (4 B zero) follow the header
+            if (!hit) {
+                const char nf[9] = {'N', 'o', 't', ' ', 'f', 'o', 'u', 'n', 'd'};
+                for (int i = 0; i < 9; i++) tx[32 + i] = (unsigned char)nf[i];
+            }
+            s_len = hit ? 36u + vlen : 41u;
+            atomicAdd(&a.stats[0], 1ull);
+            if (!hit) atomicAdd(&a.stats[1], 1ull);
+        }
+        if (hit) {
+            const unsigned char* src = a.heap + e->voff;
+            for (unsigned i = threadIdx.x; i < vlen; i += blockDim.x) tx[36 + i] = src[i];
+        }
+        // consumer call: Bar1 (the reply is complete) is kept under relaxed ordering
+        gsys_sendto(a.ctx, a.fd, tx, s_len, 0, from, *(volatile unsigned*)fromlen, gf);
+        __syncthreads();
+    }
+}
+
 }  // namespace
 
 extern "C" {
+
+int gsys_mc_build(const uint8_t* keys, const uint32_t* key_off, const uint8_t* key_len, const uint8_t* vals,
+                  const uint64_t* val_off, const uint32_t* val_len, uint32_t n, uint32_t nbuckets, uint32_t bucket_cap,
+                  void* d_entries, uint32_t* d_bucket_n, uint8_t* d_heap, uint64_t heap_bytes) {
+    if (!n || !nbuckets || !bucket_cap || !keys || !key_off || !key_len || !vals || !val_off || !val_len ||
+        !d_entries || !d_bucket_n || !d_heap)
+        return -EINVAL;
+    std::vector<McEntry> ent((size_t)nbuckets * bucket_cap);
+    memset(ent.data(), 0, ent.size() * sizeof(McEntry));
+    std::vector<uint32_t> cnt(nbuckets, 0);
+    uint64_t hend = 0;
+    for (uint32_t i = 0; i < n; i++) {
+        const unsigned kl = key_len[i];
+        if (kl < 1 || kl > MC_MAXKEY || val_len[i] > MC_MAXVAL) return -EINVAL;
+        const unsigned b = mc_hash(keys + key_off[i], kl) % nbuckets;
+        if (cnt[b] >= bucket_cap) return -E2BIG;
+        McEntry& e = ent[(size_t)b * bucket_cap + cnt[b]++];
+        unsigned char kb[32] = {0};
+        memcpy(kb, keys + key_off[i], kl);
+        memcpy(&e.k0, kb, 16);
+        memcpy(&e.k1, kb + 16, 16);
+        e.klen = kl;
+        e.vlen = val_len[i];
+        e.voff = val_off[i];
+        if (val_off[i] + val_len[i] > hend) hend = val_off[i] + val_len[i];
+    }
+    if (hend > heap_bytes) return -EINVAL;
+    if (cudaMemcpy(d_entries, ent.data(), ent.size() * sizeof(McEntry), cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(d_bucket_n, cnt.data(), nbuckets * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(d_heap, vals, hend, cudaMemcpyHostToDevice) != cudaSuccess)
+        return -EIO;
+    return 0;
+}
+
+uint64_t gsys_mc_entries_bytes(uint32_t nbuckets, uint32_t bucket_cap) {
+    return (uint64_t)nbuckets * bucket_cap * sizeof(McEntry);
+}
+
+int gsys_mc_serve(int32_t fd, const void* d_entries, const uint32_t* d_bucket_n, const uint8_t* d_heap,
+                  uint32_t nbuckets, uint32_t bucket_cap, uint32_t nwg, uint8_t* io, const uint32_t* stop,
+                  uint64_t* d_stats, uint32_t gflags, void* stream) {
+    gsys_dev_ctx* ctx = gsys_internal_ctx_d();
+    if (!ctx) return -ENODEV;
+    if (!d_entries || !d_bucket_n || !d_heap || !nbuckets || !bucket_cap || !nwg || !io || !stop || !d_stats)
+        return -EINVAL;
+    if ((gflags & GSYS_GRAN_MASK) != GSYS_WG || (gflags & GSYS_NONBLOCKING)) return -EINVAL;
+    McArgs a;
+    memset(&a, 0, sizeof a);
+    a.ctx = ctx;
+    a.entries = reinterpret_cast<const McEntry*>(d_entries);
+    a.bucket_n = d_bucket_n;
+    a.heap = d_heap;
+    a.io = io;
+    a.stop = stop;
+    a.stats = reinterpret_cast<unsigned long long*>(d_stats);
+    a.nbuckets = nbuckets;
+    a.cap = bucket_cap;
+    a.gflags = gflags;
+    a.fd = fd;
+    void* args[] = {&a};
+    return gsys_launch((const void*)mc_kernel, nwg, 1, 1, 256, 1, 1, args, 0, stream);
+}
+
+
 
 int gsys_amr_release(uint64_t host_mesh, uint32_t nblocks, uint64_t block_bytes, const uint8_t* d_levels,
                      uint32_t iters, int32_t statm_fd, uint64_t watermark_bytes, uint64_t page_bytes, float* d_field,

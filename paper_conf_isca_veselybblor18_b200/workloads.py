@@ -202,3 +202,44 @@ def signal_search_run(data_dev, nblocks: int, block_bytes: int, key: bytes, sig:
             time.sleep(0.0002)
     rc = G.gsys_wait(stream)
     return counts.numpy().copy(), got, ts, rc
+
+
+# ---------------------------------------------------------------------------- config 4 (next row)
+def mc_serve_run(keys, vals, packets, nwg: int = 8, nbuckets: int = 64, bucket_cap: int = 1024,
+                 gflags: int = G.WG | G.BLOCKING | G.RELAXED, client_threads: int = 4, window: int = 8,
+                 stream=None):
+    """Config 4: memcached-style GET server on the GPU (recvfrom/sendto issued by work-groups)
+    driven by the UDP load generator.  Returns (responses, latencies ns, client seconds, stats)."""
+    import ctypes
+    import numpy as np
+
+    from inputs import mc as MC
+    ensure_init()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    L = G.lib()
+    kb, ko, kl, vb, vo, vl = MC.pack(keys, vals)
+    ent = torch.zeros(int(L.gsys_mc_entries_bytes(nbuckets, bucket_cap)), dtype=torch.uint8, device=dev)
+    bn = torch.zeros(nbuckets, dtype=torch.int32, device=dev)
+    heap = torch.zeros(max(vb.size, 1), dtype=torch.uint8, device=dev)
+    rc = L.gsys_mc_build(kb.ctypes.data, ko.ctypes.data, kl.ctypes.data, vb.ctypes.data, vo.ctypes.data,
+                         vl.ctypes.data, len(keys), nbuckets, bucket_cap, ent.data_ptr(), bn.data_ptr(),
+                         heap.data_ptr(), heap.numel())
+    if rc:
+        raise G.GsysError(-rc, "gsys_mc_build")
+    io = torch.zeros(nwg * 8192, dtype=torch.uint8).pin_memory()
+    stop = torch.zeros(1, dtype=torch.int32).pin_memory()
+    stats = torch.zeros(4, dtype=torch.int64, device=dev)
+    sock = MC.udp_server_socket()
+    port = sock.getsockname()[1]
+    s = torch.cuda.Stream(device=dev) if stream is None else stream
+    try:
+        rc = L.gsys_mc_serve(sock.fileno(), ent.data_ptr(), bn.data_ptr(), heap.data_ptr(), nbuckets, bucket_cap, nwg,
+                             io.data_ptr(), stop.data_ptr(), stats.data_ptr(), gflags, s.cuda_stream)
+        if rc:
+            raise G.GsysError(-rc, "gsys_mc_serve")
+        resp, lat, secs = MC.run_client(port, packets, nthreads=client_threads, window=window)
+    finally:
+        stop[0] = 1
+        G.gsys_wait(s)
+        sock.close()
+    return resp, lat, secs, stats.cpu().tolist()

@@ -59,3 +59,18 @@ def test_signal_search_counts_and_ids(gflags):
     want = [oracle.count_key(data[b * bs:(b + 1) * bs], key) for b in range(nb)]
     assert counts.tolist() == want
     assert sum(want) > 0
+
+
+# ---------------------------------------------------------------------------- config 4: memcached
+@pytest.mark.parametrize("gflags", [G.WG | G.BLOCKING | G.RELAXED, G.WG | G.BLOCKING | G.STRONG])
+def test_memcached_gpu_server_matches_definition(gflags):
+    from inputs import mc as MC
+    from oracle import mc as OM
+    keys, vals = MC.dataset(4000, vlen=(64, 4096))
+    reqs = MC.requests(keys, 5000)
+    pkts = [MC.encode_get(i, k) for i, k in enumerate(reqs)]
+    resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=8, nbuckets=16, bucket_cap=1024, gflags=gflags)
+    table = dict(zip(keys, vals))
+    bad = [i for i, (p, r) in enumerate(zip(pkts, resp)) if r != OM.expected_response(p, table)]
+    assert not bad, (len(bad), bad[:5])
+    assert stats[0] == len(pkts) and stats[1] == sum(1 for k in reqs if k not in table)
