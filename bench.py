@@ -546,12 +546,14 @@ def run_memcached(a):
         reqs = MC.requests(keys, 20000)
         pkts = [MC.encode_get(i, k) for i, k in enumerate(reqs)]
         table = dict(zip(keys, vals))
-        for nwg in (4, 8, 12):
+        for nwg, send in ((4, "blocking"), (12, "blocking"), (12, "nonblocking")):
+            sg = G.WG | G.RELAXED | (G.NONBLOCKING if send == "nonblocking" else G.BLOCKING)
             resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=nwg, nbuckets=nbuckets,
-                                                    bucket_cap=per_bucket * 2, client_threads=4, window=8)
+                                                    bucket_cap=per_bucket * 2, client_threads=4, window=8,
+                                                    send_gflags=sg)
             ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
             lat_us = np.array(lat, dtype=np.float64) / 1e3
-            out["cases"].append({"server": "gpu", "elements_per_bucket": per_bucket, "work_groups": nwg,
+            out["cases"].append({"server": "gpu", "sendto": send, "elements_per_bucket": per_bucket, "work_groups": nwg,
                                  "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
                                  "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
                                  "requests": len(pkts)})

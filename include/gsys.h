@@ -80,6 +80,7 @@ enum gsys_state {
 #define GSYS_F_PRODUCER  0x100u   /* call class: producer (read-like), P20.24-29            */
 #define GSYS_F_INLINE    0x200u   /* small result goes to the slot's inline payload line    */
 #define GSYS_F_INLINE_IN 0x400u   /* small input (siginfo, sockaddr) is in the inline line   */
+#define GSYS_F_NOHINT    0x800u   /* unpredictable latency (network): poll without the learned sleep */
 
 /* Syscall numbers served (Linux x86-64). */
 #define GSYS_NR_PREAD64        17
@@ -311,8 +312,9 @@ int gsys_signal_search(const uint8_t* d_data, uint32_t nblocks, uint64_t block_b
  * d_heap (DEVICE, heap_bytes >= max(val_off+val_len)).  -E2BIG when a bucket overflows.
  * gsys_mc_serve launches nwg work-groups that loop recvfrom(fd) -> lookup -> sendto with the
  * memcached binary protocol over UDP (8-byte frame header; GET hit: status 0, 4-byte flags +
- * value; miss: status 1 + "Not found"), both calls WG-granularity, blocking, `gflags` ordering
- * (paper: weak).  io: pinned host-mapped [nwg][8192] request/reply buffers; stop: host-mapped
+ * value; miss: status 1 + "Not found"), both calls WG-granularity: recvfrom with `gflags`
+ * (blocking; paper: weak ordering), sendto with `send_gflags` (paper: blocking + weak;
+ * GSYS_NONBLOCKING lets the work-group take the next request while the reply is sent).  io: pinned host-mapped [nwg][8192] request/reply buffers; stop: host-mapped
  * u32 the host sets to 1 to end the server (checked whenever recvfrom times out -- set
  * SO_RCVTIMEO on fd); d_stats (DEVICE u64[4]): served, misses, malformed, receive timeouts.
  * Keep nwg below the service thread count: each waiting recvfrom occupies a service thread. */
@@ -323,7 +325,7 @@ int gsys_mc_build(const uint8_t* keys, const uint32_t* key_off, const uint8_t* k
                   uint64_t heap_bytes);
 int gsys_mc_serve(int32_t fd, const void* d_entries, const uint32_t* d_bucket_n, const uint8_t* d_heap,
                   uint32_t nbuckets, uint32_t bucket_cap, uint32_t nwg, uint8_t* io, const uint32_t* stop,
-                  uint64_t* d_stats, uint32_t gflags, void* stream);
+                  uint64_t* d_stats, uint32_t gflags, uint32_t send_gflags, void* stream);
 
 /* Host-side consumer for GPU-issued signals: installs an async-signal-safe SA_SIGINFO handler
  * for `sig` (SIGRTMIN..SIGRTMAX) that appends si_value.sival_int to a ring of `capacity` entries

@@ -201,7 +201,8 @@ __device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
  * the device-memory word (L2-resident; written by a stream memory operation after the DMA) or,
  * for GSYS_HOSTBUF / inline calls, the host-mapped word the service stores directly (each poll
  * is one PCIe read, so the backoff starts longer and caps at poll_ns_max). */
-__device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq, bool host) {
+__device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq, bool host,
+                                               bool nohint = false) {
     unsigned long long v;
     if (!host) {
         const unsigned long long* m = c->mirror + s;
@@ -219,7 +220,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         // more than 2 means it woke too early (grow by the extra polling time / 2), so the
         // sleep converges just below the service latency without feeding on its own length.
         const unsigned long long* m = c->hdone + s;
-        const unsigned hint = c->lat_hint[s];
+        const unsigned hint = nohint ? 0u : c->lat_hint[s];
         unsigned left = hint;
         while (left > 0) {
             const unsigned d = left > 100000u ? 100000u : left;
@@ -233,10 +234,12 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(c->poll_ns_host);
         }
-        unsigned nh = hint;
-        if (polls <= 1) nh = hint - (hint >> 2);
-        else if (polls > 2) nh = hint + (polls - 2) * (c->poll_ns_host >> 1);
-        c->lat_hint[s] = nh > 200000u ? 200000u : nh;
+        if (!nohint) {
+            unsigned nh = hint;
+            if (polls <= 1) nh = hint - (hint >> 2);
+            else if (polls > 2) nh = hint + (polls - 2) * (c->poll_ns_host >> 1);
+            c->lat_hint[s] = nh > 200000u ? 200000u : nh;
+        }
     }
     fence_acq_rel_sys();   /* acquire: the payload is visible before the completion word */
     return (long long)(int)(unsigned)(v & 0xffffffffull);
@@ -272,7 +275,7 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         st_release_gpu(&c->claim[s], 0u);
         return 0;
     }
-    long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) != 0u);
+    long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) != 0u, (flags & GSYS_F_NOHINT) != 0u);
     if (io.out != nullptr && r >= 0) {
         const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
         uint4* dst = reinterpret_cast<uint4*>(io.out);
@@ -441,14 +444,14 @@ __device__ __forceinline__ long long gsys_sendto(const gsys_dev_ctx* c, int fd, 
                                                  const void* to, unsigned tolen, unsigned gflags) {
     unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
                                (unsigned long long)(long long)flags, (unsigned long long)to, (unsigned long long)tolen};
-    return gsys::invoke(c, GSYS_NR_SENDTO, gflags, false, a);
+    return gsys::invoke(c, GSYS_NR_SENDTO, gflags | GSYS_F_NOHINT, false, a);
 }
 __device__ __forceinline__ long long gsys_recvfrom(const gsys_dev_ctx* c, int fd, void* buf, size_t n, int flags,
                                                    void* from, unsigned* fromlen, unsigned gflags) {
     unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
                                (unsigned long long)(long long)flags, (unsigned long long)from,
                                (unsigned long long)fromlen};
-    return gsys::invoke(c, GSYS_NR_RECVFROM, gflags, true, a);
+    return gsys::invoke(c, GSYS_NR_RECVFROM, gflags | GSYS_F_NOHINT, true, a);
 }
 /* rt_sigqueueinfo: the 128 B siginfo travels in the slot's inline line (copied by the caller before
  * publishing), so `info` may live anywhere the caller can read -- registers/local memory included --

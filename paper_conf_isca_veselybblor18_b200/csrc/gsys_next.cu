@@ -173,8 +173,8 @@ struct McArgs {
     unsigned char* io;              // host-mapped [nwg][MC_IO_BYTES]
     const volatile unsigned* stop;  // host-mapped stop flag
     unsigned long long* stats;      // device [4]: served, misses, malformed, recv timeouts
-    unsigned nbuckets, cap, gflags;
-    int fd;
+    unsigned nbuckets, cap, gflags, send_gflags;
+    int fd, pad_;
 };
 
 __device__ __forceinline__ unsigned be16(const unsigned char* p) { return ((unsigned)p[0] << 8) | p[1]; }
@@ -187,7 +187,8 @@ __device__ __forceinline__ void put_be32(unsigned char* p, unsigned v) {
 }
 
 __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
-    __shared__ unsigned s_found, s_len, s_keylen, s_bucket, s_ok, s_done;
+    __shared__ unsigned s_found, s_len, s_keylen, s_bucket, s_ok, s_done, s_fromlen;
+    __shared__ __align__(16) unsigned char s_rx[80];      // frame + header + extras + key (<= 32 + 16 + 32)
     __shared__ __align__(16) unsigned char s_key[MC_MAXKEY];
     unsigned char* io = a.io + (size_t)blockIdx.x * MC_IO_BYTES;
     unsigned char* rx = io + MC_RX;
@@ -207,13 +208,16 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
             if (s_done) break;
             continue;
         }
+        // the first 80 bytes of the datagram in one coalesced PCIe read (5 lanes x 16 B), then
+        // parse from shared memory -- byte-wise volatile reads would cost one round trip each
+        if (threadIdx.x < 5) reinterpret_cast<uint4*>(s_rx)[threadIdx.x] = reinterpret_cast<const uint4*>(rx)[threadIdx.x];
+        if (threadIdx.x == 5) s_fromlen = *fromlen;
+        __syncthreads();
         if (threadIdx.x == 0) {
-            const volatile unsigned char* v = rx;
+            const unsigned char* v = s_rx;
             unsigned ok = r >= 32 && v[8] == 0x80 && v[9] == 0x00;
-            unsigned char hdr[32];
-            for (int i = 0; i < 32; i++) hdr[i] = v[i];
-            const unsigned klen = be16(hdr + 10), ext = hdr[12];
-            ok = ok && klen >= 1 && klen <= MC_MAXKEY && (long long)(32 + ext + klen) <= r;
+            const unsigned klen = be16(v + 10), ext = v[12];
+            ok = ok && klen >= 1 && klen <= MC_MAXKEY && ext <= 16 && (long long)(32 + ext + klen) <= r;
             s_keylen = ok ? klen : 0u;
             for (unsigned i = 0; i < MC_MAXKEY; i++) s_key[i] = (ok && i < klen) ? v[32 + ext + i] : 0u;
             s_bucket = ok ? mc_hash(s_key, klen) % a.nbuckets : 0u;
@@ -239,9 +243,9 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
         const unsigned vlen = hit ? e->vlen : 0u;
         // reply: UDP frame header + binary response header (+ flags + value | "Not found")
         if (threadIdx.x == 0) {
-            const volatile unsigned char* v = rx;
-            unsigned char h[36];
-            for (int i = 0; i < 36; i++) h[i] = 0;
+            const unsigned char* v = s_rx;
+            __align__(16) unsigned char h[48];
+            for (int i = 0; i < 48; i++) h[i] = 0;
             h[0] = v[0]; h[1] = v[1];                 // request id
             put_be16(h + 4, 1u);                      // total datagrams
             h[8] = 0x81;                              // magic: response
@@ -250,11 +254,13 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
             put_be16(h + 14, hit ? 0u : 1u);          // status: 0 ok, 1 key not found
             put_be32(h + 16, hit ? 4u + vlen : 9u);   // total body
             for (int i = 0; i < 4; i++) h[20 + i] = v[20 + i];   // opaque
-            for (int i = 0; i < 36; i++) tx[i] = h[i];            // flags (4 B zero) follow the header
             if (!hit) {
                 const char nf[9] = {'N', 'o', 't', ' ', 'f', 'o', 'u', 'n', 'd'};
-                for (int i = 0; i < 9; i++) tx[32 + i] = (unsigned char)nf[i];
+                for (int i = 0; i < 9; i++) h[32 + i] = (unsigned char)nf[i];
             }
+            for (int i = 0; i < 2; i++) reinterpret_cast<uint4*>(tx)[i] = reinterpret_cast<const uint4*>(h)[i];
+            if (!hit) reinterpret_cast<uint4*>(tx)[2] = reinterpret_cast<const uint4*>(h)[2];
+            else *reinterpret_cast<unsigned*>(tx + 32) = 0u;     // flags
             s_len = hit ? 36u + vlen : 41u;
             atomicAdd(&a.stats[0], 1ull);
             if (!hit) atomicAdd(&a.stats[1], 1ull);
@@ -264,7 +270,7 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
             for (unsigned i = threadIdx.x; i < vlen; i += blockDim.x) tx[36 + i] = src[i];
         }
         // consumer call: Bar1 (the reply is complete) is kept under relaxed ordering
-        gsys_sendto(a.ctx, a.fd, tx, s_len, 0, from, *(volatile unsigned*)fromlen, gf);
+        gsys_sendto(a.ctx, a.fd, tx, s_len, 0, from, s_fromlen, a.send_gflags | GSYS_HOSTBUF);
         __syncthreads();
     }
 }
@@ -312,12 +318,13 @@ uint64_t gsys_mc_entries_bytes(uint32_t nbuckets, uint32_t bucket_cap) {
 
 int gsys_mc_serve(int32_t fd, const void* d_entries, const uint32_t* d_bucket_n, const uint8_t* d_heap,
                   uint32_t nbuckets, uint32_t bucket_cap, uint32_t nwg, uint8_t* io, const uint32_t* stop,
-                  uint64_t* d_stats, uint32_t gflags, void* stream) {
+                  uint64_t* d_stats, uint32_t gflags, uint32_t send_gflags, void* stream) {
     gsys_dev_ctx* ctx = gsys_internal_ctx_d();
     if (!ctx) return -ENODEV;
     if (!d_entries || !d_bucket_n || !d_heap || !nbuckets || !bucket_cap || !nwg || !io || !stop || !d_stats)
         return -EINVAL;
     if ((gflags & GSYS_GRAN_MASK) != GSYS_WG || (gflags & GSYS_NONBLOCKING)) return -EINVAL;
+    if ((send_gflags & GSYS_GRAN_MASK) != GSYS_WG) return -EINVAL;
     McArgs a;
     memset(&a, 0, sizeof a);
     a.ctx = ctx;
@@ -330,6 +337,7 @@ int gsys_mc_serve(int32_t fd, const void* d_entries, const uint32_t* d_bucket_n,
     a.nbuckets = nbuckets;
     a.cap = bucket_cap;
     a.gflags = gflags;
+    a.send_gflags = send_gflags;
     a.fd = fd;
     void* args[] = {&a};
     return gsys_launch((const void*)mc_kernel, nwg, 1, 1, 256, 1, 1, args, 0, stream);

@@ -81,7 +81,7 @@ SIGNATURES = {
     "gsys_sigsink_install": (ctypes.c_int, [_I32, _U32]),
     "gsys_mc_entries_bytes": (_U64, [_U32, _U32]),
     "gsys_mc_build": (ctypes.c_int, [_P, _P, _P, _P, _P, _P, _U32, _U32, _U32, _P, _P, _P, _U64]),
-    "gsys_mc_serve": (ctypes.c_int, [_I32, _P, _P, _P, _U32, _U32, _U32, _P, _P, _P, _U32, _P]),
+    "gsys_mc_serve": (ctypes.c_int, [_I32, _P, _P, _P, _U32, _U32, _U32, _P, _P, _P, _U32, _U32, _P]),
     "gsys_sigsink_read": (ctypes.c_int, [_P, _P, _U32]),
     "gsys_read_profile": (ctypes.c_int, [_P, ctypes.c_int]),
     "gsys_wordcount": (ctypes.c_int, [_P, _P, _U32, _U32, ctypes.c_char_p, _P, _U32, ctypes.c_char_p, _P, _U32,

@@ -207,7 +207,7 @@ def signal_search_run(data_dev, nblocks: int, block_bytes: int, key: bytes, sig:
 # ---------------------------------------------------------------------------- config 4 (next row)
 def mc_serve_run(keys, vals, packets, nwg: int = 8, nbuckets: int = 64, bucket_cap: int = 1024,
                  gflags: int = G.WG | G.BLOCKING | G.RELAXED, client_threads: int = 4, window: int = 8,
-                 stream=None):
+                 stream=None, send_gflags: int | None = None):
     """Config 4: memcached-style GET server on the GPU (recvfrom/sendto issued by work-groups)
     driven by the UDP load generator.  Returns (responses, latencies ns, client seconds, stats)."""
     import ctypes
@@ -234,7 +234,8 @@ def mc_serve_run(keys, vals, packets, nwg: int = 8, nbuckets: int = 64, bucket_c
     s = torch.cuda.Stream(device=dev) if stream is None else stream
     try:
         rc = L.gsys_mc_serve(sock.fileno(), ent.data_ptr(), bn.data_ptr(), heap.data_ptr(), nbuckets, bucket_cap, nwg,
-                             io.data_ptr(), stop.data_ptr(), stats.data_ptr(), gflags, s.cuda_stream)
+                             io.data_ptr(), stop.data_ptr(), stats.data_ptr(), gflags,
+                             gflags if send_gflags is None else send_gflags, s.cuda_stream)
         if rc:
             raise G.GsysError(-rc, "gsys_mc_serve")
         resp, lat, secs = MC.run_client(port, packets, nthreads=client_threads, window=window)

@@ -62,14 +62,16 @@ def test_signal_search_counts_and_ids(gflags):
 
 
 # ---------------------------------------------------------------------------- config 4: memcached
-@pytest.mark.parametrize("gflags", [G.WG | G.BLOCKING | G.RELAXED, G.WG | G.BLOCKING | G.STRONG])
-def test_memcached_gpu_server_matches_definition(gflags):
+@pytest.mark.parametrize("gflags,send", [(G.WG | G.BLOCKING | G.RELAXED, None), (G.WG | G.BLOCKING | G.STRONG, None),
+                                         (G.WG | G.BLOCKING | G.RELAXED, G.WG | G.NONBLOCKING | G.RELAXED)])
+def test_memcached_gpu_server_matches_definition(gflags, send):
     from inputs import mc as MC
     from oracle import mc as OM
     keys, vals = MC.dataset(4000, vlen=(64, 4096))
     reqs = MC.requests(keys, 5000)
     pkts = [MC.encode_get(i, k) for i, k in enumerate(reqs)]
-    resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=8, nbuckets=16, bucket_cap=1024, gflags=gflags)
+    resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=8, nbuckets=16, bucket_cap=1024, gflags=gflags,
+                                            send_gflags=send)
     table = dict(zip(keys, vals))
     bad = [i for i, (p, r) in enumerate(zip(pkts, resp)) if r != OM.expected_response(p, table)]
     assert not bad, (len(bad), bad[:5])
