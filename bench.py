@@ -49,7 +49,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip scan roofline / syscall-rate extras")
     ap.add_argument("--root", default=None, help="corpus directory (default /dev/shm/gsys_corpus)")
-    ap.add_argument("--mode", default="wordcount", choices=["wordcount", "syscalls", "memcached", "mm"],
+    ap.add_argument("--mode", default="wordcount", choices=["wordcount", "syscalls", "memcached", "mm", "fig8", "fig9"],
                     help="syscalls: config-2 sweep; memcached: config 4; mm: config 5 (one JSON line each)")
     return ap.parse_args()
 
@@ -184,6 +184,10 @@ def main():
         return run_memcached(a)
     if a.mode == "mm":
         return run_mm(a)
+    if a.mode == "fig8":
+        return run_fig8(a)
+    if a.mode == "fig9":
+        return run_fig9(a)
     import torch
     import torch.distributed as dist
 
@@ -636,6 +640,79 @@ def run_mm(a):
                             "ids_exact_once": sorted(got) == list(range(nb)), "digests": len(digests),
                             "overlapped_s": overlapped, "search_then_hash_s": serial,
                             "speedup": serial / overlapped if overlapped > 0 else None}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def run_fig8(a):
+    """Row f3 (sec. VII, Fig. 8): blocking x ordering of a work-group pwrite after N
+    permutation iterations on 8 KB blocks, 1024 work-items per work-group.  Reported: time per
+    permutation iteration (lower is better) for strong/weak x block/non-block."""
+    import numpy as np
+    import torch
+
+    import inputs
+    from oracle import plan
+    from paper_conf_isca_veselybblor18_b200 import gsys as G
+    from paper_conf_isca_veselybblor18_b200 import workloads as W
+
+    torch.cuda.set_device(0)
+    W.ensure_init()
+    nb, bs = 8192, 8192
+    data, perm = inputs.perm_inputs(nb, bs)
+    path = os.path.join(a.root or "/dev/shm", "gsys_fig8.bin")
+    combos = {"strong-block": G.WG | G.BLOCKING | G.STRONG, "strong-nonblock": G.WG | G.NONBLOCKING | G.STRONG,
+              "weak-block": G.WG | G.BLOCKING | G.RELAXED, "weak-nonblock": G.WG | G.NONBLOCKING | G.RELAXED}
+    out = {"mode": "fig8", "blocks": nb, "block_bytes": bs, "work_items_per_wg": 1024, "grid": 296, "rows": []}
+    for iters in (1, 2, 4, 8, 16, 32):
+        row = {"iters": iters}
+        for name, fl in combos.items():
+            W.perm_pwrite_run(data[:bs * 64], perm, iters, path, fl, bs, grid=64)
+            secs, rc = W.perm_pwrite_run(data, perm, iters, path, fl, bs, grid=296)
+            row[name + "_us_per_perm"] = secs * 1e6 / iters
+            row[name + "_ok"] = rc == 0
+        got = np.fromfile(path, dtype=np.uint8)
+        row["file_equals_cpu_permutation"] = bool(np.array_equal(got, plan.permuted_blocks(data, perm, iters, bs)))
+        out["rows"].append(row)
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def run_fig9(a):
+    """Row f4 (sec. VII, Fig. 9): host memory-copy throughput while GPU threads poll
+    N distinct 64 B lines of pinned host memory (PCIe reads) or of device memory (L2)."""
+    import threading
+
+    import numpy as np
+    import torch
+
+    from paper_conf_isca_veselybblor18_b200 import gsys as G
+
+    torch.cuda.set_device(0)
+    L = G.lib()
+    src = np.ones(256 << 20, dtype=np.uint8)
+    dst = np.empty_like(src)
+
+    def host_bw(seconds):
+        n, t0 = 0, time.perf_counter()
+        while time.perf_counter() - t0 < seconds:
+            np.copyto(dst, src)
+            n += 1
+        return n * src.nbytes * 2 / (time.perf_counter() - t0) / 1e9     # read + write bytes
+    out = {"mode": "fig9", "baseline_host_copy_GBps": host_bw(1.0), "rows": []}
+    sink = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for where in ("host", "device"):
+        for nlines in (1, 64, 1024, 4096, 16384, 65536, 262144):
+            lines = (torch.zeros(nlines * 8, dtype=torch.int64).pin_memory() if where == "host"
+                     else torch.zeros(nlines * 8, dtype=torch.int64, device="cuda"))
+            sink.zero_()
+            ns = int(1.5e9)
+            L.gsys_poll_storm(lines.data_ptr(), nlines, max(nlines, 148 * 256), ns, sink.data_ptr(), None)
+            time.sleep(0.2)
+            bw = host_bw(1.0)
+            torch.cuda.synchronize()
+            out["rows"].append({"polled": where, "lines": nlines, "gpu_threads": max(nlines, 148 * 256),
+                                "host_copy_GBps": bw, "gpu_polls_per_s": int(sink.item()) / 1.5})
     print(json.dumps(out), flush=True)
     return 0
 

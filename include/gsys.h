@@ -327,6 +327,24 @@ int gsys_mc_serve(int32_t fd, const void* d_entries, const uint32_t* d_bucket_n,
                   uint32_t nbuckets, uint32_t bucket_cap, uint32_t nwg, uint8_t* io, const uint32_t* stop,
                   uint64_t* d_stats, uint32_t gflags, uint32_t send_gflags, void* stream);
 
+/* Row f3 -- Fig. 8 study (sec. VII): `grid` work-groups of 1024 work-items each take
+ * blocks of d_in ([nblocks][block_bytes], DEVICE, block_bytes % 16 == 0, <= 16384), apply the
+ * permutation out[i] = in[d_perm[i]] `iters` times in shared memory, store the result in
+ * staging[blk] (pinned host-mapped [nblocks][block_bytes]; one line per block so a non-blocking
+ * write never races the next block) and pwrite it to fd at file_off + blk*block_bytes with
+ * `gflags` (GSYS_WG + blocking/non-blocking + strong/relaxed).  grid 0 = one work-group per block.
+ * Asynchronous; gsys_wait() drains the writes. */
+int gsys_perm_pwrite(const uint8_t* d_in, const uint16_t* d_perm, uint32_t nblocks, uint32_t block_bytes,
+                     uint32_t iters, uint8_t* staging, int32_t fd, uint64_t file_off, uint32_t gflags,
+                     uint32_t grid, void* stream);
+
+/* Row f4 -- Fig. 9 study (sec. VII, polling contention): nthreads GPU threads poll
+ * nlines distinct 64 B lines of `lines` (pinned host-mapped or DEVICE memory, nlines*64 bytes) for
+ * `ns` nanoseconds with system-scope loads; the total poll count is added to *d_sink (DEVICE
+ * u64).  Used to measure how completion polling degrades host memory throughput. */
+int gsys_poll_storm(const void* lines, uint32_t nlines, uint32_t nthreads, uint64_t ns, uint64_t* d_sink,
+                    void* stream);
+
 /* Host-side consumer for GPU-issued signals: installs an async-signal-safe SA_SIGINFO handler
  * for `sig` (SIGRTMIN..SIGRTMAX) that appends si_value.sival_int to a ring of `capacity` entries
  * (any thread of the process may take the signal); gsys_sigsink_read drains up to cap values

@@ -203,3 +203,15 @@ def signal_blocks(nblocks: int, block_bytes: int, seed: int = SEED_SIGNAL):
     """Data array for signal-search (config 5b, sec. VIII-B): synthetic text blocks."""
     buf, _, _ = gen_bytes(seed, 0, nblocks * block_bytes)
     return buf
+
+
+SEED_PERM = 9
+
+
+def perm_inputs(nblocks: int, block_bytes: int = 8192, seed: int = SEED_PERM):
+    """Fig. 8 inputs (sec. VII: "The input data array is preloaded with random values
+    and divided into 8KB blocks"): random bytes and a fixed random permutation of block positions."""
+    rng = np.random.default_rng(seed)
+    data = rng.integers(0, 256, size=nblocks * block_bytes, dtype=np.uint8)
+    perm = rng.permutation(block_bytes).astype(np.uint16)
+    return data, perm

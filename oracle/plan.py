@@ -67,3 +67,14 @@ def amr_released(levels, rss_ok=None):
             if out[b] == 0 and levels[t][b] == 0:
                 out[b] = t + 1
     return out
+
+
+def permuted_blocks(data, perm, iters: int, block_bytes: int):
+    """Fig. 8: each block permuted `iters` times, out[i] = in[perm[i]] -- the bytes the
+    GPU work-groups must have written to the file (numpy fancy indexing, one step at a time)."""
+    import numpy as np
+    blocks = np.asarray(data).reshape(-1, block_bytes)
+    out = blocks.copy()
+    for _ in range(iters):
+        out = out[:, perm]
+    return out.reshape(-1)

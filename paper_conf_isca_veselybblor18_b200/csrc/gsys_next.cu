@@ -275,9 +275,110 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
     }
 }
 
+// ------------------------------------------------------------------ row f3: Fig. 8 permutation + pwrite
+// PAPER.md:26 sec. VII "Blocking and ordering strategies": work-groups of 1024 work-items
+// independently permute 8 KB blocks (a DES-like permutation step, repeated `iters` times) and
+// write each result to a file with a work-group pwrite; blocking x ordering is the study.
+struct PermArgs {
+    const gsys_dev_ctx* ctx;
+    const unsigned char* in;          // DEVICE [nblocks][bs]
+    const unsigned short* perm;       // DEVICE [bs] permutation: out[i] = in[perm[i]]
+    unsigned char* staging;           // host-mapped [nblocks][bs] (one line per block: no reuse hazard)
+    unsigned long long file_off;
+    unsigned nblocks, bs, iters, gflags;
+    int fd, pad_;
+};
+
+__global__ void __launch_bounds__(1024) perm_kernel(PermArgs a) {
+    extern __shared__ __align__(16) unsigned char psm[];   // [bs] x 2 + perm [bs] u16
+    unsigned char* b0 = psm;
+    unsigned char* b1 = psm + a.bs;
+    unsigned short* pm = reinterpret_cast<unsigned short*>(psm + 2 * a.bs);
+    for (unsigned i = threadIdx.x; i < a.bs; i += blockDim.x) pm[i] = a.perm[i];
+    for (unsigned blk = blockIdx.x; blk < a.nblocks; blk += gridDim.x) {
+        const unsigned char* src = a.in + (size_t)blk * a.bs;
+        for (unsigned i = threadIdx.x; i < a.bs / 16u; i += blockDim.x)
+            reinterpret_cast<uint4*>(b0)[i] = reinterpret_cast<const uint4*>(src)[i];
+        __syncthreads();
+        unsigned char* cur = b0;
+        unsigned char* nxt = b1;
+        for (unsigned it = 0; it < a.iters; it++) {
+            for (unsigned i = threadIdx.x; i < a.bs; i += blockDim.x) nxt[i] = cur[pm[i]];
+            __syncthreads();
+            unsigned char* t = cur; cur = nxt; nxt = t;
+        }
+        unsigned char* out = a.staging + (size_t)blk * a.bs;
+        for (unsigned i = threadIdx.x; i < a.bs / 16u; i += blockDim.x)
+            reinterpret_cast<uint4*>(out)[i] = reinterpret_cast<const uint4*>(cur)[i];
+        // consumer call: Bar1 always (the block is complete); Bar2 only when strong
+        gsys_pwrite(a.ctx, a.fd, out, a.bs, (long long)(a.file_off + (unsigned long long)blk * a.bs),
+                    a.gflags | GSYS_HOSTBUF);
+        __syncthreads();   // both shared buffers are reused by the next block
+    }
+}
+
+// ------------------------------------------------------------------ row f4: Fig. 9 polling contention
+// PAPER.md:28 sec. VII "Polling/halt-resume and memory contention": GPU threads poll `nlines`
+// distinct 64 B lines (as completion polls would) for `ns` nanoseconds while the host measures its
+// own memory throughput.  host = 1 polls pinned host-mapped lines (each poll is a PCIe read, the
+// B200 analogue of spilling past the APU's L2); host = 0 polls device lines (L2-resident).
+__global__ void poll_kernel(const unsigned long long* lines, unsigned nlines, unsigned long long ns,
+                            unsigned long long* sink) {
+    const unsigned tid = blockIdx.x * blockDim.x + threadIdx.x;
+    const unsigned long long* p = lines + (size_t)(tid % nlines) * 8;
+    const unsigned long long end = gsys::globaltimer() + ns;
+    unsigned long long acc = 0, polls = 0;
+    while (gsys::globaltimer() < end) {
+        acc += gsys::ld_relaxed_sys(p);
+        polls++;
+    }
+    atomicAdd(sink, polls + (acc & 1ull));
+}
+
 }  // namespace
 
 extern "C" {
+
+int gsys_poll_storm(const void* lines, uint32_t nlines, uint32_t nthreads, uint64_t ns, uint64_t* d_sink,
+                    void* stream) {
+    if (!lines || !nlines || !nthreads || !d_sink) return -EINVAL;
+    const unsigned bs = 256, nb = (nthreads + bs - 1) / bs;
+    poll_kernel<<<nb, bs, 0, (cudaStream_t)stream>>>(reinterpret_cast<const unsigned long long*>(lines), nlines, ns,
+                                                    reinterpret_cast<unsigned long long*>(d_sink));
+    return cudaGetLastError() == cudaSuccess ? 0 : -EIO;
+}
+
+
+int gsys_perm_pwrite(const uint8_t* d_in, const uint16_t* d_perm, uint32_t nblocks, uint32_t block_bytes,
+                     uint32_t iters, uint8_t* staging, int32_t fd, uint64_t file_off, uint32_t gflags, uint32_t grid,
+                     void* stream) {
+    gsys_dev_ctx* ctx = gsys_internal_ctx_d();
+    if (!ctx) return -ENODEV;
+    if (!d_in || !d_perm || !staging || !nblocks || !block_bytes || block_bytes % 16 || block_bytes > 16384)
+        return -EINVAL;
+    if ((gflags & GSYS_GRAN_MASK) != GSYS_WG) return -EINVAL;
+    PermArgs a;
+    memset(&a, 0, sizeof a);
+    a.ctx = ctx;
+    a.in = d_in;
+    a.perm = d_perm;
+    a.staging = staging;
+    a.file_off = file_off;
+    a.nblocks = nblocks;
+    a.bs = block_bytes;
+    a.iters = iters;
+    a.gflags = gflags;
+    a.fd = fd;
+    const size_t smem = 4ull * block_bytes;
+    if (smem > 48 * 1024 &&
+        cudaFuncSetAttribute((const void*)perm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+            cudaSuccess)
+        return -EINVAL;
+    if (grid == 0 || grid > nblocks) grid = nblocks;
+    void* args[] = {&a};
+    return gsys_launch((const void*)perm_kernel, grid, 1, 1, 1024, 1, 1, args, smem, stream);
+}
+
 
 int gsys_mc_build(const uint8_t* keys, const uint32_t* key_off, const uint8_t* key_len, const uint8_t* vals,
                   const uint64_t* val_off, const uint32_t* val_len, uint32_t n, uint32_t nbuckets, uint32_t bucket_cap,

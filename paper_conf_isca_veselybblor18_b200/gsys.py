@@ -80,6 +80,8 @@ SIGNATURES = {
     "gsys_signal_search": (ctypes.c_int, [_P, _U32, _U64, ctypes.c_char_p, _U32, _I32, _I32, _I32, _P, _U32, _P]),
     "gsys_sigsink_install": (ctypes.c_int, [_I32, _U32]),
     "gsys_mc_entries_bytes": (_U64, [_U32, _U32]),
+    "gsys_perm_pwrite": (ctypes.c_int, [_P, _P, _U32, _U32, _U32, _P, _I32, _U64, _U32, _U32, _P]),
+    "gsys_poll_storm": (ctypes.c_int, [_P, _U32, _U32, _U64, _P, _P]),
     "gsys_mc_build": (ctypes.c_int, [_P, _P, _P, _P, _P, _P, _U32, _U32, _U32, _P, _P, _P, _U64]),
     "gsys_mc_serve": (ctypes.c_int, [_I32, _P, _P, _P, _U32, _U32, _U32, _P, _P, _P, _U32, _U32, _P]),
     "gsys_sigsink_read": (ctypes.c_int, [_P, _P, _U32]),

@@ -244,3 +244,34 @@ def mc_serve_run(keys, vals, packets, nwg: int = 8, nbuckets: int = 64, bucket_c
         G.gsys_wait(s)
         sock.close()
     return resp, lat, secs, stats.cpu().tolist()
+
+
+# ---------------------------------------------------------------------------- row f3 (Fig. 8)
+def perm_pwrite_run(data, perm, iters: int, path: str, gflags: int, block_bytes: int = 8192, grid: int = 0,
+                    stream=None):
+    """Permute every block `iters` times on the GPU and pwrite it from the work-group.
+    Returns (device seconds from launch to drained, wait rc)."""
+    import numpy as np
+    ensure_init()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    nb = len(data) // block_bytes
+    d_in = torch.from_numpy(np.ascontiguousarray(data)).to(dev)
+    d_perm = torch.from_numpy(np.ascontiguousarray(perm, dtype=np.uint16).view(np.int16)).to(dev)
+    staging = torch.zeros(nb * block_bytes, dtype=torch.uint8).pin_memory()
+    fd = os.open(path, os.O_RDWR | os.O_CREAT, 0o644)
+    try:
+        os.ftruncate(fd, nb * block_bytes)
+        s = stream or torch.cuda.current_stream()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        rc = G.lib().gsys_perm_pwrite(d_in.data_ptr(), d_perm.data_ptr(), nb, block_bytes, iters,
+                                      staging.data_ptr(), fd, 0, gflags, grid, s.cuda_stream)
+        if rc:
+            raise G.GsysError(-rc, "gsys_perm_pwrite")
+        wrc = G.gsys_wait(s)
+        e1.record(s)
+        e1.synchronize()
+    finally:
+        os.close(fd)
+    return e0.elapsed_time(e1) / 1e3, wrc

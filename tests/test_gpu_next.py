@@ -76,3 +76,18 @@ def test_memcached_gpu_server_matches_definition(gflags, send):
     bad = [i for i, (p, r) in enumerate(zip(pkts, resp)) if r != OM.expected_response(p, table)]
     assert not bad, (len(bad), bad[:5])
     assert stats[0] == len(pkts) and stats[1] == sum(1 for k in reqs if k not in table)
+
+
+# ---------------------------------------------------------------------------- row f3: Fig. 8
+@pytest.mark.parametrize("gflags", [G.WG | G.BLOCKING | G.STRONG, G.WG | G.NONBLOCKING | G.STRONG,
+                                    G.WG | G.BLOCKING | G.RELAXED, G.WG | G.NONBLOCKING | G.RELAXED])
+@pytest.mark.parametrize("iters", [1, 5])
+def test_perm_pwrite_file_equals_cpu_permutation(tmpdir_shm, gflags, iters):
+    import os
+    nb, bs = 300, 8192
+    data, perm = inputs.perm_inputs(nb, bs)
+    path = os.path.join(tmpdir_shm, f"perm_{gflags}_{iters}.bin")
+    secs, rc = W.perm_pwrite_run(data, perm, iters, path, gflags, bs, grid=148)
+    assert rc == 0
+    got = np.fromfile(path, dtype=np.uint8)
+    assert np.array_equal(got, plan.permuted_blocks(data, perm, iters, bs))
