@@ -206,14 +206,18 @@ struct WcArgs {
 };
 
 __global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
-    __shared__ int s_hit;
+    // per-chunk grep flag, double-buffered by chunk parity: thread 0 clears the next chunk's flag
+    // after reading this one, so no thread can still be touching it (racecheck-clean)
+    __shared__ int s_hit[2];
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
     ScanState S;
     unsigned* shist = load_tables(smem, a.tables, nwarps, S);
     const ScanTables& sT = *S.T;
+    if (threadIdx.x == 0) { s_hit[0] = 0; s_hit[1] = 0; }
     __syncthreads();
     unsigned char* base = a.staging + (size_t)blockIdx.x * a.stride;
+    unsigned par = 0;
     for (unsigned k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         unsigned lo = 0, hi = a.nfiles;     // largest f with chunk_base[f] <= k
         while (hi - lo > 1) {
@@ -228,7 +232,6 @@ __global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
         const long long len = e + 16 - off;
         unsigned char* dst = base + 16 - (s - off);
         const bool grep = a.file_hits != nullptr && sT.npat > 0 && *(volatile unsigned*)&a.file_hits[f] == 0u;
-        if (threadIdx.x == 0) s_hit = 0;
         // row a1-a6: one work-group pread of the chunk + halo (P32.7)
         const unsigned long long t0 = a.prof ? gsys::globaltimer() : 0ull;
         const long long r = gsys_pread(a.ctx, a.fds[f], dst, (size_t)len, off,
@@ -238,7 +241,7 @@ __global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
         if (r > 0) {
             const long long valid_end = off + r;
             const long long own_end = e < valid_end ? e : valid_end;
-            S.hit = grep ? &s_hit : nullptr;
+            S.hit = grep ? &s_hit[par] : nullptr;
             if (own_end > s) {
                 switch (a.ld_policy) {
                     case LD_SYS: scan_range<LD_SYS>(base + 16, s, own_end, valid_end, S); break;
@@ -249,7 +252,11 @@ __global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
             }
         }
         __syncthreads();   // the staging line is free again before the next chunk's pread
-        if (threadIdx.x == 0 && grep && s_hit) atomicExch(&a.file_hits[f], 1u);
+        if (threadIdx.x == 0) {
+            if (grep && s_hit[par]) atomicExch(&a.file_hits[f], 1u);
+            s_hit[par] = 0;
+        }
+        par ^= 1u;
         if (a.prof && threadIdx.x == 0) {
             const unsigned long long t2 = gsys::globaltimer();
             atomicAdd(&a.prof[0], t1 - t0);

@@ -1,0 +1,27 @@
+"""Small end-to-end run of every kernel for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+import inputs
+from paper_conf_isca_veselybblor18_b200 import gsys as G
+from paper_conf_isca_veselybblor18_b200 import workloads as W
+words, pats = inputs.dictionary(), inputs.patterns()
+d = "/dev/shm/gsys_san"
+os.makedirs(d, exist_ok=True)
+p = os.path.join(d, "f.txt")
+inputs.write_file(p, 1, 0, (1 << 20) + 77, grep_plants=True)
+for st in (G.STAGE_HOST, G.STAGE_DEVICE):
+    r = W.wordcount_files([p], words, pats, chunk=64 << 10, staging=st, blocks=8)
+    print("wc", st, int(r.hist.sum()), r.wait_rc)
+buf, _, _ = inputs.gen_bytes(2, 0, (1 << 20) + 5)
+t = torch.zeros(buf.size + 64, dtype=torch.uint8, device="cuda")
+t[:buf.size].copy_(torch.from_numpy(buf))
+h = torch.zeros(64, dtype=torch.int64, device="cuda")
+G.gsys_scan_device(t, buf.size, 4096, words, pats, h, None, 8, 512)
+torch.cuda.synchronize()
+print("scan", int(h.sum()))
+for fl in (G.WI | G.BLOCKING, G.WG | G.NONBLOCKING | G.RELAXED, G.KERNEL | G.BLOCKING | G.RELAXED):
+    n, ret, lat, _, rc = W.bench_calls("getrusage", fl, 4, 64, 2)
+    print("calls", fl, rc, int((ret == 0).sum()))
+print("ok")
