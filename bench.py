@@ -293,11 +293,26 @@ def main():
         h2d_peak = measure_h2d(dev)
         extras["scan"] = scan_roofline(G, dev, corpus, words, pats, chunk)
         extras["syscalls"] = wg_syscall_rate(G, W, dev)
+        extras["config1"] = config1_latency(G, W, dev, words, pats, a.root)
     kernel_s = dev_s / a.steps
     algo_bytes = my_bytes + sum(((s + chunk - 1) // chunk) * 17 for s in of.sizes)   # chunk + halo
     rank_achieved = algo_bytes / kernel_s / 1e9
+    traffic, sysmem_ratio = None, None
+    summ = os.path.join(ROOT, "profiles", "r01_ncu_summary.json")
+    if os.path.exists(summ):   # one ncu --set full capture of wc_kernel (64 files = 1 GiB), scaled per launch
+        wk = json.load(open(summ)).get("wc_kernel_64x16MiB_host_staging", {})
+        try:
+            cap_bytes = 64 * (16 << 20)
+            dram = float(wk["dram__bytes_read.sum"]) + float(wk["dram__bytes_write.sum"])
+            traffic = dram * algo_bytes / cap_bytes
+            sysmem_ratio = float(wk["syslts__t_sectors_aperture_sysmem_lookup_miss.sum"]) * 32 / cap_bytes
+        except (KeyError, ValueError):
+            pass
     roofline = {"bound": "host-link", "achieved": rank_achieved, "peak": h2d_peak, "unit": "GB/s",
-                "frac": (rank_achieved / h2d_peak) if h2d_peak else None, "traffic": None,
+                "frac": (rank_achieved / h2d_peak) if h2d_peak else None, "traffic": traffic,
+                "traffic_note": "HBM bytes from profiles/r01_ncu_summary.json scaled to this launch (zero-copy: "
+                                "the data never lands in HBM); system-memory sector bytes per corpus byte = "
+                                f"{sysmem_ratio}",
                 "kernel": "wc_kernel (GPU-issued WG preads + scan), one launch per step per rank",
                 "peak_source": "measured live: pinned cudaMemcpyAsync H2D, 256 MiB x 8, this box's PCIe link "
                                "(MEASURED_PEAKS.json has no host-link figure)"}
@@ -323,6 +338,7 @@ def main():
                "parity": {"hist_equals_generator_census": hist_ok},
                "secondary": {"wg_syscalls_per_s_in_wordcount": syscalls_per_step * world / (dev_s / a.steps),
                              **({"getrusage_wg": extras["syscalls"]} if "syscalls" in extras else {}),
+                             **({"config1_16MiB": extras["config1"]} if "config1" in extras else {}),
                              **({"scan_hbm": extras["scan"]} if "scan" in extras else {})},
                "service": {"threads": st["threads"], "coalesce_max": st["coalesce_max"],
                            "window_us": st["coalesce_window_us"], "bundles_per_step": st["bundles"] / a.steps,
@@ -383,6 +399,41 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
 
 
+def config1_latency(G, W, dev, words, pats, root):
+    """Config 1 (BASELINE.json configs[0]): one 16 MiB file, 64 work-groups, WG + blocking + strong:
+    device time per wordcount (the latency case: 64 preads in flight at once)."""
+    import torch
+
+    import inputs
+    path = os.path.join(root or "/dev/shm", "gsys_config1_16MiB.txt")
+    if not os.path.exists(path) or os.path.getsize(path) != (16 << 20):
+        inputs.write_file(path, inputs.SEED_FILE16M, 0, 16 << 20)
+    fd = os.open(path, os.O_RDONLY)
+    out = {}
+    try:
+        s = torch.cuda.Stream(device=dev)
+        h = torch.zeros(64, dtype=torch.int64, device=dev)
+        for name, st in (("host", G.STAGE_HOST), ("device", G.STAGE_DEVICE)):
+            ts = []
+            for rep in range(23):
+                h.zero_()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                G.gsys_wordcount([fd], [16 << 20], 256 << 10, words, pats, h, None, None,
+                                 G.WG | G.BLOCKING | G.STRONG, 0, 256, s, st)
+                G.gsys_wait(s)
+                e1.record(s)
+                e1.synchronize()
+                if rep >= 3:
+                    ts.append(e0.elapsed_time(e1))
+            ts.sort()
+            out[name] = {"ms_median": ts[len(ts) // 2], "GBps_median": (16 << 20) / (ts[len(ts) // 2] / 1e3) / 1e9,
+                         "ms_min": ts[0]}
+    finally:
+        os.close(fd)
+    return out
+
+
 def wg_syscall_rate(G, W, dev):
     """getrusage(RUSAGE_SELF) at WG granularity, blocking: 4 WGs/SM x 256 threads x 20 calls."""
     import torch
@@ -406,9 +457,11 @@ def cpu_baseline_leg(a, corpus, words, pats, chunk):
     oracle.corpus(sample[:1], words, pats, chunk=chunk, nthreads=nthr)
     _, _, secs, _ = oracle.corpus(sample, words, pats, chunk=chunk, nthreads=nthr)
     rate = oracle.syscall_rate("getrusage", nthr, 200000)
+    _, _, secs1, _ = oracle.corpus(sample[:4], words, pats, chunk=chunk, nthreads=1)
+    one_thread = sum(os.path.getsize(p) for p in sample[:4]) / secs1 / 1e9
     pread_ceiling = {str(t): oracle.pread_only(corpus.paths[:64], t, chunk) / 1e9 for t in (1, 4, 8, nthr)}
     return {"value": sbytes / secs / 1e9, "unit": "GB/s", "cores": nthr, "kind": "oracle",
-            "host_pread_only_GBps_by_threads": pread_ceiling,
+            "host_pread_only_GBps_by_threads": pread_ceiling, "value_1_thread": one_thread,
             "sample": f"{len(sample)} of {a.files} files ({sbytes / 2**20:.0f} MiB): pread + scalar wordcount + grep, "
                       f"{nthr} pthreads, {cpu_model()}",
             "getrusage_direct_calls_per_s": rate}
