@@ -10,12 +10,12 @@
 //
 // Scan (reading A9/A10, csrc/scan_core.cuh): a token is a maximal run of [A-Za-z0-9_]; it is owned
 // by the chunk that holds its first byte; a dictionary hit is a whole token byte-equal to one of
-// <= 64 words of <= 16 bytes.  Each lane takes 16 aligned bytes per step (one coalesced uint4 load;
-// the 16-byte lookahead and the byte before come from the neighbouring lanes by warp shuffle) and
-// runs them through a byte DFA built from a trie of the dictionary, held in shared memory (one
-// LDS per byte, no per-token divergence); hits go to a per-warp shared histogram.  grep tests
-// every owned position whose byte is in the first-byte range of the patterns.  No tensor cores:
-// nothing here is a contraction.
+// <= 64 words of <= 16 bytes.  A warp stages 2 KiB tiles in shared memory (cp.async, double
+// buffered); each lane runs its contiguous 64-byte span through a byte DFA built from a trie of the
+// dictionary, held transposed in shared memory (one IMAD + one LDS.U16 per byte, no per-token
+// divergence); a hit is the entry into a per-word emission state, counted once per byte pair with
+// a predicated shared RED into the warp's histogram.  grep tests every owned position whose byte
+// is in the first-byte range of the patterns.  No tensor cores: nothing here is a contraction.
 
 #include <cuda_runtime.h>
 #include <errno.h>
@@ -36,8 +36,7 @@ namespace {
 using namespace gsys_scan;
 
 struct ScanState {
-    const ScanTables* T;        // shared memory
-    const unsigned short* dfa;  // shared memory, T->nstates x NCOL
+    const ScanTables* T;        // shared memory, the transposed DFA follows it
     unsigned* whist;            // this warp's shared histogram [64]
     unsigned char* stage;       // shared memory, WARP_STAGE bytes per warp
     int* hit;                   // shared grep-hit flag of the current chunk (nullptr: no grep)
@@ -76,11 +75,19 @@ __device__ __forceinline__ unsigned ld1(const unsigned char* p) {
 
 
 
-// count a DFA emission (h = word + 1, 0 = none) without a branch: predicated shared reduction
-__device__ __forceinline__ void red_hit(unsigned* wh, unsigned h) {
-    const unsigned addr = (unsigned)__cvta_generic_to_shared(wh) + (h - 1u) * 4u;
-    asm volatile("{ .reg .pred p; setp.ne.u32 p, %1, 0; @p red.shared.add.u32 [%0], 1; }" :: "r"(addr), "r"(h)
-                 : "memory");
+// Count a DFA entry e if it is an emission (e >= emit2: word (e - emit2) / 2) without a branch: an
+// unconditional shared increment at hb + 2 e (hb = histogram address - 2 emit2), or at the warp's
+// dummy word.  (A predicated RED is compiled into a branch around the atomic plus a reconvergence
+// barrier; an unconditional increment is one ATOMS.POPC.INC, which merges lanes on one address.)
+constexpr unsigned HSTRIDE = MAXD + 4;    // per-warp shared words: histogram + dummy (+ pad)
+__device__ __forceinline__ void red_emit(unsigned hb, unsigned dummy, unsigned e, unsigned emit2) {
+    asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(e >= emit2 ? hb + 2u * e : dummy) : "memory");
+}
+// the larger of a 4-byte group's two pair maxima unconditionally, the smaller only when it is an
+// emission too (a branch taken when any lane saw two hits in 4 bytes)
+__device__ __forceinline__ void red_emit2(unsigned hb, unsigned dummy, unsigned hi, unsigned lo, unsigned emit2) {
+    red_emit(hb, dummy, hi, emit2);
+    if (lo >= emit2) asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hb + 2u * lo) : "memory");
 }
 
 // Scan positions [s, own_end) of a text whose valid bytes end at valid_end; seg0 points at the
@@ -106,9 +113,28 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
 
+// full-size copies (no src-size operand: no zero-fill bookkeeping)
+__device__ __forceinline__ void cp_async16_full(unsigned dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" :: "r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async4_full(unsigned dst, const void* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(dst), "l"(src) : "memory");
+}
+
 // issue the copies of the tile starting at `base` into buffer `buf` (shared address)
 __device__ __forceinline__ void stage_tile(unsigned buf, const unsigned char* seg0, long long s, long long base,
                                            long long valid_end, unsigned lane) {
+    if (base > 0 && base + 2048 + 16 <= valid_end) {   // interior tile: no bounds, no zero fill
+        const unsigned char* src = seg0 + (base - s);
+        const unsigned d = buf + (lane >> 2) * SLOT + 16u * (lane & 3u);
+#pragma unroll
+        for (int k = 0; k < 4; k++) cp_async16_full(d + 8u * k * SLOT, src + 512 * k + 16 * lane);
+        if (lane == 0u) {
+            cp_async16_full(buf + 32u * SLOT, src + 2048);
+            cp_async4_full(buf + 33u * SLOT, src - 4);
+        }
+        return;
+    }
 #pragma unroll
     for (int k = 0; k < 4; k++) {
         const long long p = base + 512 * k + 16 * lane;
@@ -126,14 +152,17 @@ __device__ __forceinline__ void stage_tile(unsigned buf, const unsigned char* se
     }
 }
 
-template <int P>
+template <int P, bool WIDE>
 __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                            long long valid_end, const ScanState& S) {
     const ScanTables& T = *S.T;
-    const unsigned short* dfa = S.dfa;
+    const Dfa<WIDE> D = dfa_view<WIDE>(T);
     const bool grep = S.hit != nullptr && T.npat > 0;
-    unsigned* wh = S.whist;
-    auto on_hit = [wh](unsigned h) { red_hit(wh, h); };
+    const unsigned emit2 = D.emit2;
+    const unsigned hb = (unsigned)__cvta_generic_to_shared(S.whist) - 2u * emit2;
+    const unsigned dummy = (unsigned)__cvta_generic_to_shared(S.whist + MAXD);
+    auto emit = [hb, dummy, emit2](unsigned e) { red_emit(hb, dummy, e, emit2); };
+    auto emit2x = [hb, dummy, emit2](unsigned hi, unsigned lo) { red_emit2(hb, dummy, hi, lo, emit2); };
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     unsigned char* stage = S.stage + warp * WARP_STAGE;
     const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
@@ -157,7 +186,7 @@ __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg
         const unsigned prevb = lane ? (unsigned)buf[(lane - 1u) * SLOT + 63u] : (unsigned)buf[33u * SLOT + 3u];
         const long long p0 = base + 64ll * lane;
         if (p0 < own_end) {
-            dfa_lane64(dfa, W, prevb, p0, own_end, valid_end, on_hit);
+            dfa_lane64(D, W, prevb, p0, own_end, valid_end, emit, emit2x);
             if (grep && !*(volatile int*)S.hit && grep_lane64(T, W, p0, own_end, valid_end)) *S.hit = 1;
         }
         __syncwarp();                // every lane is done with this buffer before it is refilled
@@ -168,24 +197,22 @@ __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg
 // Dynamic shared memory: [ScanTables + DFA (tables_bytes)] [per-warp histograms] [warp stages].
 __device__ __forceinline__ unsigned* load_tables(unsigned char* smem, const ScanTables* gT, unsigned nwarps,
                                                  ScanState& S) {
-    const unsigned nst = gT->nstates;
-    const size_t tb = (tables_bytes(nst) + 15) & ~(size_t)15;
+    const size_t tb = (tables_bytes(gT->nsp, gT->ncol) + 15) & ~(size_t)15;
     const uint4* src = reinterpret_cast<const uint4*>(gT);
     uint4* dst = reinterpret_cast<uint4*>(smem);
     for (unsigned i = threadIdx.x; i < tb / 16; i += blockDim.x) dst[i] = src[i];
     unsigned* shist = reinterpret_cast<unsigned*>(smem + tb);
-    for (unsigned i = threadIdx.x; i < nwarps * MAXD; i += blockDim.x) shist[i] = 0;
-    S.stage = smem + tb + nwarps * MAXD * 4;
+    for (unsigned i = threadIdx.x; i < nwarps * HSTRIDE; i += blockDim.x) shist[i] = 0;
+    S.stage = smem + tb + nwarps * HSTRIDE * 4;
     S.T = reinterpret_cast<const ScanTables*>(smem);
-    S.dfa = reinterpret_cast<const unsigned short*>(smem + sizeof(ScanTables));
-    S.whist = shist + (threadIdx.x / 32) * MAXD;
+    S.whist = shist + (threadIdx.x / 32) * HSTRIDE;
     return shist;
 }
 
 __device__ __forceinline__ void flush_hist(unsigned* shist, unsigned nwarps, unsigned ndict, unsigned long long* hist) {
     for (unsigned d = threadIdx.x; d < ndict; d += blockDim.x) {
         unsigned long long sum = 0;
-        for (unsigned w = 0; w < nwarps; w++) sum += shist[w * MAXD + d];
+        for (unsigned w = 0; w < nwarps; w++) sum += shist[w * HSTRIDE + d];
         if (sum) atomicAdd(hist + d, sum);
     }
 }
@@ -205,7 +232,7 @@ struct WcArgs {
     unsigned nfiles, nchunks, chunk, stride, gflags, host_staging, ld_policy, pad_;
 };
 
-__global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
+__global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     // per-chunk grep flag, double-buffered by chunk parity: thread 0 clears the next chunk's flag
     // after reading this one, so no thread can still be touching it (racecheck-clean)
     __shared__ int s_hit[2];
@@ -243,12 +270,7 @@ __global__ void __launch_bounds__(256, 4) wc_kernel(WcArgs a) {
             const long long own_end = e < valid_end ? e : valid_end;
             S.hit = grep ? &s_hit[par] : nullptr;
             if (own_end > s) {
-                switch (a.ld_policy) {
-                    case LD_SYS: scan_range<LD_SYS>(base + 16, s, own_end, valid_end, S); break;
-                    case LD_CA: scan_range<LD_CA>(base + 16, s, own_end, valid_end, S); break;
-                    case LD_NC: scan_range<LD_NC>(base + 16, s, own_end, valid_end, S); break;
-                    default: scan_range<LD_CG>(base + 16, s, own_end, valid_end, S); break;
-                }
+                scan_range<LD_CG, false>(base + 16, s, own_end, valid_end, S);
             }
         }
         __syncthreads();   // the staging line is free again before the next chunk's pread
@@ -292,9 +314,8 @@ __global__ void __launch_bounds__(512, 1) scan_kernel(ScanArgs a) {
     for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         const long long s = (long long)k * a.chunk;
         const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
-        if (a.ld_policy == LD_CG) scan_range<LD_CG>(a.text + s, s, e, (long long)a.n, S);
-        else if (a.ld_policy == LD_CA) scan_range<LD_CA>(a.text + s, s, e, (long long)a.n, S);
-        else scan_range<LD_NC>(a.text + s, s, e, (long long)a.n, S);
+        if (sT.ncol == NCOL_WIDE) scan_range<LD_NC, true>(a.text + s, s, e, (long long)a.n, S);
+        else scan_range<LD_NC, false>(a.text + s, s, e, (long long)a.n, S);
     }
     __syncthreads();
     flush_hist(shist, nwarps, sT.ndict, a.hist);
@@ -456,6 +477,8 @@ int ensure_hstaging(Workspace* W, size_t bytes) {
     return 0;
 }
 
+constexpr size_t kSmemDynMax = 227 * 1024 - 64;   // opt-in dynamic shared memory per block (static s_hit aside)
+
 int ensure_smem_attr(const void* fn, size_t bytes) {
     if (bytes <= 48 * 1024) return 0;
     if (bytes > 227 * 1024) return -E2BIG;
@@ -551,7 +574,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.gflags = gflags;
     if (nch == 0) return 0;
     void* args[] = {&a};
-    size_t smem = align_up(tb, 16) + (threads / 32) * (MAXD * 4 + WARP_STAGE);
+    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE);
     rc = ensure_smem_attr((const void*)wc_kernel, smem);
     if (rc) return rc;
     return gsys_launch((const void*)wc_kernel, blocks, 1, 1, threads, 1, 1, args, smem, stream);
@@ -589,20 +612,29 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
+    // 129-column table when it fits next to the warps' staging (1 block of `threads` per SM),
+    // else the 77-column one
     size_t tb = 0;
-    int rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb);
+    unsigned ncol = NCOL_WIDE;
+    int rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
     if (rc && rc != -ENOSPC) return rc;
+    if (align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE) > kSmemDynMax) {
+        ncol = NCOL_NARROW;
+        rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
+        if (rc && rc != -ENOSPC) return rc;
+    }
     size_t total = align_up(tb, 256);
     rc = ensure_upload(W, total);
     if (rc) return rc;
-    rc = build_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr);
+    rc = build_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr, ncol);
     if (rc) return rc;
     cudaStream_t s = (cudaStream_t)stream;
     cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
     cudaEventRecord(W->up_ev, s);
     unsigned long long nch = (n + chunk - 1) / chunk;
     if (nch == 0) return 0;
-    if (blocks == 0) blocks = 2u * (uint32_t)W->sms;
+    const bool blocks_auto = blocks == 0;
+    if (blocks == 0) blocks = (uint32_t)W->sms;
     if (nch < blocks) blocks = (uint32_t)nch;
     ScanArgs a;
     memset(&a, 0, sizeof a);
@@ -613,13 +645,17 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     a.hit = d_hit;
     a.nchunks = nch;
     a.chunk = chunk;
-    {
-        const char* ev = getenv("GSYS_SCAN_LD");   // diagnostics: 1 = ld.cg, 3 = ld.ca instead of ld.nc
-        a.ld_policy = ev ? (unsigned)atoi(ev) : (unsigned)LD_NC;
-    }
-    size_t smem = align_up(tb, 16) + (threads / 32) * (MAXD * 4 + WARP_STAGE);
+    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE);
     rc = ensure_smem_attr((const void*)scan_kernel, smem);
     if (rc) return rc;
+    if (blocks_auto) {   // one full wave: resident blocks per SM x SMs
+        int per_sm = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, scan_kernel, (int)threads, smem) != cudaSuccess ||
+            per_sm < 1)
+            per_sm = 1;
+        blocks = (uint32_t)per_sm * (uint32_t)W->sms;
+        if (nch < blocks) blocks = (uint32_t)nch;
+    }
     scan_kernel<<<blocks, threads, smem, s>>>(a);
     return map_cuda(cudaGetLastError());
 }

@@ -7,15 +7,24 @@
 // words of <= 16 bytes; grep -F reports whether any pattern occurs as a substring.
 //
 // Wordcount runs a byte-level DFA built from a trie of the dictionary ("search for occurrences of
-// 64 strings", PAPER.md:32 P32.6): state ROOT (at a token start), DEAD (inside a token that can no
-// longer match) and one state per dictionary prefix.  A byte b selects column clamp(b-47, 0, 76):
-// column 0 holds every byte <= '/', 76 every byte >= '{', 1..75 the bytes '0'..'z' one by one, so
-// the table needs 77 columns and no class lookup.  A non-word byte leaves any state for ROOT and,
-// from a state that spells a whole dictionary word, emits that word.  Entry (u16) = next state in
-// bits 0..8 (<= 512 states) | (word+1) in bits 9..15 (terminating entries only; their next state
-// is ROOT = 0), so one shared-memory load, one AND and one shift per byte, no per-token branch.
-// Hits are counted with a predicated shared-memory reduction on the device (no divergence).  Two
-// segments run interleaved per lane (two independent state chains) to hide the load latency.
+// 64 strings", PAPER.md:32 P32.6).  States: ROOT (at a token start), DEAD (inside a token that can
+// no longer match), one state per dictionary prefix, and one EMISSION state per dictionary word --
+// a copy of ROOT entered on the non-word byte that ends a token spelling that word.  Counting a
+// hit is therefore "the DFA entered emission state E_d", with no separate output field.
+//
+// Table layout (transposed, column-major): entry(col, state) is a u16 at byte offset
+// col * (2 * nsp) + 2 * state, and the entry's value is 2 * next_state -- the byte offset of the
+// next state inside any column.  One transition is one IMAD (col * stride + entry) and one LDS.U16.
+// nsp (states per column, padded) is = 2 mod 4, so the column stride is an odd number of 32-bit
+// words and lanes sitting in the same state but reading different bytes land on different banks.
+// Emission states are numbered last, so "entry >= emit2" (= 2 * first emission state) detects a
+// hit and, since two emissions are never adjacent (a token has >= 1 byte), the larger entry of a
+// byte pair carries the pair's only possible emission: one compare + one predicated shared RED per
+// two bytes.  Two column maps:
+//   narrow (77 columns): column = clamp(b - 47, 0, 76) -- bytes <= '/' share column 0, bytes >= '{'
+//     column 76 (fits 2 work-groups per SM next to the wordcount's staging);
+//   wide (129 columns): column = b for b < 0x80, 128 for any byte >= 0x80; a 64-byte span without
+//     a high byte (the common case, checked with one OR tree) indexes the table with the raw byte.
 // grep keeps a SWAR first-byte range filter plus a 128-bit verify per candidate.
 #pragma once
 #include <cuda_runtime.h>
@@ -53,14 +62,18 @@ inline unsigned host_funnelshift_r(unsigned lo, unsigned hi, unsigned sh) {
 
 constexpr int MAXD = 64;
 constexpr int MAXP = 8;
-constexpr int NCOL = 77;                 // DFA columns (see header)
+constexpr unsigned NCOL_NARROW = 77;    // see header
+constexpr unsigned NCOL_WIDE = 129;
 constexpr unsigned ROOT = 0u, DEAD = 1u;
-constexpr unsigned MAX_STATES = 512;    // 9-bit next-state field
+constexpr unsigned MAX_TRIE = 512;      // trie states (ROOT, DEAD, dictionary prefixes)
 
 struct ScanTables {
     uint4 pats[MAXP];           // zero-padded grep patterns
     unsigned ndict, npat;
-    unsigned nstates;           // DFA states; the table (nstates x NCOL u16) follows the struct
+    unsigned nstates;           // trie states; emission state of word d is nstates + d
+    unsigned ncol;              // NCOL_NARROW or NCOL_WIDE
+    unsigned nsp;               // states per column incl. padding (= 2 mod 4)
+    unsigned emit2;             // 2 * nstates: entries >= emit2 are emissions
     unsigned fb_lo, fb_hi;      // first-byte range of patterns (SWAR candidate filter)
     unsigned fbmap[8];          // exact first-byte bitmap
     unsigned char plen[MAXP];
@@ -68,7 +81,7 @@ struct ScanTables {
 };
 static_assert(sizeof(ScanTables) % 16 == 0, "ScanTables must keep the DFA 16-byte aligned");
 
-GSYS_HD size_t tables_bytes(unsigned nstates) { return sizeof(ScanTables) + (size_t)nstates * NCOL * 2; }
+GSYS_HD size_t tables_bytes(unsigned nsp, unsigned ncol) { return sizeof(ScanTables) + (size_t)ncol * nsp * 2; }
 
 // ------------------------------------------------------------------ helpers
 GSYS_HD unsigned compress4(unsigned m80) { return ((m80 >> 7) * 0x10204080u) >> 28; }
@@ -81,11 +94,12 @@ GSYS_HD unsigned range4(unsigned x, unsigned add_lo, unsigned add_hi) {
 GSYS_HD bool is_word_byte(unsigned c) {
     return (c - 'a' < 26u) || (c - 'A' < 26u) || (c - '0' < 10u) || c == '_';
 }
-GSYS_HD unsigned dfa_col(unsigned b) {
+GSYS_HD unsigned col_narrow(unsigned b) {
     int c = (int)b - 47;
     c = c < 0 ? 0 : c;
-    return (unsigned)(c > NCOL - 1 ? NCOL - 1 : c);
+    return (unsigned)(c > (int)NCOL_NARROW - 1 ? (int)NCOL_NARROW - 1 : c);
 }
+GSYS_HD unsigned col_wide(unsigned b) { return b < 128u ? b : 128u; }
 
 // 16 bytes of the 32-byte window (A, B) starting at byte j (0..15), little-endian
 GSYS_HD void extract16(const uint4& A, const uint4& B, unsigned j, unsigned t[4]) {
@@ -107,6 +121,22 @@ GSYS_HD void mask_len(unsigned t[4], unsigned len) {
         t[k] &= m;
     }
 }
+// byte i (0..3) of w, zero-extended (one PRMT on the device)
+GSYS_HD unsigned byte_of(unsigned w, unsigned i) {
+#ifdef __CUDA_ARCH__
+    return __byte_perm(w, 0u, 0x4440u + i);
+#else
+    return (w >> (8u * i)) & 0xffu;
+#endif
+}
+// warp-uniform "does any active lane still need this" (a lane's own flag on the host)
+GSYS_HD bool any_lane(bool p) {
+#ifdef __CUDA_ARCH__
+    return __any_sync(__activemask(), p);
+#else
+    return p;
+#endif
+}
 // byte i (0..31) of the window (A, B)
 GSYS_HD unsigned window_byte(const uint4& A, const uint4& B, unsigned i) {
     const unsigned q = i >> 2;
@@ -115,61 +145,59 @@ GSYS_HD unsigned window_byte(const uint4& A, const uint4& B, unsigned i) {
     return (w >> (8 * (i & 3u))) & 0xffu;
 }
 
-// One DFA transition; returns the word id + 1 emitted (0 = none).
-GSYS_HD unsigned dfa_step(const unsigned short* __restrict__ dfa, unsigned& st, unsigned b) {
-    const unsigned e = dfa[st * NCOL + dfa_col(b)];
-    st = e & 0x1ffu;
-    return e >> 9;
-}
-
-// Start state of a step at p0: inside a token owned by the left neighbour -> DEAD.
-GSYS_HD unsigned start_state(unsigned prevb, long long p0) {
-    return (p0 > 0 && is_word_byte(prevb)) ? DEAD : ROOT;
-}
-
-// Follow the token still open after owned byte index `from` of window (A, B) to its end.
-template <class OnHit>
-GSYS_HD void dfa_finish(const unsigned short* __restrict__ dfa, unsigned st, const uint4& A, const uint4& B,
-                        unsigned from, unsigned nvalid, OnHit&& on_hit) {
-    for (unsigned i = from; st > DEAD; i++) {
-        const unsigned b = i < nvalid ? window_byte(A, B, i) : 0u;   // past the data: terminator
-        on_hit(dfa_step(dfa, st, b));
-        if (i >= nvalid) break;
+// View of the transposed DFA (see header).  Entries are 2 * state; the DFA "state" carried by the
+// scan is the entry value itself.
+template <bool WIDE>
+struct Dfa {
+    const unsigned char* base;  // entry(col, e) at base + col * stride + e
+    unsigned stride;            // 2 * nsp
+    unsigned emit2;             // first emission entry
+    GSYS_HD static unsigned col(unsigned b) { return WIDE ? col_wide(b) : col_narrow(b); }
+    GSYS_HD unsigned at(unsigned c, unsigned e) const {
+        const unsigned v = *reinterpret_cast<const unsigned short*>(base + c * stride + e);
+#ifdef __CUDA_ARCH__
+        __builtin_assume(v < 65536u);   // lets max() of two entries skip a re-mask
+#endif
+        return v;
     }
+    GSYS_HD unsigned step(unsigned e, unsigned b) const { return at(col(b), e); }
+    // inside a token whose prefix is still a dictionary prefix (ROOT, DEAD, emissions are not)
+    GSYS_HD bool live(unsigned e) const { return e > 2u * DEAD && e < emit2; }
+};
+template <bool WIDE>
+GSYS_HD Dfa<WIDE> dfa_view(const ScanTables& T) {
+    return Dfa<WIDE>{reinterpret_cast<const unsigned char*>(&T) + sizeof(ScanTables), 2u * T.nsp, T.emit2};
 }
 
-// Two full 16-byte steps (both owned and valid for all 16 bytes) run interleaved.
-template <class OnHit>
-GSYS_HD void dfa_pair(const unsigned short* __restrict__ dfa, unsigned& s0, unsigned& s1, const uint4& A0,
-                      const uint4& A1, OnHit&& on_hit) {
-    const unsigned w0[4] = {A0.x, A0.y, A0.z, A0.w};
-    const unsigned w1[4] = {A1.x, A1.y, A1.z, A1.w};
-GSYS_UNROLL
-    for (int i = 0; i < 16; i++) {
-        const unsigned h0 = dfa_step(dfa, s0, (w0[i >> 2] >> (8 * (i & 3))) & 0xffu);
-        const unsigned h1 = dfa_step(dfa, s1, (w1[i >> 2] >> (8 * (i & 3))) & 0xffu);
-        on_hit(h0);
-        on_hit(h1);
-    }
+// Start entry of a span at p0: inside a token owned by the left neighbour -> DEAD.
+GSYS_HD unsigned start_entry(unsigned prevb, long long p0) {
+    return (p0 > 0 && is_word_byte(prevb)) ? 2u * DEAD : 2u * ROOT;
 }
 
-// One 16-byte step of the scan at text position p0:
+// One 16-byte step of the scan at text position p0 (the reference composition, host emulation):
 //   A = bytes [p0, p0+16), B = bytes [p0+16, p0+32) (zeros past valid_end), prevb = byte p0-1
 //   (meaningful when p0 > 0).  Owned token starts are the positions [p0, min(p0+16, own_end));
-//   a token owned here is followed into B until it ends (at most 16 + 1 bytes); bytes at or past
+//   a token owned here is followed into B until it ends (at most 16 more bytes); bytes at or past
 //   valid_end do not exist (end of file / short read) and terminate the token.
-// on_hit(h) receives every DFA emission value (h = word id + 1, or 0 for none) -- the device
-// counts with a predicated reduction, the host emulation with a branch.
-template <class OnHit>
-GSYS_HD void dfa_segment(const unsigned short* __restrict__ dfa, const uint4& A, const uint4& B, unsigned prevb,
-                         long long p0, long long own_end, long long valid_end, OnHit&& on_hit) {
+// emit(e) receives DFA entries; entries >= emit2 are hits of word (e - emit2) / 2.
+template <bool WIDE, class Emit>
+GSYS_HD void dfa_segment(const Dfa<WIDE>& D, const uint4& A, const uint4& B, unsigned prevb, long long p0,
+                         long long own_end, long long valid_end, Emit&& emit) {
     const long long nvalid_ll = valid_end - p0;
     const unsigned nvalid = nvalid_ll >= 32 ? 32u : (unsigned)nvalid_ll;
     const long long nown_ll = own_end - p0;
     const unsigned nown = nown_ll >= 16 ? 16u : (unsigned)nown_ll;
-    unsigned st = start_state(prevb, p0);
-    for (unsigned i = 0; i < nown && i < nvalid; i++) on_hit(dfa_step(dfa, st, window_byte(A, B, i)));
-    dfa_finish(dfa, st, A, B, nown, nvalid, on_hit);
+    unsigned e = start_entry(prevb, p0);
+    for (unsigned i = 0; i < nown && i < nvalid; i++) {
+        e = D.step(e, window_byte(A, B, i));
+        emit(e);
+    }
+    for (unsigned i = nown; D.live(e) && i < 32u; i++) {
+        const unsigned b = i < nvalid ? window_byte(A, B, i) : 0u;   // past the data: terminator
+        e = D.step(e, b);
+        emit(e);
+        if (i >= nvalid) break;
+    }
 }
 
 // grep part of a step: true if a pattern starts at an owned position of [p0, p0+16).
@@ -223,76 +251,142 @@ GSYS_HD unsigned lane_byte(const Win& W, unsigned i) {
     return window_byte(a, a, i & 15u);
 }
 
+// Transitions over the 64 bytes of W.w0..w3 (all owned and valid), emissions counted per 4 bytes.  RAW: every
+// byte is < 0x80 and the table is wide, so the byte is its own column.
+// emit2x(hi, lo): count hi if it is an emission, then lo (lo <= hi, rarely an emission).
+template <bool RAW, bool WIDE, class Emit2>
+GSYS_HD unsigned dfa_run64(const Dfa<WIDE>& D, const Win& W, unsigned e, Emit2&& emit2x) {
+GSYS_UNROLL
+    for (int k = 0; k < 4; k++) {
+        const uint4 q = W.get((unsigned)k);
+        const unsigned wv[4] = {q.x, q.y, q.z, q.w};
+GSYS_UNROLL
+        for (int j = 0; j < 4; j++) {
+            const unsigned w = wv[j];
+            const unsigned b0 = byte_of(w, 0u), b1 = byte_of(w, 1u), b2 = byte_of(w, 2u), b3 = byte_of(w, 3u);
+            const unsigned e0 = D.at(RAW ? b0 : D.col(b0), e);
+            const unsigned e1 = D.at(RAW ? b1 : D.col(b1), e0);
+            const unsigned e2 = D.at(RAW ? b2 : D.col(b2), e1);
+            e = D.at(RAW ? b3 : D.col(b3), e2);
+            // at most one of two consecutive entries is an emission, so each pair's larger entry
+            // carries its pair's emission; both pairs emit only around a 1-2 byte token
+            const unsigned m01 = e0 > e1 ? e0 : e1, m23 = e2 > e ? e2 : e;
+            emit2x(m01 > m23 ? m01 : m23, m01 > m23 ? m23 : m01);
+        }
+    }
+    return e;
+}
+
 // A lane's 64-byte span at p0: W[0..3] = bytes [p0, p0+64), W[4] = [p0+64, p0+80) (zeros past
 // valid_end).  Owned token starts: [p0, min(p0+64, own_end)); the token open at the end of the
-// owned range is followed to its end (<= 17 more bytes, all inside W[4] for a full span).
-template <class OnHit>
-GSYS_HD void dfa_lane64(const unsigned short* __restrict__ dfa, const Win& W, unsigned prevb, long long p0,
-                        long long own_end, long long valid_end, OnHit&& on_hit) {
+// owned range is followed to its end (a live prefix has <= 16 bytes, so it is resolved within the
+// 16 bytes of W[4]; a byte at or past valid_end is a terminator).
+template <bool WIDE, class Emit, class Emit2>
+GSYS_HD void dfa_lane64(const Dfa<WIDE>& D, const Win& W, unsigned prevb, long long p0, long long own_end,
+                        long long valid_end, Emit&& emit, Emit2&& emit2x) {
     const long long nvalid_ll = valid_end - p0;
     const unsigned nvalid = nvalid_ll >= 80 ? 80u : (unsigned)nvalid_ll;
     const long long nown_ll = own_end - p0;
     const unsigned nown = nown_ll >= 64 ? 64u : (unsigned)nown_ll;
-    unsigned st = start_state(prevb, p0);
+    unsigned e = start_entry(prevb, p0);
     if (nown == 64u && nvalid >= 64u) {
-GSYS_UNROLL
-        for (int k = 0; k < 4; k++) {
-            const uint4 q = W.get((unsigned)k);
-            const unsigned wv[4] = {q.x, q.y, q.z, q.w};
-GSYS_UNROLL
-            for (int i = 0; i < 16; i++) on_hit(dfa_step(dfa, st, (wv[i >> 2] >> (8 * (i & 3))) & 0xffu));
+        bool raw = false;
+        if (WIDE) {
+            const unsigned o = W.w0.x | W.w0.y | W.w0.z | W.w0.w | W.w1.x | W.w1.y | W.w1.z | W.w1.w | W.w2.x |
+                               W.w2.y | W.w2.z | W.w2.w | W.w3.x | W.w3.y | W.w3.z | W.w3.w;
+            raw = (o & 0x80808080u) == 0u;
         }
-        for (unsigned i = 64; st > DEAD; i++) {
-            const unsigned b = i < nvalid ? window_byte(W.w4, W.w4, i - 64u) : 0u;
-            on_hit(dfa_step(dfa, st, b));
-            if (i >= nvalid) break;
+        if (raw) e = dfa_run64<true>(D, W, e, emit2x);
+        else e = dfa_run64<false>(D, W, e, emit2x);
+        if (nvalid == 80u) {
+            // follow the open token through W[4] with the entry frozen at its first non-live value
+            // (ROOT, DEAD or the word's emission state), then count that one value; a span whose
+            // last entry is not live has nothing open (an emission there was counted in the loop)
+            const bool lv0 = D.live(e);
+            bool lv = lv0;
+            const unsigned w4[4] = {W.w4.x, W.w4.y, W.w4.z, W.w4.w};
+GSYS_UNROLL
+            for (int j = 0; j < 4; j++) {
+                if (!any_lane(lv)) break;
+GSYS_UNROLL
+                for (int i = 0; i < 4; i++) {
+                    const unsigned en = D.step(e, byte_of(w4[j], (unsigned)i));
+                    e = lv ? en : e;
+                    lv = D.live(e);
+                }
+            }
+            emit(lv0 ? e : 2u * ROOT);
+            return;
+        }
+        const unsigned nla = nvalid - 64u;
+        for (unsigned i = 0; i < 16u && D.live(e); i++) {
+            const unsigned b = i < nla ? window_byte(W.w4, W.w4, i) : 0u;
+            e = D.step(e, b);
+            emit(e);
         }
         return;
     }
-    for (unsigned i = 0; i < nown && i < nvalid; i++) on_hit(dfa_step(dfa, st, lane_byte(W, i)));
-    for (unsigned i = nown; st > DEAD; i++) {
-        const unsigned b = i < nvalid ? lane_byte(W, i) : 0u;
-        on_hit(dfa_step(dfa, st, b));
+    for (unsigned i = 0; i < nown && i < nvalid; i++) {
+        e = D.step(e, lane_byte(W, i));
+        emit(e);
+    }
+    for (unsigned i = nown; D.live(e) && i <= 80u; i++) {
+        const unsigned b = i < nvalid && i < 80u ? lane_byte(W, i) : 0u;
+        e = D.step(e, b);
+        emit(e);
         if (i >= nvalid) break;
     }
 }
 
 // grep over a lane's span: the four 16-byte steps with their 32-byte windows.
 GSYS_HD bool grep_lane64(const ScanTables& T, const Win& W, long long p0, long long own_end, long long valid_end) {
-    for (unsigned k = 0; k < 4; k++) {
+    if (T.npat == 0) return false;
+    if (T.fb_hi < 0x80u) {
+        // one SWAR pass over the 64 bytes: does any byte fall in the patterns' first-byte range?
+        // (7-bit test: bytes >= 0x80 may pass, the exact steps below reject them)
+        const unsigned add_lo = (0x80u - T.fb_lo) * 0x01010101u, add_hi = (0x7fu - T.fb_hi) * 0x01010101u;
+        auto r = [add_lo, add_hi](unsigned x) {
+            const unsigned lo7 = x & 0x7f7f7f7fu;
+            return (lo7 + add_lo) & ~(lo7 + add_hi);
+        };
+        const unsigned acc = r(W.w0.x) | r(W.w0.y) | r(W.w0.z) | r(W.w0.w) | r(W.w1.x) | r(W.w1.y) | r(W.w1.z) |
+                             r(W.w1.w) | r(W.w2.x) | r(W.w2.y) | r(W.w2.z) | r(W.w2.w) | r(W.w3.x) | r(W.w3.y) |
+                             r(W.w3.z) | r(W.w3.w);
+        if (!(acc & 0x80808080u)) return false;
+    }
+GSYS_UNROLL
+    for (int k = 0; k < 4; k++) {
         const long long q = p0 + 16 * k;
         if (q >= own_end) break;
-        const uint4 a = W.get(k), b = W.get(k + 1);
-        if (grep_step(T, a, b, q, own_end, valid_end)) return true;
+        if (grep_step(T, W.get((unsigned)k), W.get((unsigned)k + 1u), q, own_end, valid_end)) return true;
     }
     return false;
 }
 
 // Whole step (wordcount + grep) for one segment -- the reference composition used by the host
 // emulation; the kernels run the 64-byte lane spans above (checked equal by the CPU tests).
-template <class OnHit>
-GSYS_HD bool scan_step(const ScanTables& T, const unsigned short* __restrict__ dfa, const uint4& A, const uint4& B,
-                       unsigned prevb, long long p0, long long own_end, long long valid_end, bool grep,
-                       OnHit&& on_hit) {
-    dfa_segment(dfa, A, B, prevb, p0, own_end, valid_end, on_hit);
+template <bool WIDE, class Emit>
+GSYS_HD bool scan_step(const ScanTables& T, const Dfa<WIDE>& D, const uint4& A, const uint4& B, unsigned prevb,
+                       long long p0, long long own_end, long long valid_end, bool grep, Emit&& emit) {
+    dfa_segment(D, A, B, prevb, p0, own_end, valid_end, emit);
     return grep && grep_step(T, A, B, p0, own_end, valid_end);
 }
 
 // ------------------------------------------------------------------ host: table builder
-// Writes ScanTables followed by the DFA (nstates x NCOL u16) into `out` (tables_bytes(nstates)
-// bytes, capacity `cap`).  Dictionary words must be 1..16 bytes; a word containing a non-word
-// byte can never equal a token and gets no trie path; duplicate words count once (first wins).
-// -E2BIG when the trie needs more than 512 states (distinct prefixes + 2).
+// Writes ScanTables followed by the transposed DFA (ncol x nsp u16) into `out` (capacity `cap`;
+// the size needed is returned in *used).  Dictionary words must be 1..16 bytes; a word containing
+// a non-word byte can never equal a token and gets no trie path; duplicate words count once (the
+// first wins).  -E2BIG when the trie needs more than MAX_TRIE states (distinct prefixes + 2).
 inline int build_tables(void* out, size_t cap, const char* dict, const uint8_t* dlen, uint32_t ndict,
-                        const char* pats, const uint8_t* plen, uint32_t npat, size_t* used) {
+                        const char* pats, const uint8_t* plen, uint32_t npat, size_t* used,
+                        unsigned ncol = NCOL_NARROW) {
     if (ndict > (uint32_t)MAXD || npat > (uint32_t)MAXP) return -EINVAL;
     if (ndict && (!dict || !dlen)) return -EINVAL;
     if (npat && (!pats || !plen)) return -EINVAL;
-    // trie over the DFA columns
-    std::vector<short> child;            // [state][NCOL]
-    std::vector<unsigned char> acc;      // word id + 1 per state
-    child.assign(2 * NCOL, -1);
-    acc.assign(2, 0);
+    if (ncol != NCOL_NARROW && ncol != NCOL_WIDE) return -EINVAL;
+    // trie over byte values
+    std::vector<int> child(2 * 256, -1);   // [state][byte]
+    std::vector<unsigned char> acc(2, 0);  // word id + 1 per state
     for (uint32_t d = 0; d < ndict; d++) {
         if (dlen[d] < 1 || dlen[d] > 16) return -EINVAL;
         const unsigned char* w = (const unsigned char*)dict + 17 * d;
@@ -301,19 +395,21 @@ inline int build_tables(void* out, size_t cap, const char* dict, const uint8_t* 
         if (!ok) continue;
         unsigned s = ROOT;
         for (unsigned k = 0; k < dlen[d]; k++) {
-            const unsigned c = dfa_col(w[k]);
-            if (child[s * NCOL + c] < 0) {
-                child[s * NCOL + c] = (short)acc.size();
+            if (child[s * 256 + w[k]] < 0) {
+                child[s * 256 + w[k]] = (int)acc.size();
                 acc.push_back(0);
-                child.resize(acc.size() * NCOL, -1);
+                child.resize(acc.size() * 256, -1);
             }
-            s = (unsigned)child[s * NCOL + c];
+            s = (unsigned)child[s * 256 + w[k]];
         }
         if (!acc[s]) acc[s] = (unsigned char)(d + 1);
     }
     const unsigned nstates = (unsigned)acc.size();
-    if (nstates > MAX_STATES) return -E2BIG;     // dictionary trie too large for the 9-bit state field
-    const size_t need = tables_bytes(nstates);
+    if (nstates > MAX_TRIE) return -E2BIG;
+    const unsigned nt = nstates + ndict;   // + one emission state per word
+    unsigned nsp = nt;
+    while (nsp % 4u != 2u) nsp++;
+    const size_t need = tables_bytes(nsp, ncol);
     if (used) *used = need;
     if (!out || need > cap) return -ENOSPC;
     ScanTables* T = (ScanTables*)out;
@@ -321,15 +417,23 @@ inline int build_tables(void* out, size_t cap, const char* dict, const uint8_t* 
     T->ndict = ndict;
     T->npat = npat;
     T->nstates = nstates;
+    T->ncol = ncol;
+    T->nsp = nsp;
+    T->emit2 = 2u * nstates;
     unsigned short* dfa = (unsigned short*)((unsigned char*)out + sizeof(ScanTables));
-    for (unsigned s = 0; s < nstates; s++) {
-        for (unsigned c = 0; c < (unsigned)NCOL; c++) {
-            const unsigned b = c == 0 ? 0u : (c == NCOL - 1 ? 255u : c + 47u);   // a byte of the column
-            unsigned short e;
-            if (!is_word_byte(b)) e = (unsigned short)((s >= 2 ? acc[s] : 0u) << 9);
-            else if (s == DEAD) e = (unsigned short)DEAD;
-            else e = child[s * NCOL + c] >= 0 ? (unsigned short)child[s * NCOL + c] : (unsigned short)DEAD;
-            dfa[s * NCOL + c] = e;
+    for (unsigned c = 0; c < ncol; c++) {
+        unsigned b;   // a byte of the column
+        if (ncol == NCOL_NARROW) b = c == 0 ? 0u : (c == NCOL_NARROW - 1 ? 255u : c + 47u);
+        else b = c == 128u ? 255u : c;
+        for (unsigned s = 0; s < nsp; s++) {
+            unsigned next = ROOT;
+            if (s < nt) {
+                const unsigned r = s >= nstates ? ROOT : s;   // emission states behave as ROOT
+                if (!is_word_byte(b)) next = (r >= 2 && acc[r]) ? nstates + acc[r] - 1u : ROOT;
+                else if (r == DEAD) next = DEAD;
+                else next = child[r * 256 + b] >= 0 ? (unsigned)child[r * 256 + b] : DEAD;
+            }
+            dfa[(size_t)c * nsp + s] = (unsigned short)(2u * next);
         }
     }
     T->fb_lo = 0xff;

@@ -33,10 +33,11 @@ def emul():
 
     def run(text, words, pats, chunk):
         h0, g0 = run2(text, words, pats, chunk, 0)
-        h1, g1 = run2(text, words, pats, chunk, 1)
-        h2, g2 = run2(text, words, pats, chunk, 2)
-        assert np.array_equal(h0, h1) and g0 == g1     # paired 16-byte steps == reference composition
-        assert np.array_equal(h0, h2) and g0 == g2     # the kernels' 64-byte lane spans == reference
+        for mode in (1, 2, 3):
+            # 1: wc_kernel's 64-byte lane spans (77-column table); 2: scan_kernel's lane spans (129
+            # columns, raw-byte fast path); 3: 16-byte reference steps on the 129-column table
+            h, g = run2(text, words, pats, chunk, mode)
+            assert np.array_equal(h0, h) and g0 == g, mode
         return h0, g0
 
     def run2(text, words, pats, chunk, pairs):
