@@ -303,7 +303,7 @@ def main():
         wk = json.load(open(summ)).get("wc_kernel_64x16MiB_host_staging", {})
         try:
             cap_bytes = 64 * (16 << 20)
-            dram = float(wk["dram__bytes_read.sum"]) + float(wk["dram__bytes_write.sum"])
+            dram = float(wk["dram_read_bytes"]) + float(wk["dram_write_bytes"])
             traffic = dram * algo_bytes / cap_bytes
             sysmem_ratio = float(wk["syslts__t_sectors_aperture_sysmem_lookup_miss.sum"]) * 32 / cap_bytes
         except (KeyError, ValueError):
@@ -394,8 +394,20 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
     ach = n / t / 1e9
     del text
+    traffic, limiter = None, None
+    summ = os.path.join(ROOT, "profiles", "r01_ncu_summary.json")
+    if os.path.exists(summ):   # the ncu --set full capture of the same 1 GiB scan
+        sk = json.load(open(summ)).get("scan_kernel_1GiB", {})
+        try:
+            traffic = (float(sk["dram_read_bytes"]) + float(sk["dram_write_bytes"])) * n / (64 * (16 << 20))
+            limiter = (f"shared-memory pipe: l1tex {float(sk['l1tex__throughput.avg.pct_of_peak_sustained_active']):.0f}% "
+                       f"of peak (DFA lookups, bank conflicts), issue "
+                       f"{float(sk['smsp__issue_active.avg.pct_of_peak_sustained_active']):.0f}%")
+        except (KeyError, ValueError):
+            pass
     return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "bytes": n,
-            "ms": t * 1e3, "kernel": "scan_kernel (HBM-resident text, 2 blocks/SM x 512 threads)",
+            "traffic": traffic, "limiter": limiter, "ms": t * 1e3,
+            "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 512 threads, 129-column transposed DFA in shared memory)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
 
 

@@ -229,7 +229,8 @@ struct WcArgs {
     unsigned* file_hits;
     long long* req_ret;
     unsigned long long* prof;       // optional: [0] ns waiting in the call, [1] ns scanning, [2] chunks
-    unsigned nfiles, nchunks, chunk, stride, gflags, host_staging, ld_policy, pad_;
+    unsigned* next_chunk;           // dynamic chunk queue (zeroed before the launch)
+    unsigned nfiles, nchunks, chunk, stride, gflags, host_staging;
 };
 
 __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
@@ -245,7 +246,15 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     __syncthreads();
     unsigned char* base = a.staging + (size_t)blockIdx.x * a.stride;
     unsigned par = 0;
-    for (unsigned k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
+    // Chunks come from a global queue, not a static stride: a work-group takes the next chunk when
+    // it is done with its last one, so the ~110 chunk latencies per work-group do not add up into a
+    // tail set by the slowest of 296 work-groups.
+    __shared__ unsigned s_k;
+    for (;;) {
+        if (threadIdx.x == 0) s_k = atomicAdd(a.next_chunk, 1u);
+        __syncthreads();
+        const unsigned k = s_k;
+        if (k >= a.nchunks) break;
         unsigned lo = 0, hi = a.nfiles;     // largest f with chunk_base[f] <= k
         while (hi - lo > 1) {
             unsigned mid = (lo + hi) >> 1;
@@ -298,7 +307,7 @@ struct ScanArgs {
     unsigned long long* hist;
     unsigned* hit;
     unsigned long long nchunks;
-    unsigned chunk, ld_policy;
+    unsigned chunk, pad_;
 };
 
 __global__ void __launch_bounds__(512, 1) scan_kernel(ScanArgs a) {
@@ -420,6 +429,7 @@ struct Workspace {
     unsigned char* staging_d = nullptr;
     size_t staging_cap = 0;
     unsigned long long* prof_d = nullptr;  // wc_kernel profile counters (gsys_set_profile)
+    unsigned* next_chunk_d = nullptr;      // wc_kernel chunk queue
     bool prof_on = false;
     unsigned char* hstaging = nullptr;    // pinned, host-mapped (zero-copy staging)
     size_t hstaging_cap = 0;
@@ -567,6 +577,8 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.hist = reinterpret_cast<unsigned long long*>(d_hist);
     a.file_hits = d_file_hits;
     a.req_ret = reinterpret_cast<long long*>(d_req_ret);
+    if (!W->next_chunk_d && cudaMalloc((void**)&W->next_chunk_d, 256) != cudaSuccess) return -ENOMEM;
+    a.next_chunk = W->next_chunk_d;
     a.nfiles = nfiles;
     a.nchunks = (unsigned)nch;
     a.chunk = chunk;
@@ -577,6 +589,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE);
     rc = ensure_smem_attr((const void*)wc_kernel, smem);
     if (rc) return rc;
+    if (cudaMemsetAsync(W->next_chunk_d, 0, 4, s) != cudaSuccess) return -EIO;
     return gsys_launch((const void*)wc_kernel, blocks, 1, 1, threads, 1, 1, args, smem, stream);
 }
 

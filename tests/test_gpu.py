@@ -142,6 +142,59 @@ def test_scan_device_parity():
             assert bool(hit.item()) == oracle.grep(buf, PATS)
 
 
+def _scan_dev(buf, words, pats, chunk, threads=0):
+    size = len(buf)
+    d_text = torch.zeros(size + 64, dtype=torch.uint8, device="cuda")
+    d_text[:size].copy_(torch.from_numpy(np.frombuffer(bytes(buf), dtype=np.uint8)))
+    hist = torch.zeros(64, dtype=torch.int64, device="cuda")
+    hit = torch.zeros(1, dtype=torch.int32, device="cuda")
+    G.gsys_scan_device(d_text, size, chunk, words, pats, hist, hit, 0, threads)
+    torch.cuda.synchronize()
+    return as_u64(hist)[:len(words)], bool(hit.item())
+
+
+@pytest.mark.parametrize("threads", [0, 256])
+def test_scan_device_high_bytes(threads):
+    """Text mixing every byte value: 64-byte spans with a byte >= 0x80 leave the raw-byte fast path
+    of the 129-column table for the clamped one (and the grep prefilter sees false candidates)."""
+    rng = np.random.default_rng(11)
+    words = [b"ab", b"b", b"\xc3", b"a" * 16, b"Zq_9", b"q"]
+    pats = [b"\xc3\xa9ab", b"b q", b"Zq_9 "]
+    alpha = np.frombuffer(b"ab q_Z9\n\xc3\xa9\xff\x80", dtype=np.uint8)
+    for trial in range(4):
+        n = int(rng.integers(100_000, 400_000))
+        text = alpha[rng.integers(0, len(alpha), size=n)]
+        text[rng.integers(0, n, size=n // 3)] = rng.integers(0, 256, size=n // 3, dtype=np.uint8)
+        for chunk in (64, 4096, 256 << 10):
+            hist, hit = _scan_dev(text, words, pats, chunk, threads)
+            assert np.array_equal(hist, oracle.count_tokens(text, words)[:len(words)]), (trial, chunk)
+            assert hit == oracle.grep(text, pats)
+
+
+def test_scan_device_large_trie_uses_narrow_table():
+    """A dictionary whose 129-column table no longer fits next to 16 warps' staging (482 trie
+    states + 30 emission states) runs on the 77-column table: same counts."""
+    words = [bytes([ord("A") + i % 26 if i < 26 else ord("a") + i - 26]) + bytes((97 + (i * 7 + k) % 26) for k in range(15))
+             for i in range(30)]
+    buf, _, _ = inputs.gen_bytes(inputs.SEED_CORPUS, 5, 1 << 20)
+    text = bytearray(buf.tobytes())
+    for i, w in enumerate(words):                 # plant every word a few times, whole-token
+        for r in range(3):
+            at = 1000 + 30_000 * (i * 3 + r) % (len(text) - 40)
+            text[at:at + 18] = b" " + w + b" "
+    hist, _ = _scan_dev(bytes(text), words, [], 4096)
+    exp = oracle.count_tokens(np.frombuffer(bytes(text), dtype=np.uint8), words)[:len(words)]
+    assert np.array_equal(hist, exp) and exp.sum() >= 30
+
+
+def test_scan_device_trie_too_large_is_e2big():
+    alpha = b"ABCDEFGHIJKLMNOPQRSTUVWXYZabcdefghijklmnopqrstuvwxyz0123456789"
+    words = [alpha[i:i + 1] + b"x" * 15 for i in range(40)]       # 40 x 16 + 2 = 642 trie states > 512
+    with pytest.raises(OSError) as ei:
+        _scan_dev(b"abc def", words, [], 4096)
+    assert ei.value.errno == errno.E2BIG
+
+
 # ---------------------------------------------------------------------------- microbenchmark matrix
 VALID_CELLS = [(G.WI, G.BLOCKING, G.STRONG), (G.WI, G.NONBLOCKING, G.STRONG),
                (G.WG, G.BLOCKING, G.STRONG), (G.WG, G.BLOCKING, G.RELAXED),
