@@ -196,10 +196,17 @@ def main():
     from paper_conf_isca_veselybblor18_b200 import workloads as W
 
     rank, world, local = dist_env()
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # GSYS_BENCH_ONE_GPU=1 (test only): every rank on cuda:0 with gloo, to exercise the N > 1 path
+    # on a one-GPU box (NCCL refuses two ranks on one device)
+    one_gpu = os.environ.get("GSYS_BENCH_ONE_GPU") == "1"
+    dev_idx = 0 if one_gpu else local
+    torch.cuda.set_device(dev_idx)
+    dev = torch.device("cuda", dev_idx)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     def barrier():
         if world > 1:
@@ -250,7 +257,7 @@ def main():
         for _ in range(a.warmup):
             step()
         barrier()
-        clk = Clocks(local)
+        clk = Clocks(dev_idx)
         clk.start()
         ev0 = torch.cuda.Event(enable_timing=True)
         ev1 = torch.cuda.Event(enable_timing=True)
@@ -289,7 +296,7 @@ def main():
     # ---- roofline of the dominant kernel (wc_kernel): host-link bound
     extras = {}
     h2d_peak = None
-    if not a.no_extras:
+    if not a.no_extras and rank == 0:   # after the timed region; rank 0 alone (shared host files)
         h2d_peak = measure_h2d(dev)
         extras["scan"] = scan_roofline(G, dev, corpus, words, pats, chunk)
         extras["syscalls"] = wg_syscall_rate(G, W, dev)

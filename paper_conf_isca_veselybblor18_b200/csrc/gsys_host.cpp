@@ -150,6 +150,47 @@ enum PtrKind { PK_INVALID = 0, PK_DEVICE = 1, PK_HOST = 2 };
 
 struct Instance;
 
+// CPUs the service threads may use: the process's allowed CPUs intersected with the GPU's
+// /sys/bus/pci/devices/<bdf>/local_cpulist (its NUMA node), unless that leaves none.  Returns the
+// count and fills *out (left empty when there is no locality information).
+static int service_cpus(int dev, cpu_set_t* out) {
+    CPU_ZERO(out);
+    cpu_set_t allowed;
+    CPU_ZERO(&allowed);
+    if (sched_getaffinity(0, sizeof allowed, &allowed) != 0) return (int)std::thread::hardware_concurrency();
+    const int nall = CPU_COUNT(&allowed);
+    char bdf[32] = {0};
+    if (cudaDeviceGetPCIBusId(bdf, sizeof bdf, dev) != cudaSuccess) return nall;
+    for (char* c = bdf; *c; c++) *c = (char)((*c >= 'A' && *c <= 'F') ? *c - 'A' + 'a' : *c);
+    char path[128];
+    snprintf(path, sizeof path, "/sys/bus/pci/devices/%s/local_cpulist", bdf);
+    FILE* f = fopen(path, "r");
+    if (!f) return nall;
+    char buf[4096];
+    const size_t n = fread(buf, 1, sizeof buf - 1, f);
+    fclose(f);
+    buf[n] = 0;
+    cpu_set_t local;
+    CPU_ZERO(&local);
+    for (char* p = buf; *p;) {   // "0-27,56-83"
+        char* end;
+        const long a = strtol(p, &end, 10);
+        if (end == p) break;
+        long b = a;
+        p = end;
+        if (*p == '-') b = strtol(p + 1, &p, 10);
+        for (long c = a; c <= b && c < CPU_SETSIZE; c++) CPU_SET((int)c, &local);
+        while (*p == ',' || *p == '\n' || *p == ' ') p++;
+    }
+    CPU_AND(out, &local, &allowed);
+    const int k = CPU_COUNT(out);
+    if (k == 0 || k == nall) {   // no locality information, or every allowed CPU is local anyway
+        CPU_ZERO(out);
+        return nall;
+    }
+    return k;
+}
+
 struct Req {
     uint32_t slot, seq, nr, flags;
     uint64_t a[6];
@@ -235,6 +276,7 @@ struct Worker {
 // ------------------------------------------------------------------ instance
 struct Instance {
     int dev = -1;
+    cpu_set_t cpus;                 // service-thread CPUs (this GPU's NUMA-local ones), empty = any
     uint32_t nslots = 0;
     gsys_slot* area_h = nullptr;        // pinned, mapped
     gsys_slot* area_d = nullptr;
@@ -341,6 +383,7 @@ void Worker::run() {
     sigdelset(&ss, SIGILL);
     sigdelset(&ss, SIGABRT);
     pthread_sigmask(SIG_BLOCK, &ss, nullptr);
+    if (CPU_COUNT(&inst->cpus) > 0) sched_setaffinity(0, sizeof inst->cpus, &inst->cpus);   // NUMA-local
     cudaSetDevice(inst->dev);
     Instance* I = inst;
     uint64_t idle_since = now_ns();
@@ -966,11 +1009,21 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);
     if (cudaDeviceSynchronize() != cudaSuccess) return fail(-EIO);
 
-    // service threads
-    long cores = (long)std::thread::hardware_concurrency();
-    cpu_set_t cs;
-    if (sched_getaffinity(0, sizeof cs, &cs) == 0) cores = CPU_COUNT(&cs);
-    uint32_t nthr = (uint32_t)std::max<long>(1, std::min<long>(16, cores - 2));
+    // service threads: on the CPUs local to this GPU's PCIe root, sized for the
+    // ranks that share the host (LOCAL_WORLD_SIZE, set by torchrun)
+    const int nlocal = service_cpus(I->dev, &I->cpus);
+    uint32_t nthr;
+    {
+        const char* lw = getenv("LOCAL_WORLD_SIZE");
+        const long lws = (lw && atol(lw) > 0) ? atol(lw) : 1;
+        long allowed = (long)std::thread::hardware_concurrency();
+        cpu_set_t cs;
+        if (sched_getaffinity(0, sizeof cs, &cs) == 0) allowed = CPU_COUNT(&cs);
+        // ranks expected on this GPU's CPU set if the GPUs are spread evenly across NUMA nodes
+        const long share = std::max<long>(1, (lws * nlocal + allowed - 1) / std::max<long>(1, allowed));
+        const long per = nlocal / share;
+        nthr = (uint32_t)std::max<long>(1, std::min<long>(16, lws == 1 ? per - 2 : per - 1));
+    }
     ev = getenv("GSYS_THREADS");
     if (ev && atoi(ev) > 0) nthr = (uint32_t)atoi(ev);
     I->nthreads = nthr;
