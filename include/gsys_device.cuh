@@ -215,10 +215,11 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         }
     } else {
         // every poll is a PCIe round trip, so a waiting caller first sleeps for the slot's learned
-        // "sleep hint" and then polls at a fixed interval.  The hint adapts multiplicatively on
-        // the number of polls the wait took: 1 poll means it may have overslept (shrink by 1/4),
-        // more than 2 means it woke too early (grow by the extra polling time / 2), so the
-        // sleep converges just below the service latency without feeding on its own length.
+        // "sleep hint" and then polls at a fixed (short) interval.  The hint adapts on how the
+        // wait went: answered by the first poll means it may have overslept (shrink by 1/4); more
+        // than 2 polls means it woke too early (grow by half the time spent polling, measured on
+        // %globaltimer), so the sleep converges just below the service latency without feeding on
+        // its own length, whatever the poll interval.
         const unsigned long long* m = c->hdone + s;
         const unsigned hint = nohint ? 0u : c->lat_hint[s];
         unsigned left = hint;
@@ -228,6 +229,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             left -= d;
         }
         unsigned polls = 0;
+        const unsigned long long tp = globaltimer();
         for (;;) {
             v = ld_relaxed_sys(m);
             polls++;
@@ -235,10 +237,10 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             __nanosleep(c->poll_ns_host);
         }
         if (!nohint) {
-            unsigned nh = hint;
+            unsigned long long nh = hint;
             if (polls <= 1) nh = hint - (hint >> 2);
-            else if (polls > 2) nh = hint + (polls - 2) * (c->poll_ns_host >> 1);
-            c->lat_hint[s] = nh > 200000u ? 200000u : nh;
+            else if (polls > 2) nh = hint + ((globaltimer() - tp) >> 1);
+            c->lat_hint[s] = nh > 200000ull ? 200000u : (unsigned)nh;
         }
     }
     fence_acq_rel_sys();   /* acquire: the payload is visible before the completion word */

@@ -111,7 +111,9 @@ int main(int argc, char** argv) {
     CK(cudaEventRecord(e1));
     CK(cudaEventSynchronize(e1));
     printf("{\"variant\": \"copy_engine\", \"GBps\": %.2f}\n", reps * n / (timeit(e0, e1) / 1e3) / 1e9);
+    const bool only_mix = argc > 1;
     for (int bps : {1, 2, 4}) for (int th : {256, 512, 1024}) {
+        if (only_mix) break;
         const int blocks = sms * bps;
         k_ldg<<<blocks, th>>>((const uint4*)hd, n / 16, 4);
         CK(cudaDeviceSynchronize());
@@ -123,6 +125,7 @@ int main(int argc, char** argv) {
                reps * n / (timeit(e0, e1) / 1e3) / 1e9);
     }
     for (int bps : {1, 2, 4}) for (int th : {256, 512}) {
+        if (only_mix) break;
         const int blocks = sms * bps;
         const size_t smem = (size_t)(th / 32) * 4096;
         CK(cudaFuncSetAttribute(k_cpasync, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -137,6 +140,7 @@ int main(int argc, char** argv) {
                reps * n / (timeit(e0, e1) / 1e3) / 1e9);
     }
     for (unsigned B : {4096u, 16384u, 32768u}) for (unsigned S : {2u, 4u, 8u}) for (int bps : {1, 2}) {
+        if (only_mix) break;
         const size_t smem = (size_t)B * S;
         if (smem * bps > 200 * 1024) continue;
         const int blocks = sms * bps;
@@ -151,6 +155,32 @@ int main(int argc, char** argv) {
         CK(cudaEventSynchronize(e1));
         printf("{\"variant\": \"tma_bulk\", \"bytes\": %u, \"stages\": %u, \"blocks\": %d, \"GBps\": %.2f}\n", B, S, blocks,
                reps * n / (timeit(e0, e1) / 1e3) / 1e9);
+    }
+    // concurrency: SM reads (ldg128 over the first half) while the copy engine moves the second half
+    if (argc > 1) {
+        cudaStream_t s1, s2;
+        CK(cudaStreamCreateWithFlags(&s1, cudaStreamNonBlocking));
+        CK(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+        for (double frac_ce : {0.0, 0.1, 0.2, 0.3, 0.5}) {
+            const size_t nce = ((size_t)(n * frac_ce) / 4096) * 4096, nsm = n - nce;
+            cudaEvent_t a0, a1, b1;
+            CK(cudaEventCreate(&a0)); CK(cudaEventCreate(&a1)); CK(cudaEventCreate(&b1));
+            CK(cudaDeviceSynchronize());
+            CK(cudaEventRecord(a0, s1));
+            CK(cudaStreamWaitEvent(s2, a0, 0));
+            for (int r = 0; r < reps; r++) {
+                if (nsm) k_ldg<<<sms * 2, 512, 0, s1>>>((const uint4*)hd, nsm / 16, 4);
+                if (nce) CK(cudaMemcpyAsync(d + nsm, h + nsm, nce, cudaMemcpyHostToDevice, s2));
+            }
+            CK(cudaEventRecord(a1, s1));
+            CK(cudaEventRecord(b1, s2));
+            CK(cudaEventSynchronize(a1));
+            CK(cudaEventSynchronize(b1));
+            const float t1 = timeit(a0, a1), t2 = timeit(a0, b1);
+            const float t = t1 > t2 ? t1 : t2;
+            printf("{\"variant\": \"sm+ce\", \"ce_fraction\": %.2f, \"sm_ms\": %.3f, \"ce_ms\": %.3f, \"GBps\": %.2f}\n",
+                   frac_ce, t1 / reps, t2 / reps, reps * n / (t / 1e3) / 1e9);
+        }
     }
     fflush(stdout);
     return 0;
