@@ -622,7 +622,8 @@ def run_memcached(a):
         reqs = MC.requests(keys, 20000)
         pkts = [MC.encode_get(i, k) for i, k in enumerate(reqs)]
         table = dict(zip(keys, vals))
-        for nwg, send in ((4, "blocking"), (12, "blocking"), (12, "nonblocking")):
+        for nwg, send in ((4, "blocking"), (12, "blocking"), (12, "nonblocking"), (32, "blocking"),
+                          (32, "nonblocking"), (64, "nonblocking")):
             sg = G.WG | G.RELAXED | (G.NONBLOCKING if send == "nonblocking" else G.BLOCKING)
             resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=nwg, nbuckets=nbuckets,
                                                     bucket_cap=per_bucket * 2, client_threads=4, window=8,

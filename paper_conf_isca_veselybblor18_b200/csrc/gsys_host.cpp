@@ -197,6 +197,15 @@ struct Req {
     int64_t ret;
     bool ok;
     bool dma;      // a host->device copy was queued for this request
+    bool parked;   // blocking recvfrom on an empty socket: completed later by service_parked()
+};
+
+// A blocking recvfrom that found no datagram does not hold a service thread (reading B11): the
+// request waits here and idle threads retry it (MSG_DONTWAIT) until a datagram arrives or the
+// socket's SO_RCVTIMEO expires, so the GPU caller still sees one blocking POSIX call.
+struct Parked {
+    Req r;
+    uint64_t deadline_ns;   // UINT64_MAX: no receive timeout
 };
 
 // ------------------------------------------------------------------ worker
@@ -261,6 +270,8 @@ struct Worker {
     int64_t do_pwrite(Req& r);
     int64_t do_getrusage(Req& r);
     int64_t do_generic(Req& r);
+    int64_t do_recvfrom(Req& r, bool may_park);
+    void service_parked();
     int read_small(uintptr_t p, void* out, size_t n);
     int write_small(uintptr_t p, const void* in, size_t n);
     // queue a host->device copy; issued with the bundle's other copies by flush_copies()
@@ -319,6 +330,11 @@ struct Instance {
     std::mutex sleep_mu;
     std::condition_variable sleep_cv;
     std::atomic<int> sleepers{0};
+    std::mutex park_mu;
+    std::vector<Parked> parked;
+    std::atomic<uint32_t> nparked{0};
+    // host-store completion (args[0], state, completion word) of a request finished outside process()
+    void complete_host(const Req& r);
     uint32_t nthreads = 0;
 
     // stats
@@ -391,6 +407,12 @@ void Worker::run() {
     while (!I->stop.load(std::memory_order_relaxed)) {
         uint64_t h = I->head.load(std::memory_order_acquire);
         if (!I->ready(h)) {
+            if (I->nparked.load(std::memory_order_relaxed)) {   // parked recvfroms keep us awake
+                service_parked();
+                idle_since = now_ns();
+                _mm_pause();
+                continue;
+            }
             uint64_t k = I->kick.load(std::memory_order_relaxed);
             if (k != last_kick) { last_kick = k; idle_since = now_ns(); }
             if (now_ns() - idle_since > 2000000ull) {
@@ -423,6 +445,7 @@ void Worker::run() {
         uint64_t mb = I->st_max_bundle.load(std::memory_order_relaxed);
         while (n > mb && !I->st_max_bundle.compare_exchange_weak(mb, n)) {}
         process(h, n);
+        if (I->nparked.load(std::memory_order_relaxed)) service_parked();
         idle_since = now_ns();
     }
 }
@@ -654,37 +677,124 @@ int64_t Worker::do_generic(Req& r) {
                                r.a[4] ? salen : 0);
             return z < 0 ? -(int64_t)errno : z;
         }
-        case GSYS_NR_RECVFROM: {
-            size_t n = (size_t)r.a[2];
-            uint8_t* hp = nullptr;
-            PtrKind k = resolve((uintptr_t)r.a[1], n ? n : 1, &hp);
-            if (k == PK_INVALID) return -EFAULT;
-            uint8_t sa[128];
-            socklen_t salen = 0;
-            if (r.a[5]) {
-                uint32_t l = 0;
-                if (read_small((uintptr_t)r.a[5], &l, 4) != 0) return -EFAULT;
-                salen = std::min<uint32_t>(l, sizeof sa);
-            }
-            uint8_t* dst = hp;
-            if (k == PK_DEVICE) {
-                dst = alloc(n ? n : 1);
-                if (!dst) return -ENOMEM;
-            }
-            ssize_t z = recvfrom((int)r.a[0], dst, n, (int)r.a[3], r.a[4] ? (struct sockaddr*)sa : nullptr,
-                                 r.a[5] ? &salen : nullptr);
-            if (z < 0) return -(int64_t)errno;
-            if (k == PK_DEVICE && z > 0) h2d((void*)r.a[1], dst, (size_t)z);
-            if (r.a[4] && write_small((uintptr_t)r.a[4], sa, salen) != 0) return -EFAULT;
-            if (r.a[5]) {
-                uint32_t l = salen;
-                if (write_small((uintptr_t)r.a[5], &l, 4) != 0) return -EFAULT;
-            }
-            return z;
-        }
+        case GSYS_NR_RECVFROM:
+            return do_recvfrom(r, true);
         default:
             return -ENOSYS;
     }
+}
+
+int64_t Worker::do_recvfrom(Req& r, bool may_park) {
+    size_t n = (size_t)r.a[2];
+    uint8_t* hp = nullptr;
+    PtrKind k = resolve((uintptr_t)r.a[1], n ? n : 1, &hp);
+    if (k == PK_INVALID) return -EFAULT;
+    uint8_t sa[128];
+    socklen_t salen = 0;
+    if (r.a[5]) {
+        uint32_t l = 0;
+        if (read_small((uintptr_t)r.a[5], &l, 4) != 0) return -EFAULT;
+        salen = std::min<uint32_t>(l, sizeof sa);
+    }
+    // park only calls that complete by a host store (host buffer / non-blocking) and that asked
+    // to block; everything else keeps the plain blocking call
+    const int uflags = (int)r.a[3];
+    const bool host_done = k == PK_HOST && ((r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) || (r.flags & GSYS_NONBLOCKING));
+    const bool try_park = may_park && host_done && !(uflags & MSG_DONTWAIT);
+    uint8_t* dst = hp;
+    if (k == PK_DEVICE) {
+        dst = alloc(n ? n : 1);
+        if (!dst) return -ENOMEM;
+    }
+    ssize_t z = recvfrom((int)r.a[0], dst, n, uflags | (try_park || !may_park ? MSG_DONTWAIT : 0),
+                         r.a[4] ? (struct sockaddr*)sa : nullptr, r.a[5] ? &salen : nullptr);
+    if (z < 0) {
+        const int e = errno;
+        if (try_park && (e == EAGAIN || e == EWOULDBLOCK)) {
+            // blocking socket? (O_NONBLOCK sockets return EAGAIN at once, as POSIX says)
+            const int fl = fcntl((int)r.a[0], F_GETFL);
+            if (fl >= 0 && !(fl & O_NONBLOCK)) {
+                struct timeval tv = {0, 0};
+                socklen_t tl = sizeof tv;
+                uint64_t dl = UINT64_MAX;
+                if (getsockopt((int)r.a[0], SOL_SOCKET, SO_RCVTIMEO, &tv, &tl) == 0 && (tv.tv_sec || tv.tv_usec))
+                    dl = now_ns() + (uint64_t)tv.tv_sec * 1000000000ull + (uint64_t)tv.tv_usec * 1000ull;
+                r.parked = true;
+                std::lock_guard<std::mutex> g(inst->park_mu);
+                inst->parked.push_back(Parked{r, dl});
+                inst->nparked.fetch_add(1, std::memory_order_release);
+                return -EAGAIN;
+            }
+        }
+        return -(int64_t)e;
+    }
+    if (k == PK_DEVICE && z > 0) h2d((void*)r.a[1], dst, (size_t)z);
+    if (r.a[4] && write_small((uintptr_t)r.a[4], sa, salen) != 0) return -EFAULT;
+    if (r.a[5]) {
+        uint32_t l = salen;
+        if (write_small((uintptr_t)r.a[5], &l, 4) != 0) return -EFAULT;
+    }
+    return z;
+}
+
+// Retry parked recvfroms (FIFO): the first EAGAIN on a socket ends the pass for that socket;
+// expired timeouts complete with -EAGAIN as the blocking call would have.
+void Worker::service_parked() {
+    Instance* I = inst;
+    std::unique_lock<std::mutex> g(I->park_mu, std::try_to_lock);
+    if (!g.owns_lock() || I->parked.empty()) return;
+    const uint64_t t = now_ns();
+    int empty_fd[8];
+    int nempty = 0;
+    size_t keep = 0;
+    for (size_t i = 0; i < I->parked.size(); i++) {
+        Parked p = I->parked[i];
+        const int fd = (int)p.r.a[0];
+        bool skip = false;
+        for (int j = 0; j < nempty; j++) skip = skip || empty_fd[j] == fd;
+        int64_t ret = -EAGAIN;
+        bool fin = false;
+        if (!skip) {
+            Req r = p.r;
+            r.parked = false;
+            ret = do_recvfrom(r, false);
+            if (ret == -EAGAIN || ret == -EWOULDBLOCK) {
+                if (nempty < 8) empty_fd[nempty++] = fd;
+            } else {
+                fin = true;
+            }
+        }
+        if (!fin && t >= p.deadline_ns) { fin = true; ret = -EAGAIN; }
+        if (fin) {
+            p.r.ret = ret;
+            p.r.parked = false;
+            I->complete_host(p.r);
+        } else {
+            I->parked[keep++] = p;
+        }
+    }
+    const size_t done = I->parked.size() - keep;
+    I->parked.resize(keep);
+    if (done) I->nparked.fetch_sub((uint32_t)done, std::memory_order_release);
+}
+
+void Instance::complete_host(const Req& r) {
+    const bool blocking = !(r.flags & GSYS_NONBLOCKING);
+    gsys_slot* sl = area_h + r.slot;
+    __atomic_store_n(&sl->args[0], (uint64_t)r.ret, __ATOMIC_RELAXED);
+    if (r.ret < 0) {
+        st_errors.fetch_add(1, std::memory_order_relaxed);
+        if (!blocking) {
+            int z = 0;
+            first_err.compare_exchange_strong(z, (int)r.ret);
+        }
+    }
+    if (r.ok) {
+        __atomic_store_n(&sl->state, blocking ? (uint32_t)GSYS_FINISHED : (uint32_t)GSYS_FREE, __ATOMIC_RELEASE);
+        host_trace(r.slot, r.seq, GSYS_PROCESSING, blocking ? GSYS_FINISHED : GSYS_FREE, blocking);
+    }
+    __atomic_store_n(&hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret, __ATOMIC_RELEASE);
+    completed.fetch_add(1, std::memory_order_release);
 }
 
 void Worker::process(uint64_t h0, uint32_t n) {
@@ -704,6 +814,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         for (int k = 0; k < 6; k++) r.a[k] = sl->args[k];
         r.ret = 0;
         r.dma = false;
+        r.parked = false;
         // "atomically switches any ready system call requests to the processing state" (P24.20)
         uint32_t expect = GSYS_READY;
         r.ok = __atomic_compare_exchange_n((uint32_t*)&I->area_h[r.slot].state, &expect, (uint32_t)GSYS_PROCESSING,
@@ -804,8 +915,10 @@ void Worker::process(uint64_t h0, uint32_t n) {
     // buffers complete with a stream memory operation ordered after the DMA above.
     ops.clear();
     bool need_sync = false;
+    uint32_t nparked_here = 0;
     for (uint32_t i = 0; i < n; i++) {
         Req& r = reqs[i];
+        if (r.parked) { nparked_here++; continue; }
         const bool blocking = !(r.flags & GSYS_NONBLOCKING);
         gsys_slot* sl = I->area_h + r.slot;
         __atomic_store_n(&sl->args[0], (uint64_t)r.ret, __ATOMIC_RELAXED);
@@ -894,7 +1007,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         }
     }
     commit();
-    I->completed.fetch_add(n, std::memory_order_release);
+    I->completed.fetch_add(n - nparked_here, std::memory_order_release);
     I->st_ns_busy.fetch_add(now_ns() - t_begin, std::memory_order_relaxed);
     I->st_ns_syscall.fetch_add(t_sys, std::memory_order_relaxed);
     I->st_ns_cuda.fetch_add(t_cuda, std::memory_order_relaxed);

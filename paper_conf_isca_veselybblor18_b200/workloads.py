@@ -207,9 +207,10 @@ def signal_search_run(data_dev, nblocks: int, block_bytes: int, key: bytes, sig:
 # ---------------------------------------------------------------------------- config 4 (next row)
 def mc_serve_run(keys, vals, packets, nwg: int = 8, nbuckets: int = 64, bucket_cap: int = 1024,
                  gflags: int = G.WG | G.BLOCKING | G.RELAXED, client_threads: int = 4, window: int = 8,
-                 stream=None, send_gflags: int | None = None):
+                 stream=None, send_gflags: int | None = None, idle_s: float = 0.0):
     """Config 4: memcached-style GET server on the GPU (recvfrom/sendto issued by work-groups)
-    driven by the UDP load generator.  Returns (responses, latencies ns, client seconds, stats)."""
+    driven by the UDP load generator (after `idle_s` seconds without traffic).  Returns
+    (responses, latencies ns, client seconds, stats [requests, misses, malformed, recv EAGAINs])."""
     import ctypes
     import numpy as np
 
@@ -238,7 +239,11 @@ def mc_serve_run(keys, vals, packets, nwg: int = 8, nbuckets: int = 64, bucket_c
                              gflags if send_gflags is None else send_gflags, s.cuda_stream)
         if rc:
             raise G.GsysError(-rc, "gsys_mc_serve")
-        resp, lat, secs = MC.run_client(port, packets, nthreads=client_threads, window=window)
+        if idle_s > 0:
+            import time
+            time.sleep(idle_s)
+        resp, lat, secs = MC.run_client(port, packets, nthreads=client_threads, window=window) if packets else \
+            ([], [], 0.0)
     finally:
         stop[0] = 1
         G.gsys_wait(s)

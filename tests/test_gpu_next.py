@@ -78,6 +78,32 @@ def test_memcached_gpu_server_matches_definition(gflags, send):
     assert stats[0] == len(pkts) and stats[1] == sum(1 for k in reqs if k not in table)
 
 
+def test_memcached_more_work_groups_than_service_threads():
+    """48 work-groups blocked in recvfrom at once (> the service threads): empty-socket calls are
+    parked by the service instead of holding a thread (reading B11); every reply stays exact."""
+    from inputs import mc as MC
+    from oracle import mc as OM
+    keys, vals = MC.dataset(2000, vlen=(64, 1024))
+    reqs = MC.requests(keys, 4000)
+    pkts = [MC.encode_get(i, k) for i, k in enumerate(reqs)]
+    resp, lat, secs, stats = W.mc_serve_run(keys, vals, pkts, nwg=48, nbuckets=16, bucket_cap=512,
+                                            client_threads=8, window=8)
+    table = dict(zip(keys, vals))
+    assert all(r == OM.expected_response(p, table) for p, r in zip(pkts, resp))
+    assert stats[0] == len(pkts)
+
+
+def test_recvfrom_blocks_until_the_socket_timeout():
+    """No traffic: every GPU recvfrom on the SO_RCVTIMEO = 20 ms socket blocks (parked on the host)
+    and returns -EAGAIN once the timeout passes -- 4 work-groups x 0.3 s => at most ~60 returns,
+    and at least ~ (0.3 s / 20 ms - 1) per work-group."""
+    from inputs import mc as MC
+    keys, vals = MC.dataset(100, vlen=64)
+    resp, lat, secs, stats = W.mc_serve_run(keys, vals, [], nwg=4, nbuckets=4, bucket_cap=64, idle_s=0.3)
+    assert stats[0] == 0
+    assert 4 * 10 <= stats[3] <= 4 * 17, stats
+
+
 # ---------------------------------------------------------------------------- row f3: Fig. 8
 @pytest.mark.parametrize("gflags", [G.WG | G.BLOCKING | G.STRONG, G.WG | G.NONBLOCKING | G.STRONG,
                                     G.WG | G.BLOCKING | G.RELAXED, G.WG | G.NONBLOCKING | G.RELAXED])
