@@ -43,7 +43,8 @@ def parse():
     ap.add_argument("--order", default="relaxed", choices=["strong", "relaxed"])
     ap.add_argument("--blocks", type=int, default=296, help="work-groups (2 per SM)")
     ap.add_argument("--threads", type=int, default=256)
-    ap.add_argument("--staging", default="host", choices=["device", "host"])
+    ap.add_argument("--staging", default="host", choices=["device", "host", "mixed"])
+    ap.add_argument("--dev16", type=int, default=4, help="mixed staging: chunks per 16 on the device (DMA) path")
     ap.add_argument("--cmax", type=int, default=8, help="coalescing max bundle (P22.13)")
     ap.add_argument("--window", type=int, default=0, help="coalescing window us (P22.13)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -235,7 +236,7 @@ def main():
     W.ensure_init()
     G.gsys_set_coalesce_max(a.cmax)
     G.gsys_set_coalesce_window(a.window)
-    staging = G.STAGE_HOST if a.staging == "host" else G.STAGE_DEVICE
+    staging = {"host": G.STAGE_HOST, "device": G.STAGE_DEVICE}.get(a.staging) or G.STAGE_MIXED(a.dev16)
     stream = torch.cuda.Stream(device=dev)
     of = W.OpenFiles(mine).__enter__()
     my_bytes = sum(of.sizes)

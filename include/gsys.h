@@ -212,6 +212,9 @@ int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap);
 /* ---------------------------------------------------------------- workloads (the hot path) */
 #define GSYS_STAGE_DEVICE 0u
 #define GSYS_STAGE_HOST   1u
+/* Mixed: chunk k lands in a device line when (k mod 16) < n (copy-engine DMA), else in a host line
+ * (SM zero-copy reads); both engines then share the host link.  n in 1..15. */
+#define GSYS_STAGE_MIXED(n) (0x100u | ((n) & 15u))
 /*
  * Wordcount + grep -F -l over files read with GPU-issued preads (sec. VIII-C,
  * P32.3-9 wordcount "64 strings", "work-group granularity with blocking and weak-ordering";
@@ -228,7 +231,9 @@ int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap);
  *   staging         GSYS_STAGE_DEVICE: each work-group's pread lands in a device (HBM) line,
  *                   the host service DMAs it from its pinned bounce ring;  GSYS_STAGE_HOST: the
  *                   pread lands in a pinned host-mapped line ("syscall buffers" in system memory,
- *                   PAPER.md:24 P24.37-51) and the scan reads it over PCIe (zero-copy).
+ *                   PAPER.md:24 P24.37-51) and the scan reads it over PCIe (zero-copy);
+ *                   GSYS_STAGE_MIXED(n): n of every 16 chunks (by global chunk index) take the
+ *                   device path, the rest the host path (each work-group owns one line of each).
  *   blocks          work-groups launched (0 = 2 per SM); threads: threads per work-group
  *                   (0 = 256; multiple of 32, <= 256).
  *   d_req_ret       DEVICE int64[total chunks] (may be NULL): per-chunk pread return value.

@@ -224,13 +224,16 @@ struct WcArgs {
     const int* fds;
     const unsigned long long* sizes;
     const unsigned* chunk_base;     // [nfiles + 1] first global chunk of each file
-    unsigned char* staging;         // [gridDim.x * stride]
+    unsigned char* staging;         // [gridDim.x * stride] host-mapped (host/mixed) or device lines
+    unsigned char* staging_dev;     // [gridDim.x * stride] device lines of the mixed mode
     unsigned long long* hist;
     unsigned* file_hits;
     long long* req_ret;
     unsigned long long* prof;       // optional: [0] ns waiting in the call, [1] ns scanning, [2] chunks
     unsigned* next_chunk;           // dynamic chunk queue (zeroed before the launch)
-    unsigned nfiles, nchunks, chunk, stride, gflags, host_staging;
+    unsigned nfiles, nchunks, chunk, stride, gflags;
+    unsigned host_staging;          // 0 device, 1 host, 2 mixed
+    unsigned dev16;                 // mixed: chunks with (k mod 16) < dev16 use the device line
 };
 
 __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
@@ -244,7 +247,8 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     const ScanTables& sT = *S.T;
     if (threadIdx.x == 0) { s_hit[0] = 0; s_hit[1] = 0; }
     __syncthreads();
-    unsigned char* base = a.staging + (size_t)blockIdx.x * a.stride;
+    unsigned char* const hbase = a.staging + (size_t)blockIdx.x * a.stride;
+    unsigned char* const dbase = a.host_staging == 2u ? a.staging_dev + (size_t)blockIdx.x * a.stride : hbase;
     unsigned par = 0;
     // Chunks come from a global queue, not a static stride: a work-group takes the next chunk when
     // it is done with its last one, so the ~110 chunk latencies per work-group do not add up into a
@@ -266,12 +270,15 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
         const long long e = s + a.chunk < size ? s + a.chunk : size;
         const long long off = s ? s - 1 : 0;
         const long long len = e + 16 - off;
+        // host line (SM zero-copy reads) or device line (copy-engine DMA) for this chunk
+        const bool hostbuf = a.host_staging == 1u || (a.host_staging == 2u && (k & 15u) >= a.dev16);
+        unsigned char* const base = hostbuf ? hbase : dbase;
         unsigned char* dst = base + 16 - (s - off);
         const bool grep = a.file_hits != nullptr && sT.npat > 0 && *(volatile unsigned*)&a.file_hits[f] == 0u;
         // row a1-a6: one work-group pread of the chunk + halo (P32.7)
         const unsigned long long t0 = a.prof ? gsys::globaltimer() : 0ull;
         const long long r = gsys_pread(a.ctx, a.fds[f], dst, (size_t)len, off,
-                                       a.gflags | (a.host_staging == 1u ? GSYS_HOSTBUF : 0u));
+                                       a.gflags | (hostbuf ? GSYS_HOSTBUF : 0u));
         const unsigned long long t1 = a.prof ? gsys::globaltimer() : 0ull;
         if (threadIdx.x == 0 && a.req_ret) a.req_ret[k] = r;
         if (r > 0) {
@@ -515,7 +522,8 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     gsys_dev_ctx* ctx = gsys_internal_ctx_d();
     if (!ctx) return -ENODEV;
     if ((gflags & GSYS_GRAN_MASK) != GSYS_WG || (gflags & GSYS_NONBLOCKING)) return -EINVAL;
-    if (staging > GSYS_STAGE_HOST) return -EINVAL;
+    const bool mixed = (staging & ~15u) == GSYS_STAGE_MIXED(0) && (staging & 15u) != 0u;
+    if (staging > GSYS_STAGE_HOST && !mixed) return -EINVAL;
     if (nfiles == 0 || !fds || !sizes || !d_hist) return -EINVAL;
     if (chunk < 4096 || (chunk % 16) || chunk > (1u << 30)) return -EINVAL;
     if (threads == 0) threads = 256;
@@ -552,14 +560,17 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     cudaEventRecord(W->up_ev, s);
     size_t stride = align_up((size_t)chunk + 64, 256);
     unsigned char* stage = nullptr;
-    if (staging == GSYS_STAGE_HOST) {
+    unsigned char* stage_dev = nullptr;
+    if (staging == GSYS_STAGE_HOST || mixed) {
         rc = ensure_hstaging(W, stride * blocks);
         if (rc) return rc;
         cudaHostGetDevicePointer((void**)&stage, W->hstaging, 0);
-    } else {
+    }
+    if (staging == GSYS_STAGE_DEVICE || mixed) {
         rc = ensure_staging(W, stride * blocks);
         if (rc) return rc;
-        stage = W->staging_d;
+        if (mixed) stage_dev = W->staging_d;
+        else stage = W->staging_d;
     }
     WcArgs a;
     memset(&a, 0, sizeof a);
@@ -569,11 +580,13 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.sizes = reinterpret_cast<const unsigned long long*>(W->up_d + o_s);
     a.chunk_base = reinterpret_cast<const unsigned*>(W->up_d + o_c);
     a.staging = stage;
+    a.staging_dev = stage_dev;
     if (W->prof_on) {
         if (!W->prof_d && cudaMalloc((void**)&W->prof_d, 64) != cudaSuccess) return -ENOMEM;
         a.prof = W->prof_d;
     }
-    a.host_staging = staging == GSYS_STAGE_HOST ? 1u : 0u;
+    a.host_staging = mixed ? 2u : (staging == GSYS_STAGE_HOST ? 1u : 0u);
+    a.dev16 = mixed ? (staging & 15u) : 0u;
     a.hist = reinterpret_cast<unsigned long long*>(d_hist);
     a.file_hits = d_file_hits;
     a.req_ret = reinterpret_cast<long long*>(d_req_ret);

@@ -234,6 +234,14 @@ def pack_words(words):
 STAGE_DEVICE, STAGE_HOST = 0, 1
 
 
+def STAGE_MIXED(n: int) -> int:
+    """GSYS_STAGE_MIXED(n): n of every 16 chunks take the device line (copy-engine DMA), the rest
+    the host line (SM zero-copy reads)."""
+    if not 1 <= n <= 15:
+        raise ValueError("mixed staging share must be 1..15 (of 16)")
+    return 0x100 | n
+
+
 def gsys_wordcount(fds, sizes, chunk: int, dict_words, patterns, d_hist, d_file_hits=None, d_req_ret=None,
                    gflags: int = WG | BLOCKING | STRONG, blocks: int = 0, threads: int = 0, stream=None,
                    staging: int = STAGE_DEVICE) -> int:

@@ -55,7 +55,7 @@ def as_u64(t):
 
 
 # ---------------------------------------------------------------------------- wordcount (rows a1-a8)
-@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST, G.STAGE_MIXED(5)])
 @pytest.mark.parametrize("order", [G.STRONG, G.RELAXED])
 def test_wordcount_config1_parity(file16m, order, staging):
     """Config 1: 16 MiB file, 64 work-groups, WG + blocking (+ strong / relaxed), device or
@@ -75,7 +75,7 @@ def test_wordcount_config1_parity(file16m, order, staging):
     assert bool(res.file_hits[0]) == oracle.grep(data, PATS)
 
 
-@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST, G.STAGE_MIXED(5)])
 @pytest.mark.parametrize("chunk,blocks,threads", [(4096, 7, 64), (256 << 10, 0, 256), (64 << 10, 3, 256),
                                                   (1 << 20, 1, 128)])
 def test_wordcount_ragged_corpus(ragged_corpus, chunk, blocks, threads, staging):
@@ -343,7 +343,7 @@ def test_protocol_trace_validates(file1m):
 
 # ---------------------------------------------------------------------------- full size (config 3 shape)
 @pytest.mark.slow
-@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST, G.STAGE_MIXED(5)])
 def test_full_size_corpus_census(tmpdir_shm, staging):
     """8 GiB, 512 x 16 MiB files, the bench launch configuration: whole-corpus histogram equals
     the generator's census and grep hits equal the planted set; 4 sampled files through the oracle."""

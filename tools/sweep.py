@@ -25,7 +25,8 @@ ap.add_argument("--cmax", type=int, default=8)
 ap.add_argument("--window", type=int, default=0)
 ap.add_argument("--merge", type=int, default=1)
 ap.add_argument("--steps", type=int, default=3)
-ap.add_argument("--staging", default="device", choices=["device", "host"])
+ap.add_argument("--staging", default="device", choices=["device", "host", "mixed"])
+ap.add_argument("--dev16", type=int, default=4)
 a = ap.parse_args()
 
 corpus = inputs.make_corpus(a.files, a.file_mib << 20)
@@ -41,7 +42,7 @@ s = torch.cuda.Stream()
 h = torch.zeros(64, dtype=torch.int64, device="cuda")
 hits = torch.zeros(len(of.fds), dtype=torch.int32, device="cuda")
 with torch.cuda.stream(s):
-    stg = G.STAGE_HOST if a.staging == "host" else G.STAGE_DEVICE
+    stg = {"host": G.STAGE_HOST, "device": G.STAGE_DEVICE}.get(a.staging) or G.STAGE_MIXED(a.dev16)
     G.gsys_wordcount(of.fds, of.sizes, a.chunk_kib << 10, words, pats, h, hits, None, gflags, a.blocks, a.threads, s,
                      stg)
     G.gsys_wait(s)
