@@ -81,6 +81,8 @@ enum gsys_state {
 #define GSYS_F_INLINE    0x200u   /* small result goes to the slot's inline payload line    */
 #define GSYS_F_INLINE_IN 0x400u   /* small input (siginfo, sockaddr) is in the inline line   */
 #define GSYS_F_NOHINT    0x800u   /* unpredictable latency (network): poll without the learned sleep */
+#define GSYS_F_PULL      0x1000u  /* blocking pread: the host reads into the slot's host-mapped pull
+                                     area and the GPU copies it to the destination (reading B12)  */
 
 /* Syscall numbers served (Linux x86-64). */
 #define GSYS_NR_PREAD64        17

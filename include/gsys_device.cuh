@@ -64,6 +64,8 @@ struct gsys_dev_ctx {
     unsigned ring_mask;
     unsigned poll_ns_max;           /* backoff cap for device-memory polls                      */
     unsigned poll_ns_host;          /* poll interval for host-memory (PCIe) polls               */
+    unsigned pull_big_bytes;        /* pull area of each slot s with s % 32 == 0 (0: none)      */
+    unsigned char* pull_big;        /* host-mapped [(nslots / 32) * pull_big_bytes]            */
 };
 
 #ifdef __CUDACC__
@@ -252,13 +254,81 @@ __device__ __forceinline__ void release(const gsys_dev_ctx* c, unsigned s, unsig
     st_release_gpu(&c->claim[s], 0u);      /* "consume the result" then free (reading A3) */
 }
 
+/* ------------------------------------------------------------------ pull (reading B12)
+ * A blocking pread into memory the host cannot write cheaply (device memory) is served into a
+ * host-mapped area owned by the slot, completed with a host store, and copied to the destination
+ * by the GPU (SM reads over PCIe) -- no copy-engine transfer and no stream memory operation,
+ * whose fixed costs dominate small reads.  The area is the slot's inline line for n <= 256 B,
+ * or, for a work-group's caller (cooperative copy) in a slot with s % 32 == 0, the slot's
+ * pull_big_bytes area.  The slot stays claimed until the copy is done, so the host never
+ * refills an area that is still being read. */
+__device__ __forceinline__ const unsigned char* pull_src(const gsys_dev_ctx* c, unsigned s, unsigned long long n,
+                                                         bool coop) {
+    if (n == 0ull) return nullptr;
+    if (n <= GSYS_INLINE_BYTES) return c->inline_buf + (size_t)s * GSYS_INLINE_BYTES;
+    if (coop && (s & 31u) == 0u && n <= c->pull_big_bytes) return c->pull_big + (size_t)(s >> 5) * c->pull_big_bytes;
+    return nullptr;
+}
+
+/* 16 bytes v to d (any alignment), at most `left` of them */
+__device__ __forceinline__ void store16(unsigned char* d, const uint4& v, long long left) {
+    const uintptr_t da = (uintptr_t)d;
+    if (left >= 16 && (da & 15u) == 0u) {
+        *reinterpret_cast<uint4*>(d) = v;
+    } else if (left >= 16 && (da & 3u) == 0u) {
+        unsigned* d4 = reinterpret_cast<unsigned*>(d);
+        d4[0] = v.x; d4[1] = v.y; d4[2] = v.z; d4[3] = v.w;
+    } else {
+        const unsigned m = left >= 16 ? 16u : (unsigned)left;
+        for (unsigned b = 0; b < m; b++) {
+            const unsigned w = b < 8u ? (b < 4u ? v.x : v.y) : (b < 12u ? v.z : v.w);
+            d[b] = (unsigned char)(w >> (8u * (b & 3u)));
+        }
+    }
+}
+
+/* Copy r bytes of a pull area (16-byte aligned, host-mapped) to dst (any alignment); threads
+ * tid = 0..nt-1 share the work.  Source loads are .sys-scope (never a stale L1 line of an earlier
+ * pull of the same area) and issued four at a time per thread, so they overlap on the link. */
+__device__ __forceinline__ void pull_copy(const unsigned char* src, unsigned char* dst, long long r, unsigned tid,
+                                          unsigned nt) {
+    const unsigned n16 = (unsigned)((r + 15) >> 4);
+    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+    for (unsigned i = tid; i < n16; i += 4u * nt) {
+        const unsigned i1 = i + nt, i2 = i + 2u * nt, i3 = i + 3u * nt;
+        const uint4 v0 = ld_v4_sys(s4 + i);
+        const uint4 v1 = i1 < n16 ? ld_v4_sys(s4 + i1) : z;
+        const uint4 v2 = i2 < n16 ? ld_v4_sys(s4 + i2) : z;
+        const uint4 v3 = i3 < n16 ? ld_v4_sys(s4 + i3) : z;
+        store16(dst + 16u * i, v0, r - 16ll * i);
+        if (i1 < n16) store16(dst + 16u * i1, v1, r - 16ll * i1);
+        if (i2 < n16) store16(dst + 16u * i2, v2, r - 16ll * i2);
+        if (i3 < n16) store16(dst + 16u * i3, v3, r - 16ll * i3);
+    }
+}
+
+/* A pull the caller's scope finishes (work-group cooperative copy): filled by call_thread. */
+struct PullOut {
+    const unsigned char* src = nullptr;
+    unsigned slot = 0, seq = 0;
+};
+
 /* One thread, one request: claim -> (inline input) -> marshal -> publish -> (poll).  A non-blocking
  * request's slot is reused only after the host has served it (P24.34, A15).  io.out: for
- * GSYS_F_INLINE calls, where the host's inline result is copied after completion. */
+ * GSYS_F_INLINE calls, where the host's inline result is copied after completion.  po: when set
+ * (a work-group caller), a pulled pread's copy and the slot's release are left to the caller's
+ * scope; otherwise this thread copies (inline-size pulls only). */
 __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned nr, unsigned flags,
-                                                 const unsigned long long a[6], const InlineIO& io = InlineIO()) {
+                                                 const unsigned long long a[6], const InlineIO& io = InlineIO(),
+                                                 PullOut* po = nullptr) {
     const bool blocking = !(flags & GSYS_NONBLOCKING);
     unsigned s = claim(c, blocking);
+    const unsigned char* psrc = nullptr;
+    if (nr == GSYS_NR_PREAD64 && blocking && !(flags & GSYS_HOSTBUF)) {
+        psrc = pull_src(c, s, a[2], po != nullptr);
+        if (psrc) flags |= GSYS_F_PULL;
+    }
     if (io.in != nullptr) {   /* input payload into the inline line; published by marshal's fence */
         uint4* dst = reinterpret_cast<uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
         const unsigned char* src = reinterpret_cast<const unsigned char*>(io.in);
@@ -277,11 +347,30 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         st_release_gpu(&c->claim[s], 0u);
         return 0;
     }
-    long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) != 0u, (flags & GSYS_F_NOHINT) != 0u);
+    long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) != 0u,
+                            (flags & GSYS_F_NOHINT) != 0u);
+    if (psrc != nullptr && r > 0) {
+        if (po != nullptr) {   /* the work-group copies and releases (wg_call) */
+            po->src = psrc; po->slot = s; po->seq = seq;
+            return r;
+        }
+        pull_copy(psrc, reinterpret_cast<unsigned char*>(a[1]), r, 0u, 1u);
+    }
     if (io.out != nullptr && r >= 0) {
         const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
         uint4* dst = reinterpret_cast<uint4*>(io.out);
-        for (unsigned i = 0; i < io.out_bytes / 16u; i++) dst[i] = ld_v4_sys(src + i);
+        // loads four at a time (not one PCIe round trip per 16 B), then the stores
+        const unsigned n16 = io.out_bytes / 16u;
+        for (unsigned i = 0; i < n16; i += 4u) {
+            const uint4 v0 = ld_v4_sys(src + i);
+            const uint4 v1 = i + 1u < n16 ? ld_v4_sys(src + i + 1u) : v0;
+            const uint4 v2 = i + 2u < n16 ? ld_v4_sys(src + i + 2u) : v0;
+            const uint4 v3 = i + 3u < n16 ? ld_v4_sys(src + i + 3u) : v0;
+            dst[i] = v0;
+            if (i + 1u < n16) dst[i + 1u] = v1;
+            if (i + 2u < n16) dst[i + 2u] = v2;
+            if (i + 3u < n16) dst[i + 3u] = v3;
+        }
     }
     release(c, s, seq);
     return r;
@@ -298,18 +387,31 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
                                              const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     __shared__ long long s_ret[2];
     __shared__ unsigned s_par;
+    __shared__ const unsigned char* s_psrc[2];
+    __shared__ unsigned char* s_pdst[2];
     const bool strong = !(flags & GSYS_RELAXED);
     const bool bar1 = strong || !producer;
     const bool bar2 = strong || producer;
     const unsigned tid = block_tid();
     if (bar1) __syncthreads();
     long long r = 0;
-    if (tid == 0) r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, io);
+    PullOut po;
+    if (tid == 0) r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, io, bar2 ? &po : nullptr);
     if (bar2) {
         unsigned p = 0;
-        if (tid == 0) { p = (s_par ^ 1u) & 1u; s_par = p; s_ret[p] = r; }
+        if (tid == 0) {
+            p = (s_par ^ 1u) & 1u; s_par = p; s_ret[p] = r;
+            s_psrc[p] = po.src; s_pdst[p] = reinterpret_cast<unsigned char*>(a[1]);
+        }
         p = (unsigned)__syncthreads_or(tid == 0 ? (int)p : 0);
-        return s_ret[p];
+        const long long rv = s_ret[p];
+        const unsigned char* src = s_psrc[p];
+        if (src != nullptr) {   /* pulled pread (reading B12): the whole work-group copies */
+            pull_copy(src, s_pdst[p], rv, tid, block_threads());
+            __syncthreads();
+            if (tid == 0) release(c, po.slot, po.seq);
+        }
+        return rv;
     }
     if (tid < 32) {
         unsigned nt = block_threads();

@@ -292,6 +292,16 @@ struct Instance {
     gsys_slot* area_h = nullptr;        // pinned, mapped
     gsys_slot* area_d = nullptr;
     uint8_t* inline_h = nullptr;
+    uint8_t* pull_h = nullptr;          // pinned, mapped: [(nslots/32) * pull_bytes] (reading B12)
+    uint8_t* pull_d = nullptr;
+    uint32_t pull_bytes = 0;
+    // host address of slot s's pull area for an n-byte pread (the device's pull_src rule), or null
+    uint8_t* pull_area(uint32_t s, uint64_t n) const {
+        if (n == 0) return nullptr;
+        if (n <= GSYS_INLINE_BYTES) return inline_h + (size_t)s * GSYS_INLINE_BYTES;
+        if ((s & 31u) == 0u && n <= pull_bytes && pull_h) return pull_h + (size_t)(s >> 5) * pull_bytes;
+        return nullptr;
+    }
     uint8_t* inline_d = nullptr;
     uint64_t* ring_h = nullptr;
     uint64_t* ring_d = nullptr;
@@ -561,7 +571,14 @@ int64_t Worker::do_pread(Req& r) {
         return z < 0 ? -(int64_t)errno : 0;
     }
     uint8_t* hp = nullptr;
-    PtrKind k = resolve(buf, n, &hp);
+    PtrKind k;
+    if (r.flags & GSYS_F_PULL) {   // into the slot's pull area; the GPU copies it out (reading B12)
+        hp = inst->pull_area(r.slot, n);
+        if (!hp) return -EINVAL;
+        k = PK_HOST;
+    } else {
+        k = resolve(buf, n, &hp);
+    }
     if (k == PK_INVALID) return -EFAULT;
     inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
     if (k == PK_HOST) {
@@ -853,7 +870,9 @@ void Worker::process(uint64_t h0, uint32_t n) {
             bool okd = true;
             for (uint32_t j : mem) {
                 Req& r = reqs[midx[j]];
-                PtrKind k = r.a[2] ? resolve((uintptr_t)r.a[1], r.a[2], nullptr) : PK_INVALID;
+                PtrKind k = !r.a[2] ? PK_INVALID
+                            : (r.flags & GSYS_F_PULL) ? (I->pull_area(r.slot, r.a[2]) ? PK_HOST : PK_INVALID)
+                                                      : resolve((uintptr_t)r.a[1], r.a[2], nullptr);
                 if (k == PK_INVALID || (k == PK_HOST && r.a[2] > (64u << 10))) { okd = false; break; }
             }
             if (!okd) continue;
@@ -872,7 +891,9 @@ void Worker::process(uint64_t h0, uint32_t n) {
                 dma_flag = false;
                 if (ri > 0) {
                     uint8_t* hp = nullptr;
-                    PtrKind k = resolve((uintptr_t)r.a[1], r.a[2], &hp);
+                    PtrKind k = PK_HOST;
+                    if (r.flags & GSYS_F_PULL) hp = I->pull_area(r.slot, r.a[2]);
+                    else k = resolve((uintptr_t)r.a[1], r.a[2], &hp);
                     if (k == PK_HOST) {
                         memcpy(hp, b + mgoff_in[j], (size_t)ri);
                     } else {
@@ -933,7 +954,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         memset(&op, 0, sizeof op);
         if (blocking) {
             const uint64_t word = ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret;
-            if (r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)) {
+            if (r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) {
                 if (r.dma) { need_sync = true; continue; }
                 if (r.ok) {
                     __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
@@ -986,7 +1007,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         for (uint32_t i = 0; i < n; i++) {
             Req& r = reqs[i];
             const bool nb = (r.flags & GSYS_NONBLOCKING) != 0;
-            if (!r.dma || (!nb && !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE)))) continue;
+            if (!r.dma || (!nb && !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)))) continue;
             gsys_slot* sl = I->area_h + r.slot;
             if (r.ok) {
                 __atomic_store_n(&sl->state, nb ? (uint32_t)GSYS_FREE : (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
@@ -1069,6 +1090,19 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     if (cudaHostAlloc((void**)&I->inline_h, inl, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
     cudaHostGetDevicePointer((void**)&I->inline_d, I->inline_h, 0);
+    {   // pull areas of the slots a work-group caller lands in (s % 32 == 0): GSYS_PULL_KB, default 16
+        const char* pv = getenv("GSYS_PULL_KB");
+        const long kb = pv ? atol(pv) : 16;
+        I->pull_bytes = (kb > 0 && kb <= 1024) ? (uint32_t)kb << 10 : 0u;
+        const size_t pb = (size_t)((slots + 31) / 32) * I->pull_bytes;
+        if (pb && cudaHostAlloc((void**)&I->pull_h, pb, cudaHostAllocMapped | cudaHostAllocPortable) == cudaSuccess) {
+            cudaHostGetDevicePointer((void**)&I->pull_d, I->pull_h, 0);
+        } else {
+            cudaGetLastError();
+            I->pull_h = nullptr;
+            I->pull_bytes = 0;
+        }
+    }
     if (cudaHostAlloc((void**)&I->ring_h, (size_t)rc * 8, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
     memset(I->ring_h, 0, (size_t)rc * 8);
@@ -1121,6 +1155,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // 256 ns: a 4 KiB pread round trip drops from 16.1 to 9.9 us vs 4 us polling, and the
     // wordcount (pollers sharing the PCIe link with the scan) is unchanged (profiles/r01_latency.json)
     c.poll_ns_host = (ev && atoi(ev) > 0) ? (unsigned)atoi(ev) : 256u;
+    c.pull_big_bytes = I->pull_bytes;
+    c.pull_big = I->pull_d;
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);
     if (cudaDeviceSynchronize() != cudaSuccess) return fail(-EIO);
 
@@ -1305,6 +1341,9 @@ int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint3
     // reset the kernel-scope call sites for this launch (block rounds + per-round records)
     cudaMemsetAsync(I->kblock_d, 0, (size_t)nb * GSYS_KSITES * 4, s);
     cudaMemsetAsync(I->krounds_d, 0, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS, s);
+    // the learned pre-poll sleep (reading B3) is relearned per launch: a hint carried over from
+    // another workload's latency would make this kernel's first calls oversleep
+    cudaMemsetAsync(I->lat_hint_d, 0, (size_t)I->nslots * 4, s);
     I->gen.fetch_add(1);
     I->kick.fetch_add(1);
     if (I->sleepers.load(std::memory_order_relaxed) > 0) {
@@ -1355,6 +1394,7 @@ int gsys_shutdown(void) {
     }
     cudaFreeHost(I->area_h);
     cudaFreeHost(I->inline_h);
+    if (I->pull_h) cudaFreeHost(I->pull_h);
     cudaFreeHost(I->ring_h);
     cudaFreeHost(I->hdone_h);
     cudaFree(I->claim_d);

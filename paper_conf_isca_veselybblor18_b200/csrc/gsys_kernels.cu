@@ -374,7 +374,7 @@ __device__ unsigned long long scope_sum(const unsigned char* b, unsigned long lo
     return r;
 }
 
-__global__ void bench_kernel(BenchArgs a) {
+__global__ void __launch_bounds__(1024, 1) bench_kernel(BenchArgs a) {   // <= 64 registers: 4 x 256-thread WGs per SM
     const unsigned gran = a.gflags & GSYS_GRAN_MASK;
     const unsigned tid = threadIdx.x;
     const bool wi = gran == GSYS_WI;

@@ -362,3 +362,39 @@ def test_full_size_corpus_census(tmpdir_shm, staging):
         h, hits = oracle_hist_hits([c.paths[f]])
         r1 = W.wordcount_files([c.paths[f]], WORDS, PATS, chunk=256 << 10, staging=staging)
         assert np.array_equal(as_u64(r1.hist), h) and r1.file_hits.tolist() == hits.tolist()
+
+
+# ---------------------------------------------------------------------------- pull path (reading B12)
+@pytest.mark.parametrize("gran,length", [(G.WG, n) for n in (1, 15, 16, 255, 256, 257, 1000, 4096, 16383, 16384,
+                                                             16385, 65536)] +
+                         [(G.WI, n) for n in (1, 100, 256, 257)] + [(G.KERNEL, n) for n in (200, 3000)])
+@pytest.mark.parametrize("shift", [0, 1, 4, 8])
+def test_pread_pull_sizes(file1m, gran, length, shift):
+    """Blocking preads into device memory: <= 256 B (any caller) and work-group preads of up to
+    the slot's pull area (16 KiB) are read by the host into a host-mapped pull area and copied by
+    the GPU; longer ones take the DMA path.  Every size and destination alignment must give the
+    file's bytes, the POSIX return and the byte sums the scope computes right after the call."""
+    size = os.path.getsize(file1m)
+    data = open(file1m, "rb").read()
+    blocks, threads, iters = 3, 96, 2
+    callers = {G.WI: blocks * threads, G.WG: blocks, G.KERNEL: 1}[gran]
+    order = G.RELAXED if gran == G.KERNEL else G.STRONG
+    d_all = torch.zeros(callers * length + 64, dtype=torch.uint8, device="cuda")
+    d_buf = d_all[shift:]
+    fd = os.open(file1m, os.O_RDONLY)
+    try:
+        ncall, ret, _, sm, rc = W.bench_calls("pread", gran | G.BLOCKING | order, blocks, threads, iters, fd, length,
+                                              size, d_buf, want_sum=True)
+    finally:
+        os.close(fd)
+    assert rc == 0 and ncall == callers
+    reqs = plan.microbench_requests({G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}[gran], blocks, threads, iters,
+                                    length, size)
+    assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs]
+    assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs]
+    host = d_all.cpu().numpy()
+    assert not host[:shift].any()
+    for c in range(callers):
+        off = ((c * iters + iters - 1) * length) % size
+        want = data[off: off + length]
+        assert bytes(host[shift + c * length: shift + c * length + len(want)]) == want

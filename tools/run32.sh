@@ -1,4 +1,3 @@
 #!/bin/bash
-timeout 900 python bench.py --mode fig8 > gpurun_out/fig8.json 2> gpurun_out/fig8.err
-timeout 600 python bench.py --mode fig9 > gpurun_out/fig9.json 2> gpurun_out/fig9.err
-timeout 900 python bench.py --mode mm > gpurun_out/mm32.json 2> gpurun_out/mm32.err
+timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/pytest32.log 2>&1; echo rc=$? >> gpurun_out/pytest32.log
+timeout 900 python bench.py --mode syscalls > gpurun_out/sys32.json 2> gpurun_out/sys32.err; echo rc=$? >> gpurun_out/sys32.err

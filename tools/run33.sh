@@ -1,4 +1,3 @@
 #!/bin/bash
-for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_small.py > gpurun_out/san_$tool.log 2>&1; echo rc=$? >> gpurun_out/san_$tool.log
-done
+timeout 1500 python -m pytest tests -m gpu -q -x > gpurun_out/pytest33.log 2>&1; echo rc=$? >> gpurun_out/pytest33.log
+timeout 900 python bench.py --mode syscalls > gpurun_out/sys33.json 2> gpurun_out/sys33.err; echo rc=$? >> gpurun_out/sys33.err
