@@ -66,6 +66,7 @@ struct gsys_dev_ctx {
     unsigned poll_ns_host;          /* poll interval for host-memory (PCIe) polls               */
     unsigned pull_big_bytes;        /* pull area of each slot s with s % 32 == 0 (0: none)      */
     unsigned char* pull_big;        /* host-mapped [(nslots / 32) * pull_big_bytes]            */
+    unsigned no_hint;               /* 1: no learned pre-poll sleep (env GSYS_SLEEP_HINT=0)     */
 };
 
 #ifdef __CUDACC__
@@ -112,6 +113,9 @@ __device__ __forceinline__ uint4 ld_v4_sys(const uint4* p) {
     return v;
 }
 __device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+    unsigned long long v; asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory"); return v;
+}
 
 __device__ __forceinline__ unsigned block_tid() {
     return threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
@@ -187,7 +191,11 @@ __device__ __forceinline__ unsigned marshal(const gsys_dev_ctx* c, unsigned s, u
  * "scalar wavefront instruction" of P24.14).  Entry = (position+1) << 32 | slot, so the host
  * recognises a fresh entry without the ring ever being cleared. */
 __device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
+#if defined(GSYS_DOORBELL_SC)
     __threadfence_system();
+#else
+    fence_acq_rel_sys();   /* release: the slot line (and inline input) before the entry */
+#endif
     unsigned mask = __activemask();
     unsigned lane = laneid();
     unsigned leader = __ffs(mask) - 1u;
@@ -210,7 +218,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         const unsigned long long* m = c->mirror + s;
         unsigned ns = 64;
         for (;;) {
-            v = ld_relaxed_sys(m);
+            v = ld_acquire_sys(m);
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(ns);
             ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
@@ -223,6 +231,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         // %globaltimer), so the sleep converges just below the service latency without feeding on
         // its own length, whatever the poll interval.
         const unsigned long long* m = c->hdone + s;
+        nohint = nohint || c->no_hint;
         const unsigned hint = nohint ? 0u : c->lat_hint[s];
         unsigned left = hint;
         while (left > 0) {
@@ -233,7 +242,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         unsigned polls = 0;
         const unsigned long long tp = globaltimer();
         for (;;) {
-            v = ld_relaxed_sys(m);
+            v = ld_acquire_sys(m);
             polls++;
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(c->poll_ns_host);
@@ -245,7 +254,9 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             c->lat_hint[s] = nh > 200000ull ? 200000u : (unsigned)nh;
         }
     }
-    fence_acq_rel_sys();   /* acquire: the payload is visible before the completion word */
+    /* the polls are acquire loads: the payload (device memory after the DMA, or the inline / pull
+     * area the host wrote before its release store) is read after the completion word, with no
+     * separate system-scope fence (a MEMBAR.SYS per call) */
     return (long long)(int)(unsigned)(v & 0xffffffffull);
 }
 

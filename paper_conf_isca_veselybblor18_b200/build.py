@@ -32,13 +32,15 @@ def _stale() -> bool:
     return any(os.path.getmtime(p) > t for p in SOURCES + HEADERS + [__file__])
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = "") -> str:
+    """Compile libgsys.so; `defines`/`out` build a diagnostic variant elsewhere (tools/)."""
+    if not out and not force and not _stale():
         return LIB
     objs = []
-    build_dir = os.path.join(PKG, "build")
+    build_dir = os.path.join(PKG, "build" + ("_" + os.path.basename(out) if out else ""))
     os.makedirs(build_dir, exist_ok=True)
-    common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3,-Wall", "-I", INCLUDE, "-I", CSRC]
+    common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3,-Wall", "-I", INCLUDE, "-I", CSRC,
+              *["-D" + d for d in defines]]
     for src in SOURCES:
         obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         cmd = [NVCC, *common, *ARCH, "-c", src, "-o", obj]
@@ -48,11 +50,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
             cmd = [NVCC, "-x", "cu", *common, *ARCH, "-c", src, "-o", obj]
         subprocess.check_call(cmd)
         objs.append(obj)
-    tmp = LIB + f".tmp{os.getpid()}"
+    target = out or LIB
+    tmp = target + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs,
                            "-Xlinker", "--no-undefined", "-lpthread", "-ldl", "-lrt"])
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -1155,6 +1155,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // 256 ns: a 4 KiB pread round trip drops from 16.1 to 9.9 us vs 4 us polling, and the
     // wordcount (pollers sharing the PCIe link with the scan) is unchanged (profiles/r01_latency.json)
     c.poll_ns_host = (ev && atoi(ev) > 0) ? (unsigned)atoi(ev) : 256u;
+    ev = getenv("GSYS_SLEEP_HINT");
+    c.no_hint = (ev && atoi(ev) == 0) ? 1u : 0u;
     c.pull_big_bytes = I->pull_bytes;
     c.pull_big = I->pull_d;
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);

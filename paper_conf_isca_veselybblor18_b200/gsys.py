@@ -100,8 +100,8 @@ def lib():
     """Load libgsys.so (building it in-tree if stale).  Raises if it cannot be built/loaded."""
     global _lib
     if _lib is None:
-        path = _build.LIB
-        if not os.path.exists(path) or os.environ.get("GSYS_REBUILD"):
+        path = os.environ.get("GSYS_LIB") or _build.LIB   # GSYS_LIB: a diagnostic variant (tools/)
+        if path == _build.LIB and (not os.path.exists(path) or os.environ.get("GSYS_REBUILD")):
             _build.build()
         L = ctypes.CDLL(path)
         for name, (res, args) in SIGNATURES.items():

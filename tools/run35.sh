@@ -1,7 +1,6 @@
 #!/bin/bash
-python -c "import inputs; inputs.make_corpus(512, 16<<20)" 2>&1 | tail -1
-timeout 900 python bench.py > gpurun_out/bench35.json 2> gpurun_out/bench35.err
-timeout 900 python bench.py --mode syscalls > gpurun_out/syscalls35.json 2> gpurun_out/syscalls35.err
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --cache-control none --csv --log-file gpurun_out/launches35.csv python bench.py --steps 2 --warmup 1 --no-extras --no-cpu-baseline > gpurun_out/ncu35.log 2>&1; echo rc=$? >> gpurun_out/ncu35.log
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:scan_kernel -s 1 -c 1 -o gpurun_out/prof_scan35 python tools/prof_scan.py > gpurun_out/ncu_scan35.log 2>&1; echo rc=$? >> gpurun_out/ncu_scan35.log
-timeout 1500 ncu --set full --import-source on --clock-control none --cache-control none --replay-mode application -k regex:wc_kernel -c 1 -o gpurun_out/prof_wc35 python tools/prof_wc.py host 64 > gpurun_out/ncu_wc35.log 2>&1; echo rc=$? >> gpurun_out/ncu_wc35.log
+# sleep-hint experiment: learned hint vs none, poll interval 256 vs 1024 ns
+timeout 900 python bench.py --mode syscalls --cell-ms 60 > gpurun_out/sys35a.json 2> gpurun_out/sys35a.err
+GSYS_SLEEP_HINT=0 timeout 900 python bench.py --mode syscalls --cell-ms 60 > gpurun_out/sys35b.json 2> gpurun_out/sys35b.err
+GSYS_SLEEP_HINT=0 GSYS_POLL_NS_HOST=1024 timeout 900 python bench.py --mode syscalls --cell-ms 60 > gpurun_out/sys35c.json 2> gpurun_out/sys35c.err
+GSYS_SLEEP_HINT=0 GSYS_POLL_NS_HOST=4096 timeout 900 python bench.py --mode syscalls --cell-ms 60 > gpurun_out/sys35d.json 2> gpurun_out/sys35d.err
