@@ -67,6 +67,9 @@ struct gsys_dev_ctx {
     unsigned pull_big_bytes;        /* pull area of each slot s with s % 32 == 0 (0: none)      */
     unsigned char* pull_big;        /* host-mapped [(nslots / 32) * pull_big_bytes]            */
     unsigned no_hint;               /* 1: no learned pre-poll sleep (env GSYS_SLEEP_HINT=0)     */
+    unsigned memop_completion;      /* 1 (default): DMA'd blocking calls complete by a stream
+                                       memop into `mirror`; 0 (env GSYS_COMPLETION=host): by a
+                                       host store into `hdone` once the DMA has drained          */
 };
 
 #ifdef __CUDACC__
@@ -358,7 +361,7 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         st_release_gpu(&c->claim[s], 0u);
         return 0;
     }
-    long long r = wait_done(c, s, seq, (flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) != 0u,
+    long long r = wait_done(c, s, seq, !c->memop_completion || (flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) != 0u,
                             (flags & GSYS_F_NOHINT) != 0u);
     if (psrc != nullptr && r > 0) {
         if (po != nullptr) {   /* the work-group copies and releases (wg_call) */

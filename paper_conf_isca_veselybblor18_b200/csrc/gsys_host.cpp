@@ -325,6 +325,7 @@ struct Instance {
     gsys_dev_ctx* ctx_d = nullptr;
     cudaStream_t ctl = nullptr;
     bool mem64 = true;
+    bool memop_completion = false;      // see gsys_dev_ctx::memop_completion
 
     // service
     std::vector<Worker*> workers;
@@ -954,7 +955,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         memset(&op, 0, sizeof op);
         if (blocking) {
             const uint64_t word = ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret;
-            if (r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) {
+            if (!I->memop_completion || (r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL))) {
                 if (r.dma) { need_sync = true; continue; }
                 if (r.ok) {
                     __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
@@ -1007,7 +1008,8 @@ void Worker::process(uint64_t h0, uint32_t n) {
         for (uint32_t i = 0; i < n; i++) {
             Req& r = reqs[i];
             const bool nb = (r.flags & GSYS_NONBLOCKING) != 0;
-            if (!r.dma || (!nb && !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)))) continue;
+            if (!r.dma || (!nb && I->memop_completion && !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL))))
+                continue;
             gsys_slot* sl = I->area_h + r.slot;
             if (r.ok) {
                 __atomic_store_n(&sl->state, nb ? (uint32_t)GSYS_FREE : (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
@@ -1155,6 +1157,12 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // 256 ns: a 4 KiB pread round trip drops from 16.1 to 9.9 us vs 4 us polling, and the
     // wordcount (pollers sharing the PCIe link with the scan) is unchanged (profiles/r01_latency.json)
     c.poll_ns_host = (ev && atoi(ev) > 0) ? (unsigned)atoi(ev) : 256u;
+    ev = getenv("GSYS_COMPLETION");
+    // default memop: a host-store completion must first wait for the DMA (an event synchronize per
+    // bundle), which measured slower for device staging (42.5 vs 46.7 GB/s at 256 KiB chunks) and
+    // no faster for 4 KiB preads (profiles/r01_completion_paths.json)
+    c.memop_completion = (ev && strcmp(ev, "host") == 0) ? 0u : 1u;
+    I->memop_completion = c.memop_completion != 0;
     ev = getenv("GSYS_SLEEP_HINT");
     c.no_hint = (ev && atoi(ev) == 0) ? 1u : 0u;
     c.pull_big_bytes = I->pull_bytes;
