@@ -178,9 +178,6 @@ struct McArgs {
 };
 
 __device__ __forceinline__ unsigned be16(const unsigned char* p) { return ((unsigned)p[0] << 8) | p[1]; }
-__device__ __forceinline__ unsigned be32(const unsigned char* p) {
-    return ((unsigned)p[0] << 24) | ((unsigned)p[1] << 16) | ((unsigned)p[2] << 8) | p[3];
-}
 __device__ __forceinline__ void put_be16(unsigned char* p, unsigned v) { p[0] = (unsigned char)(v >> 8); p[1] = (unsigned char)v; }
 __device__ __forceinline__ void put_be32(unsigned char* p, unsigned v) {
     p[0] = (unsigned char)(v >> 24); p[1] = (unsigned char)(v >> 16); p[2] = (unsigned char)(v >> 8); p[3] = (unsigned char)v;
