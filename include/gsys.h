@@ -123,6 +123,11 @@ int gsys_set_coalesce_window(uint32_t us);
  * the union inside a coalesced bundle (north_star extension, reading A8). on = 0/1. */
 int gsys_set_merge(int on);
 
+/* Fault injection for tests (SURVEY.md sec. 5 "failure detection"): from now on every pread whose
+ * offset equals `offset` completes with -err without being executed (err 0 turns it off).  The
+ * GPU caller sees the POSIX error convention of reading A4/A11.  0, -ENODEV, -EINVAL. */
+int gsys_set_fault(int32_t err, int64_t offset);
+
 /* Protocol tracing (debug): on = 1 records every slot transition (GPU and host side) into
  * trace buffers readable with gsys_trace_read(); capacity = max records per side. */
 int gsys_set_trace(int on, uint32_t capacity);

@@ -198,6 +198,7 @@ struct Req {
     bool ok;
     bool dma;      // a host->device copy was queued for this request
     bool parked;   // blocking recvfrom on an empty socket: completed later by service_parked()
+    bool faulted;  // fault injection (gsys_set_fault): completed with the injected -errno, not executed
 };
 
 // A blocking recvfrom that found no datagram does not hold a service thread (reading B11): the
@@ -336,6 +337,9 @@ struct Instance {
     std::atomic<uint32_t> coalesce_max{8};
     std::atomic<uint32_t> window_us{0};
     std::atomic<int> merge{1};
+    std::atomic<int> fault_err{0};          // gsys_set_fault: preads at fault_off fail with -fault_err
+    std::atomic<int64_t> fault_off{-1};
+    std::atomic<uint64_t> st_faults{0};
     std::atomic<uint64_t> gen{1};          // pointer-cache generation
     std::atomic<uint64_t> kick{0};
     std::mutex sleep_mu;
@@ -833,6 +837,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         r.ret = 0;
         r.dma = false;
         r.parked = false;
+        r.faulted = false;
         // "atomically switches any ready system call requests to the processing state" (P24.20)
         uint32_t expect = GSYS_READY;
         r.ok = __atomic_compare_exchange_n((uint32_t*)&I->area_h[r.slot].state, &expect, (uint32_t)GSYS_PROCESSING,
@@ -842,11 +847,24 @@ void Worker::process(uint64_t h0, uint32_t n) {
         I->st_nr[nr_index(r.nr)].fetch_add(1, std::memory_order_relaxed);
     }
 
+    // ---- fault injection (tests): the pread at the chosen offset fails without being executed
+    std::vector<bool> done(n, false);
+    if (const int ferr = I->fault_err.load(std::memory_order_relaxed)) {
+        const int64_t foff = I->fault_off.load(std::memory_order_relaxed);
+        for (uint32_t i = 0; i < n; i++) {
+            Req& r = reqs[i];
+            if (r.ok && r.nr == GSYS_NR_PREAD64 && (int64_t)r.a[3] == foff) {
+                r.ret = -(int64_t)ferr;
+                r.faulted = true;
+                done[i] = true;
+                I->st_faults.fetch_add(1, std::memory_order_relaxed);
+            }
+        }
+    }
     // ---- execute: preads first through the merge planner (reading A8), then the rest in order
     midx.clear();
     for (uint32_t i = 0; i < n; i++)
-        if (reqs[i].ok && reqs[i].nr == GSYS_NR_PREAD64) midx.push_back(i);
-    std::vector<bool> done(n, false);
+        if (reqs[i].ok && reqs[i].nr == GSYS_NR_PREAD64 && !reqs[i].faulted) midx.push_back(i);
     if (midx.size() > 1 && I->merge.load(std::memory_order_relaxed)) {
         uint32_t m = (uint32_t)midx.size();
         mfd.resize(m); moff.resize(m); mlen.resize(m); morder.resize(m); mgroup.resize(m);
@@ -1265,6 +1283,15 @@ int gsys_set_coalesce_window(uint32_t us) {
     Instance* I = current();
     if (!I) return -ENODEV;
     I->window_us.store(us);
+    return 0;
+}
+
+int gsys_set_fault(int32_t err, int64_t offset) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    if (err < 0 || err > 4095) return -EINVAL;
+    I->fault_off.store(offset);
+    I->fault_err.store(err);
     return 0;
 }
 

@@ -62,6 +62,7 @@ SIGNATURES = {
     "gsys_set_coalesce_max": (ctypes.c_int, [_U32]),
     "gsys_set_coalesce_window": (ctypes.c_int, [_U32]),
     "gsys_set_merge": (ctypes.c_int, [ctypes.c_int]),
+    "gsys_set_fault": (ctypes.c_int, [ctypes.c_int32, ctypes.c_int64]),
     "gsys_set_trace": (ctypes.c_int, [ctypes.c_int, _U32]),
     "gsys_launch": (ctypes.c_int, [_P, _U32, _U32, _U32, _U32, _U32, _U32, _P, ctypes.c_size_t, _P]),
     "gsys_wait": (ctypes.c_int, [_P]),
@@ -140,6 +141,11 @@ def gsys_set_coalesce_window(us: int) -> int:
 
 def gsys_set_merge(on: bool) -> int:
     return _check(lib().gsys_set_merge(int(bool(on))), "gsys_set_merge")
+
+
+def gsys_set_fault(err: int, offset: int = -1) -> int:
+    """Test hook: preads at `offset` fail with -err (err 0 = off)."""
+    return _check(lib().gsys_set_fault(err, offset), "gsys_set_fault")
 
 
 def gsys_set_trace(on: bool, capacity: int = 0) -> int:

@@ -398,3 +398,34 @@ def test_pread_pull_sizes(file1m, gran, length, shift):
         off = ((c * iters + iters - 1) * length) % size
         want = data[off: off + length]
         assert bytes(host[shift + c * length: shift + c * length + len(want)]) == want
+
+
+# ---------------------------------------------------------------------------- fault injection
+from ownership import owned_counts  # noqa: E402
+
+
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST])
+def test_wordcount_injected_eio(file16m, staging):
+    """A failing pread (EIO injected by the service on chunk 37's request) reaches the work-group
+    as -EIO (POSIX convention), that chunk is not scanned, every other chunk is: the histogram
+    equals the oracle's whole-file counts minus the counts the failed chunk owns."""
+    p, census = file16m
+    data = open(p, "rb").read()
+    chunk = 256 << 10
+    k = 37
+    s = k * chunk
+    G.gsys_set_fault(5, s - 1)       # chunk k's request is [s - 1, e + 16)
+    try:
+        res = W.wordcount_files([p], WORDS, PATS, chunk=chunk, gflags=G.WG | G.BLOCKING | G.STRONG, staging=staging)
+    finally:
+        G.gsys_set_fault(0, -1)
+    rets = res.req_ret.tolist()
+    assert rets[k] == -5
+    reqs = plan.wordcount_chunk_requests(len(data), chunk)
+    assert [r for i, r in enumerate(rets) if i != k] == [plan.expected_pread_ret(len(data), r[3], r[4])
+                                                         for i, r in enumerate(reqs) if i != k]
+    want = oracle.count_tokens(data, WORDS) - owned_counts(data, s, min(s + chunk, len(data)), WORDS)
+    assert np.array_equal(as_u64(res.hist), want)
+    # the fault is off again: a clean run equals the census
+    res2 = W.wordcount_files([p], WORDS, PATS, chunk=chunk, staging=staging)
+    assert np.array_equal(as_u64(res2.hist), census)

@@ -254,3 +254,20 @@ def test_amr_release_rule():
     lv = [[1, 0, 2, 3], [0, 0, 1, 3], [2, 2, 0, 3]]
     assert plan.amr_released(lv) == [2, 1, 3, 0]
     assert plan.amr_released(lv, rss_ok=[False, True, True]) == [2, 2, 3, 0]
+
+
+def test_owned_counts_partition_sums_to_whole():
+    """tests/ownership.owned_counts (used by the GPU fault-injection test) is pinned here: for any
+    chunking, the per-chunk owned counts add up to the whole-text counts."""
+    from ownership import owned_counts
+    rng = np.random.default_rng(11)
+    words = [b"a", b"ab", b"ba", b"b_1", b"abc"]
+    for _ in range(300):
+        n = int(rng.integers(0, 60))
+        text = bytes(rng.choice(list(b"ab_1 ,\n"), size=n).tolist())
+        whole = oracle.count_tokens(text, words)
+        chunk = int(rng.integers(1, 12))
+        tot = np.zeros(len(words), dtype=np.uint64)
+        for s in range(0, n, chunk):
+            tot += owned_counts(text, s, min(s + chunk, n), words)
+        assert np.array_equal(tot, whole), (text, chunk)
