@@ -676,6 +676,41 @@ def run_memcached(a):
                                  "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
                                  "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
                                  "requests": len(pkts)})
+    # higher offered load (8 client sockets x 32 in flight): the GPU server with 128 work-groups
+    # against the CPU server with 4 and 8 threads (profiles/r01_memcached_load_sweep.jsonl)
+    keys, vals = MC.dataset(64 * 16 * 3 // 4, vlen=1024)
+    table = dict(zip(keys, vals))
+    pkts = [MC.encode_get(i, k) for i, k in enumerate(MC.requests(keys, 60000))]
+    kb, ko, kl, vb, vo, vl = MC.pack(keys, vals)
+    for send in ("blocking", "nonblocking"):
+        sg = G.WG | G.RELAXED | (G.NONBLOCKING if send == "nonblocking" else G.BLOCKING)
+        resp, lat, secs, _ = W.mc_serve_run(keys, vals, pkts, nwg=128, nbuckets=64, bucket_cap=32, client_threads=8,
+                                            window=32, send_gflags=sg)
+        ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
+        lat_us = np.array(lat, dtype=np.float64) / 1e3
+        out["cases"].append({"server": "gpu", "sendto": send, "elements_per_bucket": 16, "work_groups": 128,
+                             "in_flight": 256, "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
+                             "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
+                             "requests": len(pkts)})
+    for st in (4, 8):
+        sock = MC.udp_server_socket()
+        stop = ctypes.c_int(0)
+        th = threading.Thread(target=lambda: oracle.lib().oracle_mc_serve(
+            sock.fileno(), st, kb.ctypes.data, ko.ctypes.data, kl.ctypes.data, vb.ctypes.data, vo.ctypes.data,
+            vl.ctypes.data, len(keys), 64, ctypes.addressof(stop)))
+        th.start()
+        try:
+            resp, lat, secs = MC.run_client(sock.getsockname()[1], pkts, nthreads=8, window=32)
+        finally:
+            stop.value = 1
+            th.join()
+            sock.close()
+        lat_us = np.array(lat, dtype=np.float64) / 1e3
+        ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
+        out["cases"].append({"server": "cpu-oracle", "threads": st, "elements_per_bucket": 16, "in_flight": 256,
+                             "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
+                             "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
+                             "requests": len(pkts)})
     out["host_cores"] = nthr
     out["service_threads"] = G.gsys_stats()["threads"]
     print(json.dumps(out), flush=True)
