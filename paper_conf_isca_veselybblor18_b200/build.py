@@ -32,7 +32,7 @@ def _stale() -> bool:
     return any(os.path.getmtime(p) > t for p in SOURCES + HEADERS + [__file__])
 
 
-def build(force: bool = False, verbose: bool = False, defines=(), out: str = "") -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = "", host_flags=(), link=()) -> str:
     """Compile libgsys.so; `defines`/`out` build a diagnostic variant elsewhere (tools/)."""
     if not out and not force and not _stale():
         return LIB
@@ -40,7 +40,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = "")
     build_dir = os.path.join(PKG, "build" + ("_" + os.path.basename(out) if out else ""))
     os.makedirs(build_dir, exist_ok=True)
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3,-Wall", "-I", INCLUDE, "-I", CSRC,
-              *["-D" + d for d in defines]]
+              *["-D" + d for d in defines], *[x for f in host_flags for x in ("-Xcompiler", f)]]
     for src in SOURCES:
         obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         cmd = [NVCC, *common, *ARCH, "-c", src, "-o", obj]
@@ -53,7 +53,7 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str = "")
     target = out or LIB
     tmp = target + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs,
-                           "-Xlinker", "--no-undefined", "-lpthread", "-ldl", "-lrt"])
+                           "-Xlinker", "--no-undefined", "-lpthread", "-ldl", "-lrt", *link])
     os.replace(tmp, target)
     return target
 

@@ -829,11 +829,14 @@ void Worker::process(uint64_t h0, uint32_t n) {
         uint64_t e = __atomic_load_n(&I->ring_h[(h0 + i) & mask], __ATOMIC_ACQUIRE);
         Req& r = reqs[i];
         r.slot = (uint32_t)e;
-        volatile gsys_slot* sl = (volatile gsys_slot*)(I->area_h + r.slot);
-        r.nr = sl->nr;
-        r.flags = sl->flags;
-        r.seq = sl->seq;
-        for (int k = 0; k < 6; k++) r.a[k] = sl->args[k];
+        // the line was written by the GPU before its doorbell entry (fence.acq_rel.sys + the entry
+        // load above); plain atomic loads, since another worker may still be storing args[0] of the
+        // slot's previous request (ordered only through the GPU, which the C++ model cannot see)
+        gsys_slot* sl = I->area_h + r.slot;
+        r.nr = __atomic_load_n(&sl->nr, __ATOMIC_RELAXED);
+        r.flags = __atomic_load_n(&sl->flags, __ATOMIC_RELAXED);
+        r.seq = __atomic_load_n(&sl->seq, __ATOMIC_RELAXED);
+        for (int k = 0; k < 6; k++) r.a[k] = __atomic_load_n(&sl->args[k], __ATOMIC_RELAXED);
         r.ret = 0;
         r.dma = false;
         r.parked = false;
