@@ -11,9 +11,18 @@ d = "/dev/shm/gsys_san"
 os.makedirs(d, exist_ok=True)
 p = os.path.join(d, "f.txt")
 inputs.write_file(p, 1, 0, (1 << 20) + 77, grep_plants=True)
-for st in (G.STAGE_HOST, G.STAGE_DEVICE):
+for st in (G.STAGE_HOST, G.STAGE_DEVICE, G.STAGE_MIXED(5)):
     r = W.wordcount_files([p], words, pats, chunk=64 << 10, staging=st, blocks=8)
     print("wc", st, int(r.hist.sum()), r.wait_rc)
+# pull path (reading B12): 4113-byte work-group preads into unaligned device lines
+r = W.wordcount_files([p], words, pats, chunk=4096, staging=G.STAGE_DEVICE, blocks=8)
+print("wc-pull", int(r.hist.sum()), r.wait_rc)
+fd = os.open(p, os.O_RDONLY)
+dbuf = torch.zeros(64 * 1000 + 64, dtype=torch.uint8, device="cuda")
+for fl, ln in ((G.WG | G.BLOCKING, 1000), (G.WI | G.BLOCKING, 200), (G.KERNEL | G.BLOCKING | G.RELAXED, 100)):
+    n, ret, lat, sm, rc = W.bench_calls("pread", fl, 4, 64, 2, fd, ln, (1 << 20), dbuf[1:], want_sum=True)
+    print("pull", fl, rc, int((ret == ln).sum()))
+os.close(fd)
 buf, _, _ = inputs.gen_bytes(2, 0, (1 << 20) + 5)
 t = torch.zeros(buf.size + 64, dtype=torch.uint8, device="cuda")
 t[:buf.size].copy_(torch.from_numpy(buf))
