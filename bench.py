@@ -301,7 +301,7 @@ def main():
     if not a.no_extras and rank == 0:   # after the timed region; rank 0 alone (shared host files)
         h2d_peak = measure_h2d(dev)
         extras["scan"] = scan_roofline(G, dev, corpus, words, pats, chunk)
-        extras["syscalls"] = wg_syscall_rate(G, W, dev)
+        extras["syscalls"] = wg_syscall_rate(G, W, dev, corpus.paths[0])
         extras["config1"] = config1_latency(G, W, dev, words, pats, a.root)
     kernel_s = dev_s / a.steps
     algo_bytes = my_bytes + sum(((s + chunk - 1) // chunk) * 17 for s in of.sizes)   # chunk + halo
@@ -334,6 +334,11 @@ def main():
         dist.barrier()
     if rank == 0:
         syscalls_per_step = st["requests"] / a.steps
+        if cpu_baseline and "syscalls" in extras:   # WG syscall rates against the oracle's direct rates
+            for k, cell in extras["syscalls"].items():
+                base = cpu_baseline["pread4k_direct_calls_per_s" if k.startswith("pread") else
+                                    "getrusage_direct_calls_per_s"]
+                cell["frac_of_oracle_direct"] = cell["calls_per_s"] / base if base else None
         out = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": a.steps,
                "warmup": a.warmup, "ms_per_step": dev_s / a.steps * 1e3, "higher_is_better": True,
                "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
@@ -346,7 +351,7 @@ def main():
                "clocks": clocks,
                "parity": {"hist_equals_generator_census": hist_ok},
                "secondary": {"wg_syscalls_per_s_in_wordcount": syscalls_per_step * world / (dev_s / a.steps),
-                             **({"getrusage_wg": extras["syscalls"]} if "syscalls" in extras else {}),
+                             **({"syscalls_wg": extras["syscalls"]} if "syscalls" in extras else {}),
                              **({"config1_16MiB": extras["config1"]} if "config1" in extras else {}),
                              **({"scan_hbm": extras["scan"]} if "scan" in extras else {})},
                "service": {"threads": st["threads"], "coalesce_max": st["coalesce_max"],
@@ -455,19 +460,39 @@ def config1_latency(G, W, dev, words, pats, root):
     return out
 
 
-def wg_syscall_rate(G, W, dev):
-    """getrusage(RUSAGE_SELF) at WG granularity, blocking: 4 WGs/SM x 256 threads x 20 calls."""
+def wg_syscall_rate(G, W, dev, path):
+    """The metric's other half, "GPU-issued syscalls/sec (WG granularity)": 592 work-groups
+    (4/SM x 256 threads), each cell calibrated then run for >= 100 ms of calls.  getrusage blocking
+    and non-blocking; 4 KiB preads into device memory, blocking (the pull path, reading B12)."""
     import torch
-    blocks, threads, iters = 592, 256, 20
-    W.bench_calls("getrusage", G.WG | G.BLOCKING | G.RELAXED, blocks, threads, 2)
-    torch.cuda.synchronize()
-    t0 = time.perf_counter()
-    _, ret, lat, _, rc = W.bench_calls("getrusage", G.WG | G.BLOCKING | G.RELAXED, blocks, threads, iters)
-    dt = time.perf_counter() - t0
-    lat_us = (lat.double() / 1e3).cpu()
-    return {"calls_per_s": blocks * iters / dt, "callers": blocks, "iters": iters,
-            "lat_p50_us": float(lat_us.median()), "lat_p99_us": float(lat_us.quantile(0.99)),
-            "all_ok": bool((ret == 0).all())}
+    blocks, threads = 592, 256
+    size = os.path.getsize(path)
+    fd = os.open(path, os.O_RDONLY)
+    dbuf = torch.empty(blocks * 4096, dtype=torch.uint8, device=dev)
+    out = {}
+    try:
+        for name, kind, flags in (("getrusage_blocking", "getrusage", G.WG | G.BLOCKING | G.RELAXED),
+                                  ("getrusage_nonblocking", "getrusage", G.WG | G.NONBLOCKING | G.RELAXED),
+                                  ("pread4k_device_blocking", "pread", G.WG | G.BLOCKING | G.RELAXED)):
+            kw = dict(fd=fd, length=4096, size=size, d_buf=dbuf) if kind == "pread" else {}
+            iters = 20
+            for _ in range(2):   # calibration pass, then the >= 100 ms pass
+                torch.cuda.synchronize()
+                t0 = time.perf_counter()
+                _, ret, lat, _, rc = W.bench_calls(kind, flags, blocks, threads, iters, **kw)
+                dt = time.perf_counter() - t0
+                rate = blocks * iters / dt
+                iters = int(min(max(20, rate * 0.1 / blocks), 4000))
+            lat_us = (lat.double() / 1e3).cpu()
+            blocking = not (flags & G.NONBLOCKING)
+            ok = bool((ret == (4096 if kind == "pread" else 0)).all()) if blocking else bool((ret == 0).all())
+            out[name] = {"calls_per_s": rate, "callers": blocks, "seconds": dt,
+                         "lat_p50_us": float(lat_us.median()) if blocking else None,
+                         "lat_p99_us": float(lat_us.quantile(0.99)) if blocking else None,
+                         "all_ok": ok and rc == 0}
+    finally:
+        os.close(fd)
+    return out
 
 
 def cpu_baseline_leg(a, corpus, words, pats, chunk):
@@ -478,6 +503,11 @@ def cpu_baseline_leg(a, corpus, words, pats, chunk):
     oracle.corpus(sample[:1], words, pats, chunk=chunk, nthreads=nthr)
     _, _, secs, _ = oracle.corpus(sample, words, pats, chunk=chunk, nthreads=nthr)
     rate = oracle.syscall_rate("getrusage", nthr, 200000)
+    fd = os.open(corpus.paths[0], os.O_RDONLY)
+    try:
+        prate = oracle.syscall_rate("pread", nthr, 100000, fd, 4096, os.path.getsize(corpus.paths[0]))
+    finally:
+        os.close(fd)
     _, _, secs1, _ = oracle.corpus(sample[:4], words, pats, chunk=chunk, nthreads=1)
     one_thread = sum(os.path.getsize(p) for p in sample[:4]) / secs1 / 1e9
     pread_ceiling = {str(t): oracle.pread_only(corpus.paths[:64], t, chunk) / 1e9 for t in (1, 4, 8, nthr)}
@@ -485,7 +515,7 @@ def cpu_baseline_leg(a, corpus, words, pats, chunk):
             "host_pread_only_GBps_by_threads": pread_ceiling, "value_1_thread": one_thread,
             "sample": f"{len(sample)} of {a.files} files ({sbytes / 2**20:.0f} MiB): pread + scalar wordcount + grep, "
                       f"{nthr} pthreads, {cpu_model()}",
-            "getrusage_direct_calls_per_s": rate}
+            "getrusage_direct_calls_per_s": rate, "pread4k_direct_calls_per_s": prate}
 
 
 def run_syscalls(a):
