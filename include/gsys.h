@@ -128,6 +128,12 @@ int gsys_set_merge(int on);
  * GPU caller sees the POSIX error convention of reading A4/A11.  0, -ENODEV, -EINVAL. */
 int gsys_set_fault(int32_t err, int64_t offset);
 
+/* Phase diagnostics of blocking GPU calls (enabled with env GSYS_DIAG_PHASES=1 at gsys_init):
+ * out8 = {ns claiming, ns marshalling + publishing, ns waiting for completion, -, calls,
+ * ns of learned pre-poll sleep, completion polls, ns copying results + releasing}, summed over
+ * calls since the last reset.  0, -ENOTSUP (not enabled), -ENODEV, -EINVAL, -EIO. */
+int gsys_diag_phases(uint64_t* out8, int reset);
+
 /* Protocol tracing (debug): on = 1 records every slot transition (GPU and host side) into
  * trace buffers readable with gsys_trace_read(); capacity = max records per side. */
 int gsys_set_trace(int on, uint32_t capacity);

@@ -67,6 +67,7 @@ struct gsys_dev_ctx {
     unsigned pull_big_bytes;        /* pull area of each slot s with s % 32 == 0 (0: none)      */
     unsigned char* pull_big;        /* host-mapped [(nslots / 32) * pull_big_bytes]            */
     unsigned no_hint;               /* 1: no learned pre-poll sleep (env GSYS_SLEEP_HINT=0)     */
+    unsigned long long* diag;       /* device [8] phase accumulators (env GSYS_DIAG_PHASES=1) or null */
     unsigned memop_completion;      /* 1 (default): DMA'd blocking calls complete by a stream
                                        memop into `mirror`; 0 (env GSYS_COMPLETION=host): by a
                                        host store into `hdone` once the DMA has drained          */
@@ -112,6 +113,18 @@ __device__ __forceinline__ void st_v4_sys(void* p, uint4 v) {
 __device__ __forceinline__ uint4 ld_v4_sys(const uint4* p) {
     uint4 v;
     asm volatile("ld.relaxed.sys.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    return v;
+}
+/* Weak 16-byte load of a host-written result.  Used only after the caller's acquire of the
+ * completion word (ld.acquire.sys, which also invalidates this SM's L1) -- or, for the other
+ * threads of a work-group, after the Bar2 barrier that follows it -- so by the PTX memory model it
+ * observes everything the host wrote before its release store.  Weak loads of one thread are
+ * pipelined; strong .sys (or .cv) loads are issued one round trip at a time (a 144 B rusage cost
+ * 5 us that way, profiles/r01_phase_probe.jsonl). */
+__device__ __forceinline__ uint4 ld_v4_after_acquire(const uint4* p) {
+    uint4 v;
+    asm volatile("ld.global.v4.u32 {%0, %1, %2, %3}, [%4];"
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
     return v;
 }
@@ -244,12 +257,14 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         }
         unsigned polls = 0;
         const unsigned long long tp = globaltimer();
+        if (c->diag) { atomicAdd(c->diag + 5, (unsigned long long)hint); }
         for (;;) {
             v = ld_acquire_sys(m);
             polls++;
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(c->poll_ns_host);
         }
+        if (c->diag) atomicAdd(c->diag + 6, (unsigned long long)polls);
         if (!nohint) {
             unsigned long long nh = hint;
             if (polls <= 1) nh = hint - (hint >> 2);
@@ -302,8 +317,8 @@ __device__ __forceinline__ void store16(unsigned char* d, const uint4& v, long l
 }
 
 /* Copy r bytes of a pull area (16-byte aligned, host-mapped) to dst (any alignment); threads
- * tid = 0..nt-1 share the work.  Source loads are .sys-scope (never a stale L1 line of an earlier
- * pull of the same area) and issued four at a time per thread, so they overlap on the link. */
+ * tid = 0..nt-1 share the work, four pipelined loads at a time per thread (ld_v4_after_acquire:
+ * the caller acquired the completion word; the other threads follow it through Bar2). */
 __device__ __forceinline__ void pull_copy(const unsigned char* src, unsigned char* dst, long long r, unsigned tid,
                                           unsigned nt) {
     const unsigned n16 = (unsigned)((r + 15) >> 4);
@@ -311,10 +326,10 @@ __device__ __forceinline__ void pull_copy(const unsigned char* src, unsigned cha
     const uint4 z = make_uint4(0u, 0u, 0u, 0u);
     for (unsigned i = tid; i < n16; i += 4u * nt) {
         const unsigned i1 = i + nt, i2 = i + 2u * nt, i3 = i + 3u * nt;
-        const uint4 v0 = ld_v4_sys(s4 + i);
-        const uint4 v1 = i1 < n16 ? ld_v4_sys(s4 + i1) : z;
-        const uint4 v2 = i2 < n16 ? ld_v4_sys(s4 + i2) : z;
-        const uint4 v3 = i3 < n16 ? ld_v4_sys(s4 + i3) : z;
+        const uint4 v0 = ld_v4_after_acquire(s4 + i);
+        const uint4 v1 = i1 < n16 ? ld_v4_after_acquire(s4 + i1) : z;
+        const uint4 v2 = i2 < n16 ? ld_v4_after_acquire(s4 + i2) : z;
+        const uint4 v3 = i3 < n16 ? ld_v4_after_acquire(s4 + i3) : z;
         store16(dst + 16u * i, v0, r - 16ll * i);
         if (i1 < n16) store16(dst + 16u * i1, v1, r - 16ll * i1);
         if (i2 < n16) store16(dst + 16u * i2, v2, r - 16ll * i2);
@@ -337,7 +352,9 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
                                                  const unsigned long long a[6], const InlineIO& io = InlineIO(),
                                                  PullOut* po = nullptr) {
     const bool blocking = !(flags & GSYS_NONBLOCKING);
+    const unsigned long long d0 = c->diag ? globaltimer() : 0ull;
     unsigned s = claim(c, blocking);
+    const unsigned long long d1 = c->diag ? globaltimer() : 0ull;
     const unsigned char* psrc = nullptr;
     if (nr == GSYS_NR_PREAD64 && blocking && !(flags & GSYS_HOSTBUF)) {
         psrc = pull_src(c, s, a[2], po != nullptr);
@@ -361,11 +378,21 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         st_release_gpu(&c->claim[s], 0u);
         return 0;
     }
+    const unsigned long long d2 = c->diag ? globaltimer() : 0ull;
     long long r = wait_done(c, s, seq, !c->memop_completion || (flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) != 0u,
                             (flags & GSYS_F_NOHINT) != 0u);
+    if (c->diag) {   /* phase diagnostics: claim, marshal+publish, wait, (copy+release below) */
+        const unsigned long long d3 = globaltimer();
+        atomicAdd(c->diag + 0, d1 - d0);
+        atomicAdd(c->diag + 1, d2 - d1);
+        atomicAdd(c->diag + 2, d3 - d2);
+        atomicAdd(c->diag + 4, 1ull);
+        atomicAdd(c->diag + 7, (unsigned long long)-(long long)d3);   /* + end time below */
+    }
     if (psrc != nullptr && r > 0) {
         if (po != nullptr) {   /* the work-group copies and releases (wg_call) */
             po->src = psrc; po->slot = s; po->seq = seq;
+            if (c->diag) atomicAdd(c->diag + 7, globaltimer());
             return r;
         }
         pull_copy(psrc, reinterpret_cast<unsigned char*>(a[1]), r, 0u, 1u);
@@ -373,20 +400,18 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     if (io.out != nullptr && r >= 0) {
         const uint4* src = reinterpret_cast<const uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
         uint4* dst = reinterpret_cast<uint4*>(io.out);
-        // loads four at a time (not one PCIe round trip per 16 B), then the stores
+        // every piece's load is issued before the first store: one PCIe round trip for the result
         const unsigned n16 = io.out_bytes / 16u;
-        for (unsigned i = 0; i < n16; i += 4u) {
-            const uint4 v0 = ld_v4_sys(src + i);
-            const uint4 v1 = i + 1u < n16 ? ld_v4_sys(src + i + 1u) : v0;
-            const uint4 v2 = i + 2u < n16 ? ld_v4_sys(src + i + 2u) : v0;
-            const uint4 v3 = i + 3u < n16 ? ld_v4_sys(src + i + 3u) : v0;
-            dst[i] = v0;
-            if (i + 1u < n16) dst[i + 1u] = v1;
-            if (i + 2u < n16) dst[i + 2u] = v2;
-            if (i + 3u < n16) dst[i + 3u] = v3;
-        }
+        uint4 t[GSYS_INLINE_BYTES / 16];
+#pragma unroll
+        for (unsigned i = 0; i < GSYS_INLINE_BYTES / 16; i++)
+            if (i < n16) t[i] = ld_v4_after_acquire(src + i);
+#pragma unroll
+        for (unsigned i = 0; i < GSYS_INLINE_BYTES / 16; i++)
+            if (i < n16) dst[i] = t[i];
     }
     release(c, s, seq);
+    if (c->diag) atomicAdd(c->diag + 7, globaltimer());
     return r;
 }
 

@@ -327,6 +327,7 @@ struct Instance {
     cudaStream_t ctl = nullptr;
     bool mem64 = true;
     bool memop_completion = false;      // see gsys_dev_ctx::memop_completion
+    unsigned long long* diag_d = nullptr;   // GSYS_DIAG_PHASES accumulators (device)
 
     // service
     std::vector<Worker*> workers;
@@ -1184,6 +1185,12 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // no faster for 4 KiB preads (profiles/r01_completion_paths.json)
     c.memop_completion = (ev && strcmp(ev, "host") == 0) ? 0u : 1u;
     I->memop_completion = c.memop_completion != 0;
+    ev = getenv("GSYS_DIAG_PHASES");
+    if (ev && atoi(ev) > 0) {
+        if (cudaMalloc((void**)&c.diag, 64) != cudaSuccess) return fail(-ENOMEM);
+        cudaMemset(c.diag, 0, 64);
+        I->diag_d = c.diag;
+    }
     ev = getenv("GSYS_SLEEP_HINT");
     c.no_hint = (ev && atoi(ev) == 0) ? 1u : 0u;
     c.pull_big_bytes = I->pull_bytes;
@@ -1286,6 +1293,16 @@ int gsys_set_coalesce_window(uint32_t us) {
     Instance* I = current();
     if (!I) return -ENODEV;
     I->window_us.store(us);
+    return 0;
+}
+
+int gsys_diag_phases(uint64_t* out8, int reset) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    if (!I->diag_d) return -ENOTSUP;
+    if (!out8) return -EINVAL;
+    if (cudaMemcpy(out8, I->diag_d, 64, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+    if (reset && cudaMemset(I->diag_d, 0, 64) != cudaSuccess) return -EIO;
     return 0;
 }
 

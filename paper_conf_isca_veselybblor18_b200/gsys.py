@@ -63,6 +63,7 @@ SIGNATURES = {
     "gsys_set_coalesce_window": (ctypes.c_int, [_U32]),
     "gsys_set_merge": (ctypes.c_int, [ctypes.c_int]),
     "gsys_set_fault": (ctypes.c_int, [ctypes.c_int32, ctypes.c_int64]),
+    "gsys_diag_phases": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int]),
     "gsys_set_trace": (ctypes.c_int, [ctypes.c_int, _U32]),
     "gsys_launch": (ctypes.c_int, [_P, _U32, _U32, _U32, _U32, _U32, _U32, _P, ctypes.c_size_t, _P]),
     "gsys_wait": (ctypes.c_int, [_P]),
@@ -141,6 +142,16 @@ def gsys_set_coalesce_window(us: int) -> int:
 
 def gsys_set_merge(on: bool) -> int:
     return _check(lib().gsys_set_merge(int(bool(on))), "gsys_set_merge")
+
+
+def gsys_diag_phases(reset: bool = True) -> dict:
+    """Per-call phase sums of blocking calls (needs GSYS_DIAG_PHASES=1 at init)."""
+    out = (ctypes.c_uint64 * 8)()
+    _check(lib().gsys_diag_phases(out, int(bool(reset))), "gsys_diag_phases")
+    n = max(out[4], 1)
+    return {"calls": out[4], "claim_us": out[0] / n / 1e3, "publish_us": out[1] / n / 1e3,
+            "wait_us": out[2] / n / 1e3, "copy_release_us": out[7] / n / 1e3, "hint_sleep_us": out[5] / n / 1e3,
+            "polls_per_call": out[6] / n}
 
 
 def gsys_set_fault(err: int, offset: int = -1) -> int:
