@@ -128,6 +128,11 @@ __device__ __forceinline__ uint4 ld_v4_after_acquire(const uint4* p) {
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
     return v;
 }
+#ifdef GSYS_POLL_RELAXED_FENCE
+#define GSYS_POLL_LOAD ld_relaxed_sys
+#else
+#define GSYS_POLL_LOAD ld_acquire_sys
+#endif
 __device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
     unsigned long long v; asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory"); return v;
@@ -234,7 +239,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         const unsigned long long* m = c->mirror + s;
         unsigned ns = 64;
         for (;;) {
-            v = ld_acquire_sys(m);
+            v = GSYS_POLL_LOAD(m);
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(ns);
             ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
@@ -259,7 +264,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
         const unsigned long long tp = globaltimer();
         if (c->diag) { atomicAdd(c->diag + 5, (unsigned long long)hint); }
         for (;;) {
-            v = ld_acquire_sys(m);
+            v = GSYS_POLL_LOAD(m);
             polls++;
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(c->poll_ns_host);
@@ -272,6 +277,9 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             c->lat_hint[s] = nh > 200000ull ? 200000u : (unsigned)nh;
         }
     }
+#ifdef GSYS_POLL_RELAXED_FENCE
+    fence_acq_rel_sys();   /* diagnostic variant: relaxed polls + one fence (round-1 original) */
+#endif
     /* the polls are acquire loads: the payload (device memory after the DMA, or the inline / pull
      * area the host wrote before its release store) is read after the completion word, with no
      * separate system-scope fence (a MEMBAR.SYS per call) */
