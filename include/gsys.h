@@ -261,8 +261,11 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
                    uint32_t gflags, uint32_t staging, uint32_t blocks, uint32_t threads, void* stream);
 
 /* Same scan over text already resident in device memory (no syscalls): the standalone scan
- * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n]; file boundaries are not
- * modelled (one file).  Adds into d_hist; d_hit (may be NULL) set to 1 if any pattern occurs. */
+ * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n] (16-byte aligned); file
+ * boundaries are not modelled (one file).  Adds into d_hist; d_hit (may be NULL) set to 1 if any
+ * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 512, else a
+ * multiple of 32 up to 768 (the 129-column table is used when it fits beside the warps' staging,
+ * else the 77-column one).  -EINVAL on bad sizes/alignment, -ENODEV before gsys_init. */
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
                      const char* dict, const uint8_t* dlen, uint32_t ndict,
                      const char* pats, const uint8_t* plen, uint32_t npat,

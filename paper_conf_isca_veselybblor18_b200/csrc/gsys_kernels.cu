@@ -317,7 +317,7 @@ struct ScanArgs {
     unsigned chunk, pad_;
 };
 
-__global__ void __launch_bounds__(512, 1) scan_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(768, 1) scan_kernel(ScanArgs a) {
     __shared__ int s_hit;
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
@@ -634,7 +634,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
     if (threads == 0) threads = 512;
-    if (threads % 32 || threads > 512) return -EINVAL;
+    if (threads % 32 || threads > 768) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
