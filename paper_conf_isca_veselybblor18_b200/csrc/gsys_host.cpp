@@ -137,10 +137,15 @@ class BounceRing {
     void retire_front() {
         if (!q_.front().committed) commit();
         Region f = q_.front();
-        ops_->wait(f.tok);
-        if (f.last) ops_->recycle(f.tok);
+        // one wait per token: the regions of one commit share it (the driver call is not free)
+        if (!waited_valid_ || !(waited_ == f.tok)) ops_->wait(f.tok);
+        waited_ = f.tok;
+        waited_valid_ = true;
+        if (f.last) { ops_->recycle(f.tok); waited_valid_ = false; }
         q_.pop_front();
     }
+    Token waited_{};
+    bool waited_valid_ = false;
     size_t cap_, head_ = 0, npending_ = 0;
     Ops* ops_;
     std::deque<Region> q_;
