@@ -1114,18 +1114,18 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     if (cudaHostAlloc((void**)&I->area_h, area_bytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
     memset(I->area_h, 0, area_bytes);
-    cudaHostGetDevicePointer((void**)&I->area_d, I->area_h, 0);
+    if (cudaHostGetDevicePointer((void**)&I->area_d, I->area_h, 0) != cudaSuccess) return fail(-EIO);
     size_t inl = (size_t)slots * GSYS_INLINE_BYTES;
     if (cudaHostAlloc((void**)&I->inline_h, inl, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
-    cudaHostGetDevicePointer((void**)&I->inline_d, I->inline_h, 0);
+    if (cudaHostGetDevicePointer((void**)&I->inline_d, I->inline_h, 0) != cudaSuccess) return fail(-EIO);
     {   // pull areas of the slots a work-group caller lands in (s % 32 == 0): GSYS_PULL_KB, default 16
         const char* pv = getenv("GSYS_PULL_KB");
         const long kb = pv ? atol(pv) : 16;
         I->pull_bytes = (kb > 0 && kb <= 1024) ? (uint32_t)kb << 10 : 0u;
         const size_t pb = (size_t)((slots + 31) / 32) * I->pull_bytes;
         if (pb && cudaHostAlloc((void**)&I->pull_h, pb, cudaHostAllocMapped | cudaHostAllocPortable) == cudaSuccess) {
-            cudaHostGetDevicePointer((void**)&I->pull_d, I->pull_h, 0);
+            if (cudaHostGetDevicePointer((void**)&I->pull_d, I->pull_h, 0) != cudaSuccess) return fail(-EIO);
         } else {
             cudaGetLastError();
             I->pull_h = nullptr;
@@ -1135,11 +1135,11 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     if (cudaHostAlloc((void**)&I->ring_h, (size_t)rc * 8, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
     memset(I->ring_h, 0, (size_t)rc * 8);
-    cudaHostGetDevicePointer((void**)&I->ring_d, I->ring_h, 0);
+    if (cudaHostGetDevicePointer((void**)&I->ring_d, I->ring_h, 0) != cudaSuccess) return fail(-EIO);
     if (cudaHostAlloc((void**)&I->hdone_h, (size_t)slots * 8, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
     memset(I->hdone_h, 0, (size_t)slots * 8);
-    cudaHostGetDevicePointer((void**)&I->hdone_d, I->hdone_h, 0);
+    if (cudaHostGetDevicePointer((void**)&I->hdone_d, I->hdone_h, 0) != cudaSuccess) return fail(-EIO);
     if (cudaMalloc(&I->claim_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     if (cudaMalloc(&I->seqs_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     if (cudaMalloc(&I->mirror_d, (size_t)slots * 8) != cudaSuccess) return fail(-ENOMEM);
@@ -1158,7 +1158,7 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     cudaMemset(I->krounds_d, 0, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS);
     cudaMemset(I->kblock_d, 0, (size_t)I->kblock_cap * GSYS_KSITES * 4);
     if (cudaMalloc(&I->ctx_d, sizeof(gsys_dev_ctx)) != cudaSuccess) return fail(-ENOMEM);
-    cudaStreamCreateWithFlags(&I->ctl, cudaStreamNonBlocking);
+    if (cudaStreamCreateWithFlags(&I->ctl, cudaStreamNonBlocking) != cudaSuccess) return fail(-EIO);
     gsys_dev_ctx& c = I->ctx_h;
     c.area = I->area_d;
     c.inline_buf = I->inline_d;
@@ -1228,8 +1228,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
         Worker* w = new Worker();
         w->inst = I;
         w->id = (int)t;
-        cudaStreamCreateWithFlags(&w->stream, cudaStreamNonBlocking);
-        if (cudaHostAlloc((void**)&w->bounce, bcap, cudaHostAllocDefault) != cudaSuccess) return fail(-ENOMEM);
+        if (cudaStreamCreateWithFlags(&w->stream, cudaStreamNonBlocking) != cudaSuccess) { delete w; return fail(-EIO); }
+        if (cudaHostAlloc((void**)&w->bounce, bcap, cudaHostAllocDefault) != cudaSuccess) { delete w; return fail(-ENOMEM); }
         w->bcap = bcap;
         w->ring = new BounceRing<cudaEvent_t, Worker::RingOps>(bcap, &w->ring_ops);
         w->reqs.reserve(4096);
