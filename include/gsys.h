@@ -239,8 +239,12 @@ int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap);
  *   pats, plen      host arrays: npat (<= 8) grep patterns, 17-byte stride, lengths 1..16.
  *   d_hist          DEVICE uint64[ndict]: whole-token counts are ADDED (reading A9).
  *   d_file_hits     DEVICE uint32[nfiles] (may be NULL): set to 1 for files containing a pattern.
- *   gflags          GSYS_WG (the paper's configuration for wordcount) + GSYS_BLOCKING +
- *                   GSYS_STRONG or GSYS_RELAXED; anything else is -EINVAL.
+ *   gflags          GSYS_WG (the paper's configuration for wordcount) + GSYS_STRONG or
+ *                   GSYS_RELAXED, and GSYS_BLOCKING (one pread, then the scan) or GSYS_NONBLOCKING
+ *                   (each work-group prefetches its next chunk into a second line with a
+ *                   non-blocking pread before scanning the current one; the slot's one-request
+ *                   rule orders them, reading A15; per-chunk returns are 0 and errors surface at
+ *                   gsys_wait, reading A4); another granularity is -EINVAL.
  *   staging         GSYS_STAGE_DEVICE: each work-group's pread lands in a device (HBM) line,
  *                   the host service DMAs it from its pinned bounce ring;  GSYS_STAGE_HOST: the
  *                   pread lands in a pinned host-mapped line ("syscall buffers" in system memory,

@@ -234,7 +234,33 @@ struct WcArgs {
     unsigned nfiles, nchunks, chunk, stride, gflags;
     unsigned host_staging;          // 0 device, 1 host, 2 mixed
     unsigned dev16;                 // mixed: chunks with (k mod 16) < dev16 use the device line
+    unsigned prefetch;              // 1: non-blocking preads, two lines per work-group (see below)
 };
+
+// One chunk of the global chunk queue: file f, owned range [s, e), request [off, off + len).
+struct WcChunk {
+    unsigned k, f;
+    long long size, s, e, off, len;
+};
+__device__ __forceinline__ bool wc_next_chunk(const WcArgs& a, unsigned* s_k, WcChunk& c) {
+    if (threadIdx.x == 0) *s_k = atomicAdd(a.next_chunk, 1u);
+    __syncthreads();
+    c.k = *s_k;
+    __syncthreads();   // s_k may be overwritten by the next call
+    if (c.k >= a.nchunks) return false;
+    unsigned lo = 0, hi = a.nfiles;     // largest f with chunk_base[f] <= k
+    while (hi - lo > 1) {
+        unsigned mid = (lo + hi) >> 1;
+        if (a.chunk_base[mid] <= c.k) lo = mid; else hi = mid;
+    }
+    c.f = lo;
+    c.size = (long long)a.sizes[c.f];
+    c.s = (long long)(c.k - a.chunk_base[c.f]) * a.chunk;
+    c.e = c.s + a.chunk < c.size ? c.s + a.chunk : c.size;
+    c.off = c.s ? c.s - 1 : 0;
+    c.len = c.e + 16 - c.off;
+    return true;
+}
 
 __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     // per-chunk grep flag, double-buffered by chunk parity: thread 0 clears the next chunk's flag
@@ -247,9 +273,66 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     const ScanTables& sT = *S.T;
     if (threadIdx.x == 0) { s_hit[0] = 0; s_hit[1] = 0; }
     __syncthreads();
-    unsigned char* const hbase = a.staging + (size_t)blockIdx.x * a.stride;
-    unsigned char* const dbase = a.host_staging == 2u ? a.staging_dev + (size_t)blockIdx.x * a.stride : hbase;
+    const size_t lines = a.prefetch ? 2u : 1u;
+    unsigned char* const hbase = a.staging + (size_t)blockIdx.x * a.stride * lines;
+    unsigned char* const dbase = a.host_staging == 2u ? a.staging_dev + (size_t)blockIdx.x * a.stride * lines : hbase;
     unsigned par = 0;
+    __shared__ unsigned s_kq;
+    if (a.prefetch) {
+        // Non-blocking work-group preads, double-buffered (P20.34-46 "non-blocking ... the GPU
+        // continues"): the read of the next chunk is issued before this chunk is scanned.  No
+        // separate wait is needed: a slot holds one request at a time (reading A15), so the next
+        // call's claim -- the next prefetch, or a blocking 0-byte pread at the end -- returns only
+        // after the host completed this one, and Bar2 hands that to the whole work-group.  A
+        // non-blocking pread returns 0 (A4): the scan takes the bytes a regular file of stable size
+        // returns (min(len, size - off)); an error surfaces at gsys_wait.
+        WcChunk c0, c1;
+        bool have = wc_next_chunk(a, &s_kq, c0);
+        unsigned cur = 0;
+        const unsigned nbflags = (a.gflags & ~GSYS_BLOCKING) | GSYS_NONBLOCKING;
+        auto line_of = [&](const WcChunk& c, unsigned ln, bool& hostbuf) {
+            hostbuf = a.host_staging == 1u || (a.host_staging == 2u && (c.k & 15u) >= a.dev16);
+            return (hostbuf ? hbase : dbase) + (size_t)ln * a.stride;
+        };
+        if (have) {
+            bool hb;
+            unsigned char* b = line_of(c0, 0, hb);
+            const long long r = gsys_pread(a.ctx, a.fds[c0.f], b + 16 - (c0.s - c0.off), (size_t)c0.len, c0.off,
+                                           nbflags | (hb ? GSYS_HOSTBUF : 0u));
+            if (threadIdx.x == 0 && a.req_ret) a.req_ret[c0.k] = r;
+        }
+        while (have) {
+            const bool more = wc_next_chunk(a, &s_kq, c1);
+            if (more) {
+                bool hb;
+                unsigned char* b = line_of(c1, cur ^ 1u, hb);
+                const long long r = gsys_pread(a.ctx, a.fds[c1.f], b + 16 - (c1.s - c1.off), (size_t)c1.len, c1.off,
+                                               nbflags | (hb ? GSYS_HOSTBUF : 0u));
+                if (threadIdx.x == 0 && a.req_ret) a.req_ret[c1.k] = r;
+            } else {
+                gsys_pread(a.ctx, a.fds[c0.f], hbase, 0, 0, a.gflags | GSYS_HOSTBUF);   // drain the slot
+            }
+            bool hb;
+            unsigned char* base = line_of(c0, cur, hb);
+            const bool grep = a.file_hits != nullptr && sT.npat > 0 && *(volatile unsigned*)&a.file_hits[c0.f] == 0u;
+            const long long valid_end = c0.off + c0.len < c0.size ? c0.off + c0.len : c0.size;
+            const long long own_end = c0.e < valid_end ? c0.e : valid_end;
+            S.hit = grep ? &s_hit[par] : nullptr;
+            if (own_end > c0.s) scan_range<LD_CG, false>(base + 16, c0.s, own_end, valid_end, S);
+            __syncthreads();   // this line is free for the prefetch issued next iteration
+            if (threadIdx.x == 0) {
+                if (grep && s_hit[par]) atomicExch(&a.file_hits[c0.f], 1u);
+                s_hit[par] = 0;
+            }
+            par ^= 1u;
+            c0 = c1;
+            have = more;
+            cur ^= 1u;
+        }
+        __syncthreads();
+        flush_hist(shist, nwarps, sT.ndict, a.hist);
+        return;
+    }
     // Chunks come from a global queue, not a static stride: a work-group takes the next chunk when
     // it is done with its last one, so the ~110 chunk latencies per work-group do not add up into a
     // tail set by the slowest of 296 work-groups.
@@ -521,7 +604,9 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
                    uint32_t blocks, uint32_t threads, void* stream) {
     gsys_dev_ctx* ctx = gsys_internal_ctx_d();
     if (!ctx) return -ENODEV;
-    if ((gflags & GSYS_GRAN_MASK) != GSYS_WG || (gflags & GSYS_NONBLOCKING)) return -EINVAL;
+    if ((gflags & GSYS_GRAN_MASK) != GSYS_WG) return -EINVAL;
+    const bool prefetch = (gflags & GSYS_NONBLOCKING) != 0;   // non-blocking: double-buffered prefetch
+    const size_t nlines = prefetch ? 2 : 1;
     const bool mixed = (staging & ~15u) == GSYS_STAGE_MIXED(0) && (staging & 15u) != 0u;
     if (staging > GSYS_STAGE_HOST && !mixed) return -EINVAL;
     if (nfiles == 0 || !fds || !sizes || !d_hist) return -EINVAL;
@@ -562,12 +647,12 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     unsigned char* stage = nullptr;
     unsigned char* stage_dev = nullptr;
     if (staging == GSYS_STAGE_HOST || mixed) {
-        rc = ensure_hstaging(W, stride * blocks);
+        rc = ensure_hstaging(W, stride * blocks * nlines);
         if (rc) return rc;
         cudaHostGetDevicePointer((void**)&stage, W->hstaging, 0);
     }
     if (staging == GSYS_STAGE_DEVICE || mixed) {
-        rc = ensure_staging(W, stride * blocks);
+        rc = ensure_staging(W, stride * blocks * nlines);
         if (rc) return rc;
         if (mixed) stage_dev = W->staging_d;
         else stage = W->staging_d;
@@ -587,6 +672,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     }
     a.host_staging = mixed ? 2u : (staging == GSYS_STAGE_HOST ? 1u : 0u);
     a.dev16 = mixed ? (staging & 15u) : 0u;
+    a.prefetch = prefetch ? 1u : 0u;
     a.hist = reinterpret_cast<unsigned long long*>(d_hist);
     a.file_hits = d_file_hits;
     a.req_ret = reinterpret_cast<long long*>(d_req_ret);
@@ -596,7 +682,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.nchunks = (unsigned)nch;
     a.chunk = chunk;
     a.stride = (unsigned)stride;
-    a.gflags = gflags;
+    a.gflags = gflags & ~GSYS_NONBLOCKING;   // the blocking flavour; prefetch derives the rest
     if (nch == 0) return 0;
     void* args[] = {&a};
     size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE);

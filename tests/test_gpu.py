@@ -429,3 +429,33 @@ def test_wordcount_injected_eio(file16m, staging):
     # the fault is off again: a clean run equals the census
     res2 = W.wordcount_files([p], WORDS, PATS, chunk=chunk, staging=staging)
     assert np.array_equal(as_u64(res2.hist), census)
+
+
+# ---------------------------------------------------------------------------- non-blocking prefetch
+@pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST, G.STAGE_MIXED(5)])
+@pytest.mark.parametrize("chunk,blocks,threads", [(4096, 7, 64), (256 << 10, 0, 256), (1 << 20, 1, 128)])
+def test_wordcount_nonblocking_prefetch(ragged_corpus, chunk, blocks, threads, staging):
+    """WG + non-blocking: each work-group prefetches its next chunk before scanning the current one
+    (two lines, ordered by the slot's one-request rule); histogram and grep set equal the oracle,
+    every call returns 0 (reading A4) and gsys_wait reports no error."""
+    c = ragged_corpus
+    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, blocks=blocks, threads=threads,
+                            gflags=G.WG | G.NONBLOCKING | G.RELAXED, staging=staging)
+    h, hits = oracle_hist_hits(c.paths)
+    assert res.wait_rc == 0
+    assert np.array_equal(as_u64(res.hist), h)
+    assert res.file_hits.tolist() == hits.tolist()
+    assert set(res.req_ret.tolist()) <= {0}
+
+
+def test_wordcount_nonblocking_full_corpus(tmpdir_shm):
+    """The bench corpus (8 GiB) through the prefetching configuration."""
+    import shutil
+    if shutil.disk_usage(tmpdir_shm).free < (10 << 30) and not os.path.exists(os.path.join(tmpdir_shm, "full8g")):
+        pytest.skip("tmpfs too small for the 8 GiB corpus")
+    c = inputs.make_corpus(512, 16 << 20, seed=inputs.SEED_CORPUS, root=tmpdir_shm, tag="full8g")
+    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=256 << 10, blocks=296,
+                            gflags=G.WG | G.NONBLOCKING | G.RELAXED, staging=G.STAGE_HOST)
+    assert res.wait_rc == 0
+    assert np.array_equal(as_u64(res.hist), c.census)
+    assert res.file_hits.tolist() == [1 if m else 0 for m in c.pmasks]

@@ -21,6 +21,7 @@ ap.add_argument("--chunk-kib", type=int, default=256)
 ap.add_argument("--blocks", type=int, default=0)
 ap.add_argument("--threads", type=int, default=256)
 ap.add_argument("--order", default="relaxed")
+ap.add_argument("--nonblocking", type=int, default=0, help="1: WG non-blocking prefetch pipeline")
 ap.add_argument("--cmax", type=int, default=8)
 ap.add_argument("--window", type=int, default=0)
 ap.add_argument("--merge", type=int, default=1)
@@ -36,7 +37,7 @@ G.gsys_set_profile(True)
 G.gsys_set_coalesce_max(a.cmax)
 G.gsys_set_coalesce_window(a.window)
 G.gsys_set_merge(a.merge)
-gflags = G.WG | G.BLOCKING | (G.RELAXED if a.order == "relaxed" else G.STRONG)
+gflags = G.WG | (G.NONBLOCKING if a.nonblocking else G.BLOCKING) | (G.RELAXED if a.order == "relaxed" else G.STRONG)
 of = W.OpenFiles(corpus.paths).__enter__()
 s = torch.cuda.Stream()
 h = torch.zeros(64, dtype=torch.int64, device="cuda")
