@@ -103,6 +103,11 @@ __device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
 __device__ __forceinline__ void st_relaxed_sys(unsigned long long* p, unsigned long long v) {
     asm volatile("st.relaxed.sys.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ unsigned cas_acquire_gpu(unsigned* p, unsigned cmp, unsigned v) {
+    unsigned old;
+    asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "l"(p), "r"(cmp), "r"(v) : "memory");
+    return old;
+}
 __device__ __forceinline__ void st_release_gpu(unsigned* p, unsigned v) {
     asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
 }
@@ -171,11 +176,12 @@ __device__ __forceinline__ unsigned hw_slot(const gsys_dev_ctx* c) {
 __device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, bool blocking) {
     unsigned s = hw_slot(c);
     unsigned ns = 32;
-    while (atomicCAS(&c->claim[s], 0u, 1u) != 0u) {
+    /* cmp-swap with acquire semantics: the slot's previous owner's writes (seqs[s], nbpend[s],
+     * released by its st.release) are visible without a separate MEMBAR */
+    while (cas_acquire_gpu(&c->claim[s], 0u, 1u) != 0u) {
         __nanosleep(ns);
         if (ns < 1024) ns <<= 1;
     }
-    __threadfence();   /* acquire the slot's previous owner's writes (seqs[s], nbpend[s]) */
     // A non-blocking caller hands the claim back at once but the host may still be serving its
     // request (P24.34: the CPU sets the slot free): reuse waits for that completion word.
     const unsigned pend = c->nbpend[s];
@@ -289,6 +295,15 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
 __device__ __forceinline__ void release(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
     trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true);
     st_release_gpu(&c->claim[s], 0u);      /* "consume the result" then free (reading A3) */
+}
+/* Release of a blocking call that read nothing host-written after its completion: the only data
+ * the slot's next owner needs (seqs[s]) was ordered by the doorbell's fence.acq_rel.sys, and the
+ * acquire poll keeps this store after the completion, so fence + relaxed store is the release
+ * pattern already -- no second MEMBAR.  (Calls that copied an inline result or a pull area use
+ * release(): those loads must complete before the host may refill the area for the next owner.) */
+__device__ __forceinline__ void release_after_fence(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
+    trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true);
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(&c->claim[s]), "r"(0u) : "memory");
 }
 
 /* ------------------------------------------------------------------ pull (reading B12)
@@ -418,7 +433,8 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         for (unsigned i = 0; i < GSYS_INLINE_BYTES / 16; i++)
             if (i < n16) dst[i] = t[i];
     }
-    release(c, s, seq);
+    if (io.out != nullptr || psrc != nullptr) release(c, s, seq);
+    else release_after_fence(c, s, seq);
     if (c->diag) atomicAdd(c->diag + 7, globaltimer());
     return r;
 }
