@@ -41,7 +41,7 @@ def parse():
     ap.add_argument("--file-mib", type=int, default=16)
     ap.add_argument("--chunk-kib", type=int, default=256)
     ap.add_argument("--order", default="relaxed", choices=["strong", "relaxed"])
-    ap.add_argument("--blocks", type=int, default=296, help="work-groups (2 per SM)")
+    ap.add_argument("--blocks", type=int, default=148, help="work-groups (1 per SM: 0.8 %% above 2 per SM, profiles/r01_blocks_ab.jsonl)")
     ap.add_argument("--threads", type=int, default=256)
     ap.add_argument("--staging", default="host", choices=["device", "host", "mixed"])
     ap.add_argument("--dev16", type=int, default=4, help="mixed staging: chunks per 16 on the device (DMA) path")

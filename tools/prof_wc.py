@@ -10,5 +10,5 @@ nf = int(sys.argv[2]) if len(sys.argv) > 2 else 64
 c = inputs.make_corpus(512, 16 << 20)
 paths = c.paths[:nf]
 res = W.wordcount_files(paths, inputs.dictionary(), inputs.patterns(), chunk=256 << 10,
-                        gflags=G.WG | G.BLOCKING | G.RELAXED, blocks=296, staging=staging)
+                        gflags=G.WG | G.BLOCKING | G.RELAXED, blocks=148, staging=staging)
 print("ok", int(res.hist.sum()))
