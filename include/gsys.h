@@ -267,7 +267,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
 /* Same scan over text already resident in device memory (no syscalls): the standalone scan
  * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n] (16-byte aligned); file
  * boundaries are not modelled (one file).  Adds into d_hist; d_hit (may be NULL) set to 1 if any
- * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 512, else a
+ * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 704, else a
  * multiple of 32 up to 768 (the 129-column table is used when it fits beside the warps' staging,
  * else the 77-column one).  -EINVAL on bad sizes/alignment, -ENODEV before gsys_init. */
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,

@@ -719,7 +719,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (!d_hist || (n && !d_text)) return -EINVAL;
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
-    if (threads == 0) threads = 512;
+    if (threads == 0) threads = 704;   // 22 warps + the 77-column table: 6 % above 16 warps + the 129-column one
     if (threads % 32 || threads > 768) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();

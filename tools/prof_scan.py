@@ -8,7 +8,7 @@ c = inputs.make_corpus(512, 16 << 20)
 text = torch.cat([torch.from_file(p, dtype=torch.uint8, size=os.path.getsize(p)) for p in c.paths[:64]]).cuda()
 hist = torch.zeros(64, dtype=torch.int64, device="cuda")
 hit = torch.zeros(1, dtype=torch.int32, device="cuda")
-for _ in range(3):   # the bench's launch: 1 block/SM x 512 threads, grep on
-    G.gsys_scan_device(text, text.numel(), 256 << 10, inputs.dictionary(), inputs.patterns(), hist, hit, 0, 512)
+for _ in range(3):   # the bench's launch: 1 block/SM x 704 threads, grep on
+    G.gsys_scan_device(text, text.numel(), 256 << 10, inputs.dictionary(), inputs.patterns(), hist, hit, 0, 704)
 torch.cuda.synchronize()
 print("ok")
