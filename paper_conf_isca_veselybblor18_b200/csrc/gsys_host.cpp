@@ -155,6 +155,26 @@ enum PtrKind { PK_INVALID = 0, PK_DEVICE = 1, PK_HOST = 2 };
 
 struct Instance;
 
+// Statistics and completion counters are bumped by every worker for every request; one shared
+// atomic per counter bounced its cache line between the 14 service threads.  Each thread adds to
+// its own cache line (tl_shard: worker id + 1, 0 for every other thread); readers sum the shards.
+// Counters are monotonic, so a sum that reaches a value means that many increments happened.
+thread_local int tl_shard = 0;
+struct Sharded {
+    static constexpr int N = 32;
+    struct alignas(64) Cell { std::atomic<uint64_t> v{0}; };
+    Cell c[N];
+    uint64_t fetch_add(uint64_t x, std::memory_order o = std::memory_order_seq_cst) {
+        return c[tl_shard & (N - 1)].v.fetch_add(x, o);
+    }
+    uint64_t load(std::memory_order o = std::memory_order_seq_cst) const {
+        uint64_t t = 0;
+        for (const Cell& x : c) t += x.v.load(o);
+        return t;
+    }
+    void store(uint64_t) { for (Cell& x : c) x.v.store(0); }
+};
+
 // CPUs the service threads may use: the process's allowed CPUs intersected with the GPU's
 // /sys/bus/pci/devices/<bdf>/local_cpulist (its NUMA node), unless that leaves none.  Returns the
 // count and fills *out (left empty when there is no locality information).
@@ -338,14 +358,14 @@ struct Instance {
     std::vector<Worker*> workers;
     std::atomic<bool> stop{false};
     alignas(64) std::atomic<uint64_t> head{0};   // doorbell entries claimed by workers
-    std::atomic<uint64_t> completed{0};    // requests whose completion was issued
+    Sharded completed;                     // requests whose completion was issued
     std::atomic<int> first_err{0};
     std::atomic<uint32_t> coalesce_max{8};
     std::atomic<uint32_t> window_us{0};
     std::atomic<int> merge{1};
     std::atomic<int> fault_err{0};          // gsys_set_fault: preads at fault_off fail with -fault_err
     std::atomic<int64_t> fault_off{-1};
-    std::atomic<uint64_t> st_faults{0};
+    Sharded st_faults;
     std::atomic<uint64_t> gen{1};          // pointer-cache generation
     std::atomic<uint64_t> kick{0};
     std::mutex sleep_mu;
@@ -359,17 +379,17 @@ struct Instance {
     uint32_t nthreads = 0;
 
     // stats
-    std::atomic<uint64_t> st_ns_busy{0}, st_ns_syscall{0}, st_ns_cuda{0}, st_ns_wait{0};
-    std::atomic<uint64_t> st_bundles{0}, st_max_bundle{0}, st_host_preads{0}, st_merged{0},
-        st_bytes_read{0}, st_bytes_h2d{0}, st_errors{0};
-    std::atomic<uint64_t> st_nr[8];
+    Sharded st_ns_busy, st_ns_syscall, st_ns_cuda, st_ns_wait;
+    Sharded st_bundles, st_host_preads, st_merged, st_bytes_read, st_bytes_h2d, st_errors;
+    std::atomic<uint64_t> st_max_bundle{0};
+    Sharded st_nr[8];
 
     // host trace
     std::atomic<int> tracing{0};
     std::mutex trace_mu;
     std::vector<gsys_trace_rec> htrace;
 
-    Instance() { for (auto& a : st_nr) a.store(0); }
+    Instance() {}
 
     void host_trace(uint32_t s, uint32_t seq, uint8_t from, uint8_t to, bool blocking) {
         if (!tracing.load(std::memory_order_relaxed)) return;
@@ -421,6 +441,7 @@ void Worker::run() {
     sigdelset(&ss, SIGABRT);
     pthread_sigmask(SIG_BLOCK, &ss, nullptr);
     if (CPU_COUNT(&inst->cpus) > 0) sched_setaffinity(0, sizeof inst->cpus, &inst->cpus);   // NUMA-local
+    tl_shard = id + 1;
     cudaSetDevice(inst->dev);
     Instance* I = inst;
     uint64_t idle_since = now_ns();
