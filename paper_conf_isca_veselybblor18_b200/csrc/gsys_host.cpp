@@ -275,6 +275,8 @@ struct Worker {
     std::vector<int32_t> mfd; std::vector<int64_t> moff; std::vector<uint64_t> mlen;
     std::vector<uint32_t> morder, mgroup; std::vector<uint64_t> mgoff_in; std::vector<int64_t> mg_off;
     std::vector<uint64_t> mg_len; std::vector<uint32_t> midx;
+    std::vector<uint8_t> done_;                        // per-bundle scratch, reused
+    std::vector<std::vector<uint32_t>> members_;
 
     cudaEvent_t get_event() {
         if (!evpool.empty()) { cudaEvent_t e = evpool.back(); evpool.pop_back(); return e; }
@@ -878,7 +880,8 @@ void Worker::process(uint64_t h0, uint32_t n) {
     }
 
     // ---- fault injection (tests): the pread at the chosen offset fails without being executed
-    std::vector<bool> done(n, false);
+    std::vector<uint8_t>& done = done_;   // reused per bundle (no allocation per request)
+    done.assign(n, 0);
     if (const int ferr = I->fault_err.load(std::memory_order_relaxed)) {
         const int64_t foff = I->fault_off.load(std::memory_order_relaxed);
         for (uint32_t i = 0; i < n; i++) {
@@ -906,7 +909,9 @@ void Worker::process(uint64_t h0, uint32_t n) {
         int ng = gsys_plan_merge(m, mfd.data(), moff.data(), mlen.data(), bcap / 2, morder.data(), mgroup.data(),
                                  mgoff_in.data(), mg_off.data(), mg_len.data());
         // execute groups with >= 2 members on regular files whose destinations are all resolvable
-        std::vector<std::vector<uint32_t>> members(ng > 0 ? ng : 0);
+        std::vector<std::vector<uint32_t>>& members = members_;
+        if (members.size() < (size_t)(ng > 0 ? ng : 0)) members.resize(ng);
+        for (int g = 0; g < ng; g++) members[g].clear();
         for (uint32_t t = 0; t < m; t++) members[mgroup[morder[t]]].push_back(morder[t]);
         for (int g = 0; g < ng; g++) {
             auto& mem = members[g];
