@@ -370,6 +370,8 @@ struct Instance {
     Sharded st_faults;
     std::atomic<uint64_t> gen{1};          // pointer-cache generation
     std::atomic<uint64_t> kick{0};
+    std::atomic<int> idle_workers{0};      // workers that found the ring empty and claimed nothing since
+    bool share_bursts = true;              // split a burst among idle workers (env GSYS_SHARE_BURSTS=0: off)
     std::mutex sleep_mu;
     std::condition_variable sleep_cv;
     std::atomic<int> sleepers{0};
@@ -448,9 +450,11 @@ void Worker::run() {
     Instance* I = inst;
     uint64_t idle_since = now_ns();
     uint64_t last_kick = I->kick.load();
+    bool idle = false;   // counted in I->idle_workers
     while (!I->stop.load(std::memory_order_relaxed)) {
         uint64_t h = I->head.load(std::memory_order_acquire);
         if (!I->ready(h)) {
+            if (!idle) { idle = true; I->idle_workers.fetch_add(1, std::memory_order_relaxed); }
             if (I->nparked.load(std::memory_order_relaxed)) {   // parked recvfroms keep us awake
                 service_parked();
                 idle_since = now_ns();
@@ -471,11 +475,20 @@ void Worker::run() {
         }
         // claim the run of ready entries at the head (a coalesced bundle, P22.9-13)
         const uint32_t cmax = I->coalesce_max.load(std::memory_order_relaxed);
+        const uint64_t win = (uint64_t)I->window_us.load(std::memory_order_relaxed) * 1000ull;
         uint32_t n = 1;
         while (n < cmax && I->ready(h + n)) n++;
+        if (!win && n > 1 && I->share_bursts) {
+            // a bundle is served serially (P22.12): with other workers idle, share a burst among
+            // them instead of serialising it here (64 simultaneous 256 KiB preads: 8 bundles of 8
+            // on 8 workers would leave 6 idle); under load nobody is idle and bundles stay <= max
+            const uint32_t avail = (uint32_t)I->idle_workers.load(std::memory_order_relaxed) + (idle ? 0u : 1u);
+            const uint32_t share = (n + (avail ? avail : 1u) - 1u) / (avail ? avail : 1u);
+            if (share < n) n = share;
+        }
         if (!I->head.compare_exchange_strong(h, h + n, std::memory_order_acq_rel)) continue;
+        if (idle) { idle = false; I->idle_workers.fetch_sub(1, std::memory_order_relaxed); }
         // coalescing window: keep extending the run for up to window microseconds (reading A19)
-        const uint64_t win = (uint64_t)I->window_us.load(std::memory_order_relaxed) * 1000ull;
         if (win && n < cmax) {
             const uint64_t t0 = now_ns();
             while (n < cmax && now_ns() - t0 < win) {
@@ -1216,6 +1229,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // no faster for 4 KiB preads (profiles/r01_completion_paths.json)
     c.memop_completion = (ev && strcmp(ev, "host") == 0) ? 0u : 1u;
     I->memop_completion = c.memop_completion != 0;
+    ev = getenv("GSYS_SHARE_BURSTS");
+    I->share_bursts = !(ev && atoi(ev) == 0);
     ev = getenv("GSYS_DIAG_PHASES");
     if (ev && atoi(ev) > 0) {
         if (cudaMalloc((void**)&c.diag, 64) != cudaSuccess) return fail(-ENOMEM);
