@@ -372,6 +372,7 @@ struct Instance {
     std::atomic<uint64_t> kick{0};
     std::atomic<int> idle_workers{0};      // workers that found the ring empty and claimed nothing since
     bool share_bursts = true;              // split a burst among idle workers (env GSYS_SHARE_BURSTS=0: off)
+    bool big_alone = true;                 // preads > 64 KiB into host memory are claimed alone (env GSYS_BIG_ALONE=0: off)
     std::mutex sleep_mu;
     std::condition_variable sleep_cv;
     std::atomic<int> sleepers{0};
@@ -478,6 +479,16 @@ void Worker::run() {
         const uint64_t win = (uint64_t)I->window_us.load(std::memory_order_relaxed) * 1000ull;
         uint32_t n = 1;
         while (n < cmax && I->ready(h + n)) n++;
+        if (!win && n > 1 && I->big_alone) {
+            // a large pread into host memory is never merged (reading A8: it would add a memcpy), so
+            // riding in a bundle (served serially, P22.12) only holds up the requests behind it:
+            // take it alone and leave its neighbours to other workers
+            const gsys_slot* sl = I->area_h + (uint32_t)__atomic_load_n(&I->ring_h[h & (I->ring_cap - 1)], __ATOMIC_ACQUIRE);
+            if (__atomic_load_n(&sl->nr, __ATOMIC_RELAXED) == GSYS_NR_PREAD64 &&
+                (__atomic_load_n(&sl->flags, __ATOMIC_RELAXED) & GSYS_HOSTBUF) &&
+                __atomic_load_n(&sl->args[2], __ATOMIC_RELAXED) > (64u << 10))
+                n = 1;
+        }
         if (!win && n > 1 && I->share_bursts) {
             // a bundle is served serially (P22.12): with other workers idle, share a burst among
             // them instead of serialising it here (64 simultaneous 256 KiB preads: 8 bundles of 8
@@ -1229,6 +1240,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // no faster for 4 KiB preads (profiles/r01_completion_paths.json)
     c.memop_completion = (ev && strcmp(ev, "host") == 0) ? 0u : 1u;
     I->memop_completion = c.memop_completion != 0;
+    ev = getenv("GSYS_BIG_ALONE");
+    I->big_alone = !(ev && atoi(ev) == 0);
     ev = getenv("GSYS_SHARE_BURSTS");
     I->share_bursts = !(ev && atoi(ev) == 0);
     ev = getenv("GSYS_DIAG_PHASES");
