@@ -459,3 +459,36 @@ def test_wordcount_nonblocking_full_corpus(tmpdir_shm):
     assert res.wait_rc == 0
     assert np.array_equal(as_u64(res.hist), c.census)
     assert res.file_hits.tolist() == [1 if m else 0 for m in c.pmasks]
+
+
+# ---------------------------------------------------------------------------- the per-call read cap
+@pytest.mark.parametrize("hostbuf", [False, True])
+def test_pread_per_call_cap_from_gpu(tmpdir_shm, hostbuf):
+    """Reading A11: one GPU-issued pread returns what one POSIX pread returns -- a 2 GiB read is
+    capped at 0x7ffff000 bytes (Fig. 7's kernel-level read).  Device buffers are served piecewise
+    through the bounce ring and must stop at exactly the same byte; host buffers are read in place."""
+    cap = 0x7FFFF000
+    path = os.path.join(tmpdir_shm, "sparse_2g.bin")
+    with open(path, "wb") as f:
+        f.truncate((1 << 31) + 4096)
+        for off, val in ((0, 0x11), (1 << 20, 0x22), (cap - 1, 0x33), (cap, 0x44)):
+            f.seek(off)
+            f.write(bytes([val]))
+    n = 1 << 31
+    if hostbuf:
+        buf = torch.zeros(n + 16, dtype=torch.uint8).pin_memory()
+        flags = G.KERNEL | G.BLOCKING | G.RELAXED | G.HOSTBUF
+    else:
+        buf = torch.zeros(n + 16, dtype=torch.uint8, device="cuda")
+        flags = G.KERNEL | G.BLOCKING | G.RELAXED
+    fd = os.open(path, os.O_RDONLY)
+    try:
+        _, ret, _, _, rc = W.bench_calls("pread", flags, 1, 32, 1, fd, n, (1 << 31) + 4096, buf)
+    finally:
+        os.close(fd)
+        os.unlink(path)
+    assert rc == 0
+    assert ret.tolist() == [cap] == [plan.expected_pread_ret((1 << 31) + 4096, 0, n)]
+    probe = torch.tensor([0, 1 << 20, cap - 1, cap], dtype=torch.int64)
+    got = buf[probe.to(buf.device)].cpu().tolist()
+    assert got == [0x11, 0x22, 0x33, 0]      # the byte at the cap was not read
