@@ -528,11 +528,18 @@ void Worker::flush_copies() {
         cudaMemcpyAttributes attr;
         memset(&attr, 0, sizeof attr);
         attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-        size_t idx0 = 0, fail = 0;
-        if (cudaMemcpyBatchAsync(cp_dst.data(), cp_src.data(), cp_len.data(), n, &attr, &idx0, 1, &fail, stream) !=
-            cudaSuccess) {
-            cudaGetLastError();
-            for (size_t i = 0; i < n; i++) cudaMemcpyAsync(cp_dst[i], cp_src[i], cp_len[i], cudaMemcpyHostToDevice, stream);
+        // at most 128 copies per batch call: larger batches of host-to-device copies can crash the
+        // process with an Xid on this driver (B200_PROFILING.md); sources are pinned (the bounce)
+        constexpr size_t kMaxBatch = 128;
+        for (size_t b = 0; b < n; b += kMaxBatch) {
+            const size_t m = n - b < kMaxBatch ? n - b : kMaxBatch;
+            size_t idx0 = 0, fail = 0;
+            if (m == 1 || cudaMemcpyBatchAsync(cp_dst.data() + b, cp_src.data() + b, cp_len.data() + b, m, &attr, &idx0,
+                                               1, &fail, stream) != cudaSuccess) {
+                cudaGetLastError();
+                for (size_t i = b; i < b + m; i++)
+                    cudaMemcpyAsync(cp_dst[i], cp_src[i], cp_len[i], cudaMemcpyHostToDevice, stream);
+            }
         }
     }
     cp_dst.clear();
