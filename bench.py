@@ -504,7 +504,7 @@ def wg_syscall_rate(G, W, dev, path):
 def cpu_baseline_leg(a, corpus, words, pats, chunk):
     import oracle
     nthr = host_cores()
-    sample = corpus.paths[:32]
+    sample = corpus.paths[:384]   # ~6 GiB: about 10 s of the oracle on 16 threads
     sbytes = sum(os.path.getsize(p) for p in sample)
     oracle.corpus(sample[:1], words, pats, chunk=chunk, nthreads=nthr)
     _, _, secs, _ = oracle.corpus(sample, words, pats, chunk=chunk, nthreads=nthr)
