@@ -184,20 +184,35 @@ typedef struct gsys_stats {
 int gsys_stats(gsys_stats_t* out);
 int gsys_stats_reset(void);
 
-/* Trace record: one slot transition (reading: oracle/protocol.py validates these). */
+/* Trace record: one slot transition ((req, slot, from, to, actor, t); the
+ * validator is oracle/protocol.py check_trace).  The request is identified by (slot, seq).
+ * t_ns is taken where the transition becomes visible to the other actor -- after the observation
+ * it depends on (a claim after the slot was seen free, a host PROCESSING after its cmp-swap saw
+ * READY) and before the store that hands the slot on (READY before the doorbell, FINISHED / FREE
+ * before the completion word) -- so causal order implies timestamp order.  GPU records carry
+ * %globaltimer, host records CLOCK_MONOTONIC; gsys_clock_sync() relates the two. */
 typedef struct gsys_trace_rec {
     uint32_t slot;
     uint32_t seq;
     uint8_t from, to;   /* gsys_state values, `from` as observed by the actor */
     uint8_t actor;      /* 0 = GPU, 1 = host                                   */
     uint8_t blocking;   /* 1 if the request was blocking                       */
-    uint32_t pad;
+    uint32_t nr;        /* syscall number of the request                       */
+    uint64_t t_ns;      /* GPU: %globaltimer; host: CLOCK_MONOTONIC            */
 } gsys_trace_rec;
 
 /* Copy up to cap records of each side into gpu_out / host_out (host memory); returns the
  * counts through n_gpu / n_host and resets the buffers. */
 int gsys_trace_read(gsys_trace_rec* gpu_out, uint32_t gpu_cap, uint32_t* n_gpu,
                     gsys_trace_rec* host_out, uint32_t host_cap, uint32_t* n_host);
+
+/* Relate the GPU's %globaltimer to the host's CLOCK_MONOTONIC: `samples` (1..4096) ping-pongs
+ * between one GPU thread and the calling host thread through host-mapped words; for the sample
+ * with the shortest round trip, host_time = gpu_time + *offset_ns within +- *uncertainty_ns
+ * (half that round trip plus the measured %globaltimer tick).  Runs a one-thread kernel on the
+ * instance's control stream.  0, -ENODEV before gsys_init, -EINVAL, -ETIMEDOUT (no answer in 1 s),
+ * -EIO. */
+int gsys_clock_sync(uint32_t samples, int64_t* offset_ns, uint64_t* uncertainty_ns);
 
 /* Compile-time facts of this build, for tests: slot bytes, inline bytes, state count. */
 int gsys_abi_info(uint32_t* slot_bytes, uint32_t* inline_bytes, uint32_t* nstates);

@@ -13,7 +13,8 @@
 //     grow by themselves when the service is the bottleneck;
 //   * a bundle executes in (fd, offset) order (reading A8), preads of adjacent/overlapping ranges
 //     of one regular file are merged into one read of the union (north_star extension), payloads
-//     for device buffers go through a pinned bounce ring and one cudaMemcpyBatchAsync per bundle,
+//     for device buffers go through a pinned bounce ring and per-bundle async copies (runs that are
+//     contiguous on both sides go as one copy),
 //     payloads for host-mapped buffers are read in place (P24.32-35);
 //   * results go back as a completion word {seq, ret} (P24.32-34): a plain host store into pinned
 //     host-mapped memory that the GPU polls (system-memory buffers, inline results and every
@@ -264,7 +265,7 @@ struct Worker {
     };
     BounceRing<cudaEvent_t, RingOps>* ring = nullptr;
     std::vector<cudaEvent_t> evpool;
-    // copies queued for one cudaMemcpyBatchAsync per bundle
+    // copies queued per bundle; flush_copies() issues them (contiguous runs joined)
     std::vector<void*> cp_dst, cp_src;
     std::vector<size_t> cp_len;
     std::vector<Req> reqs;
@@ -522,25 +523,18 @@ void Worker::flush_copies() {
     size_t n = cp_dst.size();
     if (!n) return;
     Timer tm(t_cuda);
-    if (n == 1) {
-        cudaMemcpyAsync(cp_dst[0], cp_src[0], cp_len[0], cudaMemcpyHostToDevice, stream);
-    } else {
-        cudaMemcpyAttributes attr;
-        memset(&attr, 0, sizeof attr);
-        attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-        // at most 128 copies per batch call: larger batches of host-to-device copies can crash the
-        // process with an Xid on this driver (B200_PROFILING.md); sources are pinned (the bounce)
-        constexpr size_t kMaxBatch = 128;
-        for (size_t b = 0; b < n; b += kMaxBatch) {
-            const size_t m = n - b < kMaxBatch ? n - b : kMaxBatch;
-            size_t idx0 = 0, fail = 0;
-            if (m == 1 || cudaMemcpyBatchAsync(cp_dst.data() + b, cp_src.data() + b, cp_len.data() + b, m, &attr, &idx0,
-                                               1, &fail, stream) != cudaSuccess) {
-                cudaGetLastError();
-                for (size_t i = b; i < b + m; i++)
-                    cudaMemcpyAsync(cp_dst[i], cp_src[i], cp_len[i], cudaMemcpyHostToDevice, stream);
-            }
-        }
+    // one cudaMemcpyAsync per run of copies that are contiguous in both source and destination
+    // (a merged union read split into neighbouring work-group lines is one such run); the batched
+    // copy entry points are not used (they raised GPU faults on this pool's driver)
+    size_t i = 0;
+    while (i < n) {
+        uint8_t* d = (uint8_t*)cp_dst[i];
+        const uint8_t* sp = (const uint8_t*)cp_src[i];
+        size_t len = cp_len[i];
+        size_t j = i + 1;
+        while (j < n && (uint8_t*)cp_dst[j] == d + len && (const uint8_t*)cp_src[j] == sp + len) len += cp_len[j++];
+        cudaMemcpyAsync(d, sp, len, cudaMemcpyHostToDevice, stream);
+        i = j;
     }
     cp_dst.clear();
     cp_src.clear();
