@@ -67,7 +67,8 @@ enum gsys_state {
 #define GSYS_STRONG      0x00u
 #define GSYS_RELAXED     0x10u
 #define GSYS_WEAK        GSYS_RELAXED
-#define GSYS_SITE(k)     (((uint32_t)(k) & 63u) << 24)   /* kernel-scope call site id 0..63 */
+#define GSYS_KSITES_MAX  8u
+#define GSYS_SITE(k)     (((uint32_t)(k) & 63u) << 24)   /* kernel-scope call site 0..7; 8..63 -> -EINVAL */
 /* Completion through system memory: the caller's buffer is pinned host-mapped memory, so the
  * host service performs the call in place and signals completion with a plain store into the
  * slot's host-mapped completion word, which the GPU polls over PCIe (the paper's "CPU-GPU
@@ -83,6 +84,9 @@ enum gsys_state {
 #define GSYS_F_NOHINT    0x800u   /* unpredictable latency (network): poll without the learned sleep */
 #define GSYS_F_PULL      0x1000u  /* blocking pread: the host reads into the slot's host-mapped pull
                                      area and the GPU copies it to the destination (reading B12)  */
+#define GSYS_F_PULLB     0x2000u  /* blocking work-group pread: the host reads into its host-mapped
+                                     bounce, returns the range's device address in args[1], and the
+                                     work-group copies it out, then sets the slot free (reading B13) */
 
 /* Syscall numbers served (Linux x86-64). */
 #define GSYS_NR_PREAD64        17
@@ -128,6 +132,25 @@ int gsys_set_merge(int on);
  * GPU caller sees the POSIX error convention of reading A4/A11.  0, -ENODEV, -EINVAL. */
 int gsys_set_fault(int32_t err, int64_t offset);
 
+/* Fault injection for tests: from now on every pread whose offset equals `offset` is drained and
+ * executed but its completion is never written (a lost completion); -1 turns it off.  The GPU
+ * caller's watchdog (gsys_set_poll_timeout) then returns -ETIMEDOUT.  0, -ENODEV. */
+int gsys_set_fault_drop(int64_t offset);
+
+/* Watchdog (SURVEY.md sec. 5 "failure detection"; PAPER.md:30 P30.0 GPU timeouts, PAPER.md:22
+ * P22.0 "raise an alarm"): every GPU-side wait on the host -- the slot claim, the completion poll,
+ * a kernel-scope result, gsys_wait_token -- gives up after `ms` milliseconds (0 = never; default
+ * env GSYS_POLL_TIMEOUT_MS, else 20000) and the call returns -ETIMEDOUT.  The expired wait is
+ * logged on the device; the next gsys_wait() returns -ETIMEDOUT, copies the log (read it with
+ * gsys_watchdog_read) and, once the service has drained, returns the affected slots to free.
+ * Synchronises the device first (running kernels read the setting).  0, -ENODEV, -EIO. */
+int gsys_set_poll_timeout(uint32_t ms);
+
+/* The watchdog log as the last gsys_wait() that returned -ETIMEDOUT read it: *count expired waits
+ * and up to cap records of 4 u32 {slot, seq, nr, phase (1 claim, 2 previous non-blocking request,
+ * 3 completion, 4 kernel-scope result, 5 token)}.  Returns the number of records copied. */
+int gsys_watchdog_read(uint32_t* count, uint32_t* recs, uint32_t cap);
+
 /* Phase diagnostics of blocking GPU calls (enabled with env GSYS_DIAG_PHASES=1 at gsys_init):
  * out8 = {ns claiming, ns marshalling + publishing, ns waiting for completion, -, calls,
  * ns of learned pre-poll sleep, completion polls, ns copying results + releasing}, summed over
@@ -138,13 +161,28 @@ int gsys_diag_phases(uint64_t* out8, int reset);
  * trace buffers readable with gsys_trace_read(); capacity = max records per side. */
 int gsys_set_trace(int on, uint32_t capacity);
 
-/* Launch a kernel that may call gsys_* device functions: resets the kernel-scope call sites,
- * then cudaLaunchKernel(kernel, grid, block, args, smem_bytes, stream).  `kernel` is a
- * __global__ function pointer, `args` its argument array, `stream` a cudaStream_t (NULL = the
- * legacy default stream).  CUDA errors map to -EINVAL / -ENOMEM / -EIO. */
+/* Launch a kernel that may call gsys_* device functions: gsys_launch_begin(), then
+ * cudaLaunchKernel(kernel, grid, block, args, smem_bytes, stream).  `kernel` is a __global__
+ * function registered with libgsys's own (static) CUDA runtime -- i.e. compiled into libgsys; for a
+ * kernel compiled elsewhere use gsys_launch_cu().  `args` is its argument array, `stream` a
+ * cudaStream_t (NULL = the legacy default stream).  CUDA errors map to -EINVAL / -ENOMEM / -EIO. */
 int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz,
                 uint32_t bx, uint32_t by, uint32_t bz, void** args, size_t smem_bytes,
                 void* stream);
+
+/* The same for any kernel that includes gsys_device.cuh, compiled in another module: cu_function
+ * is its CUfunction (cudaGetFuncBySymbol in the caller's runtime, or cuModuleGetFunction); the
+ * launch goes through the driver API (cuLaunchKernel), which every runtime shares. */
+int gsys_launch_cu(void* cu_function, uint32_t gx, uint32_t gy, uint32_t gz,
+                   uint32_t bx, uint32_t by, uint32_t bz, void** args, size_t smem_bytes,
+                   void* stream);
+
+/* What gsys_launch does before the launch, for callers that launch themselves (any API, CUDA
+ * graphs included): reset the kernel-scope call-site records for a grid of `nblocks` blocks on
+ * `stream` (they are per instance: kernel-granularity calls of launches running concurrently on
+ * other streams are not supported), reset the learned completion-poll sleep, wake the service.
+ * 0, -ENODEV, -EINVAL (nblocks 0 or > 2^31), -ENOMEM. */
+int gsys_launch_begin(uint64_t nblocks, void* stream);
 
 /* Drain (sec. IX "a new function call, invoked by the CPU, that ensures all GPU
  * system calls have completed before the termination of the process", P34.9).  Waits for the

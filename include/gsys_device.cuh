@@ -32,7 +32,7 @@
 
 #include "gsys.h"
 
-#define GSYS_KSITES 8u          /* kernel-scope call sites per launch          */
+#define GSYS_KSITES GSYS_KSITES_MAX   /* kernel-scope call sites per launch (gsys.h)  */
 #define GSYS_KROUNDS 4096u      /* kernel-scope calls per site per launch      */
 
 /* Per (site, round) record of a kernel-scope call (reset by gsys_launch). */
@@ -40,6 +40,19 @@ struct gsys_kround {
     unsigned arrive;   /* blocks that reached this round of the site            */
     unsigned done;     /* 1 once the caller stored ret (producer calls)          */
     long long ret;     /* the caller's result, broadcast to the other blocks     */
+};
+
+/* Watchdog log (device memory, written by the GPU, read and cleared by gsys_wait): every wait that
+ * ran out of time (ctx->poll_timeout_ns) bumps `count` and, for the first GSYS_WD_RECS, records
+ * which slot / request / call it was and in which phase.  The slot stays claimed (poisoned) until
+ * gsys_wait has drained the service, then it is returned to free. */
+#define GSYS_WD_RECS 64u
+enum gsys_wd_phase { GSYS_WD_CLAIM = 1, GSYS_WD_NBPEND = 2, GSYS_WD_COMPLETION = 3, GSYS_WD_KERNEL = 4,
+                     GSYS_WD_TOKEN = 5 };
+struct gsys_wd_log {
+    unsigned count;
+    unsigned pad;
+    struct { unsigned slot, seq, nr, phase; } rec[GSYS_WD_RECS];
 };
 
 /* Instance context in device memory (built by gsys_init). */
@@ -71,6 +84,20 @@ struct gsys_dev_ctx {
     unsigned memop_completion;      /* 1 (default): DMA'd blocking calls complete by a stream
                                        memop into `mirror`; 0 (env GSYS_COMPLETION=host): by a
                                        host store into `hdone` once the DMA has drained          */
+    unsigned pull_bounce;           /* 1: blocking work-group preads into device memory that fit no
+                                       pull area are read into the service's host-mapped bounce
+                                       and copied by the work-group (no CUDA call in the service;
+                                       env GSYS_COMPLETION=pull)                                  */
+    unsigned long long poll_timeout_ns;  /* watchdog: a claim or completion wait longer than this
+                                       returns -ETIMEDOUT (0 = wait forever)                      */
+    gsys_wd_log* wd;                /* device: watchdog log                                       */
+};
+
+/* Explicit completion token of a non-blocking call (slot, seq): gsys_wait_token() waits for that
+ * request whatever slot the caller's next call lands in (%smid / %warpid are volatile). */
+struct gsys_token {
+    unsigned slot;
+    unsigned seq;    /* 0: no request outstanding */
 };
 
 #ifdef __CUDACC__
@@ -151,16 +178,39 @@ __device__ __forceinline__ unsigned block_linear() {
     return blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
 }
 
-/* ------------------------------------------------------------------ tracing (debug) */
+/* ------------------------------------------------------------------ tracing (debug)
+ * One record per slot transition (gsys.h gsys_trace_rec), stamped with %globaltimer where the
+ * transition becomes visible: callers stamp after the observation an edge depends on and before
+ * the store that hands the slot on. */
 __device__ __forceinline__ void trace(const gsys_dev_ctx* c, unsigned s, unsigned seq, unsigned from,
-                                      unsigned to, bool blocking) {
+                                      unsigned to, bool blocking, unsigned nr) {
     if (c->trace == nullptr) return;
+    const unsigned long long t = globaltimer();
     unsigned i = atomicAdd(c->trace_n, 1u);
     if (i < c->trace_cap) {
         gsys_trace_rec r;
         r.slot = s; r.seq = seq; r.from = (uint8_t)from; r.to = (uint8_t)to; r.actor = 0;
-        r.blocking = blocking ? 1 : 0; r.pad = 0;
+        r.blocking = blocking ? 1 : 0; r.nr = nr; r.t_ns = t;
         c->trace[i] = r;
+    }
+}
+
+/* ------------------------------------------------------------------ watchdog
+ * Every wait on another agent is bounded by ctx->poll_timeout_ns: a lost completion must not hang
+ * the GPU (PAPER.md:30 P30.0, GPU timeouts kill the application; PAPER.md:22 P22.0, a failed
+ * blocking call should "raise an alarm").  The expired wait is logged in the host-mapped log and
+ * the call returns -ETIMEDOUT; gsys_wait() reports it. */
+__device__ __forceinline__ bool expired(const gsys_dev_ctx* c, unsigned long long& t0) {
+    if (c->poll_timeout_ns == 0ull) return false;
+    const unsigned long long t = globaltimer();
+    if (t0 == 0ull) { t0 = t; return false; }
+    return t - t0 > c->poll_timeout_ns;
+}
+__device__ __forceinline__ void wd_log(const gsys_dev_ctx* c, unsigned s, unsigned seq, unsigned nr, unsigned phase) {
+    if (c->wd == nullptr) return;
+    const unsigned i = atomicAdd(&c->wd->count, 1u);
+    if (i < GSYS_WD_RECS) {
+        c->wd->rec[i].slot = s; c->wd->rec[i].seq = seq; c->wd->rec[i].nr = nr; c->wd->rec[i].phase = phase;
     }
 }
 
@@ -173,20 +223,29 @@ __device__ __forceinline__ unsigned hw_slot(const gsys_dev_ctx* c) {
     return ((smid() * 64u + warpid()) * 32u + laneid()) % c->nslots;
 }
 
-__device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, bool blocking) {
+constexpr unsigned NOSLOT = 0xffffffffu;
+
+__device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, unsigned nr) {
     unsigned s = hw_slot(c);
     unsigned ns = 32;
+    unsigned long long t0 = 0ull;
     /* cmp-swap with acquire semantics: the slot's previous owner's writes (seqs[s], nbpend[s],
      * released by its st.release) are visible without a separate MEMBAR */
     while (cas_acquire_gpu(&c->claim[s], 0u, 1u) != 0u) {
         __nanosleep(ns);
         if (ns < 1024) ns <<= 1;
+        if (expired(c, t0)) { wd_log(c, s, 0u, nr, GSYS_WD_CLAIM); return NOSLOT; }
     }
     // A non-blocking caller hands the claim back at once but the host may still be serving its
     // request (P24.34: the CPU sets the slot free): reuse waits for that completion word.
     const unsigned pend = c->nbpend[s];
     if (pend) {
-        while ((unsigned)(ld_relaxed_sys(c->hdone + s) >> 32) != pend) __nanosleep(c->poll_ns_host);
+        t0 = 0ull;
+        while ((unsigned)(ld_relaxed_sys(c->hdone + s) >> 32) != pend) {
+            __nanosleep(c->poll_ns_host);
+            // the slot stays claimed (poisoned) until gsys_wait has drained the service
+            if (expired(c, t0)) { wd_log(c, s, pend, nr, GSYS_WD_NBPEND); return NOSLOT; }
+        }
         fence_acq_rel_sys();
         c->nbpend[s] = 0u;
     }
@@ -202,13 +261,13 @@ __device__ __forceinline__ unsigned marshal(const gsys_dev_ctx* c, unsigned s, u
     unsigned seq = c->seqs[s] + 1u;
     if (seq == 0u) seq = 1u;
     c->seqs[s] = seq;
-    trace(c, s, seq, GSYS_FREE, GSYS_POPULATING, !(flags & GSYS_NONBLOCKING));
+    trace(c, s, seq, GSYS_FREE, GSYS_POPULATING, !(flags & GSYS_NONBLOCKING), nr);
     uint4* line = reinterpret_cast<uint4*>(c->area + s);
     st_v4_sys(line + 0, make_uint4((unsigned)a[0], (unsigned)(a[0] >> 32), (unsigned)a[1], (unsigned)(a[1] >> 32)));
     st_v4_sys(line + 1, make_uint4((unsigned)a[2], (unsigned)(a[2] >> 32), (unsigned)a[3], (unsigned)(a[3] >> 32)));
     st_v4_sys(line + 2, make_uint4((unsigned)a[4], (unsigned)(a[4] >> 32), (unsigned)a[5], (unsigned)(a[5] >> 32)));
     st_v4_sys(line + 3, make_uint4(nr, flags, seq, (unsigned)GSYS_READY));
-    trace(c, s, seq, GSYS_POPULATING, GSYS_READY, !(flags & GSYS_NONBLOCKING));
+    trace(c, s, seq, GSYS_POPULATING, GSYS_READY, !(flags & GSYS_NONBLOCKING), nr);
     return seq;
 }
 
@@ -236,11 +295,13 @@ __device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
 /* ------------------------------------------------------------------ a5: completion
  * Blocking callers poll the slot's completion word until it carries their sequence number:
  * the device-memory word (L2-resident; written by a stream memory operation after the DMA) or,
- * for GSYS_HOSTBUF / inline calls, the host-mapped word the service stores directly (each poll
- * is one PCIe read, so the backoff starts longer and caps at poll_ns_max). */
-__device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq, bool host,
-                                               bool nohint = false) {
+ * for GSYS_HOSTBUF / inline / pulled calls, the host-mapped word the service stores directly
+ * (each poll is one PCIe read, so the caller first sleeps a learned hint).  false: the watchdog
+ * expired (logged; the slot stays claimed). */
+__device__ __forceinline__ bool wait_done(const gsys_dev_ctx* c, unsigned s, unsigned seq, bool host, bool nohint,
+                                          unsigned nr, long long& ret) {
     unsigned long long v;
+    unsigned long long t0 = 0ull;
     if (!host) {
         const unsigned long long* m = c->mirror + s;
         unsigned ns = 64;
@@ -249,6 +310,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(ns);
             ns = ns < c->poll_ns_max ? ns << 1 : c->poll_ns_max;
+            if (expired(c, t0)) { wd_log(c, s, seq, nr, GSYS_WD_COMPLETION); return false; }
         }
     } else {
         // every poll is a PCIe round trip, so a waiting caller first sleeps for the slot's learned
@@ -274,6 +336,7 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
             polls++;
             if ((unsigned)(v >> 32) == seq) break;
             __nanosleep(c->poll_ns_host);
+            if (expired(c, t0)) { wd_log(c, s, seq, nr, GSYS_WD_COMPLETION); return false; }
         }
         if (c->diag) atomicAdd(c->diag + 6, (unsigned long long)polls);
         if (!nohint) {
@@ -289,20 +352,34 @@ __device__ __forceinline__ long long wait_done(const gsys_dev_ctx* c, unsigned s
     /* the polls are acquire loads: the payload (device memory after the DMA, or the inline / pull
      * area the host wrote before its release store) is read after the completion word, with no
      * separate system-scope fence (a MEMBAR.SYS per call) */
-    return (long long)(int)(unsigned)(v & 0xffffffffull);
+    ret = (long long)(int)(unsigned)(v & 0xffffffffull);
+    return true;
 }
 
-__device__ __forceinline__ void release(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
-    trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true);
-    st_release_gpu(&c->claim[s], 0u);      /* "consume the result" then free (reading A3) */
+/* "The work-item can consume the result and continue execution" (P24.36; reading A3): the caller
+ * returns the slot to free -- the host-visible state word of the line (a posted store) and the
+ * device claim word.  release(): after the caller read host-written data (inline result, pull
+ * area) -- the acquire/release pair orders those loads before the next owner's claim; with
+ * `bounce`, the state store is a system-scope release, because the host recycles the bounce range
+ * the work-group just copied from as soon as it sees the slot free. */
+__device__ __forceinline__ void set_state_free(const gsys_dev_ctx* c, unsigned s, bool sys_release) {
+    unsigned* st = &c->area[s].state;
+    if (sys_release) asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(st), "r"((unsigned)GSYS_FREE) : "memory");
+    else asm volatile("st.relaxed.sys.global.u32 [%0], %1;" :: "l"(st), "r"((unsigned)GSYS_FREE) : "memory");
+}
+__device__ __forceinline__ void release(const gsys_dev_ctx* c, unsigned s, unsigned seq, unsigned nr,
+                                        bool bounce = false) {
+    trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true, nr);
+    set_state_free(c, s, bounce);
+    st_release_gpu(&c->claim[s], 0u);
 }
 /* Release of a blocking call that read nothing host-written after its completion: the only data
  * the slot's next owner needs (seqs[s]) was ordered by the doorbell's fence.acq_rel.sys, and the
  * acquire poll keeps this store after the completion, so fence + relaxed store is the release
- * pattern already -- no second MEMBAR.  (Calls that copied an inline result or a pull area use
- * release(): those loads must complete before the host may refill the area for the next owner.) */
-__device__ __forceinline__ void release_after_fence(const gsys_dev_ctx* c, unsigned s, unsigned seq) {
-    trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true);
+ * pattern already -- no second MEMBAR. */
+__device__ __forceinline__ void release_after_fence(const gsys_dev_ctx* c, unsigned s, unsigned seq, unsigned nr) {
+    trace(c, s, seq, GSYS_FINISHED, GSYS_FREE, true, nr);
+    set_state_free(c, s, false);
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(&c->claim[s]), "r"(0u) : "memory");
 }
 
@@ -313,7 +390,10 @@ __device__ __forceinline__ void release_after_fence(const gsys_dev_ctx* c, unsig
  * whose fixed costs dominate small reads.  The area is the slot's inline line for n <= 256 B,
  * or, for a work-group's caller (cooperative copy) in a slot with s % 32 == 0, the slot's
  * pull_big_bytes area.  The slot stays claimed until the copy is done, so the host never
- * refills an area that is still being read. */
+ * refills an area that is still being read.  Larger work-group reads (ctx->pull_bounce) land in
+ * the serving worker's host-mapped bounce ring; the host passes the range's device address back
+ * in args[1] (the argument field "re-purposed for the return value", P24.9) and recycles the
+ * range once the work-group has set the slot free. */
 __device__ __forceinline__ const unsigned char* pull_src(const gsys_dev_ctx* c, unsigned s, unsigned long long n,
                                                          bool coop) {
     if (n == 0ull) return nullptr;
@@ -363,25 +443,32 @@ __device__ __forceinline__ void pull_copy(const unsigned char* src, unsigned cha
 /* A pull the caller's scope finishes (work-group cooperative copy): filled by call_thread. */
 struct PullOut {
     const unsigned char* src = nullptr;
-    unsigned slot = 0, seq = 0;
+    unsigned slot = 0, seq = 0, nr = 0;
+    bool bounce = false;
 };
 
 /* One thread, one request: claim -> (inline input) -> marshal -> publish -> (poll).  A non-blocking
- * request's slot is reused only after the host has served it (P24.34, A15).  io.out: for
- * GSYS_F_INLINE calls, where the host's inline result is copied after completion.  po: when set
- * (a work-group caller), a pulled pread's copy and the slot's release are left to the caller's
- * scope; otherwise this thread copies (inline-size pulls only). */
+ * request's slot is reused only after the host has served it (P24.34, A15); `tok` (may be null)
+ * receives its (slot, seq) for gsys_wait_token().  io.out: for GSYS_F_INLINE calls, where the
+ * host's inline result is copied after completion.  po: when set (a work-group caller), a pulled
+ * pread's copy and the slot's release are left to the caller's scope; otherwise this thread
+ * copies (inline-size pulls only). */
 __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned nr, unsigned flags,
                                                  const unsigned long long a[6], const InlineIO& io = InlineIO(),
-                                                 PullOut* po = nullptr) {
+                                                 PullOut* po = nullptr, gsys_token* tok = nullptr) {
     const bool blocking = !(flags & GSYS_NONBLOCKING);
     const unsigned long long d0 = c->diag ? globaltimer() : 0ull;
-    unsigned s = claim(c, blocking);
+    unsigned s = claim(c, nr);
+    if (s == NOSLOT) {
+        if (tok) { tok->slot = 0u; tok->seq = 0u; }
+        return -ETIMEDOUT;
+    }
     const unsigned long long d1 = c->diag ? globaltimer() : 0ull;
     const unsigned char* psrc = nullptr;
     if (nr == GSYS_NR_PREAD64 && blocking && !(flags & GSYS_HOSTBUF)) {
         psrc = pull_src(c, s, a[2], po != nullptr);
         if (psrc) flags |= GSYS_F_PULL;
+        else if (po != nullptr && c->pull_bounce && a[2] > 0ull) flags |= GSYS_F_PULLB;
     }
     if (io.in != nullptr) {   /* input payload into the inline line; published by marshal's fence */
         uint4* dst = reinterpret_cast<uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
@@ -398,12 +485,16 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     doorbell(c, s);
     if (!blocking) {
         c->nbpend[s] = seq;
+        if (tok) { tok->slot = s; tok->seq = seq; }
         st_release_gpu(&c->claim[s], 0u);
         return 0;
     }
     const unsigned long long d2 = c->diag ? globaltimer() : 0ull;
-    long long r = wait_done(c, s, seq, !c->memop_completion || (flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL)) != 0u,
-                            (flags & GSYS_F_NOHINT) != 0u);
+    long long r = 0;
+    if (!wait_done(c, s, seq,
+                   !c->memop_completion || (flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL | GSYS_F_PULLB)) != 0u,
+                   (flags & GSYS_F_NOHINT) != 0u, nr, r))
+        return -ETIMEDOUT;   /* slot left claimed: the host may still complete into it */
     if (c->diag) {   /* phase diagnostics: claim, marshal+publish, wait, (copy+release below) */
         const unsigned long long d3 = globaltimer();
         atomicAdd(c->diag + 0, d1 - d0);
@@ -412,9 +503,16 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         atomicAdd(c->diag + 4, 1ull);
         atomicAdd(c->diag + 7, (unsigned long long)-(long long)d3);   /* + end time below */
     }
+    if (flags & GSYS_F_PULLB) {   /* the work-group copies from the worker's bounce, then releases */
+        const uint4 a01 = ld_v4_after_acquire(reinterpret_cast<const uint4*>(c->area + s));   /* args[1] = source */
+        po->src = r > 0 ? reinterpret_cast<const unsigned char*>((uintptr_t)a01.z | ((uintptr_t)a01.w << 32)) : nullptr;
+        po->slot = s; po->seq = seq; po->nr = nr; po->bounce = true;
+        if (c->diag) atomicAdd(c->diag + 7, globaltimer());
+        return r;
+    }
     if (psrc != nullptr && r > 0) {
         if (po != nullptr) {   /* the work-group copies and releases (wg_call) */
-            po->src = psrc; po->slot = s; po->seq = seq;
+            po->src = psrc; po->slot = s; po->seq = seq; po->nr = nr; po->bounce = false;
             if (c->diag) atomicAdd(c->diag + 7, globaltimer());
             return r;
         }
@@ -433,8 +531,8 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         for (unsigned i = 0; i < GSYS_INLINE_BYTES / 16; i++)
             if (i < n16) dst[i] = t[i];
     }
-    if (io.out != nullptr || psrc != nullptr) release(c, s, seq);
-    else release_after_fence(c, s, seq);
+    if (io.out != nullptr || psrc != nullptr) release(c, s, seq, nr);
+    else release_after_fence(c, s, seq, nr);
     if (c->diag) atomicAdd(c->diag + 7, globaltimer());
     return r;
 }
@@ -447,11 +545,13 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
  * Relaxed consumer (Bar2 removed): the caller's warp waits with it and gets the result, the
  * other warps proceed at once and get 0 (reading A17, P28.3). */
 __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                             const unsigned long long a[6], const InlineIO& io = InlineIO()) {
+                                             const unsigned long long a[6], const InlineIO& io = InlineIO(),
+                                             gsys_token* tok = nullptr) {
     __shared__ long long s_ret[2];
     __shared__ unsigned s_par;
     __shared__ const unsigned char* s_psrc[2];
     __shared__ unsigned char* s_pdst[2];
+    __shared__ unsigned s_prel[2];
     const bool strong = !(flags & GSYS_RELAXED);
     const bool bar1 = strong || !producer;
     const bool bar2 = strong || producer;
@@ -459,20 +559,24 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
     if (bar1) __syncthreads();
     long long r = 0;
     PullOut po;
-    if (tid == 0) r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, io, bar2 ? &po : nullptr);
+    if (tid == 0)
+        r = call_thread(c, nr, flags | (producer ? GSYS_F_PRODUCER : 0u), a, io, bar2 ? &po : nullptr, tok);
     if (bar2) {
         unsigned p = 0;
         if (tid == 0) {
             p = (s_par ^ 1u) & 1u; s_par = p; s_ret[p] = r;
             s_psrc[p] = po.src; s_pdst[p] = reinterpret_cast<unsigned char*>(a[1]);
+            s_prel[p] = (po.src != nullptr || po.bounce) ? 1u : 0u;
         }
         p = (unsigned)__syncthreads_or(tid == 0 ? (int)p : 0);
         const long long rv = s_ret[p];
         const unsigned char* src = s_psrc[p];
-        if (src != nullptr) {   /* pulled pread (reading B12): the whole work-group copies */
+        if (src != nullptr && rv > 0) {   /* pulled pread (reading B12): the whole work-group copies */
             pull_copy(src, s_pdst[p], rv, tid, block_threads());
+        }
+        if (s_prel[p]) {   /* the work-group's copy is done: thread 0 returns the slot */
             __syncthreads();
-            if (tid == 0) release(c, po.slot, po.seq);
+            if (tid == 0) release(c, po.slot, po.seq, po.nr, po.bounce);
         }
         return rv;
     }
@@ -488,8 +592,9 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
 /* Work-item (P20.31 "work-item invocations imply strong ordering"): every calling lane issues
  * its own request; the claim spins diverge, publication and the doorbell are warp-aggregated. */
 __device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                             const unsigned long long a[6], const InlineIO& io = InlineIO()) {
-    return call_thread(c, nr, (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u), a, io);
+                                             const unsigned long long a[6], const InlineIO& io = InlineIO(),
+                                             gsys_token* tok = nullptr) {
+    return call_thread(c, nr, (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u), a, io, nullptr, tok);
 }
 
 /* Kernel (P20.16-21, P20.33): relaxed only, -EINVAL for strong (reading A13).  Per call site and
@@ -498,14 +603,15 @@ __device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr,
  * on a block that was never scheduled) and the others wait for its result -- the kernel-scope
  * "barrier after".  Consumer: the LAST block to arrive calls after every block published its
  * data (the "barrier before"), and nobody waits.  Both are deadlock-free for grids larger than
- * the co-resident capacity. */
+ * the co-resident capacity.  Sites are GSYS_SITE(0..GSYS_KSITES-1); another site is -EINVAL. */
 __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
                                                  const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     __shared__ long long s_kret[2];
     __shared__ unsigned s_kpar;
     if (!(flags & GSYS_RELAXED)) return -EINVAL;
+    const unsigned site = (flags >> 24) & 63u;
+    if (site >= GSYS_KSITES) return -EINVAL;
     const unsigned tid = block_tid();
-    const unsigned site = (flags >> 24) & (GSYS_KSITES - 1u);
     const unsigned nb = gridDim.x * gridDim.y * gridDim.z;
     const unsigned bid = block_linear();
     if (!producer) __syncthreads();     /* block-level part of the barrier before */
@@ -530,8 +636,14 @@ __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned
                         st_release_gpu(&k->done, 1u);
                     } else {
                         unsigned ns = 64;
-                        while (ld_acquire_gpu(&k->done) == 0u) { __nanosleep(ns); if (ns < 2048) ns <<= 1; }
-                        r = *(volatile long long*)&k->ret;
+                        unsigned long long t0 = 0ull;
+                        bool ok = true;
+                        while (ld_acquire_gpu(&k->done) == 0u) {
+                            __nanosleep(ns);
+                            if (ns < 2048) ns <<= 1;
+                            if (expired(c, t0)) { wd_log(c, site, round, nr, GSYS_WD_KERNEL); ok = false; break; }
+                        }
+                        r = ok ? *(volatile long long*)&k->ret : -ETIMEDOUT;
                     }
                 } else {
                     __threadfence();
@@ -560,12 +672,31 @@ __device__ __forceinline__ bool flags_valid(unsigned flags) {
 
 /* Dispatch on granularity.  Invalid granularity -> -EINVAL (uniform across the scope). */
 __device__ __forceinline__ long long invoke(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
-                                            const unsigned long long a[6], const InlineIO& io = InlineIO()) {
+                                            const unsigned long long a[6], const InlineIO& io = InlineIO(),
+                                            gsys_token* tok = nullptr) {
     switch (flags & GSYS_GRAN_MASK) {
-        case GSYS_WI: return wi_call(c, nr, flags, producer, a, io);
-        case GSYS_WG: return wg_call(c, nr, flags, producer, a, io);
+        case GSYS_WI: return wi_call(c, nr, flags, producer, a, io, tok);
+        case GSYS_WG: return wg_call(c, nr, flags, producer, a, io, tok);
         case GSYS_KERNEL: return kernel_call(c, nr, flags, producer, a, io);
         default: return -EINVAL;
+    }
+}
+
+/* Wait for the non-blocking request of `tok` (one thread's token) to complete: returns its result
+ * if the slot's completion word still carries it, 0 if a later request on the slot completed
+ * since (completions on a slot are in order, A15: ours is done, its result was overwritten --
+ * errors still reach gsys_wait, reading A4), -ETIMEDOUT from the watchdog. */
+__device__ __forceinline__ long long wait_token_thread(const gsys_dev_ctx* c, const gsys_token& tok) {
+    if (tok.seq == 0u) return 0;
+    const unsigned long long* m = c->hdone + tok.slot;
+    unsigned long long t0 = 0ull;
+    for (;;) {
+        const unsigned long long v = ld_acquire_sys(m);
+        const unsigned got = (unsigned)(v >> 32);
+        if (got == tok.seq) return (long long)(int)(unsigned)(v & 0xffffffffull);
+        if ((int)(got - tok.seq) > 0) return 0;
+        __nanosleep(c->poll_ns_host);
+        if (expired(c, t0)) { wd_log(c, tok.slot, tok.seq, 0u, GSYS_WD_TOKEN); return -ETIMEDOUT; }
     }
 }
 
@@ -577,16 +708,34 @@ __device__ __forceinline__ long long invoke(const gsys_dev_ctx* c, unsigned nr, 
  * errors at gsys_wait() (reading A4).  Producer (read-like) vs consumer (write-like) class per
  * P20.24-29; madvise and rt_sigqueueinfo are consumers (reading A7). */
 __device__ __forceinline__ long long gsys_pread(const gsys_dev_ctx* c, int fd, void* buf, size_t n, long long off,
-                                                unsigned gflags) {
+                                                unsigned gflags, gsys_token* tok = nullptr) {
     unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
                                (unsigned long long)off, 0ull, 0ull};
-    return gsys::invoke(c, GSYS_NR_PREAD64, gflags, true, a);
+    return gsys::invoke(c, GSYS_NR_PREAD64, gflags, true, a, gsys::InlineIO(), tok);
+}
+/* Completion wait on an explicit token (the trailing `tok` of a non-blocking gsys_pread / pwrite /
+ * sendto: for WG calls it must be visible to the whole work-group, e.g. __shared__; thread 0
+ * writes it).  gflags' granularity
+ * gives the scope: GSYS_WI -- the calling thread waits on its own token; GSYS_WG -- thread 0
+ * waits on *tok and every thread of the block gets the result after a barrier (all must call).
+ * GSYS_KERNEL: -EINVAL (the token lives in one block). */
+__device__ __forceinline__ long long gsys_wait_token(const gsys_dev_ctx* c, const gsys_token* tok, unsigned gflags) {
+    const unsigned g = gflags & GSYS_GRAN_MASK;
+    if (g == GSYS_WI) return gsys::wait_token_thread(c, *tok);
+    if (g != GSYS_WG) return -EINVAL;
+    __shared__ long long s_tret;
+    __syncthreads();
+    if (gsys::block_tid() == 0) s_tret = gsys::wait_token_thread(c, *tok);
+    __syncthreads();
+    const long long r = s_tret;
+    __syncthreads();
+    return r;
 }
 __device__ __forceinline__ long long gsys_pwrite(const gsys_dev_ctx* c, int fd, const void* buf, size_t n,
-                                                 long long off, unsigned gflags) {
+                                                 long long off, unsigned gflags, gsys_token* tok = nullptr) {
     unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
                                (unsigned long long)off, 0ull, 0ull};
-    return gsys::invoke(c, GSYS_NR_PWRITE64, gflags, false, a);
+    return gsys::invoke(c, GSYS_NR_PWRITE64, gflags, false, a, gsys::InlineIO(), tok);
 }
 /* getrusage: blocking calls land the 144 B struct rusage in the slot's inline line and the
  * caller copies it to `ru` (any pointer the thread can write, including local memory);
@@ -608,10 +757,11 @@ __device__ __forceinline__ long long gsys_madvise(const gsys_dev_ctx* c, void* a
     return gsys::invoke(c, GSYS_NR_MADVISE, gflags, false, a);
 }
 __device__ __forceinline__ long long gsys_sendto(const gsys_dev_ctx* c, int fd, const void* buf, size_t n, int flags,
-                                                 const void* to, unsigned tolen, unsigned gflags) {
+                                                 const void* to, unsigned tolen, unsigned gflags,
+                                                 gsys_token* tok = nullptr) {
     unsigned long long a[6] = {(unsigned long long)(long long)fd, (unsigned long long)buf, (unsigned long long)n,
                                (unsigned long long)(long long)flags, (unsigned long long)to, (unsigned long long)tolen};
-    return gsys::invoke(c, GSYS_NR_SENDTO, gflags | GSYS_F_NOHINT, false, a);
+    return gsys::invoke(c, GSYS_NR_SENDTO, gflags | GSYS_F_NOHINT, false, a, gsys::InlineIO(), tok);
 }
 __device__ __forceinline__ long long gsys_recvfrom(const gsys_dev_ctx* c, int fd, void* buf, size_t n, int flags,
                                                    void* from, unsigned* fromlen, unsigned gflags) {

@@ -70,8 +70,10 @@ def amr_released(levels, rss_ok=None):
 
 
 def permuted_blocks(data, perm, iters: int, block_bytes: int):
-    """Fig. 8: each block permuted `iters` times, out[i] = in[perm[i]] -- the bytes the
-    GPU work-groups must have written to the file (numpy fancy indexing, one step at a time)."""
+    """Fig. 8 (PAPER.md:26 P26.21-27): each block permuted `iters` times, out[i] = in[perm[i]] (a
+    DES-style gather, reading A20) -- the bytes the GPU work-groups must have written to the file
+    (numpy fancy indexing, one step at a time).  Pinned by the hand-worked example in
+    tests/golden/fig8_permutation_tiny.json."""
     import numpy as np
     blocks = np.asarray(data).reshape(-1, block_bytes)
     out = blocks.copy()

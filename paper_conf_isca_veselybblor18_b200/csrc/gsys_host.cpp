@@ -62,10 +62,15 @@ namespace {
 typedef CUresult (*PFN_batch_t)(CUstream, unsigned int, CUstreamBatchMemOpParams*, unsigned int);
 typedef CUresult (*PFN_ptrattrs_t)(unsigned int, CUpointer_attribute*, void**, CUdeviceptr);
 typedef CUresult (*PFN_devattr_t)(int*, CUdevice_attribute, CUdevice);
+typedef CUresult (*PFN_launch_t)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                                 CUstream, void**, void**);
+typedef CUresult (*PFN_funcsetattr_t)(CUfunction, CUfunction_attribute, int);
 
 PFN_batch_t p_batch = nullptr;
 PFN_ptrattrs_t p_ptrattrs = nullptr;
 PFN_devattr_t p_devattr = nullptr;
+PFN_launch_t p_launch = nullptr;
+PFN_funcsetattr_t p_funcsetattr = nullptr;
 
 inline uint64_t now_ns() {
     struct timespec ts;
@@ -113,7 +118,11 @@ class BounceRing {
     // attach one completion token to every region allocated since the previous commit
     void commit() {
         if (!npending_) return;
-        Token t = ops_->make_token();
+        commit_with(ops_->make_token());
+    }
+    // ... or a given token (a pulled bounce range: released when its slot is set free)
+    void commit_with(Token t) {
+        if (!npending_) return;
         size_t first = q_.size() - npending_;
         for (size_t i = first; i < q_.size(); i++) {
             q_[i].tok = t;
@@ -225,6 +234,8 @@ struct Req {
     bool dma;      // a host->device copy was queued for this request
     bool parked;   // blocking recvfrom on an empty socket: completed later by service_parked()
     bool faulted;  // fault injection (gsys_set_fault): completed with the injected -errno, not executed
+    bool early;    // completion already issued inside the bundle (pulled bounce reads, reading B13)
+    bool dropped;  // fault injection (gsys_set_fault_drop): drained, never completed
 };
 
 // A blocking recvfrom that found no datagram does not hold a service thread (reading B11): the
@@ -243,18 +254,30 @@ struct Worker {
     cudaStream_t stream = nullptr;
     uint8_t* bounce = nullptr;       // pinned
     size_t bcap = 0;
-    // BounceRing ops: a token is a CUDA event recorded after the queued copies were issued
+    // BounceRing ops: a token is either a CUDA event recorded after the queued copies were issued,
+    // or (pulled bounce reads, reading B13) the (slot, seq) whose work-group copies the range out
+    // and then sets the slot free
+    struct Tok {
+        cudaEvent_t ev = nullptr;
+        uint32_t slot = 0, seq = 0;
+        bool operator==(const Tok& o) const { return ev == o.ev && slot == o.slot && seq == o.seq; }
+    };
     struct RingOps {
         Worker* w;
-        cudaEvent_t make_token() {
+        Tok make_token() {
             w->flush_copies();
             Timer t(w->t_cuda);
-            cudaEvent_t e = w->get_event();
-            cudaEventRecord(e, w->stream);
-            return e;
+            Tok k;
+            k.ev = w->get_event();
+            cudaEventRecord(k.ev, w->stream);
+            return k;
         }
-        void wait(cudaEvent_t e) { Timer t(w->t_wait); cudaEventSynchronize(e); }
-        void recycle(cudaEvent_t e) { w->evpool.push_back(e); }
+        void wait(const Tok& k) {
+            Timer t(w->t_wait);
+            if (k.ev) { cudaEventSynchronize(k.ev); return; }
+            w->wait_slot_free(k.slot, k.seq);
+        }
+        void recycle(const Tok& k) { if (k.ev) w->evpool.push_back(k.ev); }
     };
     RingOps ring_ops{this};
     uint64_t t_sys = 0, t_cuda = 0, t_wait = 0;   // per-bundle timers (ns)
@@ -263,7 +286,10 @@ struct Worker {
         explicit Timer(uint64_t& a) : acc(a), t0(now_ns()) {}
         ~Timer() { acc += now_ns() - t0; }
     };
-    BounceRing<cudaEvent_t, RingOps>* ring = nullptr;
+    BounceRing<Tok, RingOps>* ring = nullptr;
+    uint8_t* bounce_d = nullptr;     // device address of the (host-mapped) bounce
+    void wait_slot_free(uint32_t slot, uint32_t seq);
+    void complete_early(Req& r);
     std::vector<cudaEvent_t> evpool;
     // copies queued per bundle; flush_copies() issues them (contiguous runs joined)
     std::vector<void*> cp_dst, cp_src;
@@ -368,6 +394,10 @@ struct Instance {
     std::atomic<int> merge{1};
     std::atomic<int> fault_err{0};          // gsys_set_fault: preads at fault_off fail with -fault_err
     std::atomic<int64_t> fault_off{-1};
+    std::atomic<int64_t> drop_off{-1};      // gsys_set_fault_drop: that pread's completion is never written
+    gsys_wd_log* wd_d = nullptr;           // device watchdog log (gsys_device.cuh)
+    std::mutex wd_mu;
+    gsys_wd_log wd_last{};                 // the log as the last gsys_wait that saw expiries read it
     Sharded st_faults;
     std::atomic<uint64_t> gen{1};          // pointer-cache generation
     std::atomic<uint64_t> kick{0};
@@ -397,12 +427,15 @@ struct Instance {
 
     Instance() {}
 
-    void host_trace(uint32_t s, uint32_t seq, uint8_t from, uint8_t to, bool blocking) {
+    // stamped after the observation the edge depends on and before the store that hands the slot
+    // back (gsys.h gsys_trace_rec)
+    void host_trace(uint32_t s, uint32_t seq, uint8_t from, uint8_t to, bool blocking, uint32_t nr) {
         if (!tracing.load(std::memory_order_relaxed)) return;
         std::lock_guard<std::mutex> g(trace_mu);
         if (htrace.size() < trace_cap) {
             gsys_trace_rec r;
-            r.slot = s; r.seq = seq; r.from = from; r.to = to; r.actor = 1; r.blocking = blocking ? 1 : 0; r.pad = 0;
+            r.slot = s; r.seq = seq; r.from = from; r.to = to; r.actor = 1; r.blocking = blocking ? 1 : 0;
+            r.nr = nr; r.t_ns = now_ns();
             htrace.push_back(r);
         }
     }
@@ -617,6 +650,32 @@ int Worker::write_small(uintptr_t p, const void* in, size_t n) {
     return -EFAULT;
 }
 
+// A pulled bounce range is free again once its work-group set the slot free (or the slot already
+// carries a newer request).  Bounded by the watchdog timeout: a work-group that died without
+// consuming its range must not wedge the worker forever.
+void Worker::wait_slot_free(uint32_t slot, uint32_t seq) {
+    const gsys_slot* sl = inst->area_h + slot;
+    const uint64_t t0 = now_ns();
+    const uint64_t lim = inst->ctx_h.poll_timeout_ns ? 2 * inst->ctx_h.poll_timeout_ns : 0;
+    for (;;) {
+        if (__atomic_load_n(&sl->state, __ATOMIC_ACQUIRE) == GSYS_FREE) return;
+        if (__atomic_load_n(&sl->seq, __ATOMIC_ACQUIRE) != seq) return;
+        if (lim && now_ns() - t0 > lim) {
+            inst->st_errors.fetch_add(1, std::memory_order_relaxed);
+            return;
+        }
+        _mm_pause();
+    }
+}
+
+// Completion of one request inside its bundle (reading B13): result, state, completion word now,
+// so its work-group can start copying while the rest of the bundle is served.
+void Worker::complete_early(Req& r) {
+    r.early = true;
+    if (r.dropped) { inst->completed.fetch_add(1, std::memory_order_release); return; }
+    inst->complete_host(r);
+}
+
 // pread(fd, buf, n, off): host-mapped buf -> read in place; device buf -> read into the pinned
 // bounce and DMA.  A request larger than the bounce is served piecewise with the POSIX result of
 // one call (stop at a short piece, cap at GSYS_PREAD_CAP, reading A11).
@@ -631,6 +690,27 @@ int64_t Worker::do_pread(Req& r) {
     }
     uint8_t* hp = nullptr;
     PtrKind k;
+    if (r.flags & GSYS_F_PULLB) {
+        // reading B13: read into this worker's host-mapped bounce, hand the range's device address
+        // back in args[1] and complete at once; the work-group copies the bytes to its buffer and
+        // sets the slot free, which releases the range (no CUDA call on this path)
+        const uint64_t want = std::min<uint64_t>(std::min<uint64_t>(n, GSYS_PREAD_CAP), bcap / 2);
+        commit();   // earlier regions of this bundle keep their own tokens
+        uint8_t* b = alloc(want);
+        if (!b) return -ENOMEM;
+        ssize_t z;
+        { Timer tm(t_sys); z = pread(fd, b, want, off); }
+        Worker::Tok t;
+        t.slot = r.slot;
+        t.seq = r.seq;
+        ring->commit_with(t);
+        inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
+        r.ret = z < 0 ? -(int64_t)errno : (int64_t)z;
+        if (z > 0) inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
+        __atomic_store_n(&inst->area_h[r.slot].args[1], (uint64_t)(uintptr_t)(bounce_d + (b - bounce)), __ATOMIC_RELAXED);
+        complete_early(r);
+        return r.ret;
+    }
     if (r.flags & GSYS_F_PULL) {   // into the slot's pull area; the GPU copies it out (reading B12)
         hp = inst->pull_area(r.slot, n);
         if (!hp) return -EINVAL;
@@ -867,7 +947,7 @@ void Instance::complete_host(const Req& r) {
     }
     if (r.ok) {
         __atomic_store_n(&sl->state, blocking ? (uint32_t)GSYS_FINISHED : (uint32_t)GSYS_FREE, __ATOMIC_RELEASE);
-        host_trace(r.slot, r.seq, GSYS_PROCESSING, blocking ? GSYS_FINISHED : GSYS_FREE, blocking);
+        host_trace(r.slot, r.seq, GSYS_PROCESSING, blocking ? GSYS_FINISHED : GSYS_FREE, blocking, r.nr);
     }
     __atomic_store_n(&hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret, __ATOMIC_RELEASE);
     completed.fetch_add(1, std::memory_order_release);
@@ -895,12 +975,14 @@ void Worker::process(uint64_t h0, uint32_t n) {
         r.dma = false;
         r.parked = false;
         r.faulted = false;
+        r.early = false;
+        r.dropped = false;
         // "atomically switches any ready system call requests to the processing state" (P24.20)
         uint32_t expect = GSYS_READY;
         r.ok = __atomic_compare_exchange_n((uint32_t*)&I->area_h[r.slot].state, &expect, (uint32_t)GSYS_PROCESSING,
                                            false, __ATOMIC_ACQ_REL, __ATOMIC_ACQUIRE);
         if (!r.ok) r.ret = -EPROTO;
-        I->host_trace(r.slot, r.seq, GSYS_READY, GSYS_PROCESSING, !(r.flags & GSYS_NONBLOCKING));
+        else I->host_trace(r.slot, r.seq, GSYS_READY, GSYS_PROCESSING, !(r.flags & GSYS_NONBLOCKING), r.nr);
         I->st_nr[nr_index(r.nr)].fetch_add(1, std::memory_order_relaxed);
     }
 
@@ -915,6 +997,16 @@ void Worker::process(uint64_t h0, uint32_t n) {
                 r.ret = -(int64_t)ferr;
                 r.faulted = true;
                 done[i] = true;
+                I->st_faults.fetch_add(1, std::memory_order_relaxed);
+            }
+        }
+    }
+    if (I->drop_off.load(std::memory_order_relaxed) >= 0) {
+        const int64_t doff = I->drop_off.load(std::memory_order_relaxed);
+        for (uint32_t i = 0; i < n; i++) {
+            Req& r = reqs[i];
+            if (r.ok && r.nr == GSYS_NR_PREAD64 && (int64_t)r.a[3] == doff) {
+                r.dropped = true;
                 I->st_faults.fetch_add(1, std::memory_order_relaxed);
             }
         }
@@ -952,7 +1044,10 @@ void Worker::process(uint64_t h0, uint32_t n) {
                 PtrKind k = !r.a[2] ? PK_INVALID
                             : (r.flags & GSYS_F_PULL) ? (I->pull_area(r.slot, r.a[2]) ? PK_HOST : PK_INVALID)
                                                       : resolve((uintptr_t)r.a[1], r.a[2], nullptr);
-                if (k == PK_INVALID || (k == PK_HOST && r.a[2] > (64u << 10))) { okd = false; break; }
+                if (k == PK_INVALID || (k == PK_HOST && r.a[2] > (64u << 10)) || (r.flags & GSYS_F_PULLB)) {
+                    okd = false;
+                    break;
+                }
             }
             if (!okd) continue;
             uint8_t* b = alloc(mg_len[g]);
@@ -1015,10 +1110,11 @@ void Worker::process(uint64_t h0, uint32_t n) {
     // buffers complete with a stream memory operation ordered after the DMA above.
     ops.clear();
     bool need_sync = false;
-    uint32_t nparked_here = 0;
+    uint32_t nparked_here = 0;   // parked or already completed: not counted below
     for (uint32_t i = 0; i < n; i++) {
         Req& r = reqs[i];
-        if (r.parked) { nparked_here++; continue; }
+        if (r.parked || r.early) { nparked_here++; continue; }
+        if (r.dropped) continue;   // fault injection: drained, the completion is never written
         const bool blocking = !(r.flags & GSYS_NONBLOCKING);
         gsys_slot* sl = I->area_h + r.slot;
         __atomic_store_n(&sl->args[0], (uint64_t)r.ret, __ATOMIC_RELAXED);
@@ -1037,14 +1133,14 @@ void Worker::process(uint64_t h0, uint32_t n) {
                 if (r.dma) { need_sync = true; continue; }
                 if (r.ok) {
                     __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
-                    I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true);
+                    I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true, r.nr);
                 }
                 __atomic_store_n(&I->hdone_h[r.slot], word, __ATOMIC_RELEASE);
                 continue;
             }
             if (r.ok) {
                 __atomic_store_n(&sl->state, (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
-                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true);
+                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FINISHED, true, r.nr);
             }
             if (I->mem64) {
                 op.writeValue.operation = CU_STREAM_MEM_OP_WRITE_VALUE_64;
@@ -1068,7 +1164,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
             if (r.dma) { need_sync = true; continue; }
             if (r.ok) {
                 __atomic_store_n(&sl->state, (uint32_t)GSYS_FREE, __ATOMIC_RELEASE);
-                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FREE, false);
+                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, GSYS_FREE, false, r.nr);
             }
             __atomic_store_n(&I->hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret,
                              __ATOMIC_RELEASE);
@@ -1086,12 +1182,13 @@ void Worker::process(uint64_t h0, uint32_t n) {
         for (uint32_t i = 0; i < n; i++) {
             Req& r = reqs[i];
             const bool nb = (r.flags & GSYS_NONBLOCKING) != 0;
+            if (r.dropped || r.early || r.parked) continue;
             if (!r.dma || (!nb && I->memop_completion && !(r.flags & (GSYS_HOSTBUF | GSYS_F_INLINE | GSYS_F_PULL))))
                 continue;
             gsys_slot* sl = I->area_h + r.slot;
             if (r.ok) {
                 __atomic_store_n(&sl->state, nb ? (uint32_t)GSYS_FREE : (uint32_t)GSYS_FINISHED, __ATOMIC_RELEASE);
-                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, nb ? GSYS_FREE : GSYS_FINISHED, !nb);
+                I->host_trace(r.slot, r.seq, GSYS_PROCESSING, nb ? GSYS_FREE : GSYS_FINISHED, !nb, r.nr);
             }
             __atomic_store_n(&I->hdone_h[r.slot], ((uint64_t)r.seq << 32) | (uint32_t)(int32_t)r.ret,
                              __ATOMIC_RELEASE);
@@ -1136,6 +1233,14 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
         if (cudaGetDriverEntryPoint("cuDeviceGetAttribute", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn)
             return -ENOTSUP;
         p_devattr = (PFN_devattr_t)fn;
+        fn = nullptr;
+        if (cudaGetDriverEntryPoint("cuLaunchKernel", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn)
+            return -ENOTSUP;
+        p_launch = (PFN_launch_t)fn;
+        fn = nullptr;
+        if (cudaGetDriverEntryPoint("cuFuncSetAttribute", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn)
+            return -ENOTSUP;
+        p_funcsetattr = (PFN_funcsetattr_t)fn;
     }
     Instance* I = new Instance();
     I->dev = dev;
@@ -1239,7 +1344,7 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // default memop: a host-store completion must first wait for the DMA (an event synchronize per
     // bundle), which measured slower for device staging (42.5 vs 46.7 GB/s at 256 KiB chunks) and
     // no faster for 4 KiB preads (profiles/r01_completion_paths.json)
-    c.memop_completion = (ev && strcmp(ev, "host") == 0) ? 0u : 1u;
+    c.memop_completion = (ev && (strcmp(ev, "host") == 0 || strcmp(ev, "pull") == 0)) ? 0u : 1u;
     I->memop_completion = c.memop_completion != 0;
     ev = getenv("GSYS_BIG_ALONE");
     I->big_alone = !(ev && atoi(ev) == 0);
@@ -1253,6 +1358,16 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     }
     ev = getenv("GSYS_SLEEP_HINT");
     c.no_hint = (ev && atoi(ev) == 0) ? 1u : 0u;
+    // reading B13: GSYS_COMPLETION=pull -- blocking work-group preads into device memory are copied
+    // out of the worker's host-mapped bounce by the work-group (no CUDA call in the service)
+    ev = getenv("GSYS_COMPLETION");
+    c.pull_bounce = (ev && strcmp(ev, "pull") == 0) ? 1u : 0u;
+    // watchdog: GSYS_POLL_TIMEOUT_MS, default 20 s, 0 = off
+    ev = getenv("GSYS_POLL_TIMEOUT_MS");
+    c.poll_timeout_ns = (unsigned long long)(ev ? atoll(ev) : 20000ll) * 1000000ull;
+    if (cudaMalloc((void**)&I->wd_d, sizeof(gsys_wd_log)) != cudaSuccess) return fail(-ENOMEM);
+    cudaMemset(I->wd_d, 0, sizeof(gsys_wd_log));
+    c.wd = I->wd_d;
     c.pull_big_bytes = I->pull_bytes;
     c.pull_big = I->pull_d;
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);
@@ -1284,9 +1399,13 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
         w->inst = I;
         w->id = (int)t;
         if (cudaStreamCreateWithFlags(&w->stream, cudaStreamNonBlocking) != cudaSuccess) { delete w; return fail(-EIO); }
-        if (cudaHostAlloc((void**)&w->bounce, bcap, cudaHostAllocDefault) != cudaSuccess) { delete w; return fail(-ENOMEM); }
+        if (cudaHostAlloc((void**)&w->bounce, bcap, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) {
+            delete w;
+            return fail(-ENOMEM);
+        }
+        if (cudaHostGetDevicePointer((void**)&w->bounce_d, w->bounce, 0) != cudaSuccess) { delete w; return fail(-EIO); }
         w->bcap = bcap;
-        w->ring = new BounceRing<cudaEvent_t, Worker::RingOps>(bcap, &w->ring_ops);
+        w->ring = new BounceRing<Worker::Tok, Worker::RingOps>(bcap, &w->ring_ops);
         w->reqs.reserve(4096);
         w->ops.reserve(8192);
         I->workers.push_back(w);
@@ -1434,20 +1553,18 @@ int gsys_trace_read(gsys_trace_rec* gpu_out, uint32_t gpu_cap, uint32_t* n_gpu, 
     return 0;
 }
 
-int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint32_t bx, uint32_t by, uint32_t bz,
-                void** args, size_t smem_bytes, void* stream) {
+int gsys_launch_begin(uint64_t nblocks, void* stream) {
     Instance* I = current();
     if (!I) return -ENODEV;
-    if (!kernel || gx == 0 || gy == 0 || gz == 0 || bx == 0 || by == 0 || bz == 0) return -EINVAL;
+    if (nblocks == 0 || nblocks > (1ull << 31)) return -EINVAL;
     cudaStream_t s = (cudaStream_t)stream;
-    uint64_t nb = (uint64_t)gx * gy * gz;
-    if (nb > (1ull << 31)) return -EINVAL;
+    const uint64_t nb = nblocks;
     if (nb > I->kblock_cap) {
         uint32_t cap = I->kblock_cap;
         while (cap < nb) cap <<= 1;
         uint32_t* nk = nullptr;
         if (cudaMalloc(&nk, (size_t)cap * GSYS_KSITES * 4) != cudaSuccess) return -ENOMEM;
-        cudaStreamSynchronize(s);
+        cudaDeviceSynchronize();   // no running kernel may still read the old array
         I->graveyard.push_back(I->kblock_d);
         I->kblock_d = nk;
         I->kblock_cap = cap;
@@ -1455,7 +1572,9 @@ int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint3
         I->ctx_h.kblock_cap = cap;
         if (cudaMemcpy(I->ctx_d, &I->ctx_h, sizeof I->ctx_h, cudaMemcpyHostToDevice) != cudaSuccess) return -EIO;
     }
-    // reset the kernel-scope call sites for this launch (block rounds + per-round records)
+    // reset the kernel-scope call sites for this launch (block rounds + per-round records); they
+    // are shared by the instance: kernel-scope calls of launches running concurrently on other
+    // streams are not supported (gsys.h)
     cudaMemsetAsync(I->kblock_d, 0, (size_t)nb * GSYS_KSITES * 4, s);
     cudaMemsetAsync(I->krounds_d, 0, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS, s);
     // the learned pre-poll sleep (reading B3) is relearned per launch: a hint carried over from
@@ -1467,8 +1586,33 @@ int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint3
         std::lock_guard<std::mutex> lk(I->sleep_mu);
         I->sleep_cv.notify_all();
     }
-    cudaError_t e = cudaLaunchKernel(kernel, dim3(gx, gy, gz), dim3(bx, by, bz), args, smem_bytes, s);
-    return cuda_err(e);
+    return cuda_err(cudaGetLastError());
+}
+
+int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint32_t bx, uint32_t by, uint32_t bz,
+                void** args, size_t smem_bytes, void* stream) {
+    if (!kernel || gx == 0 || gy == 0 || gz == 0 || bx == 0 || by == 0 || bz == 0) return -EINVAL;
+    int rc = gsys_launch_begin((uint64_t)gx * gy * gz, stream);
+    if (rc) return rc;
+    return cuda_err(cudaLaunchKernel(kernel, dim3(gx, gy, gz), dim3(bx, by, bz), args, smem_bytes,
+                                     (cudaStream_t)stream));
+}
+
+int gsys_launch_cu(void* cu_function, uint32_t gx, uint32_t gy, uint32_t gz, uint32_t bx, uint32_t by, uint32_t bz,
+                   void** args, size_t smem_bytes, void* stream) {
+    if (!cu_function || gx == 0 || gy == 0 || gz == 0 || bx == 0 || by == 0 || bz == 0) return -EINVAL;
+    int rc = gsys_launch_begin((uint64_t)gx * gy * gz, stream);
+    if (rc) return rc;
+    if (smem_bytes > 48 * 1024 &&
+        p_funcsetattr((CUfunction)cu_function, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem_bytes) !=
+            CUDA_SUCCESS)
+        return -EINVAL;
+    const CUresult r = p_launch((CUfunction)cu_function, gx, gy, gz, bx, by, bz, (unsigned)smem_bytes,
+                                (CUstream)stream, args, nullptr);
+    if (r == CUDA_SUCCESS) return 0;
+    if (r == CUDA_ERROR_INVALID_VALUE || r == CUDA_ERROR_INVALID_HANDLE) return -EINVAL;
+    if (r == CUDA_ERROR_OUT_OF_MEMORY) return -ENOMEM;
+    return -EIO;
 }
 
 int gsys_wait(void* stream) {
@@ -1477,14 +1621,156 @@ int gsys_wait(void* stream) {
     cudaError_t e = stream ? cudaStreamSynchronize((cudaStream_t)stream) : cudaDeviceSynchronize();
     if (e != cudaSuccess) return cuda_err(e);
     uint32_t tail = 0;
+    gsys_wd_log wd;
     cudaMemcpyAsync(&tail, I->tail_d, 4, cudaMemcpyDeviceToHost, I->ctl);
+    cudaMemcpyAsync(&wd, I->wd_d, sizeof wd, cudaMemcpyDeviceToHost, I->ctl);
     cudaStreamSynchronize(I->ctl);
     uint64_t h = I->head.load(std::memory_order_acquire);
     uint64_t issued = h + (uint64_t)(uint32_t)(tail - (uint32_t)h);
-    while (I->head.load(std::memory_order_acquire) < issued || I->completed.load(std::memory_order_acquire) < issued)
+    // drain: every published request served and its completion landed (P34.9).  After a watchdog
+    // expiry a request may never complete (a lost completion, a call that never returns): then
+    // the drain is bounded by the same timeout.
+    const uint64_t t0 = now_ns();
+    const uint64_t lim = wd.count ? std::max<uint64_t>(I->ctx_h.poll_timeout_ns, 1000000ull) : 0;
+    bool drained = true;
+    while (I->head.load(std::memory_order_acquire) < issued || I->completed.load(std::memory_order_acquire) < issued) {
+        if (lim && now_ns() - t0 > lim) { drained = false; break; }
         std::this_thread::yield();
+    }
     for (Worker* w : I->workers) cudaStreamSynchronize(w->stream);
+    if (wd.count) {
+        // slots whose waits expired were left claimed (the host might still complete into them);
+        // once the service is drained they are returned to free -- every slot after a
+        // device-wide wait (no kernel can hold a claim then), else the logged ones
+        if (drained) {
+            if (!stream) {
+                cudaMemsetAsync(I->claim_d, 0, (size_t)I->nslots * 4, I->ctl);
+                cudaMemsetAsync(I->nbpend_d, 0, (size_t)I->nslots * 4, I->ctl);
+            } else {
+                for (uint32_t i = 0; i < std::min<uint32_t>(wd.count, GSYS_WD_RECS); i++) {
+                    const uint32_t s = wd.rec[i].slot;
+                    if (wd.rec[i].phase == GSYS_WD_KERNEL || wd.rec[i].phase == GSYS_WD_CLAIM || s >= I->nslots) continue;
+                    cudaMemsetAsync(I->claim_d + s, 0, 4, I->ctl);
+                    cudaMemsetAsync(I->nbpend_d + s, 0, 4, I->ctl);
+                }
+            }
+        }
+        {
+            std::lock_guard<std::mutex> g(I->wd_mu);
+            I->wd_last = wd;
+        }
+        cudaMemsetAsync(I->wd_d, 0, sizeof(gsys_wd_log), I->ctl);
+        cudaStreamSynchronize(I->ctl);
+        I->first_err.store(0);
+        return -ETIMEDOUT;
+    }
     return I->first_err.exchange(0);
+}
+
+int gsys_watchdog_read(uint32_t* count, uint32_t* recs, uint32_t cap) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    std::lock_guard<std::mutex> g(I->wd_mu);
+    if (count) *count = I->wd_last.count;
+    const uint32_t k = std::min<uint32_t>(std::min<uint32_t>(I->wd_last.count, GSYS_WD_RECS), cap);
+    for (uint32_t i = 0; recs && i < k; i++) {
+        recs[4 * i + 0] = I->wd_last.rec[i].slot;
+        recs[4 * i + 1] = I->wd_last.rec[i].seq;
+        recs[4 * i + 2] = I->wd_last.rec[i].nr;
+        recs[4 * i + 3] = I->wd_last.rec[i].phase;
+    }
+    return (int)k;
+}
+
+int gsys_set_poll_timeout(uint32_t ms) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;   // running kernels read the context
+    I->ctx_h.poll_timeout_ns = (unsigned long long)ms * 1000000ull;
+    if (cudaMemcpy(I->ctx_d, &I->ctx_h, sizeof I->ctx_h, cudaMemcpyHostToDevice) != cudaSuccess) return -EIO;
+    return 0;
+}
+
+// ---------------------------------------------------------------- clock relation (trace timestamps)
+}  // extern "C"
+namespace {
+// One thread: measure the %globaltimer tick, then `samples` ping-pongs with the host through
+// host-mapped words; t[2i], t[2i+1] = GPU time before the ping and after the pong.
+__global__ void clock_sync_kernel(unsigned* ping, const unsigned* pong, unsigned long long* t, unsigned samples,
+                                  unsigned long long* tick) {
+    unsigned long long prev = gsys::globaltimer(), best = ~0ull;
+    for (int i = 0; i < 20000 && best > 1; i++) {
+        const unsigned long long x = gsys::globaltimer();
+        if (x != prev) { if (x - prev < best) best = x - prev; prev = x; }
+    }
+    *tick = best;
+    for (unsigned i = 1; i <= samples; i++) {
+        const unsigned long long g0 = gsys::globaltimer();
+        asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(ping), "r"(i) : "memory");
+        const unsigned long long tlim = g0 + 1000000000ull;
+        unsigned v;
+        do {
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(pong) : "memory");
+        } while (v != i && gsys::globaltimer() < tlim);
+        t[2 * i - 2] = g0;
+        t[2 * i - 1] = v == i ? gsys::globaltimer() : 0ull;
+        if (v != i) return;
+    }
+}
+}  // namespace
+extern "C" {
+
+int gsys_clock_sync(uint32_t samples, int64_t* offset_ns, uint64_t* uncertainty_ns) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    if (samples == 0 || samples > 4096 || !offset_ns || !uncertainty_ns) return -EINVAL;
+    const size_t bytes = 256 + 16ull * samples;
+    uint8_t* buf = nullptr;
+    if (cudaHostAlloc((void**)&buf, bytes, cudaHostAllocMapped) != cudaSuccess) return -ENOMEM;
+    memset(buf, 0, bytes);
+    uint8_t* dbuf = nullptr;
+    cudaHostGetDevicePointer((void**)&dbuf, buf, 0);
+    volatile unsigned* ping = (volatile unsigned*)buf;
+    volatile unsigned* pong = (volatile unsigned*)(buf + 64);
+    unsigned long long* tick = (unsigned long long*)(buf + 128);
+    unsigned long long* t = (unsigned long long*)(buf + 256);
+    std::vector<uint64_t> h(samples, 0);
+    clock_sync_kernel<<<1, 1, 0, I->ctl>>>((unsigned*)dbuf, (const unsigned*)(dbuf + 64),
+                                           (unsigned long long*)(dbuf + 256), samples,
+                                           (unsigned long long*)(dbuf + 128));
+    int rc = cuda_err(cudaGetLastError());
+    for (uint32_t i = 1; rc == 0 && i <= samples; i++) {
+        const uint64_t tl = now_ns() + 1000000000ull;
+        while (__atomic_load_n(ping, __ATOMIC_ACQUIRE) != i) {
+            if (now_ns() > tl) { rc = -ETIMEDOUT; break; }
+        }
+        if (rc) break;
+        h[i - 1] = now_ns();
+        __atomic_store_n(pong, i, __ATOMIC_RELEASE);
+    }
+    if (cudaStreamSynchronize(I->ctl) != cudaSuccess && rc == 0) rc = -EIO;
+    if (rc == 0) {
+        uint64_t best = ~0ull;
+        for (uint32_t i = 0; i < samples; i++) {
+            const uint64_t g0 = t[2 * i], g1 = t[2 * i + 1];
+            if (!g1 || g1 < g0) continue;
+            if (g1 - g0 < best) {
+                best = g1 - g0;
+                *offset_ns = (int64_t)(h[i] - (g0 + (g1 - g0) / 2));
+            }
+        }
+        if (best == ~0ull) rc = -EIO;
+        else *uncertainty_ns = best / 2 + *tick;
+    }
+    cudaFreeHost(buf);
+    return rc;
+}
+
+int gsys_set_fault_drop(int64_t offset) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    I->drop_off.store(offset < 0 ? -1 : offset);
+    return 0;
 }
 
 int gsys_shutdown(void) {
@@ -1523,6 +1809,7 @@ int gsys_shutdown(void) {
     cudaFree(I->krounds_d);
     cudaFree(I->kblock_d);
     cudaFree(I->ctx_d);
+    cudaFree(I->wd_d);
     if (I->gtrace_d) cudaFree(I->gtrace_d);
     if (I->gtrace_n_d) cudaFree(I->gtrace_n_d);
     for (void* p : I->graveyard) cudaFree(p);

@@ -280,12 +280,12 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     __shared__ unsigned s_kq;
     if (a.prefetch) {
         // Non-blocking work-group preads, double-buffered (P20.34-46 "non-blocking ... the GPU
-        // continues"): the read of the next chunk is issued before this chunk is scanned.  No
-        // separate wait is needed: a slot holds one request at a time (reading A15), so the next
-        // call's claim -- the next prefetch, or a blocking 0-byte pread at the end -- returns only
-        // after the host completed this one, and Bar2 hands that to the whole work-group.  A
-        // non-blocking pread returns 0 (A4): the scan takes the bytes a regular file of stable size
-        // returns (min(len, size - off)); an error surfaces at gsys_wait.
+        // continues"): the read of the next chunk is issued before this chunk is scanned, and the
+        // scan of a line starts after an explicit wait on that read's completion token (slot,
+        // seq) -- whatever slot the next call landed in (%smid / %warpid are volatile).  A
+        // non-blocking pread returns 0 (A4): the scan takes the bytes a regular file of stable
+        // size returns (min(len, size - off)); an error surfaces at gsys_wait.
+        __shared__ gsys_token s_tok[2];
         WcChunk c0, c1;
         bool have = wc_next_chunk(a, &s_kq, c0);
         unsigned cur = 0;
@@ -298,7 +298,7 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
             bool hb;
             unsigned char* b = line_of(c0, 0, hb);
             const long long r = gsys_pread(a.ctx, a.fds[c0.f], b + 16 - (c0.s - c0.off), (size_t)c0.len, c0.off,
-                                           nbflags | (hb ? GSYS_HOSTBUF : 0u));
+                                           nbflags | (hb ? GSYS_HOSTBUF : 0u), &s_tok[0]);
             if (threadIdx.x == 0 && a.req_ret) a.req_ret[c0.k] = r;
         }
         while (have) {
@@ -307,11 +307,10 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
                 bool hb;
                 unsigned char* b = line_of(c1, cur ^ 1u, hb);
                 const long long r = gsys_pread(a.ctx, a.fds[c1.f], b + 16 - (c1.s - c1.off), (size_t)c1.len, c1.off,
-                                               nbflags | (hb ? GSYS_HOSTBUF : 0u));
+                                               nbflags | (hb ? GSYS_HOSTBUF : 0u), &s_tok[cur ^ 1u]);
                 if (threadIdx.x == 0 && a.req_ret) a.req_ret[c1.k] = r;
-            } else {
-                gsys_pread(a.ctx, a.fds[c0.f], hbase, 0, 0, a.gflags | GSYS_HOSTBUF);   // drain the slot
             }
+            gsys_wait_token(a.ctx, &s_tok[cur], GSYS_WG);   // this line's bytes have landed
             bool hb;
             unsigned char* base = line_of(c0, cur, hb);
             const bool grep = a.file_hits != nullptr && sT.npat > 0 && *(volatile unsigned*)&a.file_hits[c0.f] == 0u;

@@ -187,6 +187,8 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
     __shared__ unsigned s_found, s_len, s_keylen, s_bucket, s_ok, s_done, s_fromlen;
     __shared__ __align__(16) unsigned char s_rx[80];      // frame + header + extras + key (<= 32 + 16 + 32)
     __shared__ __align__(16) unsigned char s_key[MC_MAXKEY];
+    __shared__ gsys_token s_stok;   // the previous (non-blocking) reply's sendto
+    if (threadIdx.x == 0) { s_stok.slot = 0u; s_stok.seq = 0u; }
     unsigned char* io = a.io + (size_t)blockIdx.x * MC_IO_BYTES;
     unsigned char* rx = io + MC_RX;
     unsigned char* tx = io + MC_TX;
@@ -194,6 +196,9 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
     unsigned* fromlen = reinterpret_cast<unsigned*>(io + MC_FROMLEN);
     const unsigned gf = a.gflags | GSYS_HOSTBUF;
     for (;;) {
+        // the reply buffer and `from` may still be read by the previous non-blocking sendto: wait
+        // for that request by its token, whatever slot this work-group's next call lands in
+        if (a.send_gflags & GSYS_NONBLOCKING) gsys_wait_token(a.ctx, &s_stok, GSYS_WG);
         if (threadIdx.x == 0) *(volatile unsigned*)fromlen = 128u;
         const long long r = gsys_recvfrom(a.ctx, a.fd, rx, 2048, 0, from, fromlen, gf);   // producer: Bar2
         if (r < 0) {
@@ -238,6 +243,7 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
         const bool hit = s_found != 0xffffffffu;
         const McEntry* e = hit ? B + s_found : nullptr;
         const unsigned vlen = hit ? e->vlen : 0u;
+
         // reply: UDP frame header + binary response header (+ flags + value | "Not found")
         if (threadIdx.x == 0) {
             const unsigned char* v = s_rx;
@@ -267,7 +273,7 @@ __global__ void __launch_bounds__(256) mc_kernel(McArgs a) {
             for (unsigned i = threadIdx.x; i < vlen; i += blockDim.x) tx[36 + i] = src[i];
         }
         // consumer call: Bar1 (the reply is complete) is kept under relaxed ordering
-        gsys_sendto(a.ctx, a.fd, tx, s_len, 0, from, s_fromlen, a.send_gflags | GSYS_HOSTBUF);
+        gsys_sendto(a.ctx, a.fd, tx, s_len, 0, from, s_fromlen, a.send_gflags | GSYS_HOSTBUF, &s_stok);
         __syncthreads();
     }
 }

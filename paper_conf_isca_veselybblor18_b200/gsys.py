@@ -47,7 +47,7 @@ class Stats(ctypes.Structure):
 class TraceRec(ctypes.Structure):
     _fields_ = [("slot", ctypes.c_uint32), ("seq", ctypes.c_uint32), ("frm", ctypes.c_uint8),
                 ("to", ctypes.c_uint8), ("actor", ctypes.c_uint8), ("blocking", ctypes.c_uint8),
-                ("pad", ctypes.c_uint32)]
+                ("nr", ctypes.c_uint32), ("t_ns", ctypes.c_uint64)]
 
 
 _P = ctypes.c_void_p
@@ -66,12 +66,18 @@ SIGNATURES = {
     "gsys_diag_phases": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int]),
     "gsys_set_trace": (ctypes.c_int, [ctypes.c_int, _U32]),
     "gsys_launch": (ctypes.c_int, [_P, _U32, _U32, _U32, _U32, _U32, _U32, _P, ctypes.c_size_t, _P]),
+    "gsys_launch_cu": (ctypes.c_int, [_P, _U32, _U32, _U32, _U32, _U32, _U32, _P, ctypes.c_size_t, _P]),
+    "gsys_launch_begin": (ctypes.c_int, [_U64, _P]),
     "gsys_wait": (ctypes.c_int, [_P]),
     "gsys_shutdown": (ctypes.c_int, []),
     "gsys_device_ctx": (_P, []),
     "gsys_stats": (ctypes.c_int, [_P]),
     "gsys_stats_reset": (ctypes.c_int, []),
     "gsys_trace_read": (ctypes.c_int, [_P, _U32, _P, _P, _U32, _P]),
+    "gsys_clock_sync": (ctypes.c_int, [_U32, _P, _P]),
+    "gsys_set_poll_timeout": (ctypes.c_int, [_U32]),
+    "gsys_set_fault_drop": (ctypes.c_int, [_I64]),
+    "gsys_watchdog_read": (ctypes.c_int, [_P, _P, _U32]),
     "gsys_abi_info": (ctypes.c_int, [_P, _P, _P]),
     "gsys_plan_merge": (ctypes.c_int, [_U32, _P, _P, _P, _U64, _P, _P, _P, _P, _P]),
     "gsys_split_result": (_I64, [_I64, _U64, _U64]),
@@ -164,7 +170,8 @@ def gsys_set_trace(on: bool, capacity: int = 0) -> int:
 
 
 def gsys_wait(stream=None) -> int:
-    """Drain: returns the first non-blocking -errno (or 0); raises only on CUDA errors."""
+    """Drain: returns the first non-blocking -errno, -ETIMEDOUT after a watchdog expiry, or 0;
+    raises only on CUDA errors."""
     rc = lib().gsys_wait(_stream(stream))
     if rc < 0 and -rc in (5,):   # EIO from CUDA
         raise GsysError(-rc, "gsys_wait")
@@ -190,14 +197,41 @@ def gsys_stats_reset() -> int:
 
 
 def gsys_trace_read(cap: int = 1 << 20):
+    """Both sides' trace records as tuples (slot, seq, from, to, actor, blocking, nr, t_ns); GPU
+    t_ns is %globaltimer, host t_ns CLOCK_MONOTONIC (relate them with gsys_clock_sync)."""
     g = (TraceRec * cap)()
     h = (TraceRec * cap)()
     ng = ctypes.c_uint32(0)
     nh = ctypes.c_uint32(0)
     _check(lib().gsys_trace_read(g, cap, ctypes.byref(ng), h, cap, ctypes.byref(nh)), "gsys_trace_read")
-    conv = lambda arr, n: [(r.slot, r.seq, r.frm, r.to, "gpu" if r.actor == 0 else "cpu", bool(r.blocking))  # noqa: E731
-                           for r in arr[: min(n, cap)]]
+    conv = lambda arr, n: [(r.slot, r.seq, r.frm, r.to, "gpu" if r.actor == 0 else "cpu", bool(r.blocking),  # noqa: E731
+                            r.nr, r.t_ns) for r in arr[: min(n, cap)]]
     return conv(g, ng.value), conv(h, nh.value)
+
+
+def gsys_clock_sync(samples: int = 256):
+    """(offset_ns, uncertainty_ns): host CLOCK_MONOTONIC = GPU %globaltimer + offset, +- uncertainty."""
+    off = ctypes.c_int64(0)
+    unc = ctypes.c_uint64(0)
+    _check(lib().gsys_clock_sync(samples, ctypes.byref(off), ctypes.byref(unc)), "gsys_clock_sync")
+    return off.value, unc.value
+
+
+def gsys_set_poll_timeout(ms: int) -> int:
+    return _check(lib().gsys_set_poll_timeout(ms), "gsys_set_poll_timeout")
+
+
+def gsys_set_fault_drop(offset: int) -> int:
+    """Test hook: the pread at `offset` is served but its completion is never written (-1 = off)."""
+    return _check(lib().gsys_set_fault_drop(offset), "gsys_set_fault_drop")
+
+
+def gsys_watchdog_read(cap: int = 64):
+    """(count, [(slot, seq, nr, phase)]) of the last gsys_wait that returned -ETIMEDOUT."""
+    cnt = ctypes.c_uint32(0)
+    recs = (ctypes.c_uint32 * (4 * cap))()
+    k = _check(lib().gsys_watchdog_read(ctypes.byref(cnt), recs, cap), "gsys_watchdog_read")
+    return cnt.value, [tuple(recs[4 * i: 4 * i + 4]) for i in range(k)]
 
 
 def gsys_set_profile(on: bool) -> int:

@@ -284,6 +284,43 @@ def test_errors_surface(file1m):
     assert G.gsys_wait() == 0                                     # cleared
 
 
+# ---------------------------------------------------------------------------- watchdog
+@pytest.mark.parametrize("gran,length", [(G.WG, 4096), (G.WG, 100000), (G.WI, 100)])
+def test_watchdog_lost_completion(file1m, gran, length):
+    """A completion the host never writes (gsys_set_fault_drop) must not hang the GPU: the caller's
+    wait expires with -ETIMEDOUT (PAPER.md:30 P30.0, PAPER.md:22 P22.0), gsys_wait reports it with
+    the slot / request / phase, the slot is returned to free, and the next launch is unaffected."""
+    import time
+    size = os.path.getsize(file1m)
+    fd = os.open(file1m, os.O_RDONLY)
+    blocks, threads, iters = 2, (32 if gran == G.WI else 64), 2
+    callers = blocks * threads if gran == G.WI else blocks
+    d_buf = torch.zeros(callers * length, dtype=torch.uint8, device="cuda")
+    lost = (1 * length) % size                  # caller 0, second call
+    try:
+        G.gsys_set_poll_timeout(300)
+        G.gsys_set_fault_drop(lost)
+        t0 = time.time()
+        _, ret, _, _, rc = W.bench_calls("pread", gran | G.BLOCKING, blocks, threads, iters, fd, length, size, d_buf)
+        dt = time.time() - t0
+        G.gsys_set_fault_drop(-1)
+        assert rc == -errno.ETIMEDOUT
+        cnt, recs = G.gsys_watchdog_read()
+        assert cnt == 1 and recs[0][2] == G.NR_PREAD64 and recs[0][3] == 3, (cnt, recs)
+        want = [plan.expected_pread_ret(size, (i * length) % size, length) for i in range(callers * iters)]
+        want[1] = -errno.ETIMEDOUT
+        assert ret.tolist() == want
+        assert dt < 10, dt
+        # the poisoned slot was freed: the same calls now all complete
+        _, ret, _, _, rc = W.bench_calls("pread", gran | G.BLOCKING, blocks, threads, iters, fd, length, size, d_buf)
+        assert rc == 0 and ret.tolist() == [plan.expected_pread_ret(size, (i * length) % size, length)
+                                            for i in range(callers * iters)]
+    finally:
+        G.gsys_set_fault_drop(-1)
+        G.gsys_set_poll_timeout(20000)
+        os.close(fd)
+
+
 # ---------------------------------------------------------------------------- ordering semantics
 @pytest.mark.parametrize("gran,blk,order", [(G.WG, G.BLOCKING, G.STRONG), (G.WG, G.BLOCKING, G.RELAXED),
                                             (G.WG, G.NONBLOCKING, G.RELAXED), (G.WI, G.BLOCKING, G.STRONG),
@@ -311,34 +348,74 @@ def test_pwrite_consumer_barrier(tmpdir_shm, gran, blk, order):
 
 
 # ---------------------------------------------------------------------------- protocol trace (rows a2-a5, a7)
-def test_protocol_trace_validates(file1m):
-    size = os.path.getsize(file1m)
+def _traced(run):
+    """Run `run()` with protocol tracing on; return (records, eps): records are (req=(slot, seq),
+    slot, from, to, actor, t) from both logs, unsorted, GPU times mapped onto the host clock with
+    gsys_clock_sync taken before and after; eps = the clock relation's error bound."""
+    off0, unc0 = G.gsys_clock_sync(256)
     G.gsys_set_trace(True, 1 << 16)
     try:
-        fd = os.open(file1m, os.O_RDONLY)
-        d_buf = torch.zeros(8 * 2000, dtype=torch.uint8, device="cuda")
-        try:
-            W.bench_calls("pread", G.WG | G.BLOCKING, 8, 64, 3, fd, 2000, size, d_buf)
-            W.bench_calls("getrusage", G.WG | G.NONBLOCKING | G.RELAXED, 8, 64, 2)
-            W.bench_calls("getrusage", G.WI | G.BLOCKING, 2, 64, 1)
-        finally:
-            os.close(fd)
+        run()
+        assert G.gsys_wait() == 0
         gtr, htr = G.gsys_trace_read()
     finally:
         G.gsys_set_trace(False)
-    by_req = {}
-    for rec in gtr + htr:
-        by_req.setdefault((rec[0], rec[1]), []).append(rec)
-    assert len(by_req) == 8 * 3 + 8 * 2 + 2 * 64
-    records, blocking = [], {}
-    for req, recs in by_req.items():
-        pre = [r for r in recs if r[4] == "gpu" and r[2] in (protocol.FREE, protocol.POPULATING)]
-        host = [r for r in recs if r[4] == "cpu"]
-        post = [r for r in recs if r[4] == "gpu" and r[2] == protocol.FINISHED]
-        for r in pre + host + post:
-            records.append((req, r[0], r[2], r[3], r[4]))
-        blocking[req] = recs[0][5]
-    assert protocol.check_trace(records, lambda r: blocking[r]) == len(by_req)
+    off1, unc1 = G.gsys_clock_sync(256)
+    off = (off0 + off1) // 2
+    eps = max(unc0, unc1) + abs(off1 - off0) // 2 + 1
+    recs = [((r[0], r[1]), r[0], r[2], r[3], r[4], r[7] + (off if r[4] == "gpu" else 0)) for r in gtr + htr]
+    blocking = {}
+    for r in gtr + htr:
+        blocking.setdefault((r[0], r[1]), r[5])
+    return recs, blocking, eps, gtr, htr
+
+
+def test_clock_sync_is_tight():
+    off, unc = G.gsys_clock_sync(256)
+    assert 0 < unc < 20000, unc          # a PCIe round trip: a few microseconds
+    off2, unc2 = G.gsys_clock_sync(256)
+    assert abs(off2 - off) <= unc + unc2 + 2000
+
+
+def test_protocol_trace_validates(file1m):
+    """Rows a2-a5/a7 against oracle/protocol.check_trace: the GPU and host logs as recorded
+    (never reordered), every request's path in timestamp order, one live request per slot,
+    sequence numbers growing per slot -- at WG, WI and kernel granularity, blocking and
+    non-blocking (WG non-blocking calls reuse their slot back to back: P24.11, A15)."""
+    size = os.path.getsize(file1m)
+    fd = os.open(file1m, os.O_RDONLY)
+    d_buf = torch.zeros(64 * 2000, dtype=torch.uint8, device="cuda")
+
+    def run():
+        W.bench_calls("pread", G.WG | G.BLOCKING, 8, 64, 3, fd, 2000, size, d_buf)
+        W.bench_calls("getrusage", G.WG | G.NONBLOCKING | G.RELAXED, 8, 64, 2)
+        W.bench_calls("getrusage", G.WI | G.BLOCKING, 2, 64, 1)
+        W.bench_calls("getrusage", G.KERNEL | G.BLOCKING | G.RELAXED, 4, 64, 4)
+        W.bench_calls("pread", G.KERNEL | G.NONBLOCKING | G.RELAXED, 2, 64, 3, fd, 2000, size, d_buf)
+        W.bench_calls("pread", G.WI | G.NONBLOCKING, 1, 32, 2, fd, 2000, size, d_buf)
+    try:
+        recs, blocking, eps, gtr, htr = _traced(run)
+    finally:
+        os.close(fd)
+    assert eps < 20000, eps
+    n_req = 8 * 3 + 8 * 2 + 2 * 64 + 4 + 3 + 32 * 2
+    assert len(blocking) == n_req
+    assert protocol.check_trace(recs, blocking.__getitem__, eps=eps, seq_of=lambda r: r[1]) == n_req
+    # the host-visible state word is returned to free by the GPU for blocking calls (A3) and by
+    # the host for non-blocking ones (P24.34)
+    assert sum(1 for r in gtr if r[3] == protocol.FREE) == sum(1 for b in blocking.values() if b)
+    assert sum(1 for r in htr if r[3] == protocol.FREE) == sum(1 for b in blocking.values() if not b)
+
+
+def test_protocol_trace_catches_a_reordered_log(file1m):
+    """The checker is not vacuous on real logs: moving one host pick-up before its GPU publish
+    by more than the clock error fails."""
+    recs, blocking, eps, _, _ = _traced(lambda: W.bench_calls("getrusage", G.WG | G.BLOCKING, 4, 64, 2))
+    assert protocol.check_trace(recs, blocking.__getitem__, eps=eps) == 8
+    ready = {r[0]: r[5] for r in recs if r[3] == protocol.READY}
+    bad = [r if r[3] != protocol.PROCESSING else r[:5] + (ready[r[0]] - eps - 1,) for r in recs]
+    with pytest.raises(AssertionError):
+        protocol.check_trace(bad, blocking.__getitem__, eps=eps)
 
 
 # ---------------------------------------------------------------------------- full size (config 3 shape)
@@ -492,3 +569,57 @@ def test_pread_per_call_cap_from_gpu(tmpdir_shm, hostbuf):
     probe = torch.tensor([0, 1 << 20, cap - 1, cap], dtype=torch.int64)
     got = buf[probe.to(buf.device)].cpu().tolist()
     assert got == [0x11, 0x22, 0x33, 0]      # the byte at the cap was not read
+
+
+# ---------------------------------------------------------------------------- boundary: external kernels
+@pytest.fixture(scope="module")
+def ext_lib(tmpdir_shm):
+    """tests/native/ext_kernel.cu compiled as its own module (own CUDA runtime), against
+    include/gsys_device.cuh only."""
+    import ctypes
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = os.path.join(tmpdir_shm, "libext_kernel.so")
+    subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-O2", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
+                           "-gencode", "arch=compute_100a,code=sm_100a", "-I", os.path.join(root, "include"),
+                           os.path.join(root, "tests", "native", "ext_kernel.cu"), "-o", out])
+    L = ctypes.CDLL(out)
+    L.ext_function.argtypes = [ctypes.c_void_p]
+    return L
+
+
+@pytest.mark.parametrize("nwarps,length", [(4, 3000), (8, 65536)])
+def test_external_kernel_tokens(file1m, ext_lib, nwarps, length):
+    """A kernel from another module, launched with gsys_launch_cu: non-blocking work-item preads
+    issued one after the other by different warps, each waited for by ANOTHER thread through its
+    explicit (slot, seq) token (no reliance on hardware-slot reuse, P24.11 / P20.34-38), plus a
+    blocking work-group pread; every return value and byte sum equals the direct read."""
+    import ctypes
+    size = os.path.getsize(file1m)
+    data = np.fromfile(file1m, dtype=np.uint8)
+    fn = ctypes.c_void_p(0)
+    assert ext_lib.ext_function(ctypes.byref(fn)) == 0 and fn.value
+
+    class ExtArgs(ctypes.Structure):
+        _fields_ = [("ctx", ctypes.c_void_p), ("dbuf", ctypes.c_void_p), ("ret", ctypes.c_void_p),
+                    ("sum", ctypes.c_void_p), ("size", ctypes.c_uint64), ("len", ctypes.c_uint32),
+                    ("fd", ctypes.c_int32)]
+    blocks = 6
+    n = blocks * (nwarps + 1)
+    dbuf = torch.zeros(n * length, dtype=torch.uint8, device="cuda")
+    ret = torch.full((n,), -(1 << 40), dtype=torch.int64, device="cuda")
+    sm = torch.zeros(n, dtype=torch.int64, device="cuda")
+    fd = os.open(file1m, os.O_RDONLY)
+    try:
+        a = ExtArgs(G.gsys_device_ctx(), dbuf.data_ptr(), ret.data_ptr(), sm.data_ptr(), size, length, fd)
+        argv = (ctypes.c_void_p * 1)(ctypes.cast(ctypes.pointer(a), ctypes.c_void_p))
+        rc = G.lib().gsys_launch_cu(fn, blocks, 1, 1, 32 * nwarps, 1, 1, argv, 0, None)
+        assert rc == 0
+        assert G.gsys_wait() == 0
+    finally:
+        os.close(fd)
+    for i in range(n):
+        off = (i * length) % size
+        want = data[off: off + length]
+        assert int(ret[i]) == len(want), i
+        assert int(sm[i]) == int(want.astype(np.int64).sum()), i

@@ -213,6 +213,30 @@ def test_protocol_model_paths():
     assert protocol.check_trace(tr, lambda r: dict((a, c) for a, _, c in reqs)[r], 4) == 5
     assert m.state == [protocol.FREE] * 4
     assert len(tr) == sum(len(protocol.expected_path(b)) for _, _, b in reqs)
+    # the checker takes the two actors' logs in any order: concatenated GPU log + host log
+    gpu = [r for r in tr if r[4] == "gpu"]
+    cpu = [r for r in tr if r[4] == "cpu"]
+    assert protocol.check_trace(cpu + gpu, lambda r: dict((a, c) for a, _, c in reqs)[r], 4) == 5
+
+
+def _interleaved_two_slots():
+    """A valid concurrent schedule: requests 0 (slot 0, blocking) and 1 (slot 1, non-blocking)
+    overlap in time; then request 2 reuses slot 1 after the host freed it."""
+    m = protocol.SlotMachine(2)
+    m.claim(0, 0); m.claim(1, 1); m.publish(1, 1); m.publish(0, 0)
+    m.pick_up(0, 0); m.pick_up(1, 1); m.complete(1, 1, False); m.complete(0, 0, True)
+    assert not m.claim(2, 0)                  # slot 0 still finished: the caller is delayed (P24.11)
+    m.claim(2, 1); m.consume(0, 0); m.publish(2, 1); m.pick_up(2, 1); m.complete(2, 1, True); m.consume(2, 1)
+    return m.trace, {0: True, 1: False, 2: True}
+
+
+def test_protocol_interleaved_schedule_is_valid():
+    tr, blk = _interleaved_two_slots()
+    assert protocol.check_trace(tr, blk.__getitem__, 2) == 3
+
+
+def _retime(tr, req, edge, t):
+    return [r if (r[0], r[2], r[3]) != (req,) + edge else r[:5] + (t,) for r in tr]
 
 
 def test_protocol_model_rejects_violations():
@@ -225,12 +249,63 @@ def test_protocol_model_rejects_violations():
     blk = lambda r: True  # noqa: E731
     with pytest.raises(AssertionError):                # dropped edge
         protocol.check_trace(good[:-1], blk)
+    with pytest.raises(AssertionError):                # duplicated edge
+        protocol.check_trace(good + [good[2]], blk)
     with pytest.raises(AssertionError):                # wrong actor
         bad = list(good)
-        bad[2] = bad[2][:4] + ("gpu",)
+        bad[2] = bad[2][:4] + ("gpu",) + bad[2][5:]
         protocol.check_trace(bad, blk)
     with pytest.raises(AssertionError):                # non-blocking request that waited for finished
         protocol.check_trace(good, lambda r: False)
+
+
+def test_protocol_rejects_host_pickup_before_ready():
+    tr, blk = _interleaved_two_slots()
+    t_ready = [r for r in tr if r[0] == 0 and r[3] == protocol.READY][0][5]
+    bad = _retime(tr, 0, (protocol.READY, protocol.PROCESSING), t_ready - 3)
+    with pytest.raises(AssertionError, match="precedes"):
+        protocol.check_trace(bad, blk.__getitem__)
+    # within the cross-actor clock error it is accepted, beyond it not
+    assert protocol.check_trace(bad, blk.__getitem__, eps=3) == 3
+    with pytest.raises(AssertionError, match="precedes"):
+        protocol.check_trace(bad, blk.__getitem__, eps=2)
+
+
+def test_protocol_rejects_consume_before_finish():
+    tr, blk = _interleaved_two_slots()
+    t_fin = [r for r in tr if r[0] == 2 and r[3] == protocol.FINISHED][0][5]
+    bad = _retime(tr, 2, (protocol.FINISHED, protocol.FREE), t_fin - 1)
+    with pytest.raises(AssertionError, match="precedes"):
+        protocol.check_trace(bad, blk.__getitem__)
+
+
+def test_protocol_rejects_two_live_requests_on_one_slot():
+    # request 2 claims slot 1 while request 1 (non-blocking) is still being processed there
+    m = protocol.SlotMachine(2)
+    tr, blk = _interleaved_two_slots()
+    t_free1 = [r for r in tr if r[0] == 1 and r[3] == protocol.FREE][0][5]
+    bad = _retime(tr, 2, (protocol.FREE, protocol.POPULATING), t_free1 - 2)
+    with pytest.raises(AssertionError, match="live"):
+        protocol.check_trace(bad, blk.__getitem__)
+    # the same overlap on the blocking slot: two requests on slot 0, the second claimed before
+    # the first was consumed (both GPU edges: no clock slack applies)
+    trace = m.run([(10, 0, True)]) + [(11, 0, protocol.FREE, protocol.POPULATING, "gpu", 4),
+                                     (11, 0, protocol.POPULATING, protocol.READY, "gpu", 6),
+                                     (11, 0, protocol.READY, protocol.PROCESSING, "cpu", 7),
+                                     (11, 0, protocol.PROCESSING, protocol.FINISHED, "cpu", 8),
+                                     (11, 0, protocol.FINISHED, protocol.FREE, "gpu", 9)]
+    with pytest.raises(AssertionError, match="live"):
+        protocol.check_trace(trace, lambda r: True, eps=100)
+    ok = [r if r[0] == 10 else r[:5] + (r[5] + 10,) for r in trace]
+    assert protocol.check_trace(ok, lambda r: True, eps=0) == 2
+
+
+def test_protocol_rejects_sequence_going_backwards():
+    trace = protocol.SlotMachine(1).run([((0, 5), 0, True), ((0, 4), 0, True)])
+    with pytest.raises(AssertionError, match="sequence"):
+        protocol.check_trace(trace, lambda r: True, seq_of=lambda r: r[1])
+    trace = protocol.SlotMachine(1).run([((0, 4), 0, True), ((0, 5), 0, False)])
+    assert protocol.check_trace(trace, lambda r: r[1] == 4, seq_of=lambda r: r[1]) == 2
 
 
 def test_request_count_closed_forms():
@@ -271,3 +346,41 @@ def test_owned_counts_partition_sums_to_whole():
         for s in range(0, n, chunk):
             tot += owned_counts(text, s, min(s + chunk, n), words)
         assert np.array_equal(tot, whole), (text, chunk)
+
+
+def test_permuted_blocks_hand_worked_example():
+    """plan.permuted_blocks (Fig. 8, PAPER.md:26 P26.21-27) against a hand-derived 4-block example
+    (tests/golden/fig8_permutation_tiny.json): gather direction (reading A20), one step per
+    iteration, blocks independent; the scatter direction is rejected."""
+    g = json.load(open(os.path.join(GOLDEN, "fig8_permutation_tiny.json")))
+    data = np.array(g["data"], dtype=np.uint8)
+    perm = np.array(g["perm"])
+    for k, want in g["expected"].items():
+        got = plan.permuted_blocks(data, perm, int(k), g["block_bytes"])
+        assert got.tolist() == want, k
+    assert plan.permuted_blocks(data, perm, 1, 4).tolist() != g["scatter_reading_1_step"]
+
+
+def test_permuted_blocks_group_properties():
+    """Iterations compose (p^a then p^b = p^(a+b)) and the permutation's order restores the input."""
+    rng = np.random.default_rng(5)
+    bs = 64
+    perm = rng.permutation(bs)
+    data = rng.integers(0, 256, size=4 * bs, dtype=np.uint8)
+    for a, b in [(1, 2), (3, 5), (0, 4)]:
+        once = plan.permuted_blocks(plan.permuted_blocks(data, perm, a, bs), perm, b, bs)
+        assert np.array_equal(once, plan.permuted_blocks(data, perm, a + b, bs))
+    # order of the permutation = lcm of its cycle lengths
+    import math
+    seen, lcm = np.zeros(bs, bool), 1
+    for i in range(bs):
+        if not seen[i]:
+            n, j = 0, i
+            while not seen[j]:
+                seen[j] = True
+                j = perm[j]
+                n += 1
+            lcm = lcm * n // math.gcd(lcm, n)
+    assert np.array_equal(plan.permuted_blocks(data, perm, lcm, bs), data)
+    if lcm > 1:
+        assert not np.array_equal(plan.permuted_blocks(data, perm, 1, bs), data)
