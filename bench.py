@@ -43,7 +43,9 @@ def parse():
     ap.add_argument("--order", default="relaxed", choices=["strong", "relaxed"])
     ap.add_argument("--blocks", type=int, default=148, help="work-groups (1 per SM: 0.8 %% above 2 per SM, profiles/r01_blocks_ab.jsonl)")
     ap.add_argument("--threads", type=int, default=256)
-    ap.add_argument("--staging", default="host", choices=["device", "host", "mixed"])
+    ap.add_argument("--staging", default="device", choices=["device", "host", "mixed"],
+                    help="device: preads land in HBM lines (default completion: the work-group pulls them "
+                         "from the service's host-mapped bounce, reading B13); host: zero-copy host lines")
     ap.add_argument("--dev16", type=int, default=4, help="mixed staging: chunks per 16 on the device (DMA) path")
     ap.add_argument("--cmax", type=int, default=8, help="coalescing max bundle (P22.13)")
     ap.add_argument("--window", type=int, default=0, help="coalescing window us (P22.13)")
@@ -139,7 +141,9 @@ def workload_config(a, nbytes, world):
         "staging": a.staging, "coalesce_max": a.cmax, "coalesce_window_us": a.window,
         "threads_per_wg": a.threads, "dictionary_words": 64, "grep_patterns": 8,
         "l2": "inputs larger than L2 (8 GiB corpus streamed from the host every step)",
-        "input_residency": "host page cache (tmpfs); the GPU-issued preads move it to HBM inside the timed region",
+        "input_residency": ("host page cache (tmpfs); inside the timed region the GPU-issued preads bring it "
+                            "into HBM staging lines (device staging) or the scan reads it from pinned host "
+                            "lines over PCIe (host staging)"),
         "parallelism": f"files/{world}",
     }
 
@@ -153,31 +157,67 @@ def run_reference(a):
     import oracle
     corpus = inputs.make_corpus(a.files, a.file_mib << 20, root=a.root)
     words, pats = inputs.dictionary(), inputs.patterns()
-    sample = corpus.paths[: max(1, min(len(corpus.paths), 32))]
-    sbytes = sum(os.path.getsize(p) for p in sample)
+    # each step a bounded sample of the workload: the next 32 files of the corpus (rotating, so K
+    # steps cover K x 32 different files; ~0.7 s per step on 16 host threads)
+    per = max(1, min(len(corpus.paths), 32))
     nthr = host_cores()
     for _ in range(a.warmup):
-        oracle.corpus(sample[:2], words, pats, chunk=a.chunk_kib << 10, nthreads=nthr)
-    times = []
-    for _ in range(a.steps):
+        oracle.corpus(corpus.paths[:2], words, pats, chunk=a.chunk_kib << 10, nthreads=nthr)
+    times, done = [], 0
+    for i in range(a.steps):
+        sample = [corpus.paths[(i * per + j) % len(corpus.paths)] for j in range(per)]
         _, _, secs, _ = oracle.corpus(sample, words, pats, chunk=a.chunk_kib << 10, nthreads=nthr)
         times.append(secs)
+        done += sum(os.path.getsize(p) for p in sample)
     t = sum(times)
-    value = sbytes * a.steps / t / 1e9
+    sbytes = done / a.steps
+    value = done / t / 1e9
     out = {"impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world,
            "steps": a.steps, "warmup": a.warmup, "ms_per_step": t / a.steps * 1e3, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-           "config": workload_config(a, corpus.total_bytes, world),
+           "config": {**workload_config(a, corpus.total_bytes, world),
+                      "reference_sample": f"each step times the oracle on {per} of the {a.files} files "
+                                          f"(bounded sample); value = sampled bytes / oracle time"},
            "cpu_baseline": {"value": value, "unit": "GB/s", "cores": nthr, "kind": "oracle",
-                            "sample": f"{len(sample)} of {a.files} files ({sbytes / 2**20:.0f} MiB) per step, "
-                                      f"pread + scalar wordcount + grep, {nthr} pthreads, {cpu_model()}"},
+                            "sample": f"{per} of the {a.files} files ({sbytes / 2**20:.0f} MiB) per step, the next "
+                                      f"{per} each step (rotating): pread + scalar wordcount + grep, {nthr} "
+                                      f"pthreads, {cpu_model()}"},
            "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
     return 0
 
 
+def spawn_ranks(a) -> int | None:
+    """`--gpus N` without a torchrun environment: re-launch this command as N ranks (one process per
+    GPU) under torch.distributed.run on 127.0.0.1, and return its exit code; None when already
+    inside a launch (or N == 1)."""
+    if a.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return None
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
+def check_world(a, world):
+    """The launch must match --gpus, one GPU per rank (GSYS_BENCH_ONE_GPU=1, test only: every
+    rank on cuda:0)."""
+    import torch
+    if a.gpus != world:
+        raise SystemExit(f"bench.py: --gpus {a.gpus} but the launch has {world} rank(s)")
+    if os.environ.get("GSYS_BENCH_ONE_GPU") != "1" and torch.cuda.device_count() < world:
+        raise SystemExit(f"bench.py: {world} ranks but only {torch.cuda.device_count()} visible GPU(s)")
+
+
 def main():
     a = parse()
+    rc = spawn_ranks(a)
+    if rc is not None:
+        return rc
     if a.impl == "reference":
         return run_reference(a)
     if a.mode == "syscalls":
@@ -198,6 +238,7 @@ def main():
     from paper_conf_isca_veselybblor18_b200 import workloads as W
 
     rank, world, local = dist_env()
+    check_world(a, world)
     # GSYS_BENCH_ONE_GPU=1 (test only): every rank on cuda:0 with gloo, to exercise the N > 1 path
     # on a one-GPU box (NCCL refuses two ranks on one device)
     one_gpu = os.environ.get("GSYS_BENCH_ONE_GPU") == "1"
@@ -273,13 +314,31 @@ def main():
         barrier()
         clocks = clk.stop()
         st = G.gsys_stats()
-    dev_s = max_over_ranks(ev0.elapsed_time(ev1) / 1e3)
+    my_s = ev0.elapsed_time(ev1) / 1e3
+    dev_s = max_over_ranks(my_s)
     value = corpus.total_bytes * a.steps / dev_s / 1e9
+    # per-rank rate (own bytes / own device time) and, measured by every rank at once after the
+    # timed region, the concurrent pinned H2D rate of each rank's link: the host-side ceiling of a
+    # scaling curve (all ranks share the host's page cache, DRAM and cores)
+    per_rank_local = [float(rank), my_bytes * a.steps / my_s / 1e9, float(my_bytes)]
+    if world > 1:
+        barrier()
+        conc_h2d = measure_h2d(dev)
+        t = torch.tensor(per_rank_local + [conc_h2d], dtype=torch.float64, device=dev)
+        gathered = [torch.zeros_like(t) for _ in range(world)]
+        dist.all_gather(gathered, t)
+        per_rank = [{"rank": int(g[0]), "GBps": float(g[1]), "bytes": int(g[2]),
+                     "concurrent_h2d_GBps": float(g[3])} for g in (x.cpu() for x in gathered)]
+    else:
+        per_rank = [{"rank": 0, "GBps": per_rank_local[1], "bytes": my_bytes}]
     # parity of the last step against the generator census (cheap, exact)
     if world > 1:
-        hist_ok = bool((d_all[0][:64].cpu().numpy().astype("uint64") == corpus.census).all())
+        red = d_all[0].cpu().numpy()
+        hist_ok = bool((red[:64].astype("uint64") == corpus.census).all())
+        hits_ok = red[64:].tolist() == [1 if m else 0 for m in corpus.pmasks]
     else:
         hist_ok = bool((d_hist.cpu().numpy().astype("uint64") == corpus.census).all())
+        hits_ok = d_hits[:nf].cpu().tolist() == [1 if m else 0 for m in corpus.pmasks]
 
     # ---- e2e through the public API (files in -> host histogram out), wall clock
     barrier()
@@ -349,7 +408,9 @@ def main():
                "roofline": roofline,
                "cpu_baseline": cpu_baseline,
                "clocks": clocks,
-               "parity": {"hist_equals_generator_census": hist_ok},
+               "parity": {"hist_equals_generator_census": hist_ok, **({"grep_hits_equal_plants": hits_ok}
+                                                                     if hits_ok is not None else {})},
+               "per_rank": per_rank,
                "secondary": {"wg_syscalls_per_s_in_wordcount": syscalls_per_step * world / (dev_s / a.steps),
                              **({"syscalls_wg": extras["syscalls"]} if "syscalls" in extras else {}),
                              **({"config1_16MiB": extras["config1"]} if "config1" in extras else {}),

@@ -132,6 +132,20 @@ int gsys_set_merge(int on);
  * GPU caller sees the POSIX error convention of reading A4/A11.  0, -ENODEV, -EINVAL. */
 int gsys_set_fault(int32_t err, int64_t offset);
 
+/* How blocking calls on device buffers complete (env GSYS_COMPLETION=memop|host|pull at init):
+ *   GSYS_COMPLETION_MEMOP -- payload by copy-engine DMA from the worker's pinned bounce,
+ *       completion word in device memory written by a stream memory operation after it;
+ *   GSYS_COMPLETION_HOST  -- the same DMA, then the worker waits for it and stores the host-mapped
+ *       completion word;
+ *   GSYS_COMPLETION_PULL (default) -- (reading B13) work-group preads that fit no pull area are read into the
+ *       worker's host-mapped bounce and copied out by the work-group itself; the service makes no
+ *       CUDA call while kernels wait (profiler-safe); other calls as HOST.
+ * Drains first (gsys_wait).  0, -ENODEV, -EINVAL, -EIO. */
+#define GSYS_COMPLETION_MEMOP 0u
+#define GSYS_COMPLETION_HOST  1u
+#define GSYS_COMPLETION_PULL  2u
+int gsys_set_completion(uint32_t mode);
+
 /* Fault injection for tests: from now on every pread whose offset equals `offset` is drained and
  * executed but its completion is never written (a lost completion); -1 turns it off.  The GPU
  * caller's watchdog (gsys_set_poll_timeout) then returns -ETIMEDOUT.  0, -ENODEV. */

@@ -1340,11 +1340,15 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     // 256 ns: a 4 KiB pread round trip drops from 16.1 to 9.9 us vs 4 us polling, and the
     // wordcount (pollers sharing the PCIe link with the scan) is unchanged (profiles/r01_latency.json)
     c.poll_ns_host = (ev && atoi(ev) > 0) ? (unsigned)atoi(ev) : 256u;
+    // completion path of blocking device-buffer calls (gsys.h GSYS_COMPLETION_*), env
+    // GSYS_COMPLETION=memop|host|pull.  Default pull (reading B13): the work-group copies its bytes
+    // out of the service's host-mapped bounce -- 8 GiB device-staged wordcount 50.5 GB/s vs 24.5
+    // (memop) / 23.6 (host), WG 64 KiB device preads 0.75 M/s vs 0.09 / 0.14 M/s
+    // (profiles/r02_completion_ab.jsonl); the copy-engine paths pay CUDA API calls per request.
     ev = getenv("GSYS_COMPLETION");
-    // default memop: a host-store completion must first wait for the DMA (an event synchronize per
-    // bundle), which measured slower for device staging (42.5 vs 46.7 GB/s at 256 KiB chunks) and
-    // no faster for 4 KiB preads (profiles/r01_completion_paths.json)
-    c.memop_completion = (ev && (strcmp(ev, "host") == 0 || strcmp(ev, "pull") == 0)) ? 0u : 1u;
+    const int cmode = !ev ? 2 : strcmp(ev, "memop") == 0 ? 0 : strcmp(ev, "host") == 0 ? 1 : 2;
+    c.memop_completion = cmode == 0 ? 1u : 0u;
+    c.pull_bounce = cmode == 2 ? 1u : 0u;
     I->memop_completion = c.memop_completion != 0;
     ev = getenv("GSYS_BIG_ALONE");
     I->big_alone = !(ev && atoi(ev) == 0);
@@ -1358,10 +1362,6 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     }
     ev = getenv("GSYS_SLEEP_HINT");
     c.no_hint = (ev && atoi(ev) == 0) ? 1u : 0u;
-    // reading B13: GSYS_COMPLETION=pull -- blocking work-group preads into device memory are copied
-    // out of the worker's host-mapped bounce by the work-group (no CUDA call in the service)
-    ev = getenv("GSYS_COMPLETION");
-    c.pull_bounce = (ev && strcmp(ev, "pull") == 0) ? 1u : 0u;
     // watchdog: GSYS_POLL_TIMEOUT_MS, default 20 s, 0 = off
     ev = getenv("GSYS_POLL_TIMEOUT_MS");
     c.poll_timeout_ns = (unsigned long long)(ev ? atoll(ev) : 20000ll) * 1000000ull;
@@ -1643,15 +1643,20 @@ int gsys_wait(void* stream) {
         // once the service is drained they are returned to free -- every slot after a
         // device-wide wait (no kernel can hold a claim then), else the logged ones
         if (drained) {
+            // (the host-visible state word too: a pulled bounce range waits for it, reading B13)
             if (!stream) {
                 cudaMemsetAsync(I->claim_d, 0, (size_t)I->nslots * 4, I->ctl);
                 cudaMemsetAsync(I->nbpend_d, 0, (size_t)I->nslots * 4, I->ctl);
+                for (uint32_t s = 0; s < I->nslots; s++)
+                    if (__atomic_load_n(&I->area_h[s].state, __ATOMIC_RELAXED) != GSYS_FREE)
+                        __atomic_store_n(&I->area_h[s].state, (uint32_t)GSYS_FREE, __ATOMIC_RELEASE);
             } else {
                 for (uint32_t i = 0; i < std::min<uint32_t>(wd.count, GSYS_WD_RECS); i++) {
                     const uint32_t s = wd.rec[i].slot;
                     if (wd.rec[i].phase == GSYS_WD_KERNEL || wd.rec[i].phase == GSYS_WD_CLAIM || s >= I->nslots) continue;
                     cudaMemsetAsync(I->claim_d + s, 0, 4, I->ctl);
                     cudaMemsetAsync(I->nbpend_d + s, 0, 4, I->ctl);
+                    __atomic_store_n(&I->area_h[s].state, (uint32_t)GSYS_FREE, __ATOMIC_RELEASE);
                 }
             }
         }
@@ -1764,6 +1769,20 @@ int gsys_clock_sync(uint32_t samples, int64_t* offset_ns, uint64_t* uncertainty_
     }
     cudaFreeHost(buf);
     return rc;
+}
+
+int gsys_set_completion(uint32_t mode) {
+    Instance* I = current();
+    if (!I) return -ENODEV;
+    if (mode > GSYS_COMPLETION_PULL) return -EINVAL;
+    if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;   // running kernels read the context
+    int r = gsys_wait(nullptr);
+    (void)r;
+    I->ctx_h.memop_completion = mode == GSYS_COMPLETION_MEMOP ? 1u : 0u;
+    I->ctx_h.pull_bounce = mode == GSYS_COMPLETION_PULL ? 1u : 0u;
+    I->memop_completion = I->ctx_h.memop_completion != 0;
+    if (cudaMemcpy(I->ctx_d, &I->ctx_h, sizeof I->ctx_h, cudaMemcpyHostToDevice) != cudaSuccess) return -EIO;
+    return 0;
 }
 
 int gsys_set_fault_drop(int64_t offset) {

@@ -77,6 +77,7 @@ SIGNATURES = {
     "gsys_clock_sync": (ctypes.c_int, [_U32, _P, _P]),
     "gsys_set_poll_timeout": (ctypes.c_int, [_U32]),
     "gsys_set_fault_drop": (ctypes.c_int, [_I64]),
+    "gsys_set_completion": (ctypes.c_int, [_U32]),
     "gsys_watchdog_read": (ctypes.c_int, [_P, _P, _U32]),
     "gsys_abi_info": (ctypes.c_int, [_P, _P, _P]),
     "gsys_plan_merge": (ctypes.c_int, [_U32, _P, _P, _P, _U64, _P, _P, _P, _P, _P]),
@@ -219,6 +220,14 @@ def gsys_clock_sync(samples: int = 256):
 
 def gsys_set_poll_timeout(ms: int) -> int:
     return _check(lib().gsys_set_poll_timeout(ms), "gsys_set_poll_timeout")
+
+
+COMPLETION_MEMOP, COMPLETION_HOST, COMPLETION_PULL = 0, 1, 2
+
+
+def gsys_set_completion(mode: int) -> int:
+    """Completion path of blocking device-buffer calls (include/gsys.h GSYS_COMPLETION_*)."""
+    return _check(lib().gsys_set_completion(mode), "gsys_set_completion")
 
 
 def gsys_set_fault_drop(offset: int) -> int:

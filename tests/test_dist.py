@@ -1,6 +1,7 @@
 """N > 1 plumbing on CPU (gloo, world_size 2): file sharding + the single all_reduce produce the
 whole-corpus answer.  Each rank computes its shard with the CPU oracle as a stand-in for the GPU
-kernel (the GPU path itself is covered by the -m gpu tests)."""
+kernel; the same plumbing around the real GPU path is tests/test_gpu_dist.py (-m gpu).  Also the
+bench launcher: `--gpus N` spawns N ranks, and a rank count other than --gpus is refused."""
 import os
 import socket
 
@@ -61,3 +62,32 @@ def test_shard_ranges_partition():
             assert rs[0][0] == 0 and rs[-1][1] == n
             assert all(a[1] == b[0] for a, b in zip(rs, rs[1:]))
             assert max(h - l for l, h in rs) - min(h - l for l, h in rs) <= 1
+
+
+def _bench(args, env=None, timeout=600):
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), *args], env=env, capture_output=True,
+                         text=True, timeout=timeout, cwd=root)
+    lines = [json.loads(ln) for ln in out.stdout.splitlines() if ln.startswith("{")]
+    return out, lines
+
+
+def test_bench_spawns_ranks_itself(tmpdir_shm):
+    """`bench.py --gpus 2` outside torchrun re-launches itself as 2 ranks (here the CPU reference
+    arm: rank 0 times the oracle and prints the one line, rank 1 exits 0)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    out, lines = _bench(["--impl", "reference", "--gpus", "2", "--files", "2", "--file-mib", "1", "--steps", "1",
+                         "--warmup", "1", "--root", os.path.join(tmpdir_shm, "bref")], env=env)
+    assert out.returncode == 0, out.stderr[-2000:]
+    assert len(lines) == 1 and lines[0]["impl"] == "reference" and lines[0]["n_gpus"] == 2
+
+
+def test_bench_rejects_world_mismatch(tmpdir_shm):
+    """A launch whose rank count differs from --gpus fails loudly instead of timing something else."""
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    out, _ = _bench(["--gpus", "2", "--files", "2", "--file-mib", "1", "--steps", "1", "--warmup", "3",
+                     "--no-extras", "--no-cpu-baseline", "--root", os.path.join(tmpdir_shm, "bench_mm")], env=env)
+    assert out.returncode != 0 and "--gpus 2" in (out.stderr + out.stdout)

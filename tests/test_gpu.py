@@ -623,3 +623,55 @@ def test_external_kernel_tokens(file1m, ext_lib, nwarps, length):
         want = data[off: off + length]
         assert int(ret[i]) == len(want), i
         assert int(sm[i]) == int(want.astype(np.int64).sum()), i
+
+
+# ---------------------------------------------------------------------------- completion paths (B13)
+@pytest.fixture
+def completion_mode(request):
+    G.gsys_set_completion(request.param)
+    yield request.param
+    G.gsys_set_completion(G.COMPLETION_PULL)
+
+
+@pytest.mark.parametrize("completion_mode", [G.COMPLETION_MEMOP, G.COMPLETION_HOST, G.COMPLETION_PULL], indirect=True)
+@pytest.mark.parametrize("chunk,blocks,threads,nb", [(4096, 7, 64, False), (256 << 10, 0, 256, False),
+                                                     (64 << 10, 3, 256, True), (1 << 20, 1, 128, False)])
+def test_wordcount_device_staging_completion_modes(ragged_corpus, completion_mode, chunk, blocks, threads, nb):
+    """Device staging under each completion path: a stream memop after the DMA, a host store after
+    the DMA, and the work-group copying its pulled bytes out of the service's host-mapped bounce
+    (reading B13, the default)."""
+    c = ragged_corpus
+    res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, blocks=blocks, threads=threads,
+                            gflags=G.WG | (G.NONBLOCKING if nb else G.BLOCKING) | G.RELAXED, staging=G.STAGE_DEVICE)
+    h, hits = oracle_hist_hits(c.paths)
+    assert res.wait_rc == 0
+    assert np.array_equal(as_u64(res.hist), h)
+    assert res.file_hits.tolist() == hits.tolist()
+    if not nb:
+        want = []
+        for s in c.sizes:
+            want += [plan.expected_pread_ret(s, r[3], r[4]) for r in plan.wordcount_chunk_requests(s, chunk)]
+        assert res.req_ret.tolist() == want
+
+
+@pytest.mark.parametrize("completion_mode", [G.COMPLETION_PULL], indirect=True)
+@pytest.mark.parametrize("length", [16385, 100000, 1 << 20])
+@pytest.mark.parametrize("order", [G.STRONG, G.RELAXED])
+def test_pread_pull_bounce(file1m, completion_mode, length, order):
+    """WG blocking preads into device memory past the pull areas, copied out of the bounce by the
+    work-group: every return value and the byte sum every thread computes after the call."""
+    size = os.path.getsize(file1m)
+    data = np.fromfile(file1m, dtype=np.uint8)
+    blocks, iters = 6, 3
+    d_buf = torch.zeros(blocks * length, dtype=torch.uint8, device="cuda")
+    fd = os.open(file1m, os.O_RDONLY)
+    try:
+        _, ret, _, sm, rc = W.bench_calls("pread", G.WG | G.BLOCKING | order, blocks, 128, iters, fd, length, size,
+                                          d_buf, want_sum=True)
+    finally:
+        os.close(fd)
+    assert rc == 0
+    for i in range(blocks * iters):
+        off = (i * length) % size
+        b = data[off: off + length]
+        assert int(ret[i]) == len(b) and int(sm[i]) == int(b.astype(np.int64).sum()), i
