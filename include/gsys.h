@@ -322,7 +322,10 @@ int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap);
  *                   (0 = 256; multiple of 32, <= 256).
  *   d_req_ret       DEVICE int64[total chunks] (may be NULL): per-chunk pread return value.
  *   stream          cudaStream_t to launch on.
- * Asynchronous on `stream`; call gsys_wait(stream) before reading results.  Errors: -EINVAL
+ * Asynchronous on `stream`; call gsys_wait(stream) before reading results.  Launches share the
+ * instance's workspace (chunk queue, uploads, staging lines): a call waits on the device for the
+ * previous call's kernel, on whatever stream it ran, so calls on different streams serialise
+ * rather than race.  Errors: -EINVAL
  * for bad sizes/flags, -ENODEV before gsys_init, CUDA errors as in gsys_launch.  Read errors
  * of individual chunks are visible in d_req_ret (negative) and skip the chunk's scan. */
 int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, uint32_t chunk,
@@ -334,14 +337,25 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
 /* Same scan over text already resident in device memory (no syscalls): the standalone scan
  * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n] (16-byte aligned); file
  * boundaries are not modelled (one file).  Adds into d_hist; d_hit (may be NULL) set to 1 if any
- * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 704, else a
- * multiple of 32 up to 768 (the 129-column table is used when it fits beside the warps' staging,
- * else the 77-column one).  -EINVAL on bad sizes/alignment, -ENODEV before gsys_init. */
+ * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 1024 (token scan)
+ * or 704 (DFA scan), else a multiple of 32 up to 1024 (768 for the DFA, whose 129-column table is
+ * used when it fits beside the warps' staging, else the 77-column one).  -EINVAL on bad
+ * sizes/alignment, -ENODEV before gsys_init. */
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
                      const char* dict, const uint8_t* dlen, uint32_t ndict,
                      const char* pats, const uint8_t* plen, uint32_t npat,
                      uint64_t* d_hist, uint32_t* d_hit, uint32_t blocks, uint32_t threads,
                      void* stream);
+
+/* Scan implementation used by gsys_wordcount and gsys_scan_device (row a8; both exact, reading
+ * A9/A10): GSYS_SCAN_DFA (default) -- one transposed-DFA shared-memory lookup per byte
+ * (csrc/scan_core.cuh); GSYS_SCAN_TOKEN -- SWAR word-byte masks, token starts, per-token hash
+ * lookup and byte-exact verify (csrc/tokscan.cuh; no 512-state trie limit, about half the DFA's
+ * rate on B200).  Env GSYS_SCAN=dfa|token at load.  Returns the previous implementation, -EINVAL
+ * for another value. */
+#define GSYS_SCAN_TOKEN 0
+#define GSYS_SCAN_DFA   1
+int gsys_set_scan(int impl);
 
 /* Diagnostics: when on, gsys_wordcount's work-groups accumulate (thread 0, %globaltimer) the
  * time spent inside their gsys_pread calls, the time spent scanning, and the chunk count;

@@ -20,7 +20,8 @@ LIB = os.path.join(PKG, "libgsys.so")
 SOURCES = [os.path.join(CSRC, "gsys_host.cpp"), os.path.join(CSRC, "gsys_kernels.cu"),
            os.path.join(CSRC, "gsys_next.cu")]
 HEADERS = [os.path.join(INCLUDE, "gsys.h"), os.path.join(INCLUDE, "gsys_device.cuh"),
-           os.path.join(CSRC, "gsys_internal.h"), os.path.join(CSRC, "scan_core.cuh")]
+           os.path.join(CSRC, "gsys_internal.h"), os.path.join(CSRC, "scan_core.cuh"),
+           os.path.join(CSRC, "tokscan.cuh")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

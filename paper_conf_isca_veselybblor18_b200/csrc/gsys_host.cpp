@@ -1041,13 +1041,11 @@ void Worker::process(uint64_t h0, uint32_t n) {
             bool okd = true;
             for (uint32_t j : mem) {
                 Req& r = reqs[midx[j]];
+                if (r.flags & GSYS_F_PULLB) { okd = false; break; }   // read alone into the bounce (B13)
                 PtrKind k = !r.a[2] ? PK_INVALID
                             : (r.flags & GSYS_F_PULL) ? (I->pull_area(r.slot, r.a[2]) ? PK_HOST : PK_INVALID)
                                                       : resolve((uintptr_t)r.a[1], r.a[2], nullptr);
-                if (k == PK_INVALID || (k == PK_HOST && r.a[2] > (64u << 10)) || (r.flags & GSYS_F_PULLB)) {
-                    okd = false;
-                    break;
-                }
+                if (k == PK_INVALID || (k == PK_HOST && r.a[2] > (64u << 10))) { okd = false; break; }
             }
             if (!okd) continue;
             uint8_t* b = alloc(mg_len[g]);
@@ -1943,23 +1941,53 @@ uint32_t g_sig_cap = 0;
 std::atomic<uint64_t> g_sig_dropped{0};
 
 void sigsink_handler(int, siginfo_t* si, void*) {
-    const uint64_t i = g_sig_tail.fetch_add(1, std::memory_order_relaxed);
-    if (i - g_sig_head.load(std::memory_order_relaxed) >= g_sig_cap) { g_sig_dropped.fetch_add(1); return; }
+    // reserve an entry only while the ring has room (a dropped signal must not leave a hole the
+    // reader would stop at forever)
+    const uint32_t cap = __atomic_load_n(&g_sig_cap, __ATOMIC_ACQUIRE);   // 0 while re-installing
+    int32_t* const ring = g_sig_ring;
+    uint64_t* const tsb = g_sig_ts;
+    uint64_t i = g_sig_tail.load(std::memory_order_relaxed);
+    do {
+        if (cap == 0 || i - g_sig_head.load(std::memory_order_acquire) >= cap) {
+            g_sig_dropped.fetch_add(1, std::memory_order_relaxed);
+            return;
+        }
+    } while (!g_sig_tail.compare_exchange_weak(i, i + 1, std::memory_order_acq_rel));
     struct timespec ts;
     clock_gettime(CLOCK_MONOTONIC, &ts);
-    g_sig_ts[i % g_sig_cap] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
-    __atomic_store_n(&g_sig_ring[i % g_sig_cap], si->si_value.sival_int, __ATOMIC_RELEASE);
+    tsb[i % cap] = (uint64_t)ts.tv_sec * 1000000000ull + (uint64_t)ts.tv_nsec;
+    __atomic_store_n(&ring[i % cap], si->si_value.sival_int, __ATOMIC_RELEASE);
 }
 }  // namespace
 
 int gsys_sigsink_install(int32_t sig, uint32_t capacity) {
     if (sig < SIGRTMIN || sig > SIGRTMAX || capacity == 0) return -EINVAL;
-    if (!g_sig_ring) {
-        g_sig_ring = (int32_t*)calloc(capacity, sizeof(int32_t));
-        g_sig_ts = (uint64_t*)calloc(capacity, sizeof(uint64_t));
-        if (!g_sig_ring || !g_sig_ts) return -ENOMEM;
-        for (uint32_t i = 0; i < capacity; i++) g_sig_ring[i] = INT32_MIN;
-        g_sig_cap = capacity;
+    if (!g_sig_ring || capacity > g_sig_cap) {
+        // (re)allocate with `sig` blocked in this thread; the previous ring must be drained -- a
+        // larger request replaces it only when no signal is pending in it
+        if (g_sig_ring && g_sig_tail.load() != g_sig_head.load()) return -EBUSY;
+        sigset_t ss, old;
+        sigemptyset(&ss);
+        sigaddset(&ss, sig);
+        pthread_sigmask(SIG_BLOCK, &ss, &old);
+        int32_t* ring = (int32_t*)calloc(capacity, sizeof(int32_t));
+        uint64_t* tsb = (uint64_t*)calloc(capacity, sizeof(uint64_t));
+        if (!ring || !tsb) {
+            free(ring);
+            free(tsb);
+            pthread_sigmask(SIG_SETMASK, &old, nullptr);
+            return -ENOMEM;
+        }
+        for (uint32_t i = 0; i < capacity; i++) ring[i] = INT32_MIN;
+        // handlers on other threads drop while the cap is 0; the previous ring is not freed (a
+        // handler on another thread may still hold its pointer)
+        __atomic_store_n(&g_sig_cap, 0u, __ATOMIC_RELEASE);
+        g_sig_ring = ring;
+        g_sig_ts = tsb;
+        g_sig_head.store(0);
+        g_sig_tail.store(0);
+        __atomic_store_n(&g_sig_cap, capacity, __ATOMIC_RELEASE);
+        pthread_sigmask(SIG_SETMASK, &old, nullptr);
     }
     struct sigaction sa;
     memset(&sa, 0, sizeof sa);
@@ -1974,12 +2002,14 @@ int gsys_sigsink_read(int32_t* values, uint64_t* t_ns, uint32_t cap) {
     uint32_t n = 0;
     uint64_t h = g_sig_head.load(std::memory_order_relaxed);
     const uint64_t t = g_sig_tail.load(std::memory_order_acquire);
+    const uint32_t rc = __atomic_load_n(&g_sig_cap, __ATOMIC_ACQUIRE);
+    if (rc == 0) return 0;
     while (h < t && n < cap) {
-        int32_t v = __atomic_load_n(&g_sig_ring[h % g_sig_cap], __ATOMIC_ACQUIRE);
+        int32_t v = __atomic_load_n(&g_sig_ring[h % rc], __ATOMIC_ACQUIRE);
         if (v == INT32_MIN) break;   // slot claimed by a handler that has not stored yet
         values[n] = v;
-        if (t_ns) t_ns[n] = g_sig_ts[h % g_sig_cap];
-        g_sig_ring[h % g_sig_cap] = INT32_MIN;
+        if (t_ns) t_ns[n] = g_sig_ts[h % rc];
+        g_sig_ring[h % rc] = INT32_MIN;
         n++;
         h++;
     }

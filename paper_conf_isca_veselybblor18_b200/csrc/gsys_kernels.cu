@@ -23,6 +23,7 @@
 #include <stdlib.h>
 #include <string.h>
 
+#include <atomic>
 #include <mutex>
 #include <vector>
 
@@ -30,15 +31,18 @@
 #include "gsys_device.cuh"
 #include "gsys_internal.h"
 #include "scan_core.cuh"
+#include "tokscan.cuh"
 
 namespace {
 
 using namespace gsys_scan;
 
 struct ScanState {
-    const ScanTables* T;        // shared memory, the transposed DFA follows it
+    const ScanTables* T;        // shared memory: the transposed DFA follows it (DFA scan), or the grep
+                                // part of the token tables (token scan)
+    const gsys_tok::TokTables* TT;   // shared memory: token tables (token scan) or nullptr
     unsigned* whist;            // this warp's shared histogram [64]
-    unsigned char* stage;       // shared memory, WARP_STAGE bytes per warp
+    unsigned char* stage;       // shared memory, WARP_STAGE / TWARP_STAGE bytes per warp
     int* hit;                   // shared grep-hit flag of the current chunk (nullptr: no grep)
 };
 
@@ -194,9 +198,102 @@ __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg
     cp_async_wait<0>();
 }
 
+// ------------------------------------------------------------------ token-level scan (tokscan.cuh)
+// Staging for the token scan: per 2 KiB warp tile, 32 lane slots of 80 B -- the lane's 64 bytes AND
+// the 16 bytes after them (a duplicate of the next slot's first 16 B, so a token window starting
+// anywhere in the span is contiguous in shared memory) -- then the 4 bytes before the tile.
+constexpr unsigned TSTAGE_BYTES = 32 * SLOT + 16;
+constexpr unsigned TWARP_STAGE = 2 * TSTAGE_BYTES;
+
+__device__ __forceinline__ void stage_tile_tok(unsigned buf, const unsigned char* seg0, long long s, long long base,
+                                               long long valid_end, unsigned lane) {
+    if (base > 0 && base + 2048 + 16 <= valid_end) {   // interior tile: no bounds, no zero fill
+        const unsigned char* src = seg0 + (base - s);
+        const unsigned d = buf + (lane >> 2) * SLOT + 16u * (lane & 3u);
+#pragma unroll
+        for (int k = 0; k < 4; k++) cp_async16_full(d + 8u * k * SLOT, src + 512 * k + 16 * lane);
+        cp_async16_full(buf + lane * SLOT + 64u, src + 64u * (lane + 1u));
+        if (lane == 0u) cp_async4_full(buf + 32u * SLOT, src - 4);
+        return;
+    }
+#pragma unroll
+    for (int k = 0; k < 5; k++) {
+        const long long p = k < 4 ? base + 512 * k + 16 * lane : base + 64ll * (lane + 1u);
+        const unsigned dst = k < 4 ? buf + (8u * k + (lane >> 2)) * SLOT + 16u * (lane & 3u) : buf + lane * SLOT + 64u;
+        const long long left = valid_end - p;
+        const unsigned n = left >= 16 ? 16u : (left > 0 ? (unsigned)left : 0u);
+        cp_async16(dst, seg0 + (n ? p - s : 0), n);
+    }
+    if (lane == 0u) cp_async4(buf + 32u * SLOT, seg0 + (base > 0 ? base - 4 - s : 0), base > 0 ? 4u : 0u);
+}
+
+// Token-level scan of positions [s, own_end) (same contract as scan_range): warp tiles of 2 KiB
+// staged by cp.async (double-buffered); lane l takes the 64-byte span at base + 64 l, classifies it
+// (gsys_tok::mask64), gets the lookahead mask from lane l+1 and the previous byte's class from
+// lane l-1 by shuffles, and visits the tokens it owns (gsys_tok::tok_lane64).
+__device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__ seg0, long long s, long long own_end,
+                                               long long valid_end, const ScanState& S) {
+    const gsys_tok::TokTables& T = *S.TT;
+    const bool grep = S.hit != nullptr && T.g.npat > 0;
+    const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    unsigned char* stage = S.stage + warp * TWARP_STAGE;
+    const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
+    const unsigned hs = (unsigned)__cvta_generic_to_shared(S.whist);
+    auto emit = [hs](unsigned d) { asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hs + 4u * d)); };
+    const gsys_tok::TokRegs R = gsys_tok::tok_regs(T);
+    const long long step = 2048ll * nwarps;
+    long long base = s + 2048ll * warp;
+    if (base < own_end) stage_tile_tok(stage_s, seg0, s, base, valid_end, lane);
+    cp_async_commit();
+    for (unsigned it = 0; base < own_end; base += step, it ^= 1u) {
+        const long long nxt = base + step;
+        if (nxt < own_end) stage_tile_tok(stage_s + (it ^ 1u) * TSTAGE_BYTES, seg0, s, nxt, valid_end, lane);
+        cp_async_commit();
+        cp_async_wait<1>();
+        __syncwarp();
+        const unsigned char* buf = stage + it * TSTAGE_BYTES;
+        const unsigned char* span = buf + lane * SLOT;
+        Win W;
+        W.w0 = *reinterpret_cast<const uint4*>(span);
+        W.w1 = *reinterpret_cast<const uint4*>(span + 16u);
+        W.w2 = *reinterpret_cast<const uint4*>(span + 32u);
+        W.w3 = *reinterpret_cast<const uint4*>(span + 48u);
+        W.w4 = *reinterpret_cast<const uint4*>(span + 64u);
+        const unsigned long long M = gsys_tok::mask64(W);
+        unsigned la = __shfl_down_sync(0xffffffffu, (unsigned)M & 0xffffu, 1);
+        if (lane == 31u) la = gsys_tok::mask16(W.w4);
+        unsigned pw = __shfl_up_sync(0xffffffffu, (unsigned)(M >> 63), 1);
+        if (lane == 0u) pw = base > 0 ? gsys_tok::word4(*reinterpret_cast<const unsigned*>(buf + 32u * SLOT)) >> 31 : 0u;
+        const long long p0 = base + 64ll * lane;
+        if (p0 < own_end) {
+            gsys_tok::tok_lane64(T, R, span, M, la, pw != 0u, p0, own_end, valid_end, emit);
+            if (grep && !*(volatile int*)S.hit && grep_lane64(T.g, W, p0, own_end, valid_end)) *S.hit = 1;
+        }
+        __syncwarp();
+    }
+    cp_async_wait<0>();
+}
+
+// Dynamic shared memory: [tables] [per-warp histograms] [warp stages].  Token tables when tok.
+__device__ __forceinline__ unsigned* load_tables_tok(unsigned char* smem, const gsys_tok::TokTables* gT,
+                                                     unsigned nwarps, ScanState& S) {
+    constexpr size_t tb = (sizeof(gsys_tok::TokTables) + 15) & ~(size_t)15;
+    const uint4* src = reinterpret_cast<const uint4*>(gT);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (unsigned i = threadIdx.x; i < tb / 16; i += blockDim.x) dst[i] = src[i];
+    unsigned* shist = reinterpret_cast<unsigned*>(smem + tb);
+    for (unsigned i = threadIdx.x; i < nwarps * HSTRIDE; i += blockDim.x) shist[i] = 0;
+    S.stage = smem + tb + nwarps * HSTRIDE * 4;
+    S.TT = reinterpret_cast<const gsys_tok::TokTables*>(smem);
+    S.T = &S.TT->g;
+    S.whist = shist + (threadIdx.x / 32) * HSTRIDE;
+    return shist;
+}
+
 // Dynamic shared memory: [ScanTables + DFA (tables_bytes)] [per-warp histograms] [warp stages].
 __device__ __forceinline__ unsigned* load_tables(unsigned char* smem, const ScanTables* gT, unsigned nwarps,
                                                  ScanState& S) {
+    S.TT = nullptr;
     const size_t tb = (tables_bytes(gT->nsp, gT->ncol) + 15) & ~(size_t)15;
     const uint4* src = reinterpret_cast<const uint4*>(gT);
     uint4* dst = reinterpret_cast<uint4*>(smem);
@@ -220,7 +317,8 @@ __device__ __forceinline__ void flush_hist(unsigned* shist, unsigned nwarps, uns
 // ------------------------------------------------------------------ wordcount with GPU-issued preads
 struct WcArgs {
     const gsys_dev_ctx* ctx;
-    const ScanTables* tables;
+    const ScanTables* tables;            // DFA scan
+    const gsys_tok::TokTables* ttables;  // token scan
     const int* fds;
     const unsigned long long* sizes;
     const unsigned* chunk_base;     // [nfiles + 1] first global chunk of each file
@@ -262,6 +360,14 @@ __device__ __forceinline__ bool wc_next_chunk(const WcArgs& a, unsigned* s_k, Wc
     return true;
 }
 
+template <bool TOK>
+__device__ __forceinline__ void scan_line(const unsigned char* seg0, long long s, long long own_end, long long valid_end,
+                                          const ScanState& S) {
+    if (TOK) scan_range_tok(seg0, s, own_end, valid_end, S);
+    else scan_range<LD_CG, false>(seg0, s, own_end, valid_end, S);
+}
+
+template <bool TOK>
 __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     // per-chunk grep flag, double-buffered by chunk parity: thread 0 clears the next chunk's flag
     // after reading this one, so no thread can still be touching it (racecheck-clean)
@@ -269,7 +375,7 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
     ScanState S;
-    unsigned* shist = load_tables(smem, a.tables, nwarps, S);
+    unsigned* shist = TOK ? load_tables_tok(smem, a.ttables, nwarps, S) : load_tables(smem, a.tables, nwarps, S);
     const ScanTables& sT = *S.T;
     if (threadIdx.x == 0) { s_hit[0] = 0; s_hit[1] = 0; }
     __syncthreads();
@@ -317,7 +423,7 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
             const long long valid_end = c0.off + c0.len < c0.size ? c0.off + c0.len : c0.size;
             const long long own_end = c0.e < valid_end ? c0.e : valid_end;
             S.hit = grep ? &s_hit[par] : nullptr;
-            if (own_end > c0.s) scan_range<LD_CG, false>(base + 16, c0.s, own_end, valid_end, S);
+            if (own_end > c0.s) scan_line<TOK>(base + 16, c0.s, own_end, valid_end, S);
             __syncthreads();   // this line is free for the prefetch issued next iteration
             if (threadIdx.x == 0) {
                 if (grep && s_hit[par]) atomicExch(&a.file_hits[c0.f], 1u);
@@ -367,9 +473,7 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
             const long long valid_end = off + r;
             const long long own_end = e < valid_end ? e : valid_end;
             S.hit = grep ? &s_hit[par] : nullptr;
-            if (own_end > s) {
-                scan_range<LD_CG, false>(base + 16, s, own_end, valid_end, S);
-            }
+            if (own_end > s) scan_line<TOK>(base + 16, s, own_end, valid_end, S);
         }
         __syncthreads();   // the staging line is free again before the next chunk's pread
         if (threadIdx.x == 0) {
@@ -417,6 +521,26 @@ __global__ void __launch_bounds__(768, 1) scan_kernel(ScanArgs a) {
     }
     __syncthreads();
     flush_hist(shist, nwarps, sT.ndict, a.hist);
+    if (threadIdx.x == 0 && a.hit && s_hit) atomicExch(a.hit, 1u);
+}
+
+// Token-level scan of HBM-resident text (gsys_tok): 1 block of up to 32 warps per SM.
+__global__ void __launch_bounds__(1024, 1) scan_tok_kernel(ScanArgs a) {
+    __shared__ int s_hit;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const unsigned nwarps = blockDim.x / 32;
+    ScanState S;
+    unsigned* shist = load_tables_tok(smem, reinterpret_cast<const gsys_tok::TokTables*>(a.tables), nwarps, S);
+    if (threadIdx.x == 0) s_hit = 0;
+    __syncthreads();
+    S.hit = a.hit ? &s_hit : nullptr;
+    for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
+        const long long s = (long long)k * a.chunk;
+        const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
+        scan_range_tok(a.text + s, s, e, (long long)a.n, S);
+    }
+    __syncthreads();
+    flush_hist(shist, nwarps, S.T->ndict, a.hist);
     if (threadIdx.x == 0 && a.hit && s_hit) atomicExch(a.hit, 1u);
 }
 
@@ -515,6 +639,10 @@ struct Workspace {
     unsigned char* up_d = nullptr;
     size_t up_cap = 0;
     cudaEvent_t up_ev = nullptr;
+    // recorded after every launch that uses this workspace: a later call -- on any stream -- waits
+    // for it on the device before touching the shared chunk queue, uploads or staging lines, so
+    // calls on different streams are serialised instead of racing
+    cudaEvent_t last_ev = nullptr;
     unsigned char* staging_d = nullptr;
     size_t staging_cap = 0;
     unsigned long long* prof_d = nullptr;  // wc_kernel profile counters (gsys_set_profile)
@@ -526,6 +654,13 @@ struct Workspace {
 };
 Workspace g_ws[64];
 std::mutex g_ws_mu;
+// scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.44 TB/s on the
+// 1 GiB HBM scan) or GSYS_SCAN_TOKEN (0.78 TB/s, profiles/r02_scan_ab2.jsonl); env GSYS_SCAN=dfa|token
+// at load, gsys_set_scan() at run time
+std::atomic<int> g_scan_impl{[] {
+    const char* e = getenv("GSYS_SCAN");
+    return (e && strcmp(e, "token") == 0) ? (int)GSYS_SCAN_TOKEN : (int)GSYS_SCAN_DFA;
+}()};
 
 Workspace* workspace() {
     int d = 0;
@@ -533,6 +668,7 @@ Workspace* workspace() {
     Workspace* W = &g_ws[d];
     if (!W->up_ev) {
         cudaEventCreateWithFlags(&W->up_ev, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&W->last_ev, cudaEventDisableTiming);
         cudaDeviceGetAttribute(&W->sms, cudaDevAttrMultiProcessorCount, d);
     }
     return W;
@@ -626,20 +762,24 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     cbase[nfiles] = (unsigned)nch;
     if (blocks == 0) blocks = 2u * (uint32_t)W->sms;
     if (nch < blocks) blocks = (uint32_t)(nch ? nch : 1);
-    // upload: [tables][fds][sizes][cbase]
+    // upload: [tables][fds][sizes][cbase]; token tables (default) or the byte DFA (gsys_set_scan)
+    const bool tok = g_scan_impl.load() == GSYS_SCAN_TOKEN;
     size_t tb = 0;
-    int rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb);
+    int rc = tok ? gsys_tok::build_tok_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb)
+                 : build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb);
     if (rc && rc != -ENOSPC) return rc;
     size_t o_t = 0, o_f = align_up(tb, 256), o_s = align_up(o_f + 4ull * nfiles, 256),
            o_c = align_up(o_s + 8ull * nfiles, 256), total = align_up(o_c + 4ull * (nfiles + 1), 256);
     rc = ensure_upload(W, total);
     if (rc) return rc;
-    rc = build_tables(W->up_h + o_t, tb, dict, dlen, ndict, pats, plen, npat, nullptr);
+    rc = tok ? gsys_tok::build_tok_tables(W->up_h + o_t, tb, dict, dlen, ndict, pats, plen, npat, nullptr)
+             : build_tables(W->up_h + o_t, tb, dict, dlen, ndict, pats, plen, npat, nullptr);
     if (rc) return rc;
     memcpy(W->up_h + o_f, fds, 4ull * nfiles);
     memcpy(W->up_h + o_s, sizes, 8ull * nfiles);
     memcpy(W->up_h + o_c, cbase.data(), 4ull * (nfiles + 1));
     cudaStream_t s = (cudaStream_t)stream;
+    cudaStreamWaitEvent(s, W->last_ev, 0);
     cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
     cudaEventRecord(W->up_ev, s);
     size_t stride = align_up((size_t)chunk + 64, 256);
@@ -660,6 +800,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     memset(&a, 0, sizeof a);
     a.ctx = ctx;
     a.tables = reinterpret_cast<const ScanTables*>(W->up_d + o_t);
+    a.ttables = reinterpret_cast<const gsys_tok::TokTables*>(W->up_d + o_t);
     a.fds = reinterpret_cast<const int*>(W->up_d + o_f);
     a.sizes = reinterpret_cast<const unsigned long long*>(W->up_d + o_s);
     a.chunk_base = reinterpret_cast<const unsigned*>(W->up_d + o_c);
@@ -684,11 +825,14 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     a.gflags = gflags & ~GSYS_NONBLOCKING;   // the blocking flavour; prefetch derives the rest
     if (nch == 0) return 0;
     void* args[] = {&a};
-    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE);
-    rc = ensure_smem_attr((const void*)wc_kernel, smem);
+    const void* fn = tok ? (const void*)wc_kernel<true> : (const void*)wc_kernel<false>;
+    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + (tok ? TWARP_STAGE : WARP_STAGE));
+    rc = ensure_smem_attr(fn, smem);
     if (rc) return rc;
     if (cudaMemsetAsync(W->next_chunk_d, 0, 4, s) != cudaSuccess) return -EIO;
-    return gsys_launch((const void*)wc_kernel, blocks, 1, 1, threads, 1, 1, args, smem, stream);
+    rc = gsys_launch(fn, blocks, 1, 1, threads, 1, 1, args, smem, stream);
+    cudaEventRecord(W->last_ev, s);
+    return rc;
 }
 
 int gsys_set_profile(int on) {
@@ -712,24 +856,33 @@ int gsys_read_profile(uint64_t* out3, int reset) {
     return 0;
 }
 
+int gsys_set_scan(int impl) {
+    if (impl != (int)GSYS_SCAN_TOKEN && impl != (int)GSYS_SCAN_DFA) return -EINVAL;
+    return g_scan_impl.exchange(impl);
+}
+
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const char* dict, const uint8_t* dlen,
                      uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, uint64_t* d_hist,
                      uint32_t* d_hit, uint32_t blocks, uint32_t threads, void* stream) {
     if (!d_hist || (n && !d_text)) return -EINVAL;
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
-    if (threads == 0) threads = 704;   // 22 warps + the 77-column table: 6 % above 16 warps + the 129-column one
-    if (threads % 32 || threads > 768) return -EINVAL;
+    const bool tok = g_scan_impl.load() == GSYS_SCAN_TOKEN;
+    // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 32 warps
+    if (threads == 0) threads = tok ? 1024 : 704;
+    if (threads % 32 || threads > (tok ? 1024u : 768u)) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
-    // 129-column table when it fits next to the warps' staging (1 block of `threads` per SM),
-    // else the 77-column one
+    // DFA: the 129-column table when it fits next to the warps' staging (1 block of `threads` per
+    // SM), else the 77-column one
     size_t tb = 0;
     unsigned ncol = NCOL_WIDE;
-    int rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
+    int rc = tok ? gsys_tok::build_tok_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb)
+                 : build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
     if (rc && rc != -ENOSPC) return rc;
-    if (align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE) > kSmemDynMax) {
+    const size_t per_warp = HSTRIDE * 4 + (tok ? TWARP_STAGE : WARP_STAGE);
+    if (!tok && align_up(tb, 16) + (threads / 32) * per_warp > kSmemDynMax) {
         ncol = NCOL_NARROW;
         rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
         if (rc && rc != -ENOSPC) return rc;
@@ -737,9 +890,11 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     size_t total = align_up(tb, 256);
     rc = ensure_upload(W, total);
     if (rc) return rc;
-    rc = build_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr, ncol);
+    rc = tok ? gsys_tok::build_tok_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr)
+             : build_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr, ncol);
     if (rc) return rc;
     cudaStream_t s = (cudaStream_t)stream;
+    cudaStreamWaitEvent(s, W->last_ev, 0);
     cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
     cudaEventRecord(W->up_ev, s);
     unsigned long long nch = (n + chunk - 1) / chunk;
@@ -756,19 +911,22 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     a.hit = d_hit;
     a.nchunks = nch;
     a.chunk = chunk;
-    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + WARP_STAGE);
-    rc = ensure_smem_attr((const void*)scan_kernel, smem);
+    const void* fn = tok ? (const void*)scan_tok_kernel : (const void*)scan_kernel;
+    size_t smem = align_up(tb, 16) + (threads / 32) * per_warp;
+    rc = ensure_smem_attr(fn, smem);
     if (rc) return rc;
     if (blocks_auto) {   // one full wave: resident blocks per SM x SMs
         int per_sm = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, scan_kernel, (int)threads, smem) != cudaSuccess ||
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, (int)threads, smem) != cudaSuccess ||
             per_sm < 1)
             per_sm = 1;
         blocks = (uint32_t)per_sm * (uint32_t)W->sms;
         if (nch < blocks) blocks = (uint32_t)nch;
     }
-    scan_kernel<<<blocks, threads, smem, s>>>(a);
-    return map_cuda(cudaGetLastError());
+    void* args[] = {&a};
+    rc = map_cuda(cudaLaunchKernel(fn, dim3(blocks), dim3(threads), args, smem, s));
+    cudaEventRecord(W->last_ev, s);
+    return rc;
 }
 
 int gsys_bench_calls(uint32_t kind, uint32_t gflags, uint32_t blocks, uint32_t threads, uint32_t iters, int32_t fd,

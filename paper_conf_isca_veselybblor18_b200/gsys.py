@@ -78,6 +78,7 @@ SIGNATURES = {
     "gsys_set_poll_timeout": (ctypes.c_int, [_U32]),
     "gsys_set_fault_drop": (ctypes.c_int, [_I64]),
     "gsys_set_completion": (ctypes.c_int, [_U32]),
+    "gsys_set_scan": (ctypes.c_int, [ctypes.c_int]),
     "gsys_watchdog_read": (ctypes.c_int, [_P, _P, _U32]),
     "gsys_abi_info": (ctypes.c_int, [_P, _P, _P]),
     "gsys_plan_merge": (ctypes.c_int, [_U32, _P, _P, _P, _U64, _P, _P, _P, _P, _P]),
@@ -223,6 +224,12 @@ def gsys_set_poll_timeout(ms: int) -> int:
 
 
 COMPLETION_MEMOP, COMPLETION_HOST, COMPLETION_PULL = 0, 1, 2
+SCAN_TOKEN, SCAN_DFA = 0, 1
+
+
+def gsys_set_scan(impl: int) -> int:
+    """Scan implementation (include/gsys.h GSYS_SCAN_*); returns the previous one."""
+    return _check(lib().gsys_set_scan(impl), "gsys_set_scan")
 
 
 def gsys_set_completion(mode: int) -> int:

@@ -8,6 +8,7 @@
 #include <vector>
 
 #include "scan_core.cuh"
+#include "tokscan.cuh"
 
 using namespace gsys_scan;
 
@@ -58,12 +59,52 @@ static int run(const uint8_t* text, uint64_t n, uint32_t chunk, const std::vecto
     return 0;
 }
 
+// Token-level scan (tokscan.cuh) over 64-byte lane spans exactly as the kernels run them: the span
+// mask, the lookahead mask (the kernels take it from the next lane), the previous byte's class.
+static int run_tok(const uint8_t* text, uint64_t n, uint32_t chunk, const gsys_tok::TokTables& T, uint64_t* hist,
+                   uint32_t npat, bool* any_out) {
+    std::vector<uint8_t> buf(n + 160, 'a');
+    if (n) memcpy(buf.data(), text, n);
+    bool any = false;
+    const long long N = (long long)n;
+    for (uint64_t s = 0; s < n; s += chunk) {
+        const uint64_t e = s + chunk < n ? s + chunk : n;
+        for (uint64_t p0 = s; p0 < e; p0 += 64) {
+            uint4 V[5];
+            for (int k = 0; k < 5; k++) {
+                const uint64_t q = p0 + 16 * k;
+                if (q < n) memcpy(&V[k], &buf[q], 16);
+                else V[k] = make_uint4(0, 0, 0, 0);
+            }
+            Win W{V[0], V[1], V[2], V[3], V[4]};
+            const unsigned long long M = gsys_tok::mask64(W);
+            const unsigned la = gsys_tok::mask16(W.w4);
+            const bool prev_word = p0 > 0 && is_word_byte(buf[p0 - 1]);
+            gsys_tok::tok_lane64(T, gsys_tok::tok_regs(T), &buf[p0], M, la, prev_word, (long long)p0, (long long)e, N,
+                                 [hist](unsigned d) { hist[d]++; });
+            if (npat && !any && grep_lane64(T.g, W, (long long)p0, (long long)e, N)) any = true;
+        }
+    }
+    *any_out = any;
+    return 0;
+}
+
 // mode 0: 16-byte reference steps, narrow table; 1: 64-byte lane spans, narrow table (wc_kernel);
-// 2: 64-byte lane spans, wide table (scan_kernel); 3: 16-byte reference steps, wide table.
+// 2: 64-byte lane spans, wide table (scan_kernel); 3: 16-byte reference steps, wide table;
+// 4: token-level lane spans (tokscan.cuh).
 extern "C" int scan_emul2(const uint8_t* text, uint64_t n, uint32_t chunk, const char* dict, const uint8_t* dlen,
                           uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, uint64_t* hist,
                           uint32_t* hit, int mode) {
-    if (chunk < 16 || chunk % 16 || mode < 0 || mode > 3) return -EINVAL;
+    if (chunk < 16 || chunk % 16 || mode < 0 || mode > 4) return -EINVAL;
+    if (mode == 4) {
+        std::vector<uint4> tt((sizeof(gsys_tok::TokTables) + 15) / 16);
+        int rc = gsys_tok::build_tok_tables(tt.data(), tt.size() * 16, dict, dlen, ndict, pats, plen, npat, nullptr);
+        if (rc) return rc;
+        bool any = false;
+        rc = run_tok(text, n, chunk, *reinterpret_cast<const gsys_tok::TokTables*>(tt.data()), hist, npat, &any);
+        if (hit) *hit = any ? 1u : 0u;
+        return rc;
+    }
     const bool wide = mode >= 2;
     const unsigned ncol = wide ? NCOL_WIDE : NCOL_NARROW;
     size_t tb = 0;

@@ -78,7 +78,7 @@ def test_wordcount_config1_parity(file16m, order, staging):
 @pytest.mark.parametrize("staging", [G.STAGE_DEVICE, G.STAGE_HOST, G.STAGE_MIXED(5)])
 @pytest.mark.parametrize("chunk,blocks,threads", [(4096, 7, 64), (256 << 10, 0, 256), (64 << 10, 3, 256),
                                                   (1 << 20, 1, 128)])
-def test_wordcount_ragged_corpus(ragged_corpus, chunk, blocks, threads, staging):
+def test_wordcount_ragged_corpus(ragged_corpus, scan_impl, chunk, blocks, threads, staging):
     c = ragged_corpus
     res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, blocks=blocks, threads=threads,
                             gflags=G.WG | G.BLOCKING | G.RELAXED, staging=staging)
@@ -127,7 +127,14 @@ def test_wordcount_coalescing_invariance(ragged_corpus, window, cmax, merge):
         assert st["merged"] == 0
 
 
-def test_scan_device_parity():
+@pytest.fixture(params=[G.SCAN_TOKEN, G.SCAN_DFA], ids=["token", "dfa"])
+def scan_impl(request):
+    prev = G.gsys_set_scan(request.param)
+    yield request.param
+    G.gsys_set_scan(prev)
+
+
+def test_scan_device_parity(scan_impl):
     """Scan of HBM-resident text (no syscalls), ragged size, several chunk sizes."""
     for fid, size in [(0, (8 << 20) + 13), (1, 4097), (2, 100)]:
         buf, census, _ = inputs.gen_bytes(inputs.SEED_CORPUS, fid, size, grep_plants=True)
@@ -154,7 +161,7 @@ def _scan_dev(buf, words, pats, chunk, threads=0):
 
 
 @pytest.mark.parametrize("threads", [0, 256])
-def test_scan_device_high_bytes(threads):
+def test_scan_device_high_bytes(scan_impl, threads):
     """Text mixing every byte value: 64-byte spans with a byte >= 0x80 leave the raw-byte fast path
     of the 129-column table for the clamped one (and the grep prefilter sees false candidates)."""
     rng = np.random.default_rng(11)
@@ -171,7 +178,7 @@ def test_scan_device_high_bytes(threads):
             assert hit == oracle.grep(text, pats)
 
 
-def test_scan_device_large_trie_uses_narrow_table():
+def test_scan_device_large_trie_uses_narrow_table(scan_impl):
     """A dictionary whose 129-column table no longer fits next to 16 warps' staging (482 trie
     states + 30 emission states) runs on the 77-column table: same counts."""
     words = [bytes([ord("A") + i % 26 if i < 26 else ord("a") + i - 26]) + bytes((97 + (i * 7 + k) % 26) for k in range(15))
@@ -187,12 +194,18 @@ def test_scan_device_large_trie_uses_narrow_table():
     assert np.array_equal(hist, exp) and exp.sum() >= 30
 
 
-def test_scan_device_trie_too_large_is_e2big():
+def test_scan_device_trie_too_large_is_e2big(scan_impl):
+    """The byte DFA caps the trie at 512 states (-E2BIG); the token scan has no such limit."""
     alpha = b"ABCDEFGHIJKLMNOPQRSTUVWXYZabcdefghijklmnopqrstuvwxyz0123456789"
     words = [alpha[i:i + 1] + b"x" * 15 for i in range(40)]       # 40 x 16 + 2 = 642 trie states > 512
-    with pytest.raises(OSError) as ei:
-        _scan_dev(b"abc def", words, [], 4096)
-    assert ei.value.errno == errno.E2BIG
+    text = b" ".join(words[::3]) + b" abc " + words[1] + b"x " + words[7]
+    if scan_impl == G.SCAN_DFA:
+        with pytest.raises(OSError) as ei:
+            _scan_dev(text, words, [], 4096)
+        assert ei.value.errno == errno.E2BIG
+    else:
+        hist, _ = _scan_dev(text, words, [], 4096)
+        assert np.array_equal(hist, oracle.count_tokens(np.frombuffer(text, dtype=np.uint8), words)[:len(words)])
 
 
 # ---------------------------------------------------------------------------- microbenchmark matrix
@@ -675,3 +688,32 @@ def test_pread_pull_bounce(file1m, completion_mode, length, order):
         off = (i * length) % size
         b = data[off: off + length]
         assert int(ret[i]) == len(b) and int(sm[i]) == int(b.astype(np.int64).sum()), i
+
+
+def test_wordcount_calls_on_two_streams(ragged_corpus):
+    """Back-to-back launches on two streams share the workspace safely: both results
+    equal the oracle."""
+    c = ragged_corpus
+    h, hits = oracle_hist_hits(c.paths)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    outs = []
+    with W.OpenFiles(c.paths) as of:
+        for s in (s1, s2, s1, s2):
+            d_hist = torch.zeros(64, dtype=torch.int64, device="cuda")
+            d_hits = torch.zeros(len(c.paths), dtype=torch.int32, device="cuda")
+            G.gsys_wordcount(of.fds, of.sizes, 16 << 10, WORDS, PATS, d_hist, d_hits, None,
+                             G.WG | G.BLOCKING | G.RELAXED, 5, 128, s, G.STAGE_DEVICE)
+            outs.append((d_hist, d_hits))
+        assert G.gsys_wait() == 0
+    for d_hist, d_hits in outs:
+        assert np.array_equal(as_u64(d_hist), h)
+        assert d_hits.cpu().tolist() == hits.tolist()
+
+
+def test_kernel_call_sites(file1m):
+    """Kernel-scope call sites are GSYS_SITE(0..7); a larger site id is -EINVAL (it used
+    to alias site k mod 8)."""
+    _, ret, _, _, rc = W.bench_calls("getrusage", G.KERNEL | G.BLOCKING | G.RELAXED | G.SITE(7), 4, 64, 3)
+    assert rc == 0 and ret.tolist() == [0, 0, 0]
+    _, ret, _, _, rc = W.bench_calls("getrusage", G.KERNEL | G.BLOCKING | G.RELAXED | G.SITE(9), 4, 64, 2)
+    assert ret.tolist() == [-errno.EINVAL] * 2

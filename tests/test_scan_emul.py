@@ -1,6 +1,7 @@
 """CPU checks of the CUDA path's scan logic (no GPU): tests/native/scan_emul.cu compiles the same
-csrc/scan_core.cuh the sm_100a kernels use into a host library that walks the chunks/threads'
-16-byte steps sequentially; results must equal the oracle bit-exactly."""
+csrc/scan_core.cuh (byte DFA) and csrc/tokscan.cuh (token-level scan) the sm_100a kernels use into a
+host library that walks the chunks/lane spans sequentially; results must equal the oracle
+bit-exactly."""
 import ctypes
 import os
 import subprocess
@@ -16,7 +17,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SRC = os.path.join(HERE, "native", "scan_emul.cu")
 LIB = os.path.join(HERE, "native", "libscanemul.so")
-DEPS = [SRC, os.path.join(ROOT, "paper_conf_isca_veselybblor18_b200", "csrc", "scan_core.cuh")]
+DEPS = [SRC, os.path.join(ROOT, "paper_conf_isca_veselybblor18_b200", "csrc", "scan_core.cuh"),
+        os.path.join(ROOT, "paper_conf_isca_veselybblor18_b200", "csrc", "tokscan.cuh")]
 
 
 @pytest.fixture(scope="module")
@@ -33,9 +35,10 @@ def emul():
 
     def run(text, words, pats, chunk):
         h0, g0 = run2(text, words, pats, chunk, 0)
-        for mode in (1, 2, 3):
+        for mode in (1, 2, 3, 4):
             # 1: wc_kernel's 64-byte lane spans (77-column table); 2: scan_kernel's lane spans (129
-            # columns, raw-byte fast path); 3: 16-byte reference steps on the 129-column table
+            # columns, raw-byte fast path); 3: 16-byte reference steps on the 129-column table;
+            # 4: the token-level lane spans (tokscan.cuh)
             h, g = run2(text, words, pats, chunk, mode)
             assert np.array_equal(h0, h) and g0 == g, mode
         return h0, g0

@@ -36,3 +36,26 @@ def test_sigsink_receives_values():
         n = L.gsys_sigsink_read(vals, None, 512)
         got += [vals[i] for i in range(n)]
     assert sorted(got) == sent
+
+
+def test_sigsink_overflow_does_not_wedge_the_ring():
+    """Signals that arrive while the ring is full are dropped without leaving a hole: after the
+    reader drains it, later signals arrive again (the reader used to stop forever)."""
+    L = G.lib()
+    sig = signal.SIGRTMIN + 6
+    assert L.gsys_sigsink_install(sig, 256) == 0
+    vals = (ctypes.c_int32 * 1024)()
+    while L.gsys_sigsink_read(vals, None, 1024) > 0:
+        pass
+    for v in range(300):                       # 44 more than the ring holds
+        assert _queue(sig, v) == 0
+    time.sleep(0.05)
+    n = L.gsys_sigsink_read(vals, None, 1024)
+    assert n == 256 and [vals[i] for i in range(n)] == list(range(256))
+    for v in range(1000, 1010):
+        assert _queue(sig, v) == 0
+    got, deadline = [], time.time() + 5
+    while len(got) < 10 and time.time() < deadline:
+        k = L.gsys_sigsink_read(vals, None, 1024)
+        got += [vals[i] for i in range(k)]
+    assert got == list(range(1000, 1010))
