@@ -362,6 +362,7 @@ def main():
         extras["scan"] = scan_roofline(G, dev, corpus, words, pats, chunk)
         extras["syscalls"] = wg_syscall_rate(G, W, dev, corpus.paths[0])
         extras["config1"] = config1_latency(G, W, dev, words, pats, a.root)
+        extras["fig10"] = fig10_coalescing(G, W, dev, corpus.paths[0])
     kernel_s = dev_s / a.steps
     algo_bytes = my_bytes + sum(((s + chunk - 1) // chunk) * 17 for s in of.sizes)   # chunk + halo
     rank_achieved = algo_bytes / kernel_s / 1e9
@@ -414,7 +415,9 @@ def main():
                "secondary": {"wg_syscalls_per_s_in_wordcount": syscalls_per_step * world / (dev_s / a.steps),
                              **({"syscalls_wg": extras["syscalls"]} if "syscalls" in extras else {}),
                              **({"config1_16MiB": extras["config1"]} if "config1" in extras else {}),
-                             **({"scan_hbm": extras["scan"]} if "scan" in extras else {})},
+                             **({"scan_hbm": extras["scan"]} if "scan" in extras else {}),
+                             **({"fig10_coalescing": extras["fig10"]} if "fig10" in extras else {})},
+               "service_path": service_path(a, st),
                "service": {"threads": st["threads"], "coalesce_max": st["coalesce_max"],
                            "window_us": st["coalesce_window_us"], "bundles_per_step": st["bundles"] / a.steps,
                            "merged_per_step": st["merged"] / a.steps,
@@ -424,6 +427,53 @@ def main():
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def service_path(a, st):
+    """Which service path the timed steps took (from the service counters)."""
+    if a.staging == "device":
+        how = ("device staging, pull completion (reading B13): a service worker preads each work-group's "
+               "chunk into its host-mapped bounce and completes with a host store; the work-group copies "
+               "the bytes into its HBM line and scans them there; the service makes no CUDA call")
+    elif a.staging == "host":
+        how = ("host staging: a service worker preads each chunk straight into the work-group's pinned "
+               "host-mapped line and completes with a host store; the scan reads the line over PCIe")
+    else:
+        how = "mixed staging: some chunks by copy-engine DMA into HBM lines, the rest zero-copy host lines"
+    return {"description": how, "requests_per_step": st["requests"] / a.steps,
+            "bundles_per_step": st["bundles"] / a.steps, "merged_requests_per_step": st["merged"] / a.steps,
+            "merge_note": "adjacent work-group halo reads are not merged on this path: each lands in its own "
+                          "bounce range that its work-group releases (merging is exercised by the coalescing "
+                          "invariance tests and by fig10_coalescing)"}
+
+
+def fig10_coalescing(G, W, dev, path):
+    """Fig. 10 analogue (PAPER.md:28 P28.12-19) in the driver's run: WG blocking preads of 64 B and
+    1 KiB into device memory, 592 work-groups x 40 calls, coalescing max 1 vs 8."""
+    import torch
+    size = os.path.getsize(path)
+    fd = os.open(path, os.O_RDONLY)
+    dbuf = torch.empty(592 * 1024, dtype=torch.uint8, device=dev)
+    rows = []
+    try:
+        for length in (64, 1024):
+            for cmax in (1, 8):
+                G.gsys_set_coalesce_max(cmax)
+                W.bench_calls("pread", G.WG | G.BLOCKING | G.RELAXED, 592, 256, 2, fd, length, size, dbuf)
+                G.gsys_stats_reset()
+                t0 = time.perf_counter()
+                _, ret, _, _, rc = W.bench_calls("pread", G.WG | G.BLOCKING | G.RELAXED, 592, 256, 40, fd, length,
+                                                 size, dbuf)
+                dt = time.perf_counter() - t0
+                st = G.gsys_stats()
+                rows.append({"bytes_per_call": length, "coalesce_max": cmax, "calls_per_s": 592 * 40 / dt,
+                             "ns_per_byte": dt * 1e9 / (592 * 40 * length), "bundles": st["bundles"],
+                             "max_bundle": st["max_bundle"], "merged": st["merged"],
+                             "ok": bool((ret == length).all()) and rc == 0})
+    finally:
+        G.gsys_set_coalesce_max(8)
+        os.close(fd)
+    return rows
 
 
 def measure_h2d(dev):
@@ -927,7 +977,7 @@ def run_fig9(a):
             n += 1
         return n * src.nbytes * 2 / (time.perf_counter() - t0) / 1e9     # read + write bytes
     out = {"mode": "fig9", "baseline_host_copy_GBps": host_bw(1.0), "rows": []}
-    sink = torch.zeros(1, dtype=torch.int64, device="cuda")
+    sink = torch.zeros(2, dtype=torch.int64, device="cuda")
     for where in ("host", "device"):
         for nlines in (1, 64, 1024, 4096, 16384, 65536, 262144):
             lines = (torch.zeros(nlines * 8, dtype=torch.int64).pin_memory() if where == "host"
@@ -939,7 +989,7 @@ def run_fig9(a):
             bw = host_bw(1.0)
             torch.cuda.synchronize()
             out["rows"].append({"polled": where, "lines": nlines, "gpu_threads": max(nlines, 148 * 256),
-                                "host_copy_GBps": bw, "gpu_polls_per_s": int(sink.item()) / 1.5})
+                                "host_copy_GBps": bw, "gpu_polls_per_s": int(sink[0].item()) / 1.5})
     print(json.dumps(out), flush=True)
     return 0
 

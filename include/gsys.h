@@ -445,9 +445,10 @@ int gsys_perm_pwrite(const uint8_t* d_in, const uint16_t* d_perm, uint32_t nbloc
                      uint32_t grid, void* stream);
 
 /* Row f4 -- Fig. 9 study (sec. VII, polling contention): nthreads GPU threads poll
- * nlines distinct 64 B lines of `lines` (pinned host-mapped or DEVICE memory, nlines*64 bytes) for
- * `ns` nanoseconds with system-scope loads; the total poll count is added to *d_sink (DEVICE
- * u64).  Used to measure how completion polling degrades host memory throughput. */
+ * nlines distinct 64 B lines of `lines` (pinned host-mapped or DEVICE memory, nlines*64 bytes; the
+ * first u64 of each line is read) for `ns` nanoseconds with system-scope loads; d_sink (DEVICE
+ * u64[2]): [0] += total polls, [1] = max(value seen) -- a host store made during the storm must be
+ * observed.  Used to measure how completion polling degrades host memory throughput. */
 int gsys_poll_storm(const void* lines, uint32_t nlines, uint32_t nthreads, uint64_t ns, uint64_t* d_sink,
                     void* stream);
 

@@ -330,12 +330,14 @@ __global__ void poll_kernel(const unsigned long long* lines, unsigned nlines, un
     const unsigned tid = blockIdx.x * blockDim.x + threadIdx.x;
     const unsigned long long* p = lines + (size_t)(tid % nlines) * 8;
     const unsigned long long end = gsys::globaltimer() + ns;
-    unsigned long long acc = 0, polls = 0;
+    unsigned long long mx = 0, polls = 0;
     while (gsys::globaltimer() < end) {
-        acc += gsys::ld_relaxed_sys(p);
+        const unsigned long long v = gsys::ld_relaxed_sys(p);   // system scope: sees host stores
+        mx = v > mx ? v : mx;
         polls++;
     }
-    atomicAdd(sink, polls + (acc & 1ull));
+    atomicAdd(sink, polls);
+    atomicMax(sink + 1, mx);
 }
 
 }  // namespace

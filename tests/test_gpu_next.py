@@ -117,3 +117,32 @@ def test_perm_pwrite_file_equals_cpu_permutation(tmpdir_shm, gflags, iters):
     assert rc == 0
     got = np.fromfile(path, dtype=np.uint8)
     assert np.array_equal(got, plan.permuted_blocks(data, perm, iters, bs))
+
+
+@pytest.mark.parametrize("where", ["host", "device"])
+def test_poll_storm_observes_stores(where):
+    """Row f4 (Fig. 9, PAPER.md:28 P28.7-11): GPU threads polling lines with system-scope loads
+    keep polling for the requested time and observe a store the host makes during the storm (the
+    visibility the completion polls of a5 rely on)."""
+    import threading
+    import time
+    n = 64
+    lines = (torch.zeros(n * 8, dtype=torch.int64).pin_memory() if where == "host"
+             else torch.zeros(n * 8, dtype=torch.int64, device="cuda"))
+    sink = torch.zeros(2, dtype=torch.int64, device="cuda")
+    s = torch.cuda.Stream()
+    nthreads = 148 * 64
+    t0 = time.perf_counter()
+    assert G.lib().gsys_poll_storm(lines.data_ptr(), n, nthreads, int(300e6), sink.data_ptr(), s.cuda_stream) == 0
+    time.sleep(0.1)
+    if where == "host":
+        lines[::8] = 7                                       # plain host stores into pinned memory
+    else:
+        s2 = torch.cuda.Stream()
+        with torch.cuda.stream(s2):
+            lines[::8].fill_(7)                              # a concurrent kernel's stores
+    s.synchronize()
+    dt = time.perf_counter() - t0
+    polls, seen = int(sink[0]), int(sink[1])
+    assert seen == 7, seen
+    assert polls >= nthreads and 0.25 < dt < 5, (polls, dt)

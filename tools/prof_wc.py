@@ -1,4 +1,5 @@
-"""Single wordcount launch for ncu (application replay): 64 x 16 MiB files, host staging."""
+"""Single wordcount launch for ncu (application replay): the first N (default 64) of the bench's
+512 x 16 MiB files; argv[1] = device (default pull completion) | host staging."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
