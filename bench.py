@@ -366,22 +366,23 @@ def main():
     kernel_s = dev_s / a.steps
     algo_bytes = my_bytes + sum(((s + chunk - 1) // chunk) * 17 for s in of.sizes)   # chunk + halo
     rank_achieved = algo_bytes / kernel_s / 1e9
-    traffic, sysmem_ratio = None, None
-    summ = os.path.join(ROOT, "profiles", "r01_ncu_summary.json")
-    if os.path.exists(summ):   # one ncu --set full capture of wc_kernel (64 files = 1 GiB), scaled per launch
-        wk = json.load(open(summ)).get("wc_kernel_64x16MiB_host_staging", {})
+    traffic, traffic_src = None, None
+    summ = os.path.join(ROOT, "profiles", "r02_ncu_summary.json")
+    label = {"device": "wc_kernel_64x16MiB_device_pull", "host": "wc_kernel_64x16MiB_host_staging"}.get(a.staging)
+    if label and os.path.exists(summ):   # ncu capture of wc_kernel over 64 of the files (1 GiB), scaled per launch
+        wk = json.load(open(summ)).get(label, {})
         try:
             cap_bytes = 64 * (16 << 20)
-            dram = float(wk["dram_read_bytes"]) + float(wk["dram_write_bytes"])
+            dram = float(wk["dram__bytes_read.sum"]) + float(wk["dram__bytes_write.sum"])
             traffic = dram * algo_bytes / cap_bytes
-            sysmem_ratio = float(wk["syslts__t_sectors_aperture_sysmem_lookup_miss.sum"]) * 32 / cap_bytes
+            traffic_src = f"profiles/r02_ncu_summary.json[{label}]"
         except (KeyError, ValueError):
             pass
     roofline = {"bound": "host-link", "achieved": rank_achieved, "peak": h2d_peak, "unit": "GB/s",
                 "frac": (rank_achieved / h2d_peak) if h2d_peak else None, "traffic": traffic,
-                "traffic_note": "HBM bytes from profiles/r01_ncu_summary.json scaled to this launch (zero-copy: "
-                                "the data never lands in HBM); system-memory sector bytes per corpus byte = "
-                                f"{sysmem_ratio}",
+                "traffic_note": f"dram__bytes_read.sum + dram__bytes_write.sum of {traffic_src} (ncu application "
+                                "replay, 1 GiB) scaled to this launch: the staging lines stay in L2, so HBM "
+                                "traffic is ~0; the algorithmic bytes cross the host link once",
                 "kernel": "wc_kernel (GPU-issued WG preads + scan), one launch per step per rank",
                 "peak_source": "measured live: pinned cudaMemcpyAsync H2D, 256 MiB x 8, this box's PCIe link "
                                "(MEASURED_PEAKS.json has no host-link figure)"}
@@ -530,8 +531,22 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
                        f"{float(sk['smsp__issue_active.avg.pct_of_peak_sustained_active']):.0f}%")
         except (KeyError, ValueError):
             pass
+    # compute-side roofline: one random 16-bit shared-memory gather per byte (the DFA
+    # lookup), against the measured random-gather rate of tools/probes/b200_probes.cu
+    compute = None
+    probes = os.path.join(ROOT, "profiles", "r02_probes.jsonl")
+    if os.path.exists(probes):
+        for ln in open(probes):
+            try:
+                r = json.loads(ln)
+            except ValueError:
+                continue
+            if r.get("probe") == "smem" and "random gather" in r.get("op", ""):
+                compute = {"bound": "smem random gather (1 DFA lookup per byte)", "achieved": n / t,
+                           "peak": r["lookups_per_s"], "unit": "lookups/s", "frac": n / t / r["lookups_per_s"],
+                           "peak_source": "profiles/r02_probes.jsonl (tools/probes/b200_probes.cu)"}
     return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "bytes": n,
-            "traffic": traffic, "limiter": limiter, "ms": t * 1e3,
+            "traffic": traffic, "limiter": limiter, "ms": t * 1e3, "compute_roofline": compute,
             "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 704 threads (22 warps), 77-column transposed DFA in shared memory; 6 % above 512 threads with the 129-column table, profiles/r01_scan_threads_sweep.jsonl)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
 

@@ -1,4 +1,4 @@
-"""Config 1 (16 MiB, 64 WGs, WG + blocking + strong, host staging): where the ~0.6 ms goes --
+"""Config 1 (16 MiB, 64 WGs, WG + blocking + strong): where the time goes per chunk size, WG size and staging --
 per-chunk time in the call vs scanning (gsys_set_profile), kernel vs launch overheads."""
 import json
 import os
@@ -21,15 +21,16 @@ words, pats = inputs.dictionary(), inputs.patterns()
 s = torch.cuda.Stream()
 h = torch.zeros(64, dtype=torch.int64, device="cuda")
 G.gsys_set_profile(True)
-for threads in (256, 128, 64):
+cells = [(t, ck, st) for st in (G.STAGE_HOST, G.STAGE_DEVICE) for ck in (256, 128, 64) for t in (256, 128)]
+for threads, ck, staging in cells:
     res = []
     for rep in range(13):
         G.gsys_read_profile(True)
         G.gsys_stats_reset()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(s)
-        G.gsys_wordcount([fd], [16 << 20], 256 << 10, words, pats, h, None, None, G.WG | G.BLOCKING | G.STRONG, 0,
-                         threads, s, G.STAGE_HOST)
+        G.gsys_wordcount([fd], [16 << 20], ck << 10, words, pats, h, None, None, G.WG | G.BLOCKING | G.STRONG, 64,
+                         threads, s, staging)
         e1.record(s)
         G.gsys_wait(s)
         e1.synchronize()
@@ -40,5 +41,6 @@ for threads in (256, 128, 64):
                         "scan_us_per_chunk": pf["scan_ns"] / max(pf["chunks"], 1) / 1e3, "bundles": st["bundles"],
                         "svc_sys_us_per_call": st["ns_syscall"] / 1e3 / 64})
     res.sort(key=lambda r: r["ms"])
-    print(json.dumps({"threads": threads, **res[len(res) // 2]}), flush=True)
+    print(json.dumps({"threads": threads, "chunk_kib": ck, "staging": "host" if staging == G.STAGE_HOST else "device",
+                      "chunks": (16 << 10) // ck, **res[len(res) // 2]}), flush=True)
 os.close(fd)
