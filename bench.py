@@ -305,6 +305,7 @@ def main():
         ev0 = torch.cuda.Event(enable_timing=True)
         ev1 = torch.cuda.Event(enable_timing=True)
         G.gsys_stats_reset()
+        req0 = G.gsys_stats()["requests"]   # the drained-request counter is cumulative
         barrier()
         ev0.record(stream)
         for _ in range(a.steps):
@@ -314,6 +315,7 @@ def main():
         barrier()
         clocks = clk.stop()
         st = G.gsys_stats()
+        st["requests"] -= req0
     my_s = ev0.elapsed_time(ev1) / 1e3
     dev_s = max_over_ranks(my_s)
     value = corpus.total_bytes * a.steps / dev_s / 1e9

@@ -48,6 +48,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <deque>
+#include <memory>
 #include <mutex>
 #include <numeric>
 #include <thread>
@@ -246,6 +247,23 @@ struct Parked {
     uint64_t deadline_ns;   // UINT64_MAX: no receive timeout
 };
 
+// A large pread served by several workers at once (reading B14): when other workers are idle, the
+// worker that drained the request cuts its byte range into pieces that idle workers read in
+// parallel; whoever finishes the last piece assembles the single-call POSIX result (the bytes up to
+// the first short piece, or the first piece's error) and issues the completion with a host store.
+// Still one request and one completion: the GPU caller sees one blocking pread.
+struct Split {
+    Req r;
+    int fd = -1;
+    uint8_t* dst = nullptr;
+    int64_t off = 0;
+    uint64_t n = 0, piece = 0;
+    uint32_t np = 0;
+    std::atomic<uint32_t> next{0};   // next piece to claim
+    std::atomic<uint32_t> done{0};   // pieces finished
+    std::vector<int64_t> ret;
+};
+
 // ------------------------------------------------------------------ worker
 struct Worker {
     Instance* inst = nullptr;
@@ -290,6 +308,7 @@ struct Worker {
     uint8_t* bounce_d = nullptr;     // device address of the (host-mapped) bounce
     void wait_slot_free(uint32_t slot, uint32_t seq);
     void complete_early(Req& r);
+    bool try_split(Req& r, int fd, uint8_t* dst, uint64_t n, int64_t off);
     std::vector<cudaEvent_t> evpool;
     // copies queued per bundle; flush_copies() issues them (contiguous runs joined)
     std::vector<void*> cp_dst, cp_src;
@@ -395,6 +414,14 @@ struct Instance {
     std::atomic<int> fault_err{0};          // gsys_set_fault: preads at fault_off fail with -fault_err
     std::atomic<int64_t> fault_off{-1};
     std::atomic<int64_t> drop_off{-1};      // gsys_set_fault_drop: that pread's completion is never written
+    // split preads (reading B14): queue of ranges with pieces left, shared by all workers
+    std::mutex split_mu;
+    std::deque<std::shared_ptr<Split>> splits;
+    std::atomic<int> nsplits{0};
+    uint64_t split_min = 128u << 10;      // env GSYS_SPLIT_KB (0 = never split)
+    Sharded st_split;                      // preads served in pieces
+    bool run_piece(Split& sp, uint32_t i);
+    bool help_split();
     gsys_wd_log* wd_d = nullptr;           // device watchdog log (gsys_device.cuh)
     std::mutex wd_mu;
     gsys_wd_log wd_last{};                 // the log as the last gsys_wait that saw expiries read it
@@ -490,6 +517,10 @@ void Worker::run() {
         uint64_t h = I->head.load(std::memory_order_acquire);
         if (!I->ready(h)) {
             if (!idle) { idle = true; I->idle_workers.fetch_add(1, std::memory_order_relaxed); }
+            if (I->nsplits.load(std::memory_order_relaxed) && I->help_split()) {   // pieces of a split pread
+                idle_since = now_ns();
+                continue;
+            }
             if (I->nparked.load(std::memory_order_relaxed)) {   // parked recvfroms keep us awake
                 service_parked();
                 idle_since = now_ns();
@@ -676,6 +707,34 @@ void Worker::complete_early(Req& r) {
     inst->complete_host(r);
 }
 
+// Split a large pread among idle workers (reading B14).  Returns true when the request was handed
+// to the split machinery: its completion is then issued by the worker that finishes the last piece.
+bool Worker::try_split(Req& r, int fd, uint8_t* dst, uint64_t n, int64_t off) {
+    Instance* I = inst;
+    if (!I->split_min || n < I->split_min || r.dropped || r.faulted || !r.ok) return false;
+    const int idle = I->idle_workers.load(std::memory_order_relaxed);
+    if (idle < 1) return false;
+    uint32_t np = (uint32_t)std::min<uint64_t>(std::min<uint64_t>((uint64_t)idle + 1, n / (32u << 10)), 16);
+    if (np < 2) return false;
+    auto sp = std::make_shared<Split>();
+    sp->r = r;
+    sp->fd = fd;
+    sp->dst = dst;
+    sp->off = off;
+    sp->n = n;
+    sp->piece = ((n + np - 1) / np + 4095) & ~(uint64_t)4095;
+    sp->np = (uint32_t)((n + sp->piece - 1) / sp->piece);
+    sp->ret.assign(sp->np, 0);
+    r.early = true;   // completed by the last piece's worker
+    {
+        std::lock_guard<std::mutex> g(I->split_mu);
+        I->splits.push_back(sp);
+        I->nsplits.fetch_add(1, std::memory_order_release);
+    }
+    { Timer tm(t_sys); while (I->run_piece(*sp, sp->next.fetch_add(1, std::memory_order_acq_rel))) {} }
+    return true;
+}
+
 // pread(fd, buf, n, off): host-mapped buf -> read in place; device buf -> read into the pinned
 // bounce and DMA.  A request larger than the bounce is served piecewise with the POSIX result of
 // one call (stop at a short piece, cap at GSYS_PREAD_CAP, reading A11).
@@ -698,16 +757,17 @@ int64_t Worker::do_pread(Req& r) {
         commit();   // earlier regions of this bundle keep their own tokens
         uint8_t* b = alloc(want);
         if (!b) return -ENOMEM;
-        ssize_t z;
-        { Timer tm(t_sys); z = pread(fd, b, want, off); }
         Worker::Tok t;
         t.slot = r.slot;
         t.seq = r.seq;
         ring->commit_with(t);
+        __atomic_store_n(&inst->area_h[r.slot].args[1], (uint64_t)(uintptr_t)(bounce_d + (b - bounce)), __ATOMIC_RELAXED);
+        if (try_split(r, fd, b, want, off)) return 0;
+        ssize_t z;
+        { Timer tm(t_sys); z = pread(fd, b, want, off); }
         inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
         r.ret = z < 0 ? -(int64_t)errno : (int64_t)z;
         if (z > 0) inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
-        __atomic_store_n(&inst->area_h[r.slot].args[1], (uint64_t)(uintptr_t)(bounce_d + (b - bounce)), __ATOMIC_RELAXED);
         complete_early(r);
         return r.ret;
     }
@@ -719,6 +779,9 @@ int64_t Worker::do_pread(Req& r) {
         k = resolve(buf, n, &hp);
     }
     if (k == PK_INVALID) return -EFAULT;
+    if (k == PK_HOST && (r.flags & (GSYS_HOSTBUF | GSYS_F_PULL)) &&
+        try_split(r, fd, hp, std::min<uint64_t>(n, GSYS_PREAD_CAP), off))   // one call returns <= the cap (A11)
+        return 0;
     inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
     if (k == PK_HOST) {
         ssize_t z;
@@ -932,6 +995,45 @@ void Worker::service_parked() {
     const size_t done = I->parked.size() - keep;
     I->parked.resize(keep);
     if (done) I->nparked.fetch_sub((uint32_t)done, std::memory_order_release);
+}
+
+// One piece of a split pread; the worker finishing the last piece completes the request.
+bool Instance::run_piece(Split& sp, uint32_t i) {
+    if (i >= sp.np) return false;
+    const uint64_t lo = (uint64_t)i * sp.piece;
+    const uint64_t len = std::min<uint64_t>(sp.piece, sp.n - lo);
+    const ssize_t z = pread(sp.fd, sp.dst + lo, len, sp.off + (int64_t)lo);
+    sp.ret[i] = z < 0 ? -(int64_t)errno : (int64_t)z;
+    st_host_preads.fetch_add(1, std::memory_order_relaxed);
+    if (sp.done.fetch_add(1, std::memory_order_acq_rel) + 1 == sp.np) {
+        int64_t total = 0;
+        for (uint32_t k = 0; k < sp.np; k++) {
+            const uint64_t lk = std::min<uint64_t>(sp.piece, sp.n - (uint64_t)k * sp.piece);
+            if (sp.ret[k] < 0) { if (k == 0) total = sp.ret[0]; break; }
+            total += sp.ret[k];
+            if ((uint64_t)sp.ret[k] < lk) break;   // short piece: the single call would stop here
+        }
+        if (total > 0) st_bytes_read.fetch_add((uint64_t)total, std::memory_order_relaxed);
+        st_split.fetch_add(1, std::memory_order_relaxed);
+        sp.r.ret = total;
+        complete_host(sp.r);
+    }
+    return true;
+}
+
+// An idle worker takes one piece of the oldest split that still has pieces left.
+bool Instance::help_split() {
+    std::shared_ptr<Split> sp;
+    {
+        std::lock_guard<std::mutex> g(split_mu);
+        while (!splits.empty() && splits.front()->next.load(std::memory_order_relaxed) >= splits.front()->np) {
+            splits.pop_front();
+            nsplits.fetch_sub(1, std::memory_order_relaxed);
+        }
+        if (splits.empty()) return false;
+        sp = splits.front();
+    }
+    return run_piece(*sp, sp->next.fetch_add(1, std::memory_order_acq_rel));
 }
 
 void Instance::complete_host(const Req& r) {
@@ -1350,6 +1452,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     I->memop_completion = c.memop_completion != 0;
     ev = getenv("GSYS_BIG_ALONE");
     I->big_alone = !(ev && atoi(ev) == 0);
+    ev = getenv("GSYS_SPLIT_KB");
+    if (ev) I->split_min = (uint64_t)atoll(ev) << 10;
     ev = getenv("GSYS_SHARE_BURSTS");
     I->share_bursts = !(ev && atoi(ev) == 0);
     ev = getenv("GSYS_DIAG_PHASES");
