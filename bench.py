@@ -364,6 +364,8 @@ def main():
         extras["scan"] = scan_roofline(G, dev, corpus, words, pats, chunk)
         extras["syscalls"] = wg_syscall_rate(G, W, dev, corpus.paths[0])
         extras["config1"] = config1_latency(G, W, dev, words, pats, a.root)
+        for v in extras["config1"].values():
+            v["frac_of_h2d"] = v["GBps_median"] / h2d_peak if h2d_peak else None
         extras["fig10"] = fig10_coalescing(G, W, dev, corpus.paths[0])
     kernel_s = dev_s / a.steps
     algo_bytes = my_bytes + sum(((s + chunk - 1) // chunk) * 17 for s in of.sizes)   # chunk + halo
@@ -560,14 +562,16 @@ def config1_latency(G, W, dev, words, pats, root):
 
     import inputs
     path = os.path.join(root or "/dev/shm", "gsys_config1_16MiB.txt")
-    if not os.path.exists(path) or os.path.getsize(path) != (16 << 20):
-        inputs.write_file(path, inputs.SEED_FILE16M, 0, 16 << 20)
+    census, _ = inputs.write_file(path, inputs.SEED_FILE16M, 0, 16 << 20)
     fd = os.open(path, os.O_RDONLY)
     out = {}
     try:
         s = torch.cuda.Stream(device=dev)
         h = torch.zeros(64, dtype=torch.int64, device=dev)
-        for name, st in (("host", G.STAGE_HOST), ("device", G.STAGE_DEVICE)):
+        # 64 work-groups each take chunks from the file's queue: 64 KiB chunks (4 blocking preads
+        # per work-group) keep the link busier than one 256 KiB read each (profiles/r02_config1_sweep.jsonl)
+        for name, st, ck in (("host", G.STAGE_HOST, 64), ("host_256k", G.STAGE_HOST, 256),
+                             ("device", G.STAGE_DEVICE, 64)):
             ts, ws = [], []
             for rep in range(23):
                 h.zero_()
@@ -575,8 +579,8 @@ def config1_latency(G, W, dev, words, pats, root):
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 t0 = time.perf_counter()
                 e0.record(s)
-                G.gsys_wordcount([fd], [16 << 20], 256 << 10, words, pats, h, None, None,
-                                 G.WG | G.BLOCKING | G.STRONG, 0, 256, s, st)
+                G.gsys_wordcount([fd], [16 << 20], ck << 10, words, pats, h, None, None,
+                                 G.WG | G.BLOCKING | G.STRONG, 64, 256, s, st)
                 e1.record(s)          # device time: table upload + the kernel (its 64 preads inside)
                 G.gsys_wait(s)
                 _ = h.cpu()           # wall time: the call until the histogram is on the host
@@ -588,7 +592,8 @@ def config1_latency(G, W, dev, words, pats, root):
             ts.sort()
             ws.sort()
             out[name] = {"ms_median": ts[len(ts) // 2], "GBps_median": (16 << 20) / (ts[len(ts) // 2] / 1e3) / 1e9,
-                         "ms_min": ts[0], "wall_ms_median": ws[len(ws) // 2]}
+                         "ms_min": ts[0], "wall_ms_median": ws[len(ws) // 2], "chunk": ck << 10, "work_groups": 64,
+                         "parity": bool((h.cpu().numpy().astype("uint64") == census).all())}
     finally:
         os.close(fd)
     return out

@@ -1655,7 +1655,8 @@ int gsys_trace_read(gsys_trace_rec* gpu_out, uint32_t gpu_cap, uint32_t* n_gpu, 
     return 0;
 }
 
-int gsys_launch_begin(uint64_t nblocks, void* stream) {
+}  // extern "C"
+static int launch_begin_impl(uint64_t nblocks, void* stream, bool ksites) {
     Instance* I = current();
     if (!I) return -ENODEV;
     if (nblocks == 0 || nblocks > (1ull << 31)) return -EINVAL;
@@ -1676,9 +1677,11 @@ int gsys_launch_begin(uint64_t nblocks, void* stream) {
     }
     // reset the kernel-scope call sites for this launch (block rounds + per-round records); they
     // are shared by the instance: kernel-scope calls of launches running concurrently on other
-    // streams are not supported (gsys.h)
-    cudaMemsetAsync(I->kblock_d, 0, (size_t)nb * GSYS_KSITES * 4, s);
-    cudaMemsetAsync(I->krounds_d, 0, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS, s);
+    // streams are not supported (gsys.h).  Library kernels that make no kernel-scope call skip it.
+    if (ksites) {
+        cudaMemsetAsync(I->kblock_d, 0, (size_t)nb * GSYS_KSITES * 4, s);
+        cudaMemsetAsync(I->krounds_d, 0, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS, s);
+    }
     // the learned pre-poll sleep (reading B3) is relearned per launch: a hint carried over from
     // another workload's latency would make this kernel's first calls oversleep
     cudaMemsetAsync(I->lat_hint_d, 0, (size_t)I->nslots * 4, s);
@@ -1690,6 +1693,18 @@ int gsys_launch_begin(uint64_t nblocks, void* stream) {
     }
     return cuda_err(cudaGetLastError());
 }
+
+int gsys_internal_launch(const void* kernel, uint32_t grid, uint32_t block, void** args, size_t smem, void* stream,
+                         bool kernel_sites) {
+    if (!kernel || grid == 0 || block == 0) return -EINVAL;
+    int rc = launch_begin_impl(grid, stream, kernel_sites);
+    if (rc) return rc;
+    return cuda_err(cudaLaunchKernel(kernel, dim3(grid), dim3(block), args, smem, (cudaStream_t)stream));
+}
+
+extern "C" {
+
+int gsys_launch_begin(uint64_t nblocks, void* stream) { return launch_begin_impl(nblocks, stream, true); }
 
 int gsys_launch(const void* kernel, uint32_t gx, uint32_t gy, uint32_t gz, uint32_t bx, uint32_t by, uint32_t bz,
                 void** args, size_t smem_bytes, void* stream) {

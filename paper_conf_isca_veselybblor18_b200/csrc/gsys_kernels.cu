@@ -643,6 +643,12 @@ struct Workspace {
     // for it on the device before touching the shared chunk queue, uploads or staging lines, so
     // calls on different streams are serialised instead of racing
     cudaEvent_t last_ev = nullptr;
+    // the scan tables of the last (dictionary, patterns, implementation, columns) built on the host:
+    // building them (trie + DFA fill, or the hash search) costs more CPU time than a config-1 kernel
+    // runs, so repeated calls with the same dictionary reuse the blob
+    struct TabCache { std::vector<uint8_t> key, blob; unsigned char* d = nullptr; size_t dcap = 0; };
+    TabCache tcache[4];
+    unsigned tcache_next = 0;
     unsigned char* staging_d = nullptr;
     size_t staging_cap = 0;
     unsigned long long* prof_d = nullptr;  // wc_kernel profile counters (gsys_set_profile)
@@ -672,6 +678,53 @@ Workspace* workspace() {
         cudaDeviceGetAttribute(&W->sms, cudaDevAttrMultiProcessorCount, d);
     }
     return W;
+}
+
+// The scan tables for (impl, ncol, dictionary, patterns): from the cache, else built.  Returns the
+// cache entry (host blob, a 16-byte multiple, and its device copy) or nullptr with *rc set.
+Workspace::TabCache* scan_tables(Workspace* W, bool tok, unsigned ncol, const char* dict, const uint8_t* dlen,
+                                 uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, int* rc) {
+    std::vector<uint8_t> key;
+    key.reserve(16 + 18u * (ndict + npat));
+    const uint32_t hdr[4] = {tok ? 1u : 0u, ncol, ndict, npat};
+    key.insert(key.end(), (const uint8_t*)hdr, (const uint8_t*)hdr + sizeof hdr);
+    if (ndict && dict && dlen) {
+        key.insert(key.end(), (const uint8_t*)dict, (const uint8_t*)dict + 17ull * ndict);
+        key.insert(key.end(), dlen, dlen + ndict);
+    }
+    if (npat && pats && plen) {
+        key.insert(key.end(), (const uint8_t*)pats, (const uint8_t*)pats + 17ull * npat);
+        key.insert(key.end(), plen, plen + npat);
+    }
+    for (auto& c : W->tcache)
+        if (!c.blob.empty() && c.key == key) { *rc = 0; return &c; }
+    size_t tb = 0;
+    int r = tok ? gsys_tok::build_tok_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb)
+                : build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
+    if (r && r != -ENOSPC) { *rc = r; return nullptr; }
+    std::vector<uint8_t> blob((tb + 15) & ~(size_t)15, 0);
+    r = tok ? gsys_tok::build_tok_tables(blob.data(), blob.size(), dict, dlen, ndict, pats, plen, npat, nullptr)
+            : build_tables(blob.data(), blob.size(), dict, dlen, ndict, pats, plen, npat, nullptr, ncol);
+    if (r) { *rc = r; return nullptr; }
+    auto& c = W->tcache[W->tcache_next++ % 4];
+    // the entry's device copy may be in use by a running kernel: wait for the last launch first
+    cudaEventSynchronize(W->last_ev);
+    if (c.dcap < blob.size()) {
+        if (c.d) cudaFree(c.d);
+        c.d = nullptr;
+        c.dcap = 0;
+        if (cudaMalloc((void**)&c.d, blob.size()) != cudaSuccess) { *rc = -ENOMEM; c.blob.clear(); return nullptr; }
+        c.dcap = blob.size();
+    }
+    if (cudaMemcpy(c.d, blob.data(), blob.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
+        *rc = -EIO;
+        c.blob.clear();
+        return nullptr;
+    }
+    c.key.swap(key);
+    c.blob.swap(blob);
+    *rc = 0;
+    return &c;
 }
 
 int ensure_upload(Workspace* W, size_t bytes) {
@@ -764,16 +817,14 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     if (nch < blocks) blocks = (uint32_t)(nch ? nch : 1);
     // upload: [tables][fds][sizes][cbase]; token tables (default) or the byte DFA (gsys_set_scan)
     const bool tok = g_scan_impl.load() == GSYS_SCAN_TOKEN;
-    size_t tb = 0;
-    int rc = tok ? gsys_tok::build_tok_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb)
-                 : build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb);
-    if (rc && rc != -ENOSPC) return rc;
-    size_t o_t = 0, o_f = align_up(tb, 256), o_s = align_up(o_f + 4ull * nfiles, 256),
+    int rc = 0;
+    Workspace::TabCache* tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);
+    if (!tc) return rc;
+    const size_t tb = tc->blob.size();
+    // upload: [fds][sizes][cbase] (the tables are already on the device)
+    size_t o_f = 0, o_s = align_up(o_f + 4ull * nfiles, 256),
            o_c = align_up(o_s + 8ull * nfiles, 256), total = align_up(o_c + 4ull * (nfiles + 1), 256);
     rc = ensure_upload(W, total);
-    if (rc) return rc;
-    rc = tok ? gsys_tok::build_tok_tables(W->up_h + o_t, tb, dict, dlen, ndict, pats, plen, npat, nullptr)
-             : build_tables(W->up_h + o_t, tb, dict, dlen, ndict, pats, plen, npat, nullptr);
     if (rc) return rc;
     memcpy(W->up_h + o_f, fds, 4ull * nfiles);
     memcpy(W->up_h + o_s, sizes, 8ull * nfiles);
@@ -799,8 +850,8 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     WcArgs a;
     memset(&a, 0, sizeof a);
     a.ctx = ctx;
-    a.tables = reinterpret_cast<const ScanTables*>(W->up_d + o_t);
-    a.ttables = reinterpret_cast<const gsys_tok::TokTables*>(W->up_d + o_t);
+    a.tables = reinterpret_cast<const ScanTables*>(tc->d);
+    a.ttables = reinterpret_cast<const gsys_tok::TokTables*>(tc->d);
     a.fds = reinterpret_cast<const int*>(W->up_d + o_f);
     a.sizes = reinterpret_cast<const unsigned long long*>(W->up_d + o_s);
     a.chunk_base = reinterpret_cast<const unsigned*>(W->up_d + o_c);
@@ -830,7 +881,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     rc = ensure_smem_attr(fn, smem);
     if (rc) return rc;
     if (cudaMemsetAsync(W->next_chunk_d, 0, 4, s) != cudaSuccess) return -EIO;
-    rc = gsys_launch(fn, blocks, 1, 1, threads, 1, 1, args, smem, stream);
+    rc = gsys_internal_launch(fn, blocks, threads, args, smem, stream, false);   // no kernel-scope calls
     cudaEventRecord(W->last_ev, s);
     return rc;
 }
@@ -876,27 +927,17 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (!W) return -ENODEV;
     // DFA: the 129-column table when it fits next to the warps' staging (1 block of `threads` per
     // SM), else the 77-column one
-    size_t tb = 0;
-    unsigned ncol = NCOL_WIDE;
-    int rc = tok ? gsys_tok::build_tok_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb)
-                 : build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
-    if (rc && rc != -ENOSPC) return rc;
+    int rc = 0;
+    Workspace::TabCache* tc = scan_tables(W, tok, NCOL_WIDE, dict, dlen, ndict, pats, plen, npat, &rc);
+    if (!tc) return rc;
     const size_t per_warp = HSTRIDE * 4 + (tok ? TWARP_STAGE : WARP_STAGE);
-    if (!tok && align_up(tb, 16) + (threads / 32) * per_warp > kSmemDynMax) {
-        ncol = NCOL_NARROW;
-        rc = build_tables(nullptr, 0, dict, dlen, ndict, pats, plen, npat, &tb, ncol);
-        if (rc && rc != -ENOSPC) return rc;
+    if (!tok && tc->blob.size() + (threads / 32) * per_warp > kSmemDynMax) {
+        tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);
+        if (!tc) return rc;
     }
-    size_t total = align_up(tb, 256);
-    rc = ensure_upload(W, total);
-    if (rc) return rc;
-    rc = tok ? gsys_tok::build_tok_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr)
-             : build_tables(W->up_h, tb, dict, dlen, ndict, pats, plen, npat, nullptr, ncol);
-    if (rc) return rc;
+    const size_t tb = tc->blob.size();
     cudaStream_t s = (cudaStream_t)stream;
     cudaStreamWaitEvent(s, W->last_ev, 0);
-    cudaMemcpyAsync(W->up_d, W->up_h, total, cudaMemcpyHostToDevice, s);
-    cudaEventRecord(W->up_ev, s);
     unsigned long long nch = (n + chunk - 1) / chunk;
     if (nch == 0) return 0;
     const bool blocks_auto = blocks == 0;
@@ -904,7 +945,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (nch < blocks) blocks = (uint32_t)nch;
     ScanArgs a;
     memset(&a, 0, sizeof a);
-    a.tables = reinterpret_cast<const ScanTables*>(W->up_d);
+    a.tables = reinterpret_cast<const ScanTables*>(tc->d);
     a.text = d_text;
     a.n = n;
     a.hist = reinterpret_cast<unsigned long long*>(d_hist);
