@@ -241,6 +241,7 @@ __device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__
     const unsigned hs = (unsigned)__cvta_generic_to_shared(S.whist);
     auto emit = [hs](unsigned d) { asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hs + 4u * d)); };
     const gsys_tok::TokRegs R = gsys_tok::tok_regs(T);
+    const unsigned one = T.one;
     const long long step = 2048ll * nwarps;
     long long base = s + 2048ll * warp;
     if (base < own_end) stage_tile_tok(stage_s, seg0, s, base, valid_end, lane);
@@ -259,7 +260,7 @@ __device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__
         W.w2 = *reinterpret_cast<const uint4*>(span + 32u);
         W.w3 = *reinterpret_cast<const uint4*>(span + 48u);
         W.w4 = *reinterpret_cast<const uint4*>(span + 64u);
-        const unsigned long long M = gsys_tok::mask64(W);
+        const unsigned long long M = gsys_tok::mask64(W, one);
         unsigned la = __shfl_down_sync(0xffffffffu, (unsigned)M & 0xffffu, 1);
         if (lane == 31u) la = gsys_tok::mask16(W.w4);
         unsigned pw = __shfl_up_sync(0xffffffffu, (unsigned)(M >> 63), 1);

@@ -16,6 +16,8 @@
 // in distinct slots), then verified byte-exactly -- about four shared-memory accesses per token
 // (mean token 5.8 bytes plus separators) instead of one per byte.
 #pragma once
+#include <stddef.h>
+
 #include "scan_core.cuh"
 
 namespace gsys_tok {
@@ -34,26 +36,30 @@ struct TokTables {
     unsigned ndict;
     unsigned lenmask;           // bit L: some matchable dictionary word has length L (1..16)
     unsigned m[5];              // hash multipliers (bytes 0-3, 4-7, 8-11, 12-15, length)
-    unsigned pad_;
+    unsigned one;               // 1 (a run-time constant: see word4)
     unsigned char klen[MAXD];
     unsigned char slot[HSIZE];  // 0: empty, else word index + 1
 };
 static_assert(sizeof(TokTables) % 16 == 0, "TokTables must keep 16-byte alignment");
 
-GSYS_HD unsigned tok_hash(const unsigned m[5], unsigned a, unsigned b, unsigned c, unsigned d, unsigned len) {
-    return ((a * m[0]) ^ (b * m[1]) ^ (c * m[2]) ^ (d * m[3]) ^ (len * m[4])) >> (32u - HBITS);
+// Slot of a token: its first 8 bytes (zero-padded) and its length.  The builder requires the
+// matchable words to differ in (first 8 bytes, length) -- bytes 8..15 are only verified.
+GSYS_HD unsigned tok_hash(const unsigned m[5], unsigned a, unsigned b, unsigned len) {
+    return ((a * m[0]) ^ (b * m[1]) ^ (len * m[4])) >> (32u - HBITS);
 }
 
 // Word bytes of a little-endian 4-byte group: bit 7 of byte i set iff byte i is in [0-9A-Za-z_]
 // (bytes >= 0x80 are not).  Per byte, 7-bit adds that cannot carry across bytes.
-GSYS_HD unsigned word4(unsigned w) {
+// `one` == 1 at run time: the adds become IMADs (x * one + c) and run on the FMA pipe, next to the
+// LOP3s on the ALU pipe (the token scan is ALU-pipe bound: B200 issues 16 ALU lanes per SMSP).
+GSYS_HD unsigned word4(unsigned w, unsigned one = 1u) {
     const unsigned a = w & 0x7f7f7f7fu;
     const unsigned x = a | 0x20202020u;                  // letters folded to lower case
-    const unsigned g1 = x + 0x1f1f1f1fu;                 // x >= 0x61
-    const unsigned g2 = x + 0x05050505u;                 // x >= 0x7b
-    const unsigned g3 = a + 0x50505050u;                 // a >= 0x30
-    const unsigned g4 = a + 0x46464646u;                 // a >= 0x3a
-    const unsigned nu = (a ^ 0x5f5f5f5fu) + 0x7f7f7f7fu; // a != '_'
+    const unsigned g1 = x * one + 0x1f1f1f1fu;           // x >= 0x61
+    const unsigned g2 = x * one + 0x05050505u;           // x >= 0x7b
+    const unsigned g3 = a * one + 0x50505050u;           // a >= 0x30
+    const unsigned g4 = a * one + 0x46464646u;           // a >= 0x3a
+    const unsigned nu = (a ^ 0x5f5f5f5fu) * one + 0x7f7f7f7fu; // a != '_'
     // letter: x in [0x61, 0x7a] (no digit or '_' maps there); digit: a in [0x30, 0x39]
     const unsigned v = (g1 & ~g2) | (g3 & ~g4);
     return (v | ~nu) & ~w & 0x80808080u;
@@ -75,13 +81,23 @@ GSYS_HD unsigned pack16(unsigned c0, unsigned c1, unsigned c2, unsigned c3) {
 #endif
 }
 
-GSYS_HD unsigned mask16(const uint4& q) { return pack16(word4(q.x), word4(q.y), word4(q.z), word4(q.w)); }
+GSYS_HD unsigned mask16(const uint4& q, unsigned one = 1u) {
+    return pack16(word4(q.x, one), word4(q.y, one), word4(q.z, one), word4(q.w, one));
+}
 
 // Word-byte mask of the lane's 64-byte span W.w0..w3 (bit i = byte p0 + i).
-GSYS_HD unsigned long long mask64(const Win& W) {
-    const unsigned a = mask16(W.w0) | (mask16(W.w1) << 16);
-    const unsigned b = mask16(W.w2) | (mask16(W.w3) << 16);
+GSYS_HD unsigned long long mask64(const Win& W, unsigned one = 1u) {
+    const unsigned a = mask16(W.w0, one) | (mask16(W.w1, one) << 16);
+    const unsigned b = mask16(W.w2, one) | (mask16(W.w3, one) << 16);
     return (unsigned long long)a | ((unsigned long long)b << 32);
+}
+
+GSYS_HD unsigned ctz32(unsigned x) {
+#ifdef __CUDA_ARCH__
+    return (unsigned)__ffs((int)x) - 1u;
+#else
+    return (unsigned)__builtin_ctz(x);
+#endif
 }
 
 GSYS_HD unsigned ctz64(unsigned long long x) {
@@ -116,10 +132,22 @@ GSYS_HD void load8(const unsigned char* p, unsigned& lo, unsigned& hi) {
     hi = GSYS_FSHR(u1, u2, sh);
 }
 
-// Keep the first n (0..8) bytes of (lo, hi).
+// 0xffffffff >> s with s clamped to [0, 32] (32 or more: 0)
+GSYS_HD unsigned shr_ones(int s) {
+    s = s < 0 ? 0 : s;
+#ifdef __CUDA_ARCH__
+    unsigned r;
+    asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(0xffffffffu), "r"((unsigned)s));   // PTX clamps shifts >= 32
+    return r;
+#else
+    return s >= 32 ? 0u : 0xffffffffu >> s;
+#endif
+}
+
+// Keep the first n (n >= 1) bytes of (lo, hi): bytes 0..3 in lo, 4..7 in hi.
 GSYS_HD void keep8(unsigned& lo, unsigned& hi, unsigned n) {
-    lo &= n >= 4u ? 0xffffffffu : ((1u << (8u * n)) - 1u);
-    hi &= n >= 8u ? 0xffffffffu : (n <= 4u ? 0u : ((1u << (8u * (n - 4u))) - 1u));
+    lo &= shr_ones(32 - 8 * (int)n);
+    hi &= shr_ones(64 - 8 * (int)n);
 }
 
 // The tokens owned by one lane span.  span: the span's bytes p0.. in memory (at least 96 readable
@@ -129,12 +157,80 @@ GSYS_HD void keep8(unsigned& lo, unsigned& hi, unsigned n) {
 // may run up to 16 bytes into the lookahead (longer ones cannot match).  emit(d): one hit of word d.
 // Table fields a lane keeps in registers for the whole scan.
 struct TokRegs {
-    unsigned lenmask, m0, m1, m2, m3, m4;
+    unsigned lenmask, m0, m1, m4;
+    unsigned tabs;   // device: shared-space address of the TokTables (explicit ld.shared lookups)
 };
 GSYS_HD TokRegs tok_regs(const TokTables& T) {
-    return TokRegs{T.lenmask, T.m[0], T.m[1], T.m[2], T.m[3], T.m[4]};
+#ifdef __CUDA_ARCH__
+    const unsigned tabs = (unsigned)__cvta_generic_to_shared(&T);
+#else
+    const unsigned tabs = 0u;
+#endif
+    return TokRegs{T.lenmask & 0x1fffeu, T.m[0], T.m[1], T.m[4], tabs};
 }
 
+// Table lookups: shared-space loads on the device (the generic form recomputes the shared window
+// base per access), plain reads on the host.
+GSYS_HD unsigned tok_slot(const TokTables& T, const TokRegs& R, unsigned h) {
+#ifdef __CUDA_ARCH__
+    unsigned v;
+    asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(R.tabs + (unsigned)offsetof(TokTables, slot) + h));
+    return v & 0xffu;
+#else
+    (void)R;
+    return T.slot[h];
+#endif
+}
+GSYS_HD void tok_key(const TokTables& T, const TokRegs& R, unsigned d, uint4& k, unsigned& klen) {
+#ifdef __CUDA_ARCH__
+    asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(k.x), "=r"(k.y), "=r"(k.z), "=r"(k.w)
+        : "r"(R.tabs + (unsigned)offsetof(TokTables, key) + 16u * d));
+    asm("ld.shared.u8 %0, [%1];" : "=r"(klen) : "r"(R.tabs + (unsigned)offsetof(TokTables, klen) + d));
+    klen &= 0xffu;
+#else
+    (void)R;
+    k = T.key[d];
+    klen = T.klen[d];
+#endif
+}
+
+// The tokens starting at the positions set in S (bit q = byte 32*half + q of the span): lo, hi are
+// the word-byte mask of that half and of the 32 bytes after it, so the run of word bytes from q is
+// one funnel shift away; a token of 32+ word bytes leaves no zero in the window (length > 16).
+template <class Emit>
+GSYS_HD void tok_visit(const TokTables& T, const TokRegs& R, const unsigned char* span, unsigned half, unsigned S,
+                       unsigned lo, unsigned hi, Emit&& emit) {
+    while (S) {
+        const unsigned q = ctz32(S);
+        S &= S - 1u;
+        const unsigned w = GSYS_FSHR(lo, hi, q);
+        const unsigned len = ~w ? ctz32(~w) : 32u;
+        if (!((R.lenmask >> (len & 31u)) & 1u) || len > 16u) continue;
+        const unsigned char* t = span + 32u * half + q;
+        unsigned a, b;
+        load8(t, a, b);
+        keep8(a, b, len);
+        const unsigned id = tok_slot(T, R, ((a * R.m0) ^ (b * R.m1) ^ (len * R.m4)) >> (32u - HBITS));
+        if (!id) continue;
+        uint4 k;
+        unsigned klen;
+        tok_key(T, R, id - 1u, k, klen);
+        if (klen != len || k.x != a || k.y != b) continue;
+        if (len > 8u) {   // bytes 8..15: only for the few long words
+            unsigned c, d;
+            load8(t + 8u, c, d);
+            keep8(c, d, len - 8u);
+            if (k.z != c || k.w != d) continue;
+        }
+        emit(id - 1u);
+    }
+}
+
+// The tokens owned by one lane span.  span: the span's bytes p0.. in memory (at least 80 readable
+// bytes; bytes at or past valid_end are never part of a token because the masks exclude them);
+// M: word-byte mask of the 64 span bytes; la: the mask of the 16 bytes after them; prev_word:
+// byte p0-1 exists and is a word byte.  Owned token starts are [p0, min(p0+64, own_end)); a token
+// may run up to 16 bytes into the lookahead (longer ones cannot match).  emit(d): one hit of word d.
 template <class Emit>
 GSYS_HD void tok_lane64(const TokTables& T, const TokRegs& R, const unsigned char* span, unsigned long long M,
                         unsigned la, bool prev_word, long long p0, long long own_end, long long valid_end,
@@ -145,40 +241,17 @@ GSYS_HD void tok_lane64(const TokTables& T, const TokRegs& R, const unsigned cha
         if (nv < 64u) { M &= nv ? (~0ull >> (64u - nv)) : 0ull; la = 0u; }
         else la &= (1u << (nv - 64u)) - 1u;
     }
-    unsigned long long S = M & ~((M << 1) | (prev_word ? 1ull : 0ull));
+    const unsigned m0 = (unsigned)M, m1 = (unsigned)(M >> 32), m2 = la & 0xffffu;
+    unsigned s0 = m0 & ~((m0 << 1) | (prev_word ? 1u : 0u));
+    unsigned s1 = m1 & ~((m1 << 1) | (m0 >> 31));
     const long long nown_ll = own_end - p0;
-    if (nown_ll < 64) S &= nown_ll <= 0 ? 0ull : (~0ull >> (64u - (unsigned)nown_ll));
-    // token ends (last word byte): in the span, then in the lookahead.  Starts and ends alternate,
-    // so the k-th owned start pairs with the k-th end once the end of a token begun before p0 (if
-    // the span opens inside one) is dropped; a token still open at byte 79 is longer than 16.
-    unsigned long long E = M & ~((M >> 1) | ((unsigned long long)(la & 1u) << 63));
-    unsigned Ela = la & ~(la >> 1);
-    if (prev_word && (M & 1ull)) {
-        if (E) E &= E - 1ull;
-        else Ela &= Ela - 1u;
+    if (nown_ll < 64) {
+        const unsigned no = nown_ll <= 0 ? 0u : (unsigned)nown_ll;
+        s0 &= no >= 32u ? 0xffffffffu : ((1u << no) - 1u);
+        s1 &= no <= 32u ? 0u : ((1u << (no - 32u)) - 1u);
     }
-    const unsigned lenmask = R.lenmask & 0x1fffeu;   // lengths 1..16
-    while (S) {
-        const unsigned p = ctz64(S);
-        S &= S - 1ull;
-        unsigned q;
-        if (E) { q = ctz64(E); E &= E - 1ull; }
-        else { q = Ela ? 64u + ctz64(Ela) : 128u; Ela &= Ela - 1u; }
-        const unsigned len = q - p + 1u;
-        if (!((lenmask >> (len & 31u)) & 1u) || len > 31u) continue;
-        unsigned a, b, c = 0u, d = 0u;
-        load8(span + p, a, b);
-        keep8(a, b, len);
-        if (len > 8u) {
-            load8(span + p + 8u, c, d);
-            keep8(c, d, len - 8u);
-        }
-        const unsigned h = ((a * R.m0) ^ (b * R.m1) ^ (c * R.m2) ^ (d * R.m3) ^ (len * R.m4)) >> (32u - HBITS);
-        const unsigned id = T.slot[h];
-        if (!id) continue;
-        const uint4 k = T.key[id - 1u];
-        if (T.klen[id - 1u] == len && k.x == a && k.y == b && k.z == c && k.w == d) emit(id - 1u);
-    }
+    tok_visit(T, R, span, 0u, s0, m0, m1, emit);
+    tok_visit(T, R, span, 1u, s1, m1, m2, emit);
 }
 
 // ------------------------------------------------------------------ host: table builder
@@ -195,6 +268,7 @@ inline int build_tok_tables(void* out, size_t cap, const char* dict, const uint8
     TokTables* T = (TokTables*)out;
     memset(T, 0, sizeof *T);
     T->ndict = ndict;
+    T->one = 1u;
     bool match[MAXD] = {false};
     for (uint32_t d = 0; d < ndict; d++) {
         if (dlen[d] < 1 || dlen[d] > 16) return -EINVAL;
@@ -210,6 +284,12 @@ inline int build_tok_tables(void* out, size_t cap, const char* dict, const uint8
         match[d] = ok;
         if (ok) T->lenmask |= 1u << dlen[d];
     }
+    // the slot is chosen by (first 8 bytes, length): two matchable words sharing both cannot be told
+    // apart by the table -- the byte DFA handles such dictionaries
+    for (uint32_t d = 0; d < ndict; d++)
+        for (uint32_t e = 0; match[d] && e < d; e++)
+            if (match[e] && T->klen[e] == T->klen[d] && T->key[e].x == T->key[d].x && T->key[e].y == T->key[d].y)
+                return -E2BIG;
     unsigned long long x = 0x9E3779B97F4A7C15ull;
     bool placed = false;
     for (int attempt = 0; attempt < 100000 && !placed; attempt++) {
@@ -222,7 +302,7 @@ inline int build_tok_tables(void* out, size_t cap, const char* dict, const uint8
         for (uint32_t d = 0; d < ndict && placed; d++) {
             if (!match[d]) continue;
             const uint4 k = T->key[d];
-            const unsigned h = tok_hash(T->m, k.x, k.y, k.z, k.w, T->klen[d]);
+            const unsigned h = tok_hash(T->m, k.x, k.y, T->klen[d]);
             if (T->slot[h]) placed = false;
             else T->slot[h] = (unsigned char)(d + 1);
         }
