@@ -84,9 +84,12 @@ enum gsys_state {
 #define GSYS_F_NOHINT    0x800u   /* unpredictable latency (network): poll without the learned sleep */
 #define GSYS_F_PULL      0x1000u  /* blocking pread: the host reads into the slot's host-mapped pull
                                      area and the GPU copies it to the destination (reading B12)  */
-#define GSYS_F_PULLB     0x2000u  /* blocking work-group pread: the host reads into its host-mapped
-                                     bounce, returns the range's device address in args[1], and the
-                                     work-group copies it out, then sets the slot free (reading B13) */
+#define GSYS_F_PULLB     0x2000u  /* blocking pread: the host reads into its host-mapped bounce,
+                                     returns the range's device address in args[1], and the caller
+                                     (its work-group) copies it out, then sets the slot free (B13)  */
+#define GSYS_F_DEFER     0x4000u  /* non-blocking pread into device memory: the host reads into a
+                                     host-mapped range and leaves a deferred-pull record; a token
+                                     wait or gsys_wait's flush kernel copies it (reading B15)      */
 
 /* Syscall numbers served (Linux x86-64). */
 #define GSYS_NR_PREAD64        17
@@ -201,8 +204,10 @@ int gsys_launch_begin(uint64_t nblocks, void* stream);
 /* Drain (sec. IX "a new function call, invoked by the CPU, that ensures all GPU
  * system calls have completed before the termination of the process", P34.9).  Waits for the
  * stream (NULL = whole device), then until every request the device has published is processed
- * and its completion (DMA + state write) has landed.  Returns 0, or the first -errno recorded
- * for a non-blocking call since the previous gsys_wait (reading A4), which it then clears. */
+ * and its completion (DMA + state write) has landed.  A device-wide wait (NULL) also lands the
+ * deferred pulls of non-blocking device-buffer preads that no gsys_wait_token() consumed (reading
+ * B15: one flush kernel copies them all).  Returns 0, or the first -errno recorded for a
+ * non-blocking call since the previous gsys_wait (reading A4), which it then clears. */
 int gsys_wait(void* stream);
 
 /* gsys_wait(NULL), stop the service threads, free everything.  Idempotent: 0 if not initialised. */
@@ -231,6 +236,9 @@ typedef struct gsys_stats {
     uint32_t slots;           /* syscall-area slots                              */
     uint32_t coalesce_max;
     uint32_t coalesce_window_us;
+    uint64_t split;           /* preads served in pieces by several workers (B14) */
+    uint64_t deferred;        /* non-blocking preads served as deferred pulls (B15) */
+    uint64_t flushed;         /* ... of which landed by gsys_wait's flush kernel   */
 } gsys_stats_t;
 
 int gsys_stats(gsys_stats_t* out);

@@ -55,6 +55,18 @@ struct gsys_wd_log {
     struct { unsigned slot, seq, nr, phase; } rec[GSYS_WD_RECS];
 };
 
+/* Deferred pull of a non-blocking pread into device memory (reading B15): the service reads into
+ * a host-mapped range and records it here, at the request's doorbell-ring position; whoever needs
+ * the bytes -- a gsys_wait_token() on the request, or gsys_wait()'s flush kernel -- copies them to
+ * dst and sets `consumed`, which recycles the range.  tag = position + 1 once written. */
+struct gsys_nbrec {
+    unsigned long long src;   /* device address of the host-mapped range, 0: nothing to copy */
+    unsigned long long dst;
+    long long ret;            /* pread result: bytes to copy when > 0                        */
+    unsigned tag;
+    unsigned consumed;        /* written 1 by the copier (GPU or flush kernel)                */
+};
+
 /* Instance context in device memory (built by gsys_init). */
 struct gsys_dev_ctx {
     gsys_slot* area;                /* host-mapped [nslots] syscall area                    */
@@ -91,13 +103,17 @@ struct gsys_dev_ctx {
     unsigned long long poll_timeout_ns;  /* watchdog: a claim or completion wait longer than this
                                        returns -ETIMEDOUT (0 = wait forever)                      */
     gsys_wd_log* wd;                /* device: watchdog log                                       */
+    gsys_nbrec* nbrec;              /* host-mapped [ring_mask+1]: deferred-pull records (B15)     */
 };
 
-/* Explicit completion token of a non-blocking call (slot, seq): gsys_wait_token() waits for that
- * request whatever slot the caller's next call lands in (%smid / %warpid are volatile). */
+/* Explicit completion token of a non-blocking call (slot, seq, ring position): gsys_wait_token()
+ * waits for that request whatever slot the caller's next call lands in (%smid / %warpid are
+ * volatile), and finishes its deferred pull if it has one. */
 struct gsys_token {
     unsigned slot;
     unsigned seq;    /* 0: no request outstanding */
+    unsigned pos;    /* the request's doorbell-ring position: names its deferred-pull record */
+    unsigned pad_;
 };
 
 #ifdef __CUDACC__
@@ -276,7 +292,7 @@ __device__ __forceinline__ unsigned marshal(const gsys_dev_ctx* c, unsigned s, u
  * taken with one warp-aggregated atomicAdd for all lanes of the warp calling together (the
  * "scalar wavefront instruction" of P24.14).  Entry = (position+1) << 32 | slot, so the host
  * recognises a fresh entry without the ring ever being cleared. */
-__device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
+__device__ __forceinline__ unsigned doorbell(const gsys_dev_ctx* c, unsigned s) {
 #if defined(GSYS_DOORBELL_SC)
     __threadfence_system();
 #else
@@ -290,6 +306,7 @@ __device__ __forceinline__ void doorbell(const gsys_dev_ctx* c, unsigned s) {
     base = __shfl_sync(mask, base, leader);
     unsigned pos = base + (unsigned)__popc(mask & lanemask_lt());
     st_relaxed_sys(c->ring + (pos & c->ring_mask), ((unsigned long long)(pos + 1u) << 32) | s);
+    return pos;
 }
 
 /* ------------------------------------------------------------------ a5: completion
@@ -440,6 +457,21 @@ __device__ __forceinline__ void pull_copy(const unsigned char* src, unsigned cha
     }
 }
 
+/* One thread copies r bytes of a host-mapped area (16-byte aligned) to dst: eight 16-byte loads in
+ * flight per round trip over PCIe. */
+__device__ __forceinline__ void pull_copy_thread(const unsigned char* src, unsigned char* dst, long long r) {
+    const unsigned n16 = (unsigned)((r + 15) >> 4);
+    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    for (unsigned i = 0; i < n16; i += 8u) {
+        uint4 v[8];
+#pragma unroll
+        for (unsigned k = 0; k < 8u; k++) v[k] = i + k < n16 ? ld_v4_after_acquire(s4 + i + k) : make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+        for (unsigned k = 0; k < 8u; k++)
+            if (i + k < n16) store16(dst + 16u * (i + k), v[k], r - 16ll * (i + k));
+    }
+}
+
 /* A pull the caller's scope finishes (work-group cooperative copy): filled by call_thread. */
 struct PullOut {
     const unsigned char* src = nullptr;
@@ -465,10 +497,15 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     }
     const unsigned long long d1 = c->diag ? globaltimer() : 0ull;
     const unsigned char* psrc = nullptr;
+    // non-blocking pread into device memory: served into a host-mapped range and pulled later (B15)
+    if (nr == GSYS_NR_PREAD64 && !blocking && !(flags & GSYS_HOSTBUF) && c->nbrec != nullptr && a[2] > 0ull)
+        flags |= GSYS_F_DEFER;
     if (nr == GSYS_NR_PREAD64 && blocking && !(flags & GSYS_HOSTBUF)) {
         psrc = pull_src(c, s, a[2], po != nullptr);
         if (psrc) flags |= GSYS_F_PULL;
-        else if (po != nullptr && c->pull_bounce && a[2] > 0ull) flags |= GSYS_F_PULLB;
+        // bounce pull (B13): a work-group copies cooperatively; a lone caller (work-item, kernel
+        // scope) copies itself, which pays only up to 64 KiB (larger reads keep the DMA path)
+        else if (c->pull_bounce && a[2] > 0ull && (po != nullptr || a[2] <= (64ull << 10))) flags |= GSYS_F_PULLB;
     }
     if (io.in != nullptr) {   /* input payload into the inline line; published by marshal's fence */
         uint4* dst = reinterpret_cast<uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
@@ -482,10 +519,10 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         flags |= GSYS_F_INLINE_IN;
     }
     unsigned seq = marshal(c, s, nr, flags, a);
-    doorbell(c, s);
+    const unsigned pos = doorbell(c, s);
     if (!blocking) {
         c->nbpend[s] = seq;
-        if (tok) { tok->slot = s; tok->seq = seq; }
+        if (tok) { tok->slot = s; tok->seq = seq; tok->pos = pos; }
         st_release_gpu(&c->claim[s], 0u);
         return 0;
     }
@@ -503,10 +540,17 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
         atomicAdd(c->diag + 4, 1ull);
         atomicAdd(c->diag + 7, (unsigned long long)-(long long)d3);   /* + end time below */
     }
-    if (flags & GSYS_F_PULLB) {   /* the work-group copies from the worker's bounce, then releases */
+    if (flags & GSYS_F_PULLB) {   /* copy from the worker's bounce (the work-group, or this thread), then release */
         const uint4 a01 = ld_v4_after_acquire(reinterpret_cast<const uint4*>(c->area + s));   /* args[1] = source */
-        po->src = r > 0 ? reinterpret_cast<const unsigned char*>((uintptr_t)a01.z | ((uintptr_t)a01.w << 32)) : nullptr;
-        po->slot = s; po->seq = seq; po->nr = nr; po->bounce = true;
+        const unsigned char* src =
+            r > 0 ? reinterpret_cast<const unsigned char*>((uintptr_t)a01.z | ((uintptr_t)a01.w << 32)) : nullptr;
+        if (po != nullptr) {
+            po->src = src; po->slot = s; po->seq = seq; po->nr = nr; po->bounce = true;
+            if (c->diag) atomicAdd(c->diag + 7, globaltimer());
+            return r;
+        }
+        if (src != nullptr) pull_copy_thread(src, reinterpret_cast<unsigned char*>(a[1]), r);
+        release(c, s, seq, nr, true);
         if (c->diag) atomicAdd(c->diag + 7, globaltimer());
         return r;
     }
@@ -685,19 +729,49 @@ __device__ __forceinline__ long long invoke(const gsys_dev_ctx* c, unsigned nr, 
 /* Wait for the non-blocking request of `tok` (one thread's token) to complete: returns its result
  * if the slot's completion word still carries it, 0 if a later request on the slot completed
  * since (completions on a slot are in order, A15: ours is done, its result was overwritten --
- * errors still reach gsys_wait, reading A4), -ETIMEDOUT from the watchdog. */
-__device__ __forceinline__ long long wait_token_thread(const gsys_dev_ctx* c, const gsys_token& tok) {
+ * errors still reach gsys_wait, reading A4), -ETIMEDOUT from the watchdog.  *rec receives the
+ * request's deferred-pull record when it has bytes still to copy (B15), else nullptr. */
+__device__ __forceinline__ long long wait_token_thread(const gsys_dev_ctx* c, const gsys_token& tok,
+                                                       const gsys_nbrec** rec = nullptr) {
+    if (rec) *rec = nullptr;
     if (tok.seq == 0u) return 0;
     const unsigned long long* m = c->hdone + tok.slot;
     unsigned long long t0 = 0ull;
+    long long r = 0;
     for (;;) {
         const unsigned long long v = ld_acquire_sys(m);
         const unsigned got = (unsigned)(v >> 32);
-        if (got == tok.seq) return (long long)(int)(unsigned)(v & 0xffffffffull);
-        if ((int)(got - tok.seq) > 0) return 0;
+        if (got == tok.seq) { r = (long long)(int)(unsigned)(v & 0xffffffffull); break; }
+        if ((int)(got - tok.seq) > 0) break;
         __nanosleep(c->poll_ns_host);
         if (expired(c, t0)) { wd_log(c, tok.slot, tok.seq, 0u, GSYS_WD_TOKEN); return -ETIMEDOUT; }
     }
+    if (rec && c->nbrec) {
+        // the record is written before the completion word (acquired above)
+        const gsys_nbrec* q = c->nbrec + (tok.pos & c->ring_mask);
+        const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);   /* {ret, tag, consumed} */
+        const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));       /* {src, dst}           */
+        if (t.z == tok.pos + 1u && t.w == 0u && (h.x | h.y) != 0u && (long long)((unsigned long long)t.x |
+                                                                                 ((unsigned long long)t.y << 32)) > 0)
+            *rec = q;
+    }
+    return r;
+}
+
+/* Copy a deferred pull (threads tid = 0..nt-1 of the caller's scope), then mark it consumed. */
+__device__ __forceinline__ void finish_deferred(const gsys_nbrec* q, unsigned tid, unsigned nt) {
+    const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
+    const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);
+    const unsigned char* src = reinterpret_cast<const unsigned char*>((unsigned long long)h.x |
+                                                                      ((unsigned long long)h.y << 32));
+    unsigned char* dst = reinterpret_cast<unsigned char*>((unsigned long long)h.z | ((unsigned long long)h.w << 32));
+    const long long r = (long long)((unsigned long long)t.x | ((unsigned long long)t.y << 32));
+    if (nt == 1u) pull_copy_thread(src, dst, r);
+    else pull_copy(src, dst, r, tid, nt);
+}
+__device__ __forceinline__ void mark_consumed(const gsys_nbrec* q) {
+    unsigned* cons = const_cast<unsigned*>(&q->consumed);
+    asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(cons), "r"(1u) : "memory");
 }
 
 }  // namespace gsys
@@ -721,13 +795,25 @@ __device__ __forceinline__ long long gsys_pread(const gsys_dev_ctx* c, int fd, v
  * GSYS_KERNEL: -EINVAL (the token lives in one block). */
 __device__ __forceinline__ long long gsys_wait_token(const gsys_dev_ctx* c, const gsys_token* tok, unsigned gflags) {
     const unsigned g = gflags & GSYS_GRAN_MASK;
-    if (g == GSYS_WI) return gsys::wait_token_thread(c, *tok);
+    if (g == GSYS_WI) {
+        const gsys_nbrec* q = nullptr;
+        const long long r = gsys::wait_token_thread(c, *tok, &q);
+        if (q) { gsys::finish_deferred(q, 0u, 1u); gsys::mark_consumed(q); }
+        return r;
+    }
     if (g != GSYS_WG) return -EINVAL;
     __shared__ long long s_tret;
+    __shared__ const gsys_nbrec* s_trec;
     __syncthreads();
-    if (gsys::block_tid() == 0) s_tret = gsys::wait_token_thread(c, *tok);
+    if (gsys::block_tid() == 0) s_tret = gsys::wait_token_thread(c, *tok, &s_trec);
     __syncthreads();
     const long long r = s_tret;
+    const gsys_nbrec* q = s_trec;
+    if (q) {   /* the deferred pull (B15): the whole work-group copies, thread 0 marks it consumed */
+        gsys::finish_deferred(q, gsys::block_tid(), gsys::block_threads());
+        __syncthreads();
+        if (gsys::block_tid() == 0) gsys::mark_consumed(q);
+    }
     __syncthreads();
     return r;
 }

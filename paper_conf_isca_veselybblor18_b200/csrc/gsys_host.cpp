@@ -52,6 +52,7 @@
 #include <mutex>
 #include <numeric>
 #include <thread>
+#include <unordered_set>
 #include <vector>
 
 #include "gsys.h"
@@ -229,6 +230,7 @@ static int service_cpus(int dev, cpu_set_t* out) {
 
 struct Req {
     uint32_t slot, seq, nr, flags;
+    uint32_t pos;  // doorbell-ring position (names the deferred-pull record, B15)
     uint64_t a[6];
     int64_t ret;
     bool ok;
@@ -262,6 +264,40 @@ struct Split {
     std::atomic<uint32_t> next{0};   // next piece to claim
     std::atomic<uint32_t> done{0};   // pieces finished
     std::vector<int64_t> ret;
+};
+
+// Host-mapped ranges holding deferred pulls (reading B15), handed out in ring order and recycled in
+// order once their record says consumed.  alloc() never waits: when the oldest range is still
+// unconsumed the caller falls back to the copy-engine path.
+struct DeferRing {
+    uint8_t* h = nullptr;      // pinned, mapped
+    uint8_t* d = nullptr;      // its device address
+    size_t cap = 0, head = 0;
+    struct Region { size_t lo, hi; uint32_t pos; };
+    std::deque<Region> q;
+    std::mutex mu;             // q is also read by gsys_wait's flush
+    gsys_nbrec* recs = nullptr;
+    uint32_t mask = 0;
+    bool consumed(const Region& g) const {
+        const gsys_nbrec& r = recs[g.pos & mask];
+        return __atomic_load_n(&r.consumed, __ATOMIC_ACQUIRE) != 0u || __atomic_load_n(&r.tag, __ATOMIC_ACQUIRE) != g.pos + 1u;
+    }
+    // offset of n free bytes, or ~0
+    size_t alloc(size_t n, uint32_t pos) {
+        n = (n + 255) & ~(size_t)255;
+        if (n > cap) return ~(size_t)0;
+        std::lock_guard<std::mutex> g(mu);
+        while (!q.empty() && consumed(q.front())) q.pop_front();
+        size_t lo = head;
+        if (lo + n > cap) {   // wrap: the previous lap's tail must be free
+            for (const Region& r : q) if (r.lo >= head) return ~(size_t)0;
+            lo = 0;
+        }
+        for (const Region& r : q) if (r.lo < lo + n && lo < r.hi) return ~(size_t)0;
+        q.push_back(Region{lo, lo + n, pos});
+        head = lo + n;
+        return lo;
+    }
 };
 
 // ------------------------------------------------------------------ worker
@@ -306,6 +342,8 @@ struct Worker {
     };
     BounceRing<Tok, RingOps>* ring = nullptr;
     uint8_t* bounce_d = nullptr;     // device address of the (host-mapped) bounce
+    DeferRing defer;                 // deferred pulls of non-blocking preads (B15)
+    bool try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret);
     void wait_slot_free(uint32_t slot, uint32_t seq);
     void complete_early(Req& r);
     bool try_split(Req& r, int fd, uint8_t* dst, uint64_t n, int64_t off);
@@ -420,6 +458,12 @@ struct Instance {
     std::atomic<int> nsplits{0};
     uint64_t split_min = 128u << 10;      // env GSYS_SPLIT_KB (0 = never split)
     Sharded st_split;                      // preads served in pieces
+    Sharded st_deferred;                   // non-blocking preads served as deferred pulls (B15)
+    Sharded st_flushed;                    // ... of which copied by gsys_wait's flush
+    gsys_nbrec* nbrec_h = nullptr;         // pinned, mapped [ring_cap]: deferred-pull records
+    gsys_nbrec* nbrec_d = nullptr;
+    int flush_deferred(cudaStream_t st);   // copy the deferred pulls nobody has consumed yet (in order)
+    std::mutex flush_mu;
     bool run_piece(Split& sp, uint32_t i);
     bool help_split();
     gsys_wd_log* wd_d = nullptr;           // device watchdog log (gsys_device.cuh)
@@ -735,6 +779,46 @@ bool Worker::try_split(Req& r, int fd, uint8_t* dst, uint64_t n, int64_t off) {
     return true;
 }
 
+// Non-blocking pread into device memory (reading B15): read into a host-mapped range and record
+// {src, dst, ret} at the request's ring position before the completion is published; the bytes
+// reach dst when a token wait or gsys_wait's flush copies them.  false: not deferred (host
+// destination, or no free range), serve it the usual way.
+bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
+    if (!defer.h) return false;
+    uintptr_t dst = (uintptr_t)r.a[1];
+    uint8_t* hp = nullptr;
+    if (resolve(dst, n, &hp) != PK_DEVICE) return false;
+    const uint64_t want = std::min<uint64_t>(std::min<uint64_t>(n, GSYS_PREAD_CAP), defer.cap);
+    size_t o = defer.alloc(want, r.pos);
+    if (o == ~(size_t)0) {
+        // full of pulls nobody has consumed yet: give token waiters a moment, then land every pending
+        // pull in request order with one flush kernel (a CUDA launch from the service: only on
+        // overflow) -- never a copy-engine fallback, which could land this request before an older
+        // deferred one into the same buffer
+        const uint64_t t0 = now_ns();
+        while ((o = defer.alloc(want, r.pos)) == ~(size_t)0 && now_ns() - t0 < 200000ull) _mm_pause();
+        if (o == ~(size_t)0) {
+            Timer tm(t_cuda);
+            inst->flush_deferred(stream);
+            o = defer.alloc(want, r.pos);
+        }
+        if (o == ~(size_t)0) return false;   // larger than the whole range store
+    }
+    ssize_t z;
+    { Timer tm(t_sys); z = pread(fd, defer.h + o, want, off); }
+    inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
+    *ret = z < 0 ? -(int64_t)errno : (int64_t)z;
+    if (z > 0) inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
+    gsys_nbrec& rec = inst->nbrec_h[r.pos & (inst->ring_cap - 1)];
+    __atomic_store_n(&rec.src, z > 0 ? (uint64_t)(uintptr_t)(defer.d + o) : 0ull, __ATOMIC_RELAXED);
+    __atomic_store_n(&rec.dst, (uint64_t)dst, __ATOMIC_RELAXED);
+    __atomic_store_n(&rec.ret, (long long)*ret, __ATOMIC_RELAXED);
+    __atomic_store_n(&rec.consumed, 0u, __ATOMIC_RELAXED);
+    __atomic_store_n(&rec.tag, r.pos + 1u, __ATOMIC_RELEASE);   // published with the completion word after it
+    inst->st_deferred.fetch_add(1, std::memory_order_relaxed);
+    return true;
+}
+
 // pread(fd, buf, n, off): host-mapped buf -> read in place; device buf -> read into the pinned
 // bounce and DMA.  A request larger than the bounce is served piecewise with the POSIX result of
 // one call (stop at a short piece, cap at GSYS_PREAD_CAP, reading A11).
@@ -770,6 +854,10 @@ int64_t Worker::do_pread(Req& r) {
         if (z > 0) inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
         complete_early(r);
         return r.ret;
+    }
+    if ((r.flags & GSYS_F_DEFER) && !r.dropped) {
+        int64_t dret = 0;
+        if (try_defer(r, fd, n, off, &dret)) return dret;
     }
     if (r.flags & GSYS_F_PULL) {   // into the slot's pull area; the GPU copies it out (reading B12)
         hp = inst->pull_area(r.slot, n);
@@ -1065,6 +1153,7 @@ void Worker::process(uint64_t h0, uint32_t n) {
         uint64_t e = __atomic_load_n(&I->ring_h[(h0 + i) & mask], __ATOMIC_ACQUIRE);
         Req& r = reqs[i];
         r.slot = (uint32_t)e;
+        r.pos = (uint32_t)(h0 + i);
         // the line was written by the GPU before its doorbell entry (fence.acq_rel.sys + the entry
         // load above); plain atomic loads, since another worker may still be storing args[0] of the
         // slot's previous request (ordered only through the GPU, which the C++ model cannot see)
@@ -1392,6 +1481,12 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
         return fail(-ENOMEM);
     memset(I->ring_h, 0, (size_t)rc * 8);
     if (cudaHostGetDevicePointer((void**)&I->ring_d, I->ring_h, 0) != cudaSuccess) return fail(-EIO);
+    // deferred-pull records, one per ring position (B15)
+    if (cudaHostAlloc((void**)&I->nbrec_h, (size_t)rc * sizeof(gsys_nbrec), cudaHostAllocMapped | cudaHostAllocPortable) !=
+        cudaSuccess)
+        return fail(-ENOMEM);
+    memset(I->nbrec_h, 0, (size_t)rc * sizeof(gsys_nbrec));
+    if (cudaHostGetDevicePointer((void**)&I->nbrec_d, I->nbrec_h, 0) != cudaSuccess) return fail(-EIO);
     if (cudaHostAlloc((void**)&I->hdone_h, (size_t)slots * 8, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
         return fail(-ENOMEM);
     memset(I->hdone_h, 0, (size_t)slots * 8);
@@ -1470,6 +1565,9 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     if (cudaMalloc((void**)&I->wd_d, sizeof(gsys_wd_log)) != cudaSuccess) return fail(-ENOMEM);
     cudaMemset(I->wd_d, 0, sizeof(gsys_wd_log));
     c.wd = I->wd_d;
+    ev = getenv("GSYS_DEFER_MB");   // per worker; 0 = non-blocking device-buffer preads by DMA
+    const size_t defer_mb = ev ? (size_t)atoll(ev) : 16;
+    c.nbrec = defer_mb ? (gsys_nbrec*)I->nbrec_d : nullptr;
     c.pull_big_bytes = I->pull_bytes;
     c.pull_big = I->pull_d;
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);
@@ -1506,6 +1604,17 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
             return fail(-ENOMEM);
         }
         if (cudaHostGetDevicePointer((void**)&w->bounce_d, w->bounce, 0) != cudaSuccess) { delete w; return fail(-EIO); }
+        if (defer_mb) {
+            w->defer.cap = defer_mb << 20;
+            if (cudaHostAlloc((void**)&w->defer.h, w->defer.cap, cudaHostAllocMapped | cudaHostAllocPortable) !=
+                    cudaSuccess ||
+                cudaHostGetDevicePointer((void**)&w->defer.d, w->defer.h, 0) != cudaSuccess) {
+                delete w;
+                return fail(-ENOMEM);
+            }
+            w->defer.recs = I->nbrec_h;
+            w->defer.mask = rc - 1;
+        }
         w->bcap = bcap;
         w->ring = new BounceRing<Worker::Tok, Worker::RingOps>(bcap, &w->ring_ops);
         w->reqs.reserve(4096);
@@ -1732,6 +1841,66 @@ int gsys_launch_cu(void* cu_function, uint32_t gx, uint32_t gy, uint32_t gz, uin
     return -EIO;
 }
 
+}  // extern "C"
+namespace {
+struct FlushRec { unsigned long long src, dst; long long ret; const unsigned* consumed; };
+// gsys_wait's flush of deferred pulls (B15): block b copies record b (the request's bytes from the
+// host-mapped range to its device destination) and marks it consumed.
+__global__ void flush_kernel(const FlushRec* list, unsigned n) {
+    for (unsigned b = blockIdx.x; b < n; b += gridDim.x) {
+        const FlushRec f = list[b];
+        gsys::pull_copy(reinterpret_cast<const unsigned char*>(f.src), reinterpret_cast<unsigned char*>(f.dst), f.ret,
+                        threadIdx.x, blockDim.x);
+        __syncthreads();
+        if (threadIdx.x == 0)
+            asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(f.consumed), "r"(1u) : "memory");
+    }
+}
+}  // namespace
+
+int Instance::flush_deferred(cudaStream_t st) {
+    std::lock_guard<std::mutex> fg(flush_mu);
+    std::vector<std::pair<uint32_t, FlushRec>> all;   // (ring position, record)
+    for (Worker* w : workers) {
+        if (!w->defer.h) continue;
+        std::lock_guard<std::mutex> g(w->defer.mu);
+        for (const DeferRing::Region& rg : w->defer.q) {
+            gsys_nbrec& r = nbrec_h[rg.pos & (ring_cap - 1)];
+            if (w->defer.consumed(rg) || !r.src || r.ret <= 0) continue;
+            all.push_back({rg.pos, FlushRec{r.src, r.dst, r.ret, &nbrec_d[rg.pos & (ring_cap - 1)].consumed}});
+        }
+    }
+    if (all.empty()) return 0;
+    // in request order; reads into the same destination go in separate passes, so the last one
+    // issued is the one that stays (one caller's back-to-back reads into one buffer)
+    std::sort(all.begin(), all.end(), [](const auto& a, const auto& b) { return (int32_t)(a.first - b.first) < 0; });
+    FlushRec* lh = nullptr;
+    FlushRec* ld = nullptr;
+    if (cudaHostAlloc((void**)&lh, all.size() * sizeof(FlushRec), cudaHostAllocMapped) != cudaSuccess) return -ENOMEM;
+    cudaHostGetDevicePointer((void**)&ld, lh, 0);
+    size_t n = 0, start = 0;
+    std::unordered_set<unsigned long long> dsts;
+    auto launch = [&]() {
+        if (n == start) return;
+        const unsigned cnt = (unsigned)(n - start);
+        flush_kernel<<<std::min<unsigned>(cnt, 4096), 256, 0, st>>>(ld + start, cnt);
+        start = n;
+        dsts.clear();
+    };
+    for (const auto& pr : all) {
+        if (dsts.count(pr.second.dst)) launch();
+        dsts.insert(pr.second.dst);
+        lh[n++] = pr.second;
+    }
+    launch();
+    cudaError_t e = cudaStreamSynchronize(st);
+    cudaFreeHost(lh);
+    st_flushed.fetch_add(all.size(), std::memory_order_relaxed);
+    return e == cudaSuccess ? 0 : -EIO;
+}
+
+extern "C" {
+
 int gsys_wait(void* stream) {
     Instance* I = current();
     if (!I) return -ENODEV;
@@ -1755,6 +1924,13 @@ int gsys_wait(void* stream) {
         std::this_thread::yield();
     }
     for (Worker* w : I->workers) cudaStreamSynchronize(w->stream);
+    // deferred pulls nobody waited for on the GPU land now (B15) -- at a device-wide wait only:
+    // then no kernel can be copying a record or reusing its destination concurrently
+    int ferr = (drained && !stream) ? I->flush_deferred(I->ctl) : 0;
+    if (ferr) {
+        int z = 0;
+        I->first_err.compare_exchange_strong(z, ferr);
+    }
     if (wd.count) {
         // slots whose waits expired were left claimed (the host might still complete into them);
         // once the service is drained they are returned to free -- every slot after a
@@ -1929,6 +2105,7 @@ int gsys_shutdown(void) {
         for (auto e : w->evpool) cudaEventDestroy(e);
         cudaStreamDestroy(w->stream);
         cudaFreeHost(w->bounce);
+        if (w->defer.h) cudaFreeHost(w->defer.h);
         delete w;
     }
     cudaFreeHost(I->area_h);
@@ -1936,6 +2113,7 @@ int gsys_shutdown(void) {
     if (I->pull_h) cudaFreeHost(I->pull_h);
     cudaFreeHost(I->ring_h);
     cudaFreeHost(I->hdone_h);
+    cudaFreeHost(I->nbrec_h);
     cudaFree(I->claim_d);
     cudaFree(I->seqs_d);
     cudaFree(I->mirror_d);
@@ -1983,6 +2161,9 @@ int gsys_stats(gsys_stats_t* out) {
     out->slots = I->nslots;
     out->coalesce_max = I->coalesce_max.load();
     out->coalesce_window_us = I->window_us.load();
+    out->split = I->st_split.load();
+    out->deferred = I->st_deferred.load();
+    out->flushed = I->st_flushed.load();
     return 0;
 }
 
@@ -2000,6 +2181,9 @@ int gsys_stats_reset(void) {
     I->st_bytes_read.store(0);
     I->st_bytes_h2d.store(0);
     I->st_errors.store(0);
+    I->st_split.store(0);
+    I->st_deferred.store(0);
+    I->st_flushed.store(0);
     for (auto& a : I->st_nr) a.store(0);
     return 0;
 }

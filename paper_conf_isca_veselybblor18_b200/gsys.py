@@ -35,7 +35,8 @@ class Stats(ctypes.Structure):
                 ("per_nr", ctypes.c_uint64 * 8), ("ns_busy", ctypes.c_uint64), ("ns_syscall", ctypes.c_uint64),
                 ("ns_cuda", ctypes.c_uint64), ("ns_bounce_wait", ctypes.c_uint64),
                 ("threads", ctypes.c_uint32), ("slots", ctypes.c_uint32),
-                ("coalesce_max", ctypes.c_uint32), ("coalesce_window_us", ctypes.c_uint32)]
+                ("coalesce_max", ctypes.c_uint32), ("coalesce_window_us", ctypes.c_uint32),
+                ("split", ctypes.c_uint64), ("deferred", ctypes.c_uint64), ("flushed", ctypes.c_uint64)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_ if k != "per_nr"}

@@ -717,3 +717,63 @@ def test_kernel_call_sites(file1m):
     assert rc == 0 and ret.tolist() == [0, 0, 0]
     _, ret, _, _, rc = W.bench_calls("getrusage", G.KERNEL | G.BLOCKING | G.RELAXED | G.SITE(9), 4, 64, 2)
     assert ret.tolist() == [-errno.EINVAL] * 2
+
+
+# ---------------------------------------------------------------------------- deferred pulls (B15)
+def test_nonblocking_device_preads_are_deferred_and_land(file1m):
+    """Non-blocking WG and WI preads into device memory are served as deferred pulls (no
+    copy-engine transfer per request) and land by the device-wide gsys_wait: every buffer holds the
+    bytes of the caller's last read, as with the DMA path."""
+    size = os.path.getsize(file1m)
+    data = open(file1m, "rb").read()
+    for gran, blocks, threads in ((G.WG, 32, 128), (G.WI, 2, 64)):
+        iters, length = 3, 4096
+        callers = blocks if gran == G.WG else blocks * threads
+        d_buf = torch.zeros(callers * length, dtype=torch.uint8, device="cuda")
+        fd = os.open(file1m, os.O_RDONLY)
+        G.gsys_stats_reset()
+        try:
+            _, ret, _, _, rc = W.bench_calls("pread", gran | G.NONBLOCKING, blocks, threads, iters, fd, length, size,
+                                             d_buf)
+        finally:
+            os.close(fd)
+        st = G.gsys_stats()
+        assert rc == 0 and ret.tolist() == [0] * (callers * iters)
+        assert st["deferred"] == callers * iters and st["flushed"] == callers * iters, st
+        host = d_buf.cpu().numpy()
+        for c in range(callers):
+            off = ((c * iters + iters - 1) * length) % size
+            want = data[off: off + length]
+            assert bytes(host[c * length: c * length + len(want)]) == want, c
+
+
+def test_deferred_pull_ring_overflow_flushes(tmpdir_shm, file1m):
+    """With a 1 MiB deferred range store per worker, 64 KiB non-blocking preads overflow it: the
+    service lands the pending pulls in request order (one flush kernel) and goes on deferring;
+    every buffer still ends with the caller's last read (a fresh process: the size is fixed at init)."""
+    import subprocess
+    import sys
+    code = f"""
+import os, sys, numpy as np, torch
+sys.path.insert(0, {repr(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))})
+from paper_conf_isca_veselybblor18_b200 import gsys as G, workloads as W
+W.ensure_init()
+p = {file1m!r}
+size = os.path.getsize(p); data = open(p, 'rb').read()
+blocks, iters, length = 64, 2, 65536
+d = torch.zeros(blocks * length, dtype=torch.uint8, device='cuda')
+fd = os.open(p, os.O_RDONLY)
+_, ret, _, _, rc = W.bench_calls('pread', G.WG | G.NONBLOCKING, blocks, 64, iters, fd, length, size, d)
+os.close(fd)
+st = G.gsys_stats()
+h = d.cpu().numpy()
+for c in range(blocks):
+    off = ((c * iters + iters - 1) * length) % size
+    want = data[off: off + length]
+    assert bytes(h[c * length: c * length + len(want)]) == want, c
+assert rc == 0 and st['deferred'] == blocks * iters and st['flushed'] > 0, st
+print('ok', st['deferred'], st['flushed'])
+"""
+    env = dict(os.environ, GSYS_DEFER_MB="1", GSYS_THREADS="4")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-3000:]

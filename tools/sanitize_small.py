@@ -33,4 +33,33 @@ print("scan", int(h.sum()))
 for fl in (G.WI | G.BLOCKING, G.WG | G.NONBLOCKING | G.RELAXED, G.KERNEL | G.BLOCKING | G.RELAXED):
     n, ret, lat, _, rc = W.bench_calls("getrusage", fl, 4, 64, 2)
     print("calls", fl, rc, int((ret == 0).sum()))
+# round 2: pull completion from the bounce (default; large chunks), non-blocking prefetch waiting on
+# explicit tokens, token-level scan, split large preads, both completion modes of device staging
+for ck in (256 << 10, 64 << 10):
+    r = W.wordcount_files([p], words, pats, chunk=ck, staging=G.STAGE_DEVICE, blocks=4)
+    print("wc-pullb", ck, int(r.hist.sum()), r.wait_rc)
+    r = W.wordcount_files([p], words, pats, chunk=ck, staging=G.STAGE_DEVICE, blocks=4,
+                          gflags=G.WG | G.NONBLOCKING | G.RELAXED)
+    print("wc-prefetch", ck, int(r.hist.sum()), r.wait_rc)
+prev = G.gsys_set_scan(G.SCAN_TOKEN)
+r = W.wordcount_files([p], words, pats, chunk=64 << 10, staging=G.STAGE_DEVICE, blocks=4)
+print("wc-token", int(r.hist.sum()), r.wait_rc)
+h.zero_()
+G.gsys_scan_device(t, buf.size, 4096, words, pats, h, None, 8, 512)
+torch.cuda.synchronize()
+print("scan-token", int(h.sum()))
+G.gsys_set_scan(prev)
+G.gsys_set_completion(G.COMPLETION_MEMOP)
+r = W.wordcount_files([p], words, pats, chunk=64 << 10, staging=G.STAGE_DEVICE, blocks=4)
+print("wc-memop", int(r.hist.sum()), r.wait_rc)
+G.gsys_set_completion(G.COMPLETION_PULL)
+fd = os.open(p, os.O_RDONLY)
+big = torch.zeros((1 << 20) + 64, dtype=torch.uint8, device="cuda")
+n, ret, lat, sm, rc = W.bench_calls("pread", G.WG | G.BLOCKING, 1, 128, 1, fd, 1 << 20, (1 << 20) + 77, big, want_sum=True)
+print("split", rc, int(ret[0]))
+# deferred pulls (B15): non-blocking device-buffer preads landed by gsys_wait's flush kernel
+small = torch.zeros(8 * 4096, dtype=torch.uint8, device="cuda")
+n, ret, lat, sm, rc = W.bench_calls("pread", G.WG | G.NONBLOCKING, 8, 64, 2, fd, 4096, (1 << 20) + 77, small)
+print("deferred", rc, G.gsys_stats()["deferred"])
+os.close(fd)
 print("ok")
