@@ -59,6 +59,8 @@
 #include "gsys_device.cuh"
 #include "gsys_internal.h"
 
+int preload_flush_kernel();   // below, next to the flush kernel
+
 namespace {
 
 typedef CUresult (*PFN_batch_t)(CUstream, unsigned int, CUstreamBatchMemOpParams*, unsigned int);
@@ -464,6 +466,9 @@ struct Instance {
     gsys_nbrec* nbrec_d = nullptr;
     int flush_deferred(cudaStream_t st);   // copy the deferred pulls nobody has consumed yet (in order)
     std::mutex flush_mu;
+    void* flush_buf = nullptr;             // pinned, mapped: the flush kernel's record list
+    size_t flush_cap = 0;
+    std::vector<void*> flush_old;
     bool run_piece(Split& sp, uint32_t i);
     bool help_split();
     gsys_wd_log* wd_d = nullptr;           // device watchdog log (gsys_device.cuh)
@@ -813,7 +818,7 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
     __atomic_store_n(&rec.src, z > 0 ? (uint64_t)(uintptr_t)(defer.d + o) : 0ull, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.dst, (uint64_t)dst, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.ret, (long long)*ret, __ATOMIC_RELAXED);
-    __atomic_store_n(&rec.consumed, 0u, __ATOMIC_RELAXED);
+    __atomic_store_n(&rec.consumed, z > 0 ? 0u : 1u, __ATOMIC_RELAXED);   // nothing to copy: free at once
     __atomic_store_n(&rec.tag, r.pos + 1u, __ATOMIC_RELEASE);   // published with the completion word after it
     inst->st_deferred.fetch_add(1, std::memory_order_relaxed);
     return true;
@@ -1232,7 +1237,9 @@ void Worker::process(uint64_t h0, uint32_t n) {
             bool okd = true;
             for (uint32_t j : mem) {
                 Req& r = reqs[midx[j]];
-                if (r.flags & GSYS_F_PULLB) { okd = false; break; }   // read alone into the bounce (B13)
+                // read alone into the bounce (B13) / a deferred range (B15): a merged read would land
+                // by DMA, out of order with the deferred pulls
+                if (r.flags & (GSYS_F_PULLB | GSYS_F_DEFER)) { okd = false; break; }
                 PtrKind k = !r.a[2] ? PK_INVALID
                             : (r.flags & GSYS_F_PULL) ? (I->pull_area(r.slot, r.a[2]) ? PK_HOST : PK_INVALID)
                                                       : resolve((uintptr_t)r.a[1], r.a[2], nullptr);
@@ -1571,6 +1578,7 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.pull_big_bytes = I->pull_bytes;
     c.pull_big = I->pull_d;
     if (cudaMemcpy(I->ctx_d, &c, sizeof c, cudaMemcpyHostToDevice) != cudaSuccess) return fail(-EIO);
+    if (preload_flush_kernel() != 0) return fail(-EIO);
     if (cudaDeviceSynchronize() != cudaSuccess) return fail(-EIO);
 
     // service threads: on the CPUs local to this GPU's PCIe root, sized for the
@@ -1858,6 +1866,14 @@ __global__ void flush_kernel(const FlushRec* list, unsigned n) {
 }
 }  // namespace
 
+// The flush kernel is launched by service threads while an application kernel may be waiting on
+// the service: with lazy module loading its first launch would wait for the running kernels, so
+// gsys_init loads it up front.
+int preload_flush_kernel() {
+    cudaFuncAttributes fa;
+    return cudaFuncGetAttributes(&fa, (const void*)flush_kernel) == cudaSuccess ? 0 : -EIO;
+}
+
 int Instance::flush_deferred(cudaStream_t st) {
     std::lock_guard<std::mutex> fg(flush_mu);
     std::vector<std::pair<uint32_t, FlushRec>> all;   // (ring position, record)
@@ -1874,9 +1890,19 @@ int Instance::flush_deferred(cudaStream_t st) {
     // in request order; reads into the same destination go in separate passes, so the last one
     // issued is the one that stays (one caller's back-to-back reads into one buffer)
     std::sort(all.begin(), all.end(), [](const auto& a, const auto& b) { return (int32_t)(a.first - b.first) < 0; });
-    FlushRec* lh = nullptr;
+    // the record list lives in a grow-only pinned buffer: freeing pinned memory synchronises the
+    // device, which must not happen here while a kernel may be waiting on this service
+    if (flush_cap < all.size()) {
+        size_t cap = std::max<size_t>(4096, flush_cap * 2);
+        while (cap < all.size()) cap *= 2;
+        void* nb = nullptr;
+        if (cudaHostAlloc(&nb, cap * sizeof(FlushRec), cudaHostAllocMapped) != cudaSuccess) return -ENOMEM;
+        if (flush_buf) flush_old.push_back(flush_buf);   // freed at shutdown
+        flush_buf = nb;
+        flush_cap = cap;
+    }
+    FlushRec* lh = (FlushRec*)flush_buf;
     FlushRec* ld = nullptr;
-    if (cudaHostAlloc((void**)&lh, all.size() * sizeof(FlushRec), cudaHostAllocMapped) != cudaSuccess) return -ENOMEM;
     cudaHostGetDevicePointer((void**)&ld, lh, 0);
     size_t n = 0, start = 0;
     std::unordered_set<unsigned long long> dsts;
@@ -1894,7 +1920,6 @@ int Instance::flush_deferred(cudaStream_t st) {
     }
     launch();
     cudaError_t e = cudaStreamSynchronize(st);
-    cudaFreeHost(lh);
     st_flushed.fetch_add(all.size(), std::memory_order_relaxed);
     return e == cudaSuccess ? 0 : -EIO;
 }
@@ -2114,6 +2139,8 @@ int gsys_shutdown(void) {
     cudaFreeHost(I->ring_h);
     cudaFreeHost(I->hdone_h);
     cudaFreeHost(I->nbrec_h);
+    if (I->flush_buf) cudaFreeHost(I->flush_buf);
+    for (void* p : I->flush_old) cudaFreeHost(p);
     cudaFree(I->claim_d);
     cudaFree(I->seqs_d);
     cudaFree(I->mirror_d);

@@ -770,7 +770,9 @@ h = d.cpu().numpy()
 for c in range(blocks):
     off = ((c * iters + iters - 1) * length) % size
     want = data[off: off + length]
-    assert bytes(h[c * length: c * length + len(want)]) == want, c
+    got = bytes(h[c * length: c * length + len(want)])
+    which = [r for r in range(iters) if got == data[((c * iters + r) * length) % size:][:len(want)]]
+    assert got == want, (c, which, st)
 assert rc == 0 and st['deferred'] == blocks * iters and st['flushed'] > 0, st
 print('ok', st['deferred'], st['flushed'])
 """
