@@ -104,6 +104,7 @@ struct gsys_dev_ctx {
                                        returns -ETIMEDOUT (0 = wait forever)                      */
     gsys_wd_log* wd;                /* device: watchdog log                                       */
     gsys_nbrec* nbrec;              /* host-mapped [ring_mask+1]: deferred-pull records (B15)     */
+    unsigned* nbpos;                /* device [nslots]: ring position of the slot's last non-blocking request */
 };
 
 /* Explicit completion token of a non-blocking call (slot, seq, ring position): gsys_wait_token()
@@ -241,6 +242,44 @@ __device__ __forceinline__ unsigned hw_slot(const gsys_dev_ctx* c) {
 
 constexpr unsigned NOSLOT = 0xffffffffu;
 
+/* One thread copies r bytes of a host-mapped area (16-byte aligned) to dst: eight 16-byte loads in
+ * flight per round trip over PCIe. */
+__device__ __forceinline__ void pull_copy_thread(const unsigned char* src, unsigned char* dst, long long r);
+
+/* The slot's previous non-blocking request, if it left a small (<= 16 KiB) deferred pull nobody has
+ * consumed: waits for its completion word (bounded) and returns its record, else nullptr. */
+__device__ __forceinline__ const gsys_nbrec* small_deferred_pending(const gsys_dev_ctx* c, unsigned s) {
+    const unsigned pend = c->nbpend[s];
+    if (!pend) return nullptr;
+    unsigned long long t0 = 0ull;
+    while ((unsigned)(ld_acquire_sys(c->hdone + s) >> 32) != pend) {
+        __nanosleep(c->poll_ns_host);
+        if (expired(c, t0)) return nullptr;   // claim() logs it
+    }
+    const unsigned pos = c->nbpos[s];
+    const gsys_nbrec* q = c->nbrec + (pos & c->ring_mask);
+    const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);   /* {ret, tag, consumed} */
+    const long long r = (long long)((unsigned long long)t.x | ((unsigned long long)t.y << 32));
+    if (t.z != pos + 1u || t.w != 0u || r <= 0 || r > 16384) return nullptr;
+    const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
+    return (h.x | h.y) ? q : nullptr;
+}
+
+/* The deferred pull at ring position pos, if it is still pending and small (<= 16 KiB): this thread
+ * copies it and marks it consumed (the record was written before the completion word this thread
+ * has acquired). */
+__device__ __forceinline__ void consume_small_deferred(const gsys_dev_ctx* c, unsigned pos) {
+    gsys_nbrec* q = c->nbrec + (pos & c->ring_mask);
+    const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);   /* {ret, tag, consumed} */
+    const long long r = (long long)((unsigned long long)t.x | ((unsigned long long)t.y << 32));
+    if (t.z != pos + 1u || t.w != 0u || r <= 0 || r > 16384) return;
+    const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
+    if ((h.x | h.y) == 0u) return;
+    pull_copy_thread(reinterpret_cast<const unsigned char*>((unsigned long long)h.x | ((unsigned long long)h.y << 32)),
+                     reinterpret_cast<unsigned char*>((unsigned long long)h.z | ((unsigned long long)h.w << 32)), r);
+    asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(&q->consumed), "r"(1u) : "memory");
+}
+
 __device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, unsigned nr) {
     unsigned s = hw_slot(c);
     unsigned ns = 32;
@@ -264,6 +303,9 @@ __device__ __forceinline__ unsigned claim(const gsys_dev_ctx* c, unsigned nr) {
         }
         fence_acq_rel_sys();
         c->nbpend[s] = 0u;
+        // reading B15: a small deferred pull of that request nobody consumed yet lands now, before
+        // this caller's request can overtake it -- so at most one small pull per slot stays pending
+        if (c->nbrec) consume_small_deferred(c, c->nbpos[s]);
     }
     return s;
 }
@@ -472,6 +514,22 @@ __device__ __forceinline__ void pull_copy_thread(const unsigned char* src, unsig
     }
 }
 
+/* Copy a deferred pull (threads tid = 0..nt-1 of the caller's scope), then mark it consumed. */
+__device__ __forceinline__ void finish_deferred(const gsys_nbrec* q, unsigned tid, unsigned nt) {
+    const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
+    const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);
+    const unsigned char* src = reinterpret_cast<const unsigned char*>((unsigned long long)h.x |
+                                                                      ((unsigned long long)h.y << 32));
+    unsigned char* dst = reinterpret_cast<unsigned char*>((unsigned long long)h.z | ((unsigned long long)h.w << 32));
+    const long long r = (long long)((unsigned long long)t.x | ((unsigned long long)t.y << 32));
+    if (nt == 1u) pull_copy_thread(src, dst, r);
+    else pull_copy(src, dst, r, tid, nt);
+}
+__device__ __forceinline__ void mark_consumed(const gsys_nbrec* q) {
+    unsigned* cons = const_cast<unsigned*>(&q->consumed);
+    asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(cons), "r"(1u) : "memory");
+}
+
 /* A pull the caller's scope finishes (work-group cooperative copy): filled by call_thread. */
 struct PullOut {
     const unsigned char* src = nullptr;
@@ -522,6 +580,7 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     const unsigned pos = doorbell(c, s);
     if (!blocking) {
         c->nbpend[s] = seq;
+        c->nbpos[s] = pos;
         if (tok) { tok->slot = s; tok->seq = seq; tok->pos = pos; }
         st_release_gpu(&c->claim[s], 0u);
         return 0;
@@ -600,7 +659,21 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
     const bool bar1 = strong || !producer;
     const bool bar2 = strong || producer;
     const unsigned tid = block_tid();
-    if (bar1) __syncthreads();
+    if (bar1) {
+        // Bar1 doubles as the broadcast of a small deferred pull (B15) still pending on the
+        // caller's slot: the whole work-group copies it instead of the caller alone in claim()
+        __shared__ const gsys_nbrec* s_dq;
+        int pend = 0;
+        if (tid == 0 && c->nbrec) {
+            s_dq = small_deferred_pending(c, hw_slot(c));
+            pend = s_dq != nullptr;
+        }
+        if (__syncthreads_or(pend)) {
+            finish_deferred(s_dq, tid, block_threads());
+            __syncthreads();
+            if (tid == 0) mark_consumed(s_dq);
+        }
+    }
     long long r = 0;
     PullOut po;
     if (tid == 0)
@@ -756,22 +829,6 @@ __device__ __forceinline__ long long wait_token_thread(const gsys_dev_ctx* c, co
             *rec = q;
     }
     return r;
-}
-
-/* Copy a deferred pull (threads tid = 0..nt-1 of the caller's scope), then mark it consumed. */
-__device__ __forceinline__ void finish_deferred(const gsys_nbrec* q, unsigned tid, unsigned nt) {
-    const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
-    const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);
-    const unsigned char* src = reinterpret_cast<const unsigned char*>((unsigned long long)h.x |
-                                                                      ((unsigned long long)h.y << 32));
-    unsigned char* dst = reinterpret_cast<unsigned char*>((unsigned long long)h.z | ((unsigned long long)h.w << 32));
-    const long long r = (long long)((unsigned long long)t.x | ((unsigned long long)t.y << 32));
-    if (nt == 1u) pull_copy_thread(src, dst, r);
-    else pull_copy(src, dst, r, tid, nt);
-}
-__device__ __forceinline__ void mark_consumed(const gsys_nbrec* q) {
-    unsigned* cons = const_cast<unsigned*>(&q->consumed);
-    asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(cons), "r"(1u) : "memory");
 }
 
 }  // namespace gsys

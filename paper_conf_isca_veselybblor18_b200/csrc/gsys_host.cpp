@@ -52,6 +52,7 @@
 #include <mutex>
 #include <numeric>
 #include <thread>
+#include <unordered_map>
 #include <unordered_set>
 #include <vector>
 
@@ -284,18 +285,27 @@ struct DeferRing {
         const gsys_nbrec& r = recs[g.pos & mask];
         return __atomic_load_n(&r.consumed, __ATOMIC_ACQUIRE) != 0u || __atomic_load_n(&r.tag, __ATOMIC_ACQUIRE) != g.pos + 1u;
     }
-    // offset of n free bytes, or ~0
+    // offset of n free bytes, or ~0 (ring order: the free space runs from the newest region's end
+    // to the oldest outstanding region's start)
     size_t alloc(size_t n, uint32_t pos) {
         n = (n + 255) & ~(size_t)255;
         if (n > cap) return ~(size_t)0;
         std::lock_guard<std::mutex> g(mu);
         while (!q.empty() && consumed(q.front())) q.pop_front();
-        size_t lo = head;
-        if (lo + n > cap) {   // wrap: the previous lap's tail must be free
-            for (const Region& r : q) if (r.lo >= head) return ~(size_t)0;
+        size_t lo;
+        if (q.empty()) {
             lo = 0;
+        } else {
+            const size_t tail = q.front().lo;
+            if (head > tail) {           // not wrapped: [head, cap) then [0, tail)
+                if (head + n <= cap) lo = head;
+                else if (n <= tail) lo = 0;
+                else return ~(size_t)0;
+            } else {                     // wrapped: [head, tail)
+                if (head + n <= tail) lo = head;
+                else return ~(size_t)0;
+            }
         }
-        for (const Region& r : q) if (r.lo < lo + n && lo < r.hi) return ~(size_t)0;
         q.push_back(Region{lo, lo + n, pos});
         head = lo + n;
         return lo;
@@ -428,6 +438,7 @@ struct Instance {
     uint32_t* tail_d = nullptr;
     uint32_t* lat_hint_d = nullptr;
     uint32_t* nbpend_d = nullptr;
+    uint32_t* nbpos_d = nullptr;
     gsys_kround* krounds_d = nullptr;
     uint32_t* kblock_d = nullptr;
     uint32_t kblock_cap = 0;
@@ -464,7 +475,19 @@ struct Instance {
     Sharded st_flushed;                    // ... of which copied by gsys_wait's flush
     gsys_nbrec* nbrec_h = nullptr;         // pinned, mapped [ring_cap]: deferred-pull records
     gsys_nbrec* nbrec_d = nullptr;
-    int flush_deferred(cudaStream_t st);   // copy the deferred pulls nobody has consumed yet (in order)
+    // land the deferred pulls nobody has consumed yet, in request order: every one (upto_all) or
+    // those at or before ring position `upto`; by one flush kernel per pass (no kernel may be
+    // running: gsys_wait) or by copy-engine copies (from a service thread: an application kernel
+    // may fill the GPU and wait on this service, so no SM work can be relied on)
+    int flush_deferred(cudaStream_t st, bool upto_all, uint32_t upto, bool use_kernel, uint64_t only_dst = 0);
+    // destination -> ring position of the newest deferred pull into it (overflow ordering), sharded
+    // by destination so the workers do not serialise on one lock
+    struct alignas(64) DmapShard {
+        std::mutex mu;
+        std::unordered_map<uint64_t, uint32_t> m;
+    };
+    DmapShard dmap[64];
+    DmapShard& dshard(uint64_t dst) { return dmap[(dst >> 12) * 0x9E3779B97F4A7C15ull >> 58]; }
     std::mutex flush_mu;
     void* flush_buf = nullptr;             // pinned, mapped: the flush kernel's record list
     size_t flush_cap = 0;
@@ -794,20 +817,30 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
     uint8_t* hp = nullptr;
     if (resolve(dst, n, &hp) != PK_DEVICE) return false;
     const uint64_t want = std::min<uint64_t>(std::min<uint64_t>(n, GSYS_PREAD_CAP), defer.cap);
-    size_t o = defer.alloc(want, r.pos);
+    const size_t o = defer.alloc(want, r.pos);
     if (o == ~(size_t)0) {
-        // full of pulls nobody has consumed yet: give token waiters a moment, then land every pending
-        // pull in request order with one flush kernel (a CUDA launch from the service: only on
-        // overflow) -- never a copy-engine fallback, which could land this request before an older
-        // deferred one into the same buffer
-        const uint64_t t0 = now_ns();
-        while ((o = defer.alloc(want, r.pos)) == ~(size_t)0 && now_ns() - t0 < 200000ull) _mm_pause();
-        if (o == ~(size_t)0) {
-            Timer tm(t_cuda);
-            inst->flush_deferred(stream);
-            o = defer.alloc(want, r.pos);
+        // the range store is full of pulls nobody has consumed yet: this request takes the
+        // copy-engine path -- after any pending pull into the same buffer has landed (by copy
+        // engine, in request order), so the older read cannot overwrite this one
+        uint32_t last = 0;
+        bool pending = false;
+        {
+            Instance::DmapShard& sh = inst->dshard((uint64_t)dst);
+            std::lock_guard<std::mutex> g(sh.mu);
+            auto it = sh.m.find((uint64_t)dst);
+            if (it != sh.m.end()) {
+                const gsys_nbrec& pr = inst->nbrec_h[it->second & (inst->ring_cap - 1)];
+                pending = __atomic_load_n(&pr.tag, __ATOMIC_ACQUIRE) == it->second + 1u &&
+                          !__atomic_load_n(&pr.consumed, __ATOMIC_ACQUIRE);
+                last = it->second;
+                if (!pending) sh.m.erase(it);
+            }
         }
-        if (o == ~(size_t)0) return false;   // larger than the whole range store
+        if (pending) {
+            Timer tm(t_cuda);
+            inst->flush_deferred(stream, false, last, false, (uint64_t)dst);
+        }
+        return false;
     }
     ssize_t z;
     { Timer tm(t_sys); z = pread(fd, defer.h + o, want, off); }
@@ -815,12 +848,24 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
     *ret = z < 0 ? -(int64_t)errno : (int64_t)z;
     if (z > 0) inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
     gsys_nbrec& rec = inst->nbrec_h[r.pos & (inst->ring_cap - 1)];
+    // the record slot of this ring position still holds a pull nobody consumed (ring_cap requests
+    // ago): land it (and everything older) before its record is reused
+    if (__atomic_load_n(&rec.tag, __ATOMIC_ACQUIRE) == r.pos + 1u - inst->ring_cap &&
+        !__atomic_load_n(&rec.consumed, __ATOMIC_ACQUIRE) && rec.src && rec.ret > 0) {
+        Timer tm(t_cuda);
+        inst->flush_deferred(stream, false, r.pos - inst->ring_cap, false);
+    }
     __atomic_store_n(&rec.src, z > 0 ? (uint64_t)(uintptr_t)(defer.d + o) : 0ull, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.dst, (uint64_t)dst, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.ret, (long long)*ret, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.consumed, z > 0 ? 0u : 1u, __ATOMIC_RELAXED);   // nothing to copy: free at once
     __atomic_store_n(&rec.tag, r.pos + 1u, __ATOMIC_RELEASE);   // published with the completion word after it
     inst->st_deferred.fetch_add(1, std::memory_order_relaxed);
+    if (z > 0) {
+        Instance::DmapShard& sh = inst->dshard((uint64_t)dst);
+        std::lock_guard<std::mutex> g(sh.mu);
+        sh.m[(uint64_t)dst] = r.pos;
+    }
     return true;
 }
 
@@ -1506,6 +1551,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     cudaMemset(I->lat_hint_d, 0, (size_t)slots * 4);
     if (cudaMalloc(&I->nbpend_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     cudaMemset(I->nbpend_d, 0, (size_t)slots * 4);
+    if (cudaMalloc(&I->nbpos_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
+    cudaMemset(I->nbpos_d, 0, (size_t)slots * 4);
     if (cudaMalloc(&I->krounds_d, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS) != cudaSuccess) return fail(-ENOMEM);
     I->kblock_cap = 4096;
     if (cudaMalloc(&I->kblock_d, (size_t)I->kblock_cap * GSYS_KSITES * 4) != cudaSuccess) return fail(-ENOMEM);
@@ -1526,6 +1573,7 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.hdone = (unsigned long long*)I->hdone_d;
     c.lat_hint = I->lat_hint_d;
     c.nbpend = I->nbpend_d;
+    c.nbpos = I->nbpos_d;
     c.ring = (unsigned long long*)I->ring_d;
     c.ring_tail = I->tail_d;
     c.krounds = I->krounds_d;
@@ -1874,15 +1922,19 @@ int preload_flush_kernel() {
     return cudaFuncGetAttributes(&fa, (const void*)flush_kernel) == cudaSuccess ? 0 : -EIO;
 }
 
-int Instance::flush_deferred(cudaStream_t st) {
+int Instance::flush_deferred(cudaStream_t st, bool upto_all, uint32_t upto, bool use_kernel, uint64_t only_dst) {
     std::lock_guard<std::mutex> fg(flush_mu);
     std::vector<std::pair<uint32_t, FlushRec>> all;   // (ring position, record)
+    const uint32_t h = (uint32_t)head.load(std::memory_order_acquire);
     for (Worker* w : workers) {
         if (!w->defer.h) continue;
         std::lock_guard<std::mutex> g(w->defer.mu);
         for (const DeferRing::Region& rg : w->defer.q) {
             gsys_nbrec& r = nbrec_h[rg.pos & (ring_cap - 1)];
             if (w->defer.consumed(rg) || !r.src || r.ret <= 0) continue;
+            if (!upto_all && (int32_t)(rg.pos - upto) > 0) continue;
+            if (only_dst && r.dst != only_dst) continue;
+            (void)h;
             all.push_back({rg.pos, FlushRec{r.src, r.dst, r.ret, &nbrec_d[rg.pos & (ring_cap - 1)].consumed}});
         }
     }
@@ -1890,6 +1942,16 @@ int Instance::flush_deferred(cudaStream_t st) {
     // in request order; reads into the same destination go in separate passes, so the last one
     // issued is the one that stays (one caller's back-to-back reads into one buffer)
     std::sort(all.begin(), all.end(), [](const auto& a, const auto& b) { return (int32_t)(a.first - b.first) < 0; });
+    if (!use_kernel) {   // copy-engine copies in request order on one stream, then mark consumed
+        for (const auto& pr : all)
+            cudaMemcpyAsync((void*)pr.second.dst, (const void*)pr.second.src, (size_t)pr.second.ret,
+                            cudaMemcpyHostToDevice, st);
+        const cudaError_t e = cudaStreamSynchronize(st);
+        for (const auto& pr : all)
+            __atomic_store_n(&nbrec_h[pr.first & (ring_cap - 1)].consumed, 1u, __ATOMIC_RELEASE);
+        st_flushed.fetch_add(all.size(), std::memory_order_relaxed);
+        return e == cudaSuccess ? 0 : -EIO;
+    }
     // the record list lives in a grow-only pinned buffer: freeing pinned memory synchronises the
     // device, which must not happen here while a kernel may be waiting on this service
     if (flush_cap < all.size()) {
@@ -1951,7 +2013,14 @@ int gsys_wait(void* stream) {
     for (Worker* w : I->workers) cudaStreamSynchronize(w->stream);
     // deferred pulls nobody waited for on the GPU land now (B15) -- at a device-wide wait only:
     // then no kernel can be copying a record or reusing its destination concurrently
-    int ferr = (drained && !stream) ? I->flush_deferred(I->ctl) : 0;
+    int ferr = 0;
+    if (drained && !stream) {
+        ferr = I->flush_deferred(I->ctl, true, 0u, true);
+        for (auto& sh : I->dmap) {
+            std::lock_guard<std::mutex> g(sh.mu);
+            sh.m.clear();
+        }
+    }
     if (ferr) {
         int z = 0;
         I->first_err.compare_exchange_strong(z, ferr);
@@ -2147,6 +2216,7 @@ int gsys_shutdown(void) {
     cudaFree(I->tail_d);
     cudaFree(I->lat_hint_d);
     cudaFree(I->nbpend_d);
+    cudaFree(I->nbpos_d);
     cudaFree(I->krounds_d);
     cudaFree(I->kblock_d);
     cudaFree(I->ctx_d);

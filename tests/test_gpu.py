@@ -722,8 +722,9 @@ def test_kernel_call_sites(file1m):
 # ---------------------------------------------------------------------------- deferred pulls (B15)
 def test_nonblocking_device_preads_are_deferred_and_land(file1m):
     """Non-blocking WG and WI preads into device memory are served as deferred pulls (no
-    copy-engine transfer per request) and land by the device-wide gsys_wait: every buffer holds the
-    bytes of the caller's last read, as with the DMA path."""
+    copy-engine transfer per request): each lands when its caller's next call claims the slot, the
+    last ones by the device-wide gsys_wait's flush; every buffer holds the bytes of the caller's
+    last read, as with the DMA path."""
     size = os.path.getsize(file1m)
     data = open(file1m, "rb").read()
     for gran, blocks, threads in ((G.WG, 32, 128), (G.WI, 2, 64)):
@@ -739,7 +740,8 @@ def test_nonblocking_device_preads_are_deferred_and_land(file1m):
             os.close(fd)
         st = G.gsys_stats()
         assert rc == 0 and ret.tolist() == [0] * (callers * iters)
-        assert st["deferred"] == callers * iters and st["flushed"] == callers * iters, st
+        # earlier pulls land when the caller's next call claims the slot, the last ones by the flush
+        assert st["deferred"] == callers * iters and 0 < st["flushed"] <= callers * iters, st
         host = d_buf.cpu().numpy()
         for c in range(callers):
             off = ((c * iters + iters - 1) * length) % size
@@ -747,9 +749,9 @@ def test_nonblocking_device_preads_are_deferred_and_land(file1m):
             assert bytes(host[c * length: c * length + len(want)]) == want, c
 
 
-def test_deferred_pull_ring_overflow_flushes(tmpdir_shm, file1m):
+def test_deferred_pull_ring_overflow_falls_back(tmpdir_shm, file1m):
     """With a 1 MiB deferred range store per worker, 64 KiB non-blocking preads overflow it: the
-    service lands the pending pulls in request order (one flush kernel) and goes on deferring;
+    rest take the copy-engine path, each after any pending pull into the same buffer has landed;
     every buffer still ends with the caller's last read (a fresh process: the size is fixed at init)."""
     import subprocess
     import sys
@@ -773,7 +775,7 @@ for c in range(blocks):
     got = bytes(h[c * length: c * length + len(want)])
     which = [r for r in range(iters) if got == data[((c * iters + r) * length) % size:][:len(want)]]
     assert got == want, (c, which, st)
-assert rc == 0 and st['deferred'] == blocks * iters and st['flushed'] > 0, st
+assert rc == 0 and 0 < st['deferred'] < blocks * iters and st['flushed'] > 0, st
 print('ok', st['deferred'], st['flushed'])
 """
     env = dict(os.environ, GSYS_DEFER_MB="1", GSYS_THREADS="4")
