@@ -556,14 +556,19 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     const unsigned long long d1 = c->diag ? globaltimer() : 0ull;
     const unsigned char* psrc = nullptr;
     // non-blocking pread into device memory: served into a host-mapped range and pulled later (B15)
-    if (nr == GSYS_NR_PREAD64 && !blocking && !(flags & GSYS_HOSTBUF) && c->nbrec != nullptr && a[2] > 0ull)
+    // (work-item and work-group callers; a kernel-scope call is one thread the whole grid waits on:
+    // it keeps the copy engine)
+    const unsigned gran = flags & GSYS_GRAN_MASK;
+    if (nr == GSYS_NR_PREAD64 && !blocking && !(flags & GSYS_HOSTBUF) && c->nbrec != nullptr && a[2] > 0ull &&
+        gran != GSYS_KERNEL)
         flags |= GSYS_F_DEFER;
     if (nr == GSYS_NR_PREAD64 && blocking && !(flags & GSYS_HOSTBUF)) {
         psrc = pull_src(c, s, a[2], po != nullptr);
         if (psrc) flags |= GSYS_F_PULL;
-        // bounce pull (B13): a work-group copies cooperatively; a lone caller (work-item, kernel
-        // scope) copies itself, which pays only up to 64 KiB (larger reads keep the DMA path)
-        else if (c->pull_bounce && a[2] > 0ull && (po != nullptr || a[2] <= (64ull << 10))) flags |= GSYS_F_PULLB;
+        // bounce pull (B13): a work-group copies cooperatively; a work-item caller copies itself,
+        // which pays only up to 64 KiB (larger reads, and kernel-scope calls, keep the DMA path)
+        else if (c->pull_bounce && a[2] > 0ull && (po != nullptr || (gran == GSYS_WI && a[2] <= (64ull << 10))))
+            flags |= GSYS_F_PULLB;
     }
     if (io.in != nullptr) {   /* input payload into the inline line; published by marshal's fence */
         uint4* dst = reinterpret_cast<uint4*>(c->inline_buf + (size_t)s * GSYS_INLINE_BYTES);
