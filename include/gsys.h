@@ -143,7 +143,7 @@ int gsys_set_fault(int32_t err, int64_t offset);
  *   GSYS_COMPLETION_PULL (default) -- (reading B13) work-group preads that fit no pull area are read into the
  *       worker's host-mapped bounce and copied out by the work-group itself; the service makes no
  *       CUDA call while kernels wait (profiler-safe); other calls as HOST.
- * Drains first (gsys_wait).  0, -ENODEV, -EINVAL, -EIO. */
+ * Synchronises the device first (running kernels read the setting).  0, -ENODEV, -EINVAL, -EIO. */
 #define GSYS_COMPLETION_MEMOP 0u
 #define GSYS_COMPLETION_HOST  1u
 #define GSYS_COMPLETION_PULL  2u

@@ -2163,8 +2163,7 @@ int gsys_set_completion(uint32_t mode) {
     if (!I) return -ENODEV;
     if (mode > GSYS_COMPLETION_PULL) return -EINVAL;
     if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;   // running kernels read the context
-    int r = gsys_wait(nullptr);
-    (void)r;
+    // (requests carry their completion path in their flags: the service needs no drain here)
     I->ctx_h.memop_completion = mode == GSYS_COMPLETION_MEMOP ? 1u : 0u;
     I->ctx_h.pull_bounce = mode == GSYS_COMPLETION_PULL ? 1u : 0u;
     I->memop_completion = I->ctx_h.memop_completion != 0;
