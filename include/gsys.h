@@ -363,6 +363,8 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
  * for another value. */
 #define GSYS_SCAN_TOKEN 0
 #define GSYS_SCAN_DFA   1
+#define GSYS_SCAN_DFA_LDGSTS 2   /* the DFA scan with per-lane cp.async staging even when env
+                                    GSYS_SCAN_TMA=1 selects bulk-copy staging for GSYS_SCAN_DFA */
 int gsys_set_scan(int impl);
 
 /* Diagnostics: when on, gsys_wordcount's work-groups accumulate (thread 0, %globaltimer) the

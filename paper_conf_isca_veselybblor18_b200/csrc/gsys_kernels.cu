@@ -275,6 +275,109 @@ __device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__
     cp_async_wait<0>();
 }
 
+// ------------------------------------------------------------------ TMA-staged DFA scan (HBM text)
+// The same slot layout as stage_tile, filled by the bulk-copy engine instead of per-lane cp.async
+// (LDGSTS occupies the LSU pipe the DFA's shared-memory gathers are bound by): lane l copies its
+// 64 bytes into slot l, lane 0 the 16 bytes after the tile into slot 32 and the 16 bytes before it
+// into the prev area; completion is an mbarrier transaction count per buffer.  Tiles at the ends
+// of the text (zero fill, no bytes before position 0) are copied by the lanes themselves.
+constexpr unsigned MSTAGE_BYTES = 33 * SLOT + 32;      // slots + 16 B before the tile + the mbarrier
+constexpr unsigned MWARP_STAGE = 2 * MSTAGE_BYTES;
+constexpr unsigned MPREV = 33 * SLOT;                   // 16 bytes before the tile
+constexpr unsigned MBAR = 33 * SLOT + 16;               // 8-byte mbarrier
+
+__device__ __forceinline__ void mbar_init(unsigned bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_arrive(unsigned bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned bar, unsigned parity) {
+    asm volatile("{\n .reg .pred p;\n WAIT_%=:\n"
+                 " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+                 " @!p bra WAIT_%=;\n}" :: "r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_copy(unsigned dst, const void* src, unsigned bytes, unsigned bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+
+// Stage the tile at `base` into buffer `buf` (shared address); its mbarrier completes either way.
+__device__ __forceinline__ void stage_tile_tma(unsigned buf, const unsigned char* seg0, long long s, long long base,
+                                               long long valid_end, unsigned lane) {
+    const unsigned bar = buf + MBAR;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // our generic reads of buf come first
+    if (base > 0 && base + 2048 + 16 <= valid_end) {
+        const unsigned char* src = seg0 + (base - s);
+        if (lane == 0u) mbar_expect_arrive(bar, 32u * 64u + 32u);
+        __syncwarp();
+        bulk_copy(buf + lane * SLOT, src + 64u * lane, 64u, bar);
+        if (lane == 0u) {
+            bulk_copy(buf + 32u * SLOT, src + 2048, 16u, bar);
+            bulk_copy(buf + MPREV, src - 16, 16u, bar);
+        }
+        return;
+    }
+    // ends of the text: lanes copy (zero fill past valid_end, nothing before position 0)
+    unsigned char* b = reinterpret_cast<unsigned char*>(__cvta_shared_to_generic(buf));
+    for (unsigned k = 0; k < 64u; k++) {
+        const long long p = base + 64ll * lane + k;
+        b[lane * SLOT + k] = p < valid_end ? seg0[p - s] : 0u;
+    }
+    if (lane < 16u) {
+        const long long p = base + 2048 + lane;
+        b[32u * SLOT + lane] = p < valid_end ? seg0[p - s] : 0u;
+        const long long q = base - 16 + lane;
+        b[MPREV + lane] = (q >= 0 && base > 0) ? seg0[q - s] : 0u;
+    }
+    __syncwarp();
+    if (lane == 0u) mbar_arrive(bar);
+}
+
+template <bool WIDE>
+__device__ __forceinline__ void scan_range_tma(const unsigned char* __restrict__ seg0, long long s, long long own_end,
+                                               long long valid_end, const ScanState& S, unsigned& phase) {
+    const ScanTables& T = *S.T;
+    const Dfa<WIDE> D = dfa_view<WIDE>(T);
+    const bool grep = S.hit != nullptr && T.npat > 0;
+    const unsigned emit2 = D.emit2;
+    const unsigned hb = (unsigned)__cvta_generic_to_shared(S.whist) - 2u * emit2;
+    const unsigned dummy = (unsigned)__cvta_generic_to_shared(S.whist + MAXD);
+    auto emit = [hb, dummy, emit2](unsigned e) { red_emit(hb, dummy, e, emit2); };
+    auto emit2x = [hb, dummy, emit2](unsigned hi, unsigned lo) { red_emit2(hb, dummy, hi, lo, emit2); };
+    const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    unsigned char* stage = S.stage + warp * MWARP_STAGE;
+    const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
+    const long long step = 2048ll * nwarps;
+    long long base = s + 2048ll * warp;
+    if (base < own_end) stage_tile_tma(stage_s, seg0, s, base, valid_end, lane);
+    unsigned it = 0;
+    for (; base < own_end; base += step, it ^= 1u) {
+        const long long nxt = base + step;
+        if (nxt < own_end) stage_tile_tma(stage_s + (it ^ 1u) * MSTAGE_BYTES, seg0, s, nxt, valid_end, lane);
+        mbar_wait(stage_s + it * MSTAGE_BYTES + MBAR, (phase >> it) & 1u);
+        phase ^= 1u << it;
+        const unsigned char* buf = stage + it * MSTAGE_BYTES;
+        Win W;
+        W.w0 = *reinterpret_cast<const uint4*>(buf + lane * SLOT);
+        W.w1 = *reinterpret_cast<const uint4*>(buf + lane * SLOT + 16u);
+        W.w2 = *reinterpret_cast<const uint4*>(buf + lane * SLOT + 32u);
+        W.w3 = *reinterpret_cast<const uint4*>(buf + lane * SLOT + 48u);
+        W.w4 = *reinterpret_cast<const uint4*>(buf + (lane + 1u) * SLOT);
+        const unsigned prevb = lane ? (unsigned)buf[(lane - 1u) * SLOT + 63u] : (unsigned)buf[MPREV + 15u];
+        const long long p0 = base + 64ll * lane;
+        if (p0 < own_end) {
+            dfa_lane64(D, W, prevb, p0, own_end, valid_end, emit, emit2x);
+            if (grep && !*(volatile int*)S.hit && grep_lane64(T, W, p0, own_end, valid_end)) *S.hit = 1;
+        }
+        __syncwarp();                // every lane is done with this buffer before it is refilled
+    }
+    (void)it;   // `phase` tracks each buffer's mbarrier parity across ranges
+}
+
 // Dynamic shared memory: [tables] [per-warp histograms] [warp stages].  Token tables when tok.
 __device__ __forceinline__ unsigned* load_tables_tok(unsigned char* smem, const gsys_tok::TokTables* gT,
                                                      unsigned nwarps, ScanState& S) {
@@ -525,6 +628,36 @@ __global__ void __launch_bounds__(768, 1) scan_kernel(ScanArgs a) {
     if (threadIdx.x == 0 && a.hit && s_hit) atomicExch(a.hit, 1u);
 }
 
+// The byte-DFA scan with bulk-copy (TMA) staging.
+__global__ void __launch_bounds__(768, 1) scan_tma_kernel(ScanArgs a) {
+    __shared__ int s_hit;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const unsigned nwarps = blockDim.x / 32;
+    ScanState S;
+    unsigned* shist = load_tables(smem, a.tables, nwarps, S);
+    const ScanTables& sT = *S.T;
+    if (threadIdx.x == 0) s_hit = 0;
+    const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    if (lane == 0u) {
+        const unsigned st = (unsigned)__cvta_generic_to_shared(S.stage + warp * MWARP_STAGE);
+        mbar_init(st + MBAR);
+        mbar_init(st + MSTAGE_BYTES + MBAR);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    S.hit = a.hit ? &s_hit : nullptr;
+    unsigned phase = 0;
+    for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
+        const long long s = (long long)k * a.chunk;
+        const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
+        if (sT.ncol == NCOL_WIDE) scan_range_tma<true>(a.text + s, s, e, (long long)a.n, S, phase);
+        else scan_range_tma<false>(a.text + s, s, e, (long long)a.n, S, phase);
+    }
+    __syncthreads();
+    flush_hist(shist, nwarps, sT.ndict, a.hist);
+    if (threadIdx.x == 0 && a.hit && s_hit) atomicExch(a.hit, 1u);
+}
+
 // Token-level scan of HBM-resident text (gsys_tok): 1 block of up to 32 warps per SM.
 __global__ void __launch_bounds__(1024, 1) scan_tok_kernel(ScanArgs a) {
     __shared__ int s_hit;
@@ -664,6 +797,13 @@ std::mutex g_ws_mu;
 // scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.44 TB/s on the
 // 1 GiB HBM scan) or GSYS_SCAN_TOKEN (0.78 TB/s, profiles/r02_scan_ab2.jsonl); env GSYS_SCAN=dfa|token
 // at load, gsys_set_scan() at run time
+// bulk-copy (TMA) staging of the HBM DFA scan (env GSYS_SCAN_TMA=1): measured 1.13-1.17 TB/s vs
+// 1.46 with per-lane cp.async (profiles/r02_scan_staging_ab.jsonl: 33 small bulk copies per 2 KiB
+// tile cost more than the LSU slots they free), so off by default
+std::atomic<int> g_scan_tma{[] {
+    const char* e = getenv("GSYS_SCAN_TMA");
+    return (e && atoi(e) == 1) ? 1 : 0;
+}()};
 std::atomic<int> g_scan_impl{[] {
     const char* e = getenv("GSYS_SCAN");
     return (e && strcmp(e, "token") == 0) ? (int)GSYS_SCAN_TOKEN : (int)GSYS_SCAN_DFA;
@@ -909,7 +1049,7 @@ int gsys_read_profile(uint64_t* out3, int reset) {
 }
 
 int gsys_set_scan(int impl) {
-    if (impl != (int)GSYS_SCAN_TOKEN && impl != (int)GSYS_SCAN_DFA) return -EINVAL;
+    if (impl != (int)GSYS_SCAN_TOKEN && impl != (int)GSYS_SCAN_DFA && impl != (int)GSYS_SCAN_DFA_LDGSTS) return -EINVAL;
     return g_scan_impl.exchange(impl);
 }
 
@@ -919,7 +1059,8 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if (!d_hist || (n && !d_text)) return -EINVAL;
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
-    const bool tok = g_scan_impl.load() == GSYS_SCAN_TOKEN;
+    const int impl = g_scan_impl.load();
+    const bool tok = impl == GSYS_SCAN_TOKEN;
     // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 32 warps
     if (threads == 0) threads = tok ? 1024 : 704;
     if (threads % 32 || threads > (tok ? 1024u : 768u)) return -EINVAL;
@@ -931,7 +1072,8 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     int rc = 0;
     Workspace::TabCache* tc = scan_tables(W, tok, NCOL_WIDE, dict, dlen, ndict, pats, plen, npat, &rc);
     if (!tc) return rc;
-    const size_t per_warp = HSTRIDE * 4 + (tok ? TWARP_STAGE : WARP_STAGE);
+    const bool tma = impl == GSYS_SCAN_DFA && g_scan_tma.load();
+    const size_t per_warp = HSTRIDE * 4 + (tok ? TWARP_STAGE : tma ? MWARP_STAGE : WARP_STAGE);
     if (!tok && tc->blob.size() + (threads / 32) * per_warp > kSmemDynMax) {
         tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);
         if (!tc) return rc;
@@ -953,7 +1095,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     a.hit = d_hit;
     a.nchunks = nch;
     a.chunk = chunk;
-    const void* fn = tok ? (const void*)scan_tok_kernel : (const void*)scan_kernel;
+    const void* fn = tok ? (const void*)scan_tok_kernel : tma ? (const void*)scan_tma_kernel : (const void*)scan_kernel;
     size_t smem = align_up(tb, 16) + (threads / 32) * per_warp;
     rc = ensure_smem_attr(fn, smem);
     if (rc) return rc;

@@ -127,7 +127,7 @@ def test_wordcount_coalescing_invariance(ragged_corpus, window, cmax, merge):
         assert st["merged"] == 0
 
 
-@pytest.fixture(params=[G.SCAN_TOKEN, G.SCAN_DFA], ids=["token", "dfa"])
+@pytest.fixture(params=[G.SCAN_TOKEN, G.SCAN_DFA, G.SCAN_DFA_LDGSTS], ids=["token", "dfa", "dfa_ldgsts"])
 def scan_impl(request):
     prev = G.gsys_set_scan(request.param)
     yield request.param
@@ -199,7 +199,7 @@ def test_scan_device_trie_too_large_is_e2big(scan_impl):
     alpha = b"ABCDEFGHIJKLMNOPQRSTUVWXYZabcdefghijklmnopqrstuvwxyz0123456789"
     words = [alpha[i:i + 1] + b"x" * 15 for i in range(40)]       # 40 x 16 + 2 = 642 trie states > 512
     text = b" ".join(words[::3]) + b" abc " + words[1] + b"x " + words[7]
-    if scan_impl == G.SCAN_DFA:
+    if scan_impl != G.SCAN_TOKEN:
         with pytest.raises(OSError) as ei:
             _scan_dev(text, words, [], 4096)
         assert ei.value.errno == errno.E2BIG
