@@ -359,12 +359,12 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
  * A9/A10): GSYS_SCAN_DFA (default) -- one transposed-DFA shared-memory lookup per byte
  * (csrc/scan_core.cuh); GSYS_SCAN_TOKEN -- SWAR word-byte masks, token starts, per-token hash
  * lookup and byte-exact verify (csrc/tokscan.cuh; no 512-state trie limit, about half the DFA's
- * rate on B200).  Env GSYS_SCAN=dfa|token at load.  Returns the previous implementation, -EINVAL
+ * rate on B200).  Env GSYS_SCAN=dfa|token|dfa_tma at load.  Returns the previous implementation, -EINVAL
  * for another value. */
 #define GSYS_SCAN_TOKEN 0
 #define GSYS_SCAN_DFA   1
-#define GSYS_SCAN_DFA_LDGSTS 2   /* the DFA scan with per-lane cp.async staging even when env
-                                    GSYS_SCAN_TMA=1 selects bulk-copy staging for GSYS_SCAN_DFA */
+#define GSYS_SCAN_DFA_TMA 2   /* gsys_scan_device: the DFA scan with bulk-copy (TMA) staging of its
+                                 tiles (slower on B200; the wordcount treats it as GSYS_SCAN_DFA) */
 int gsys_set_scan(int impl);
 
 /* Diagnostics: when on, gsys_wordcount's work-groups accumulate (thread 0, %globaltimer) the

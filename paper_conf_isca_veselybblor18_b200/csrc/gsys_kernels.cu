@@ -797,16 +797,10 @@ std::mutex g_ws_mu;
 // scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.44 TB/s on the
 // 1 GiB HBM scan) or GSYS_SCAN_TOKEN (0.78 TB/s, profiles/r02_scan_ab2.jsonl); env GSYS_SCAN=dfa|token
 // at load, gsys_set_scan() at run time
-// bulk-copy (TMA) staging of the HBM DFA scan (env GSYS_SCAN_TMA=1): measured 1.13-1.17 TB/s vs
-// 1.46 with per-lane cp.async (profiles/r02_scan_staging_ab.jsonl: 33 small bulk copies per 2 KiB
-// tile cost more than the LSU slots they free), so off by default
-std::atomic<int> g_scan_tma{[] {
-    const char* e = getenv("GSYS_SCAN_TMA");
-    return (e && atoi(e) == 1) ? 1 : 0;
-}()};
 std::atomic<int> g_scan_impl{[] {
     const char* e = getenv("GSYS_SCAN");
-    return (e && strcmp(e, "token") == 0) ? (int)GSYS_SCAN_TOKEN : (int)GSYS_SCAN_DFA;
+    return (e && strcmp(e, "token") == 0) ? (int)GSYS_SCAN_TOKEN
+           : (e && strcmp(e, "dfa_tma") == 0) ? (int)GSYS_SCAN_DFA_TMA : (int)GSYS_SCAN_DFA;
 }()};
 
 Workspace* workspace() {
@@ -1049,7 +1043,7 @@ int gsys_read_profile(uint64_t* out3, int reset) {
 }
 
 int gsys_set_scan(int impl) {
-    if (impl != (int)GSYS_SCAN_TOKEN && impl != (int)GSYS_SCAN_DFA && impl != (int)GSYS_SCAN_DFA_LDGSTS) return -EINVAL;
+    if (impl != (int)GSYS_SCAN_TOKEN && impl != (int)GSYS_SCAN_DFA && impl != (int)GSYS_SCAN_DFA_TMA) return -EINVAL;
     return g_scan_impl.exchange(impl);
 }
 
@@ -1072,7 +1066,10 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     int rc = 0;
     Workspace::TabCache* tc = scan_tables(W, tok, NCOL_WIDE, dict, dlen, ndict, pats, plen, npat, &rc);
     if (!tc) return rc;
-    const bool tma = impl == GSYS_SCAN_DFA && g_scan_tma.load();
+    // bulk-copy (TMA) staging: measured 1.13-1.17 TB/s vs 1.46 with per-lane cp.async
+    // (profiles/r02_scan_staging_ab.jsonl: 33 small bulk copies per 2 KiB tile cost more than the
+    // LSU slots they free), so it is the opt-in GSYS_SCAN_DFA_TMA
+    const bool tma = impl == GSYS_SCAN_DFA_TMA;
     const size_t per_warp = HSTRIDE * 4 + (tok ? TWARP_STAGE : tma ? MWARP_STAGE : WARP_STAGE);
     if (!tok && tc->blob.size() + (threads / 32) * per_warp > kSmemDynMax) {
         tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);

@@ -225,7 +225,7 @@ def gsys_set_poll_timeout(ms: int) -> int:
 
 
 COMPLETION_MEMOP, COMPLETION_HOST, COMPLETION_PULL = 0, 1, 2
-SCAN_TOKEN, SCAN_DFA, SCAN_DFA_LDGSTS = 0, 1, 2
+SCAN_TOKEN, SCAN_DFA, SCAN_DFA_TMA = 0, 1, 2
 
 
 def gsys_set_scan(impl: int) -> int:

@@ -127,7 +127,7 @@ def test_wordcount_coalescing_invariance(ragged_corpus, window, cmax, merge):
         assert st["merged"] == 0
 
 
-@pytest.fixture(params=[G.SCAN_TOKEN, G.SCAN_DFA, G.SCAN_DFA_LDGSTS], ids=["token", "dfa", "dfa_ldgsts"])
+@pytest.fixture(params=[G.SCAN_TOKEN, G.SCAN_DFA, G.SCAN_DFA_TMA], ids=["token", "dfa", "dfa_tma"])
 def scan_impl(request):
     prev = G.gsys_set_scan(request.param)
     yield request.param

@@ -18,8 +18,8 @@ text = torch.cat([torch.from_file(p, dtype=torch.uint8, size=os.path.getsize(p))
 n = text.numel()
 words, pats = inputs.dictionary(), inputs.patterns()
 want_hit = int(any(c.pmasks[:64]))
-cells = [(G.SCAN_TOKEN, 1024, 256)] + [(G.SCAN_DFA, t, 256) for t in (704, 512, 768)] + \
-        [(G.SCAN_DFA_LDGSTS, 704, 256)]
+cells = [(G.SCAN_TOKEN, 1024, 256)] + [(G.SCAN_DFA_TMA, t, 256) for t in (704, 512, 768)] + \
+        [(G.SCAN_DFA, 704, 256)]
 for impl, threads, ck in cells:
     G.gsys_set_scan(impl)
     chunk = ck << 10
@@ -37,7 +37,7 @@ for impl, threads, ck in cells:
     e1.record()
     e1.synchronize()
     t = e0.elapsed_time(e1) / 1e3 / reps
-    print(json.dumps({"impl": {G.SCAN_TOKEN: "token", G.SCAN_DFA: "dfa_tma", G.SCAN_DFA_LDGSTS: "dfa_ldgsts"}[impl],
+    print(json.dumps({"impl": {G.SCAN_TOKEN: "token", G.SCAN_DFA_TMA: "dfa_tma", G.SCAN_DFA: "dfa_ldgsts"}[impl],
                       "threads": threads, "chunk": chunk,
                       "ms": t * 1e3, "GBps": n / t / 1e9, "parity": ok}), flush=True)
 G.gsys_set_scan(G.SCAN_DFA)
