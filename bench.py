@@ -382,6 +382,19 @@ def main():
             traffic_src = f"profiles/r02_ncu_summary.json[{label}]"
         except (KeyError, ValueError):
             pass
+    # the host-side co-bound: ~3 bytes of host DRAM traffic per corpus byte (pread reads the page
+    # cache and writes the bounce, the GPU reads the bounce over PCIe) against the box's measured
+    # memcpy bandwidth (tools/probes/host_membw.c, profiles/r02_host_membw.jsonl)
+    host_mem = None
+    hm = os.path.join(ROOT, "profiles", "r02_host_membw.jsonl")
+    if os.path.exists(hm):
+        try:
+            peak_h = max(json.loads(ln)["GBps_read_plus_write"] for ln in open(hm) if ln.strip())
+            host_mem = {"bound": "host DRAM (3 B per corpus byte)", "achieved": 3 * rank_achieved, "peak": peak_h,
+                        "unit": "GB/s", "frac": 3 * rank_achieved / peak_h,
+                        "peak_source": "profiles/r02_host_membw.jsonl (16-thread memcpy, read + write)"}
+        except (ValueError, KeyError):
+            pass
     roofline = {"bound": "host-link", "achieved": rank_achieved, "peak": h2d_peak, "unit": "GB/s",
                 "frac": (rank_achieved / h2d_peak) if h2d_peak else None, "traffic": traffic,
                 "traffic_note": f"dram__bytes_read.sum + dram__bytes_write.sum of {traffic_src} (ncu application "
@@ -421,7 +434,8 @@ def main():
                              **({"syscalls_wg": extras["syscalls"]} if "syscalls" in extras else {}),
                              **({"config1_16MiB": extras["config1"]} if "config1" in extras else {}),
                              **({"scan_hbm": extras["scan"]} if "scan" in extras else {}),
-                             **({"fig10_coalescing": extras["fig10"]} if "fig10" in extras else {})},
+                             **({"fig10_coalescing": extras["fig10"]} if "fig10" in extras else {}),
+                             **({"host_memory_roofline": host_mem} if host_mem else {})},
                "service_path": service_path(a, st),
                "service": {"threads": st["threads"], "coalesce_max": st["coalesce_max"],
                            "window_us": st["coalesce_window_us"], "bundles_per_step": st["bundles"] / a.steps,
