@@ -11,17 +11,21 @@
  *                                                                       P24.15, P24.32-36
  *   a6 post-call barrier + result broadcast                             P22.41-42, P28.2-3
  *
- * B200 mapping: the syscall area and doorbell ring live in pinned,
- * host-mapped memory (posted PCIe writes from the GPU, cache-resident for the host); the claim
- * words, per-slot sequence numbers and completion words live in device memory, so GPU-GPU
- * arbitration (atomicCAS) and completion polling stay in L2 instead of crossing PCIe (the
- * paper's Fig. 9 polling-contention problem, PAPER.md:28 P28.7-11).  The host writes a
- * completion word {seq, ret} with a CUDA stream memory operation ordered after the payload
- * DMA, so a thread that observes its seq also observes the pread bytes.
+ * B200 mapping: the syscall area, doorbell ring, completion words `hdone` and
+ * the pull areas live in pinned host-mapped memory (posted PCIe writes from the GPU, cache-resident
+ * for the host); the claim words and per-slot sequence numbers live in device memory, so GPU-GPU
+ * arbitration (atomicCAS) stays in L2 (Table-IV analogue: a cmp-swap costs ~0.4 us there, ~1.2 us
+ * on host memory).  The host completes a request by storing {seq, ret} into `hdone` after the
+ * result (and any pulled bytes) -- the caller's acquire load of its seq makes them visible; the
+ * alternative copy-engine paths complete through `mirror` (stream memop) or `hdone` after the DMA.
+ * Device-buffer preads are pulled by the caller out of host-mapped memory (B12/B13), non-blocking
+ * ones deferred until a token wait, the slot's next claim or gsys_wait (B15).
  *
  * Usage: every device function takes the instance context `const gsys_dev_ctx*` (from
  * gsys_device_ctx()).  Calls of WG granularity must be reached by every thread of the block,
- * calls of KERNEL granularity by every thread of every block (reading A16).
+ * calls of KERNEL granularity by every thread of every block (reading A16).  Non-blocking calls
+ * may hand back a `gsys_token` (trailing argument) for gsys_wait_token().  Every wait on the host is
+ * bounded by the instance's watchdog (-ETIMEDOUT, gsys_set_poll_timeout).
  */
 #ifndef GSYS_DEVICE_CUH
 #define GSYS_DEVICE_CUH
