@@ -204,9 +204,9 @@ int gsys_launch_begin(uint64_t nblocks, void* stream);
 /* Drain (sec. IX "a new function call, invoked by the CPU, that ensures all GPU
  * system calls have completed before the termination of the process", P34.9).  Waits for the
  * stream (NULL = whole device), then until every request the device has published is processed
- * and its completion (DMA + state write) has landed.  A device-wide wait (NULL) also lands the
- * deferred pulls of non-blocking device-buffer preads that no gsys_wait_token() consumed (reading
- * B15: one flush kernel copies them all).  Returns 0, or the first -errno recorded for a
+ * and its completion (DMA + state write) has landed, including the deferred pulls of non-blocking
+ * device-buffer preads that no gsys_wait_token() or slot claim consumed (reading B15: one flush
+ * kernel copies them all, in request order).  Returns 0, or the first -errno recorded for a
  * non-blocking call since the previous gsys_wait (reading A4), which it then clears. */
 int gsys_wait(void* stream);
 

@@ -109,6 +109,7 @@ struct gsys_dev_ctx {
     gsys_wd_log* wd;                /* device: watchdog log                                       */
     gsys_nbrec* nbrec;              /* host-mapped [ring_mask+1]: deferred-pull records (B15)     */
     unsigned* nbpos;                /* device [nslots]: ring position of the slot's last non-blocking request */
+    unsigned* nbclaim;              /* device [ring_mask+1]: position + 1 of the record whose copy is claimed */
 };
 
 /* Explicit completion token of a non-blocking call (slot, seq, ring position): gsys_wait_token()
@@ -250,8 +251,32 @@ constexpr unsigned NOSLOT = 0xffffffffu;
  * flight per round trip over PCIe. */
 __device__ __forceinline__ void pull_copy_thread(const unsigned char* src, unsigned char* dst, long long r);
 
+/* Exactly one GPU copier per deferred pull (a token wait, the slot's next claim, gsys_wait's
+ * flush kernel may all find it pending): the winner of this device-memory cmp-swap copies; the
+ * others wait until it is consumed (so their caller can rely on the bytes). */
+__device__ __forceinline__ bool claim_record(const gsys_dev_ctx* c, unsigned pos) {
+    unsigned* w = c->nbclaim + (pos & c->ring_mask);
+    unsigned old = *(volatile unsigned*)w;
+    while (old != pos + 1u) {
+        const unsigned prev = atomicCAS(w, old, pos + 1u);
+        if (prev == old) return true;
+        old = prev;
+    }
+    return false;
+}
+__device__ __forceinline__ void wait_consumed(const gsys_dev_ctx* c, const gsys_nbrec* q) {
+    unsigned long long t0 = 0ull;
+    const unsigned long long* w = reinterpret_cast<const unsigned long long*>(&q->tag);   /* {tag, consumed} */
+    while ((unsigned)(ld_acquire_sys(w) >> 32) == 0u) {
+        __nanosleep(c->poll_ns_host);
+        if (expired(c, t0)) return;
+    }
+}
+
 /* The slot's previous non-blocking request, if it left a small (<= 16 KiB) deferred pull nobody has
- * consumed: waits for its completion word (bounded) and returns its record, else nullptr. */
+ * consumed: waits for its completion word (bounded) and returns its record, claimed for the
+ * caller's scope to copy, else nullptr (nothing pending, or another copier had it: then it has
+ * landed). */
 __device__ __forceinline__ const gsys_nbrec* small_deferred_pending(const gsys_dev_ctx* c, unsigned s) {
     const unsigned pend = c->nbpend[s];
     if (!pend) return nullptr;
@@ -266,7 +291,10 @@ __device__ __forceinline__ const gsys_nbrec* small_deferred_pending(const gsys_d
     const long long r = (long long)((unsigned long long)t.x | ((unsigned long long)t.y << 32));
     if (t.z != pos + 1u || t.w != 0u || r <= 0 || r > 16384) return nullptr;
     const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
-    return (h.x | h.y) ? q : nullptr;
+    if ((h.x | h.y) == 0u) return nullptr;
+    if (claim_record(c, pos)) return q;
+    wait_consumed(c, q);
+    return nullptr;
 }
 
 /* The deferred pull at ring position pos, if it is still pending and small (<= 16 KiB): this thread
@@ -279,6 +307,7 @@ __device__ __forceinline__ void consume_small_deferred(const gsys_dev_ctx* c, un
     if (t.z != pos + 1u || t.w != 0u || r <= 0 || r > 16384) return;
     const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));
     if ((h.x | h.y) == 0u) return;
+    if (!claim_record(c, pos)) { wait_consumed(c, q); return; }
     pull_copy_thread(reinterpret_cast<const unsigned char*>((unsigned long long)h.x | ((unsigned long long)h.y << 32)),
                      reinterpret_cast<unsigned char*>((unsigned long long)h.z | ((unsigned long long)h.w << 32)), r);
     asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(&q->consumed), "r"(1u) : "memory");
@@ -834,8 +863,10 @@ __device__ __forceinline__ long long wait_token_thread(const gsys_dev_ctx* c, co
         const uint4 t = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q) + 1);   /* {ret, tag, consumed} */
         const uint4 h = ld_v4_after_acquire(reinterpret_cast<const uint4*>(q));       /* {src, dst}           */
         if (t.z == tok.pos + 1u && t.w == 0u && (h.x | h.y) != 0u && (long long)((unsigned long long)t.x |
-                                                                                 ((unsigned long long)t.y << 32)) > 0)
-            *rec = q;
+                                                                                 ((unsigned long long)t.y << 32)) > 0) {
+            if (claim_record(c, tok.pos)) *rec = q;    /* this waiter's scope copies it */
+            else wait_consumed(c, q);                  /* another copier has it: wait for the bytes */
+        }
     }
     return r;
 }

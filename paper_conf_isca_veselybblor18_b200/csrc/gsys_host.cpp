@@ -439,6 +439,7 @@ struct Instance {
     uint32_t* lat_hint_d = nullptr;
     uint32_t* nbpend_d = nullptr;
     uint32_t* nbpos_d = nullptr;
+    uint32_t* nbclaim_d = nullptr;
     gsys_kround* krounds_d = nullptr;
     uint32_t* kblock_d = nullptr;
     uint32_t kblock_cap = 0;
@@ -1553,6 +1554,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     cudaMemset(I->nbpend_d, 0, (size_t)slots * 4);
     if (cudaMalloc(&I->nbpos_d, (size_t)slots * 4) != cudaSuccess) return fail(-ENOMEM);
     cudaMemset(I->nbpos_d, 0, (size_t)slots * 4);
+    if (cudaMalloc(&I->nbclaim_d, (size_t)rc * 4) != cudaSuccess) return fail(-ENOMEM);
+    cudaMemset(I->nbclaim_d, 0, (size_t)rc * 4);
     if (cudaMalloc(&I->krounds_d, sizeof(gsys_kround) * GSYS_KSITES * GSYS_KROUNDS) != cudaSuccess) return fail(-ENOMEM);
     I->kblock_cap = 4096;
     if (cudaMalloc(&I->kblock_d, (size_t)I->kblock_cap * GSYS_KSITES * 4) != cudaSuccess) return fail(-ENOMEM);
@@ -1574,6 +1577,7 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.lat_hint = I->lat_hint_d;
     c.nbpend = I->nbpend_d;
     c.nbpos = I->nbpos_d;
+    c.nbclaim = I->nbclaim_d;
     c.ring = (unsigned long long*)I->ring_d;
     c.ring_tail = I->tail_d;
     c.krounds = I->krounds_d;
@@ -1899,17 +1903,23 @@ int gsys_launch_cu(void* cu_function, uint32_t gx, uint32_t gy, uint32_t gz, uin
 
 }  // extern "C"
 namespace {
-struct FlushRec { unsigned long long src, dst; long long ret; const unsigned* consumed; };
-// gsys_wait's flush of deferred pulls (B15): block b copies record b (the request's bytes from the
-// host-mapped range to its device destination) and marks it consumed.
-__global__ void flush_kernel(const FlushRec* list, unsigned n) {
+struct FlushRec { unsigned long long src, dst; long long ret; const unsigned* consumed; unsigned pos, pad_; };
+// gsys_wait's flush of deferred pulls (B15): block b takes record b -- unless a GPU consumer
+// (token wait, slot claim) already claimed it -- copies the request's bytes from the host-mapped
+// range to its device destination and marks it consumed.
+__global__ void flush_kernel(const gsys_dev_ctx* c, const FlushRec* list, unsigned n) {
+    __shared__ int s_mine;
     for (unsigned b = blockIdx.x; b < n; b += gridDim.x) {
         const FlushRec f = list[b];
-        gsys::pull_copy(reinterpret_cast<const unsigned char*>(f.src), reinterpret_cast<unsigned char*>(f.dst), f.ret,
-                        threadIdx.x, blockDim.x);
+        if (threadIdx.x == 0) s_mine = gsys::claim_record(c, f.pos);
         __syncthreads();
-        if (threadIdx.x == 0)
+        if (s_mine)
+            gsys::pull_copy(reinterpret_cast<const unsigned char*>(f.src), reinterpret_cast<unsigned char*>(f.dst),
+                            f.ret, threadIdx.x, blockDim.x);
+        __syncthreads();
+        if (threadIdx.x == 0 && s_mine)
             asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(f.consumed), "r"(1u) : "memory");
+        __syncthreads();
     }
 }
 }  // namespace
@@ -1935,7 +1945,7 @@ int Instance::flush_deferred(cudaStream_t st, bool upto_all, uint32_t upto, bool
             if (!upto_all && (int32_t)(rg.pos - upto) > 0) continue;
             if (only_dst && r.dst != only_dst) continue;
             (void)h;
-            all.push_back({rg.pos, FlushRec{r.src, r.dst, r.ret, &nbrec_d[rg.pos & (ring_cap - 1)].consumed}});
+            all.push_back({rg.pos, FlushRec{r.src, r.dst, r.ret, &nbrec_d[rg.pos & (ring_cap - 1)].consumed, rg.pos, 0u}});
         }
     }
     if (all.empty()) return 0;
@@ -1971,7 +1981,7 @@ int Instance::flush_deferred(cudaStream_t st, bool upto_all, uint32_t upto, bool
     auto launch = [&]() {
         if (n == start) return;
         const unsigned cnt = (unsigned)(n - start);
-        flush_kernel<<<std::min<unsigned>(cnt, 4096), 256, 0, st>>>(ld + start, cnt);
+        flush_kernel<<<std::min<unsigned>(cnt, 4096), 256, 0, st>>>(ctx_d, ld + start, cnt);
         start = n;
         dsts.clear();
     };
@@ -2011,10 +2021,11 @@ int gsys_wait(void* stream) {
         std::this_thread::yield();
     }
     for (Worker* w : I->workers) cudaStreamSynchronize(w->stream);
-    // deferred pulls nobody waited for on the GPU land now (B15) -- at a device-wide wait only:
-    // then no kernel can be copying a record or reusing its destination concurrently
+    // deferred pulls nobody waited for on the GPU land now (B15).  Kernels on other streams may
+    // still consume records themselves: every GPU copier claims a record in device memory first,
+    // so the flush kernel takes only the ones nobody else has
     int ferr = 0;
-    if (drained && !stream) {
+    if (drained) {
         ferr = I->flush_deferred(I->ctl, true, 0u, true);
         for (auto& sh : I->dmap) {
             std::lock_guard<std::mutex> g(sh.mu);
@@ -2216,6 +2227,7 @@ int gsys_shutdown(void) {
     cudaFree(I->lat_hint_d);
     cudaFree(I->nbpend_d);
     cudaFree(I->nbpos_d);
+    cudaFree(I->nbclaim_d);
     cudaFree(I->krounds_d);
     cudaFree(I->kblock_d);
     cudaFree(I->ctx_d);

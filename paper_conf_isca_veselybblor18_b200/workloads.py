@@ -117,7 +117,10 @@ def bench_calls(kind: str, gflags: int, blocks: int, threads: int, iters: int, f
     d_ret = torch.full((n,), -(1 << 40), dtype=torch.int64, device=dev) if want_ret else None
     d_lat = torch.zeros(n, dtype=torch.int64, device=dev) if want_lat else None
     d_sum = torch.zeros(n, dtype=torch.int64, device=dev) if want_sum else None
-    stream = stream or torch.cuda.current_stream()
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    else:   # the outputs were initialised on the current stream
+        stream.wait_stream(torch.cuda.current_stream())
     G.gsys_bench_calls(kind, gflags, blocks, threads, iters, fd, length, size, d_buf, d_ret, d_lat, d_sum, stream)
     rc = G.gsys_wait(stream)
     return callers, d_ret, d_lat, d_sum, rc

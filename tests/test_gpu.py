@@ -720,13 +720,16 @@ def test_kernel_call_sites(file1m):
 
 
 # ---------------------------------------------------------------------------- deferred pulls (B15)
-def test_nonblocking_device_preads_are_deferred_and_land(file1m):
+@pytest.mark.parametrize("side_stream", [False, True])
+def test_nonblocking_device_preads_are_deferred_and_land(file1m, side_stream):
     """Non-blocking WG and WI preads into device memory are served as deferred pulls (no
     copy-engine transfer per request): each lands when its caller's next call claims the slot, the
-    last ones by the device-wide gsys_wait's flush; every buffer holds the bytes of the caller's
-    last read, as with the DMA path."""
+    last ones by gsys_wait's flush -- device-wide, or scoped to a side stream (every GPU copier
+    claims a record first, reading B15); every buffer holds the bytes of the caller's last read,
+    as with the DMA path."""
     size = os.path.getsize(file1m)
     data = open(file1m, "rb").read()
+    stream = torch.cuda.Stream() if side_stream else None
     for gran, blocks, threads in ((G.WG, 32, 128), (G.WI, 2, 64)):
         iters, length = 3, 4096
         callers = blocks if gran == G.WG else blocks * threads
@@ -735,10 +738,11 @@ def test_nonblocking_device_preads_are_deferred_and_land(file1m):
         G.gsys_stats_reset()
         try:
             _, ret, _, _, rc = W.bench_calls("pread", gran | G.NONBLOCKING, blocks, threads, iters, fd, length, size,
-                                             d_buf)
+                                             d_buf, stream=stream)
         finally:
             os.close(fd)
         st = G.gsys_stats()
+        torch.cuda.synchronize()
         assert rc == 0 and ret.tolist() == [0] * (callers * iters)
         # earlier pulls land when the caller's next call claims the slot, the last ones by the flush
         assert st["deferred"] == callers * iters and 0 < st["flushed"] <= callers * iters, st
