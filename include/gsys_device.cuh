@@ -598,9 +598,12 @@ __device__ __forceinline__ long long call_thread(const gsys_dev_ctx* c, unsigned
     if (nr == GSYS_NR_PREAD64 && blocking && !(flags & GSYS_HOSTBUF)) {
         psrc = pull_src(c, s, a[2], po != nullptr);
         if (psrc) flags |= GSYS_F_PULL;
-        // bounce pull (B13): a work-group copies cooperatively; a work-item caller copies itself,
-        // which pays only up to 64 KiB (larger reads, and kernel-scope calls, keep the DMA path)
-        else if (c->pull_bounce && a[2] > 0ull && (po != nullptr || (gran == GSYS_WI && a[2] <= (64ull << 10))))
+        // bounce pull (B13): a work-group copies cooperatively; work-item callers copy with their
+        // converged warp (or alone), which pays only up to 64 KiB; a kernel-scope call is copied by
+        // the calling block, up to 1 MiB (larger reads keep the DMA path)
+        else if (c->pull_bounce && a[2] > 0ull &&
+                 ((po != nullptr && gran == GSYS_WG) || (gran == GSYS_WI && a[2] <= (64ull << 10)) ||
+                  (po != nullptr && gran == GSYS_KERNEL && a[2] <= (1ull << 20))))
             flags |= GSYS_F_PULLB;
     }
     if (io.in != nullptr) {   /* input payload into the inline line; published by marshal's fence */
@@ -746,10 +749,52 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
 
 /* Work-item (P20.31 "work-item invocations imply strong ordering"): every calling lane issues
  * its own request; the claim spins diverge, publication and the doorbell are warp-aggregated. */
+/* Blocking device-buffer preads of a warp's converged lanes: each lane's request is pulled (B12,
+ * B13) and the lanes copy every payload together -- 16-byte pieces spread over the lanes, one PCIe
+ * round trip per 512 B instead of a lone thread's loop -- then each returns its own slot. */
 __device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
                                              const unsigned long long a[6], const InlineIO& io = InlineIO(),
                                              gsys_token* tok = nullptr) {
-    return call_thread(c, nr, (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u), a, io, nullptr, tok);
+    const unsigned f = (flags & ~GSYS_RELAXED) | (producer ? GSYS_F_PRODUCER : 0u);
+    const bool coop = nr == GSYS_NR_PREAD64 && !(flags & (GSYS_NONBLOCKING | GSYS_HOSTBUF));
+    const bool nbdev = nr == GSYS_NR_PREAD64 && (flags & GSYS_NONBLOCKING) && !(flags & GSYS_HOSTBUF) &&
+                       c->nbrec != nullptr;
+    const unsigned am = __activemask();
+    const unsigned m = __ballot_sync(am, coop);
+    const unsigned mnb = __ballot_sync(am, nbdev);
+    if (nbdev) {
+        // a small deferred pull (B15) still pending on a lane's slot is copied by the converged
+        // lanes together before the claims, instead of by its lane alone inside claim()
+        const gsys_nbrec* q = small_deferred_pending(c, hw_slot(c));
+        __syncwarp(mnb);   /* each lane's acquire of its record before the others read its bytes */
+        unsigned todo = __ballot_sync(mnb, q != nullptr);
+        const unsigned rank = __popc(mnb & lanemask_lt()), nt = __popc(mnb);
+        while (todo) {
+            const int k = __ffs(todo) - 1;
+            todo &= todo - 1u;
+            finish_deferred(reinterpret_cast<const gsys_nbrec*>(__shfl_sync(mnb, (unsigned long long)q, k)), rank, nt);
+        }
+        __syncwarp(mnb);
+        if (q) mark_consumed(q);
+    }
+    if (!coop) return call_thread(c, nr, f, a, io, nullptr, tok);
+    PullOut po;
+    const long long r = call_thread(c, nr, f, a, io, &po, tok);
+    __syncwarp(m);   /* every lane's completion acquired before any lane reads another's payload */
+    unsigned todo = __ballot_sync(m, po.src != nullptr && r > 0);
+    const unsigned rank = __popc(m & lanemask_lt()), nt = __popc(m);
+    while (todo) {
+        const int k = __ffs(todo) - 1;
+        todo &= todo - 1u;
+        const unsigned char* src =
+            reinterpret_cast<const unsigned char*>(__shfl_sync(m, (unsigned long long)po.src, k));
+        unsigned char* dst = reinterpret_cast<unsigned char*>(__shfl_sync(m, a[1], k));
+        const long long n = __shfl_sync(m, r, k);
+        pull_copy(src, dst, n, rank, nt);
+    }
+    __syncwarp(m);   /* the copies are done: the slots (and their bounce ranges) can be returned */
+    if (po.src != nullptr || po.bounce) release(c, po.slot, po.seq, po.nr, po.bounce);
+    return r;
 }
 
 /* Kernel (P20.16-21, P20.33): relaxed only, -EINVAL for strong (reading A13).  Per call site and
@@ -763,6 +808,12 @@ __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned
                                                  const unsigned long long a[6], const InlineIO& io = InlineIO()) {
     __shared__ long long s_kret[2];
     __shared__ unsigned s_kpar;
+    __shared__ const unsigned char* s_ksrc;
+    __shared__ unsigned s_kslot, s_kseq, s_knr, s_kbounce;
+    __shared__ unsigned char* s_kdst;
+    __shared__ gsys_kround* s_kround;
+    __shared__ long long s_kpo_ret;
+    int kcopy = 0;
     if (!(flags & GSYS_RELAXED)) return -EINVAL;
     const unsigned site = (flags >> 24) & 63u;
     if (site >= GSYS_KSITES) return -EINVAL;
@@ -785,10 +836,19 @@ __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned
                 if (producer) {
                     unsigned t = atomicAdd(&k->arrive, 1u);
                     if (t == 0u) {
-                        r = call_thread(c, nr, flags | GSYS_F_PRODUCER, a, io);
-                        k->ret = r;
-                        __threadfence();
-                        st_release_gpu(&k->done, 1u);
+                        PullOut po;
+                        r = call_thread(c, nr, flags | GSYS_F_PRODUCER, a, io, &po);
+                        if (po.src != nullptr || po.bounce) {   /* pulled: the block copies, then publishes */
+                            s_ksrc = po.src; s_kslot = po.slot; s_kseq = po.seq; s_knr = po.nr;
+                            s_kbounce = po.bounce ? 1u : 0u;
+                            s_kdst = reinterpret_cast<unsigned char*>(a[1]);
+                            s_kround = k;
+                            kcopy = 1;
+                        } else {
+                            k->ret = r;
+                            __threadfence();
+                            st_release_gpu(&k->done, 1u);
+                        }
                     } else {
                         unsigned ns = 64;
                         unsigned long long t0 = 0ull;
@@ -812,6 +872,19 @@ __device__ __forceinline__ long long kernel_call(const gsys_dev_ctx* c, unsigned
         }
     }
     if (producer) {
+        if (__syncthreads_or(kcopy)) {   /* the first arriver's pulled pread: the whole block copies */
+            if (tid == 0) s_kpo_ret = r;
+            __syncthreads();
+            const long long rv = s_kpo_ret;
+            if (s_ksrc != nullptr && rv > 0) pull_copy(s_ksrc, s_kdst, rv, tid, block_threads());
+            __syncthreads();
+            if (tid == 0) {
+                release(c, s_kslot, s_kseq, s_knr, s_kbounce != 0u);
+                s_kround->ret = r;
+                __threadfence();
+                st_release_gpu(&s_kround->done, 1u);
+            }
+        }
         unsigned p = 0;
         if (tid == 0) { p = (s_kpar ^ 1u) & 1u; s_kpar = p; s_kret[p] = r; }
         p = (unsigned)__syncthreads_or(tid == 0 ? (int)p : 0);
