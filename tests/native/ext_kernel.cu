@@ -54,6 +54,52 @@ __global__ void ext_nb_relay(ExtArgs a) {
     if (threadIdx.x == 0) { a.ret[j] = r; a.sum[j] = s_sum; }
 }
 
+// Work-item blocking preads into device memory from a partial, diverged set of lanes (thread t
+// calls unless t % 3 == 0) with per-lane lengths around the warp-copy limit (lengths from `lens`,
+// indexed by lane), then one kernel-scope blocking pread of klen bytes into kbuf that every block
+// sums after the call (the first-arriving block copied it before releasing the others).
+struct MixArgs {
+    const gsys_dev_ctx* ctx;
+    unsigned char* dbuf;        // [threads_total * stride]
+    long long* ret;             // [threads_total] (-2^40 if the thread did not call)
+    unsigned long long* sum;    // [threads_total]
+    const unsigned* lens;       // [32]
+    unsigned char* kbuf;        // [klen]
+    long long* kret;            // [blocks]
+    unsigned long long* ksum;   // [blocks]
+    unsigned long long size, stride, klen;
+    int fd;
+};
+
+__global__ void ext_wi_mixed(MixArgs a) {
+    const unsigned long long t = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const unsigned lane = threadIdx.x % 32;
+    if (t % 3 != 0) {
+        const unsigned len = a.lens[lane];
+        const long long off = (long long)((t * 4099ull) % a.size);
+        const long long r = gsys_pread(a.ctx, a.fd, a.dbuf + t * a.stride, len, off, GSYS_WI | GSYS_BLOCKING);
+        unsigned long long acc = 0;
+        for (long long k = 0; k < (r > 0 ? r : 0); k++) acc += a.dbuf[t * a.stride + k];
+        a.ret[t] = r;
+        a.sum[t] = acc;
+    }
+    __syncthreads();
+    const long long r = gsys_pread(a.ctx, a.fd, a.kbuf, a.klen, 12345, GSYS_KERNEL | GSYS_BLOCKING | GSYS_RELAXED);
+    __shared__ unsigned long long s_sum;
+    if (threadIdx.x == 0) s_sum = 0;
+    __syncthreads();
+    unsigned long long acc = 0;
+    for (long long k = threadIdx.x; k < (r > 0 ? r : 0); k += blockDim.x) acc += a.kbuf[k];
+    atomicAdd(&s_sum, acc);
+    __syncthreads();
+    if (threadIdx.x == 0) { a.kret[blockIdx.x] = r; a.ksum[blockIdx.x] = s_sum; }
+}
+
+extern "C" int ext_function_mixed(void** f) {
+    return cudaGetFuncBySymbol(reinterpret_cast<cudaFunction_t*>(f), reinterpret_cast<const void*>(ext_wi_mixed)) ==
+                   cudaSuccess ? 0 : -1;
+}
+
 extern "C" int ext_function(void** f) {
     return cudaGetFuncBySymbol(reinterpret_cast<cudaFunction_t*>(f), reinterpret_cast<const void*>(ext_nb_relay)) ==
                    cudaSuccess ? 0 : -1;

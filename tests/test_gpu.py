@@ -638,6 +638,58 @@ def test_external_kernel_tokens(file1m, ext_lib, nwarps, length):
         assert int(sm[i]) == int(want.astype(np.int64).sum()), i
 
 
+@pytest.mark.parametrize("klen", [3000, 1 << 20, (1 << 20) + 5])
+def test_warp_and_block_copied_device_preads(file1m, ext_lib, klen):
+    """Blocking work-item preads into device memory from a diverged subset of lanes, with lengths
+    on both sides of the warp-copy limit (64 KiB) and zero: the converged lanes copy each other's
+    payloads (B13).  Then a kernel-scope pread that the first-arriving block copies (<= 1 MiB) or
+    the copy engine serves (> 1 MiB): every block sees the bytes after the call."""
+    import ctypes
+    size = os.path.getsize(file1m)
+    data = np.fromfile(file1m, dtype=np.uint8)
+    fn = ctypes.c_void_p(0)
+    ext_lib.ext_function_mixed.argtypes = [ctypes.c_void_p]
+    assert ext_lib.ext_function_mixed(ctypes.byref(fn)) == 0 and fn.value
+
+    class MixArgs(ctypes.Structure):
+        _fields_ = [("ctx", ctypes.c_void_p), ("dbuf", ctypes.c_void_p), ("ret", ctypes.c_void_p),
+                    ("sum", ctypes.c_void_p), ("lens", ctypes.c_void_p), ("kbuf", ctypes.c_void_p),
+                    ("kret", ctypes.c_void_p), ("ksum", ctypes.c_void_p), ("size", ctypes.c_uint64),
+                    ("stride", ctypes.c_uint64), ("klen", ctypes.c_uint64), ("fd", ctypes.c_int32)]
+    lens_h = [0, 1, 15, 16, 17, 100, 4096, 5000, 16384, 16385, 65535, 65536, 65537, 70000, 256, 257] * 2
+    blocks, threads, stride = 5, 96, 70016
+    nt = blocks * threads
+    lens = torch.tensor(lens_h, dtype=torch.int32, device="cuda")
+    dbuf = torch.zeros(nt * stride, dtype=torch.uint8, device="cuda")
+    ret = torch.full((nt,), -(1 << 40), dtype=torch.int64, device="cuda")
+    sm = torch.zeros(nt, dtype=torch.int64, device="cuda")
+    kbuf = torch.zeros(klen, dtype=torch.uint8, device="cuda")
+    kret = torch.zeros(blocks, dtype=torch.int64, device="cuda")
+    ksum = torch.zeros(blocks, dtype=torch.int64, device="cuda")
+    torch.cuda.synchronize()
+    fd = os.open(file1m, os.O_RDONLY)
+    try:
+        a = MixArgs(G.gsys_device_ctx(), dbuf.data_ptr(), ret.data_ptr(), sm.data_ptr(), lens.data_ptr(),
+                    kbuf.data_ptr(), kret.data_ptr(), ksum.data_ptr(), size, stride, klen, fd)
+        argv = (ctypes.c_void_p * 1)(ctypes.cast(ctypes.pointer(a), ctypes.c_void_p))
+        assert G.lib().gsys_launch_cu(fn, blocks, 1, 1, threads, 1, 1, argv, 0, None) == 0
+        assert G.gsys_wait() == 0
+    finally:
+        os.close(fd)
+    ret_h, sm_h = ret.cpu().numpy(), sm.cpu().numpy()
+    for t in range(nt):
+        if t % 3 == 0:
+            assert ret_h[t] == -(1 << 40), t
+            continue
+        off = (t * 4099) % size
+        want = data[off: off + lens_h[t % 32]]
+        assert ret_h[t] == len(want), (t, ret_h[t], len(want))
+        assert sm_h[t] == int(want.astype(np.int64).sum()), t
+    kwant = data[12345: 12345 + klen]
+    assert kret.cpu().tolist() == [len(kwant)] * blocks
+    assert ksum.cpu().tolist() == [int(kwant.astype(np.int64).sum())] * blocks
+
+
 # ---------------------------------------------------------------------------- completion paths (B13)
 @pytest.fixture
 def completion_mode(request):
