@@ -61,5 +61,14 @@ print("split", rc, int(ret[0]))
 small = torch.zeros(8 * 4096, dtype=torch.uint8, device="cuda")
 n, ret, lat, sm, rc = W.bench_calls("pread", G.WG | G.NONBLOCKING, 8, 64, 2, fd, 4096, (1 << 20) + 77, small)
 print("deferred", rc, G.gsys_stats()["deferred"])
+# warp-copied work-item pulls, block-copied kernel-scope pulls, warp-consumed deferred pulls,
+# a stream-scoped flush
+mid = torch.zeros(4 * 64 * 5000, dtype=torch.uint8, device="cuda")
+for fl, ln in ((G.WI | G.BLOCKING, 5000), (G.KERNEL | G.BLOCKING | G.RELAXED, 100000), (G.WI | G.NONBLOCKING, 4096)):
+    n, ret, lat, sm, rc = W.bench_calls("pread", fl, 4, 64, 2, fd, ln, (1 << 20) + 77, mid)
+    print("coop", fl, rc, int((ret >= 0).sum()))
+side = torch.cuda.Stream()
+n, ret, lat, sm, rc = W.bench_calls("pread", G.WG | G.NONBLOCKING, 8, 64, 2, fd, 4096, (1 << 20) + 77, small, stream=side)
+print("stream-flush", rc)
 os.close(fd)
 print("ok")
