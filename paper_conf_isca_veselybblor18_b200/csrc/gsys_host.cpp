@@ -287,28 +287,31 @@ struct DeferRing {
     }
     // offset of n free bytes, or ~0 (ring order: the free space runs from the newest region's end
     // to the oldest outstanding region's start)
+    // Consumed regions are retired lazily -- only when the free space cannot take n bytes -- so
+    // a request reads no GPU-written record line unless the ring has to make room.
     size_t alloc(size_t n, uint32_t pos) {
         n = (n + 255) & ~(size_t)255;
         if (n > cap) return ~(size_t)0;
         std::lock_guard<std::mutex> g(mu);
-        while (!q.empty() && consumed(q.front())) q.pop_front();
-        size_t lo;
-        if (q.empty()) {
-            lo = 0;
-        } else {
-            const size_t tail = q.front().lo;
-            if (head > tail) {           // not wrapped: [head, cap) then [0, tail)
-                if (head + n <= cap) lo = head;
-                else if (n <= tail) lo = 0;
-                else return ~(size_t)0;
-            } else {                     // wrapped: [head, tail)
-                if (head + n <= tail) lo = head;
-                else return ~(size_t)0;
-            }
+        size_t lo = fit(n);
+        while (lo == ~(size_t)0 && !q.empty() && consumed(q.front())) {
+            q.pop_front();
+            lo = fit(n);
         }
+        if (lo == ~(size_t)0) return lo;
         q.push_back(Region{lo, lo + n, pos});
         head = lo + n;
         return lo;
+    }
+    size_t fit(size_t n) const {
+        if (q.empty()) return 0;
+        const size_t tail = q.front().lo;
+        if (head > tail) {               // not wrapped: [head, cap) then [0, tail)
+            if (head + n <= cap) return head;
+            if (n <= tail) return 0;
+            return ~(size_t)0;
+        }
+        return head + n <= tail ? head : ~(size_t)0;   // wrapped: [head, tail)
     }
 };
 
@@ -355,6 +358,11 @@ struct Worker {
     BounceRing<Tok, RingOps>* ring = nullptr;
     uint8_t* bounce_d = nullptr;     // device address of the (host-mapped) bounce
     DeferRing defer;                 // deferred pulls of non-blocking preads (B15)
+    // destination -> ring position of the newest deferred pull this worker served into it
+    // (overflow ordering).  Written by this worker only, so its lines stay in this core's cache;
+    // the rare overflow reader takes every worker's lock and the newest pending entry
+    std::mutex dmu;
+    std::unordered_map<uint64_t, uint32_t> dmap;
     bool try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret);
     void wait_slot_free(uint32_t slot, uint32_t seq);
     void complete_early(Req& r);
@@ -481,14 +489,6 @@ struct Instance {
     // running: gsys_wait) or by copy-engine copies (from a service thread: an application kernel
     // may fill the GPU and wait on this service, so no SM work can be relied on)
     int flush_deferred(cudaStream_t st, bool upto_all, uint32_t upto, bool use_kernel, uint64_t only_dst = 0);
-    // destination -> ring position of the newest deferred pull into it (overflow ordering), sharded
-    // by destination so the workers do not serialise on one lock
-    struct alignas(64) DmapShard {
-        std::mutex mu;
-        std::unordered_map<uint64_t, uint32_t> m;
-    };
-    DmapShard dmap[64];
-    DmapShard& dshard(uint64_t dst) { return dmap[(dst >> 12) * 0x9E3779B97F4A7C15ull >> 58]; }
     std::mutex flush_mu;
     void* flush_buf = nullptr;             // pinned, mapped: the flush kernel's record list
     size_t flush_cap = 0;
@@ -825,17 +825,16 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
         // engine, in request order), so the older read cannot overwrite this one
         uint32_t last = 0;
         bool pending = false;
-        {
-            Instance::DmapShard& sh = inst->dshard((uint64_t)dst);
-            std::lock_guard<std::mutex> g(sh.mu);
-            auto it = sh.m.find((uint64_t)dst);
-            if (it != sh.m.end()) {
-                const gsys_nbrec& pr = inst->nbrec_h[it->second & (inst->ring_cap - 1)];
-                pending = __atomic_load_n(&pr.tag, __ATOMIC_ACQUIRE) == it->second + 1u &&
-                          !__atomic_load_n(&pr.consumed, __ATOMIC_ACQUIRE);
-                last = it->second;
-                if (!pending) sh.m.erase(it);
-            }
+        for (Worker* w : inst->workers) {
+            std::lock_guard<std::mutex> g(w->dmu);
+            auto it = w->dmap.find((uint64_t)dst);
+            if (it == w->dmap.end()) continue;
+            const gsys_nbrec& pr = inst->nbrec_h[it->second & (inst->ring_cap - 1)];
+            const bool p = __atomic_load_n(&pr.tag, __ATOMIC_ACQUIRE) == it->second + 1u &&
+                           !__atomic_load_n(&pr.consumed, __ATOMIC_ACQUIRE);
+            if (!p) { w->dmap.erase(it); continue; }
+            if (!pending || (int32_t)(it->second - last) > 0) last = it->second;
+            pending = true;
         }
         if (pending) {
             Timer tm(t_cuda);
@@ -863,9 +862,8 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
     __atomic_store_n(&rec.tag, r.pos + 1u, __ATOMIC_RELEASE);   // published with the completion word after it
     inst->st_deferred.fetch_add(1, std::memory_order_relaxed);
     if (z > 0) {
-        Instance::DmapShard& sh = inst->dshard((uint64_t)dst);
-        std::lock_guard<std::mutex> g(sh.mu);
-        sh.m[(uint64_t)dst] = r.pos;
+        std::lock_guard<std::mutex> g(dmu);
+        dmap[(uint64_t)dst] = r.pos;
     }
     return true;
 }
@@ -2027,9 +2025,9 @@ int gsys_wait(void* stream) {
     int ferr = 0;
     if (drained) {
         ferr = I->flush_deferred(I->ctl, true, 0u, true);
-        for (auto& sh : I->dmap) {
-            std::lock_guard<std::mutex> g(sh.mu);
-            sh.m.clear();
+        for (Worker* w : I->workers) {
+            std::lock_guard<std::mutex> g(w->dmu);
+            w->dmap.clear();
         }
     }
     if (ferr) {
