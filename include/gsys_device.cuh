@@ -714,6 +714,19 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
             __syncthreads();
             if (tid == 0) mark_consumed(s_dq);
         }
+    } else if (c->nbrec && tid < 32u && nr == GSYS_NR_PREAD64 && !(flags & GSYS_HOSTBUF)) {
+        // relaxed producer (no barrier before the call): warp 0 -- converged here, every thread of
+        // the work-group makes the call -- lands such a pull instead of the caller alone in claim()
+        const unsigned nt = block_threads();
+        const unsigned wm = nt >= 32u ? 0xffffffffu : ((1u << nt) - 1u);
+        const gsys_nbrec* q = tid == 0 ? small_deferred_pending(c, hw_slot(c)) : nullptr;
+        q = reinterpret_cast<const gsys_nbrec*>(__shfl_sync(wm, (unsigned long long)q, 0));
+        if (q) {
+            __syncwarp(wm);
+            finish_deferred(q, tid, __popc(wm));
+            __syncwarp(wm);
+            if (tid == 0) mark_consumed(q);
+        }
     }
     long long r = 0;
     PullOut po;
