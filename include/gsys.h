@@ -312,7 +312,7 @@ int gsys_selftest_bounce(uint64_t seed, uint32_t iters, uint64_t cap);
  *                   read with one work-group pread of [max(s-1,0), e+16) (reading A10).
  *   dict, dlen      host arrays: ndict (<= 64) words, 17-byte stride, lengths 1..16.
  *   pats, plen      host arrays: npat (<= 8) grep patterns, 17-byte stride, lengths 1..16.
- *   d_hist          DEVICE uint64[ndict]: whole-token counts are ADDED (reading A9).
+ *   d_hist          DEVICE uint64[ndict]: whole-token counts are ADDED (reading A9); may be NULL when ndict == 0.
  *   d_file_hits     DEVICE uint32[nfiles] (may be NULL): set to 1 for files containing a pattern.
  *   gflags          GSYS_WG (the paper's configuration for wordcount) + GSYS_STRONG or
  *                   GSYS_RELAXED, and GSYS_BLOCKING (one pread, then the scan) or GSYS_NONBLOCKING
@@ -344,7 +344,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
 
 /* Same scan over text already resident in device memory (no syscalls): the standalone scan
  * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n] (16-byte aligned); file
- * boundaries are not modelled (one file).  Adds into d_hist; d_hit (may be NULL) set to 1 if any
+ * boundaries are not modelled (one file).  Adds into d_hist (NULL allowed when ndict == 0); d_hit (may be NULL) set to 1 if any
  * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 1024 (token scan)
  * or 704 (DFA scan), else a multiple of 32 up to 1024 (768 for the DFA, whose 129-column table is
  * used when it fits beside the warps' staging, else the 77-column one).  -EINVAL on bad

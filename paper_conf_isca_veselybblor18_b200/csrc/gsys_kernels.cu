@@ -932,7 +932,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     const size_t nlines = prefetch ? 2 : 1;
     const bool mixed = (staging & ~15u) == GSYS_STAGE_MIXED(0) && (staging & 15u) != 0u;
     if (staging > GSYS_STAGE_HOST && !mixed) return -EINVAL;
-    if (nfiles == 0 || !fds || !sizes || !d_hist) return -EINVAL;
+    if (nfiles == 0 || !fds || !sizes || (!d_hist && ndict)) return -EINVAL;
     if (chunk < 4096 || (chunk % 16) || chunk > (1u << 30)) return -EINVAL;
     if (threads == 0) threads = 256;
     if (threads % 32 || threads > 256) return -EINVAL;
@@ -1050,7 +1050,7 @@ int gsys_set_scan(int impl) {
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const char* dict, const uint8_t* dlen,
                      uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, uint64_t* d_hist,
                      uint32_t* d_hit, uint32_t blocks, uint32_t threads, void* stream) {
-    if (!d_hist || (n && !d_text)) return -EINVAL;
+    if ((!d_hist && ndict) || (n && !d_text)) return -EINVAL;
     if (chunk < 16 || chunk % 16) return -EINVAL;
     if ((uintptr_t)d_text % 16) return -EINVAL;
     const int impl = g_scan_impl.load();

@@ -93,6 +93,27 @@ def test_wordcount_ragged_corpus(ragged_corpus, scan_impl, chunk, blocks, thread
     assert res.req_ret.tolist() == want
 
 
+@pytest.mark.parametrize("words,pats", [([], []), ([b"the"], []), ([], [b"the "])], ids=["none", "no-pats", "no-words"])
+def test_wordcount_degenerate_dictionaries(ragged_corpus, scan_impl, words, pats):
+    """The GPU-issued pread path with an empty dictionary and / or no grep patterns: counts and
+    per-file hits equal the oracle's (zeros where there is nothing to look for), every pread return
+    still equals the plan's."""
+    c = ragged_corpus
+    res = W.wordcount_files(c.paths, words, pats, chunk=64 << 10, gflags=G.WG | G.BLOCKING | G.RELAXED)
+    assert res.wait_rc == 0
+    h, hits, _, _ = oracle.corpus(c.paths, words, pats, nthreads=4)
+    assert np.array_equal(as_u64(res.hist)[:len(words)], np.asarray(h)[:len(words)])
+    assert int(as_u64(res.hist)[len(words):].sum()) == 0
+    if pats:
+        assert res.file_hits.tolist() == hits.tolist()
+    else:   # no patterns: no per-file hit vector (the oracle's is all zero)
+        assert res.file_hits is None and int(hits.sum()) == 0
+    want = []
+    for s in c.sizes:
+        want += [plan.expected_pread_ret(s, r[3], r[4]) for r in plan.wordcount_chunk_requests(s, 64 << 10)]
+    assert res.req_ret.tolist() == want
+
+
 def test_wordcount_grep_corpus(tmpdir_shm):
     c = inputs.make_corpus(48, 128 << 10, seed=inputs.SEED_CORPUS, root=tmpdir_shm, tag="grep48")
     res = W.wordcount_files(c.paths, WORDS, PATS, chunk=32 << 10)
@@ -176,6 +197,32 @@ def test_scan_device_high_bytes(scan_impl, threads):
             hist, hit = _scan_dev(text, words, pats, chunk, threads)
             assert np.array_equal(hist, oracle.count_tokens(text, words)[:len(words)]), (trial, chunk)
             assert hit == oracle.grep(text, pats)
+
+
+@pytest.mark.parametrize("words,pats", [
+    ([], []),                                                    # nothing to count or find
+    ([b"the", b"a", b"the", b"x y", b"a-b", b"_", b"9", b"A"], [b"q"]),   # duplicate (first wins),
+    # words with a non-word byte (never a whole token), one-byte words, case sensitivity
+    ([b"abcdefghijklmnop", b"abcdefghijklmno", b"abcdefgh", b"abcdefghi"], [b"abcdefghijklmnop"]),
+], ids=["empty", "dup-nonword-short", "shared-prefixes"])
+@pytest.mark.parametrize("size", [0, 1, 15, 16, 17, 63, 64, 65, 2047, 2048, 2049, 70_001])
+def test_scan_device_degenerate(scan_impl, words, pats, size):
+    """Degenerate dictionaries (empty; a duplicate word, which counts once -- the oracle's first
+    match wins; words containing a non-word byte, which never equal a token; 1-byte and 16-byte
+    words; words that are prefixes of one another) on texts of 0..70 KB around the 16-byte step,
+    the 64-byte lane span and the 2 KiB warp tile."""
+    rng = np.random.default_rng(size + 7 * len(words))
+    vocab = [b"the", b"a", b"_", b"9", b"A", b"x", b"y", b"ab", b"abcdefgh", b"abcdefghi", b"abcdefghijklmno",
+             b"abcdefghijklmnop", b"abcdefghijklmnopq", b"The", b"a_b"]
+    seps = [b" ", b"-", b"\n", b" y ", b"--"]
+    out = bytearray()
+    while len(out) < size:
+        out += vocab[int(rng.integers(len(vocab)))] + seps[int(rng.integers(len(seps)))]
+    text = bytes(out[:size])
+    hist, hit = _scan_dev(text, words, pats, 4096 if size > 4096 else 16)
+    arr = np.frombuffer(text, dtype=np.uint8)
+    assert np.array_equal(hist, oracle.count_tokens(arr, words)[:len(words)])
+    assert hit == oracle.grep(arr, pats)
 
 
 def test_scan_device_large_trie_uses_narrow_table(scan_impl):
