@@ -269,6 +269,48 @@ def file1m(tmpdir_shm):
     return p
 
 
+def test_concurrent_granularities_on_streams(file1m):
+    """Four call kernels in flight at once on their own streams -- work-item non-blocking and
+    blocking device preads, work-group non-blocking relaxed device preads, kernel-scope blocking
+    preads -- sharing the slots, the service, the bounce rings and the deferred store; one
+    device-wide gsys_wait.  Every blocking return and byte sum equals the direct read, every
+    buffer ends with its caller's last read."""
+    size = os.path.getsize(file1m)
+    data = open(file1m, "rb").read()
+    cells = [(G.WI | G.NONBLOCKING, 4, 128, 3, 3000), (G.WI | G.BLOCKING, 3, 96, 2, 4096),
+             (G.WG | G.NONBLOCKING | G.RELAXED, 24, 128, 4, 8192), (G.KERNEL | G.BLOCKING | G.RELAXED, 5, 64, 3, 70000)]
+    fd = os.open(file1m, os.O_RDONLY)
+    runs = []
+    try:
+        for fl, blocks, threads, iters, length in cells:
+            gran = fl & 7
+            callers = blocks * threads if gran == G.WI else blocks if gran == G.WG else 1
+            n = callers * iters
+            buf = torch.zeros(callers * length + 64, dtype=torch.uint8, device="cuda")
+            ret = torch.full((n,), -(1 << 40), dtype=torch.int64, device="cuda")
+            sm = torch.zeros(n, dtype=torch.int64, device="cuda")
+            runs.append((fl, blocks, threads, iters, length, callers, buf, ret, sm, torch.cuda.Stream()))
+        torch.cuda.synchronize()
+        for fl, blocks, threads, iters, length, callers, buf, ret, sm, st in runs:
+            G.gsys_bench_calls("pread", fl, blocks, threads, iters, fd, length, size, buf, ret, None, sm, st)
+        assert G.gsys_wait() == 0
+    finally:
+        os.close(fd)
+    for fl, blocks, threads, iters, length, callers, buf, ret, sm, st in runs:
+        gran = {G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}[fl & 7]
+        reqs = plan.microbench_requests(gran, blocks, threads, iters, length, size)
+        if not (fl & G.NONBLOCKING):
+            assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs], gran
+            assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs], gran
+        else:
+            assert ret.tolist() == [0] * len(reqs), gran
+        host = buf.cpu().numpy()
+        for c in range(callers):
+            off = ((c * iters + iters - 1) * length) % size
+            want = data[off: off + length]
+            assert bytes(host[c * length: c * length + len(want)]) == want, (gran, c)
+
+
 @pytest.mark.parametrize("gran,blk,order", VALID_CELLS)
 def test_bench_pread_matrix(file1m, gran, blk, order):
     size = os.path.getsize(file1m)
