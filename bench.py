@@ -817,9 +817,13 @@ def run_memcached(a):
     from paper_conf_isca_veselybblor18_b200 import workloads as W
 
     torch.cuda.set_device(0)
+    nthr = host_cores()
+    # the load generator (up to 8 client threads) runs on the same host: the service gets the
+    # other cores, as the CPU server's 8 threads do -- busy-polling service threads on cores the
+    # client needs would measure the oversubscription, not the server (tools/mc_threads_sweep.py)
+    os.environ.setdefault("GSYS_THREADS", str(max(2, nthr - 8)))
     W.ensure_init()
     out = {"mode": "memcached", "metric": "GET requests/s (binary memcached over UDP loopback)", "cases": []}
-    nthr = host_cores()
     for per_bucket in (16, 1024):
         nbuckets = 64
         nkeys = nbuckets * per_bucket * 3 // 4
