@@ -761,10 +761,12 @@ __device__ __forceinline__ long long wg_call(const gsys_dev_ctx* c, unsigned nr,
 }
 
 /* Work-item (P20.31 "work-item invocations imply strong ordering"): every calling lane issues
- * its own request; the claim spins diverge, publication and the doorbell are warp-aggregated. */
-/* Blocking device-buffer preads of a warp's converged lanes: each lane's request is pulled (B12,
- * B13) and the lanes copy every payload together -- 16-byte pieces spread over the lanes, one PCIe
- * round trip per 512 B instead of a lone thread's loop -- then each returns its own slot. */
+ * its own request; the claim spins diverge, publication and the doorbell are warp-aggregated.
+ * Device-buffer preads are copied by the lanes of the warp that reach the call together:
+ * blocking ones are pulled (B12, B13) and the lanes copy every payload together -- 16-byte pieces
+ * spread over the lanes, one PCIe round trip per 512 B instead of a lone thread's loop -- before
+ * each returns its own slot; for non-blocking ones the lanes land the small deferred pulls (B15)
+ * their slots still hold, together, before claiming. */
 __device__ __forceinline__ long long wi_call(const gsys_dev_ctx* c, unsigned nr, unsigned flags, bool producer,
                                              const unsigned long long a[6], const InlineIO& io = InlineIO(),
                                              gsys_token* tok = nullptr) {
