@@ -863,6 +863,38 @@ def run_memcached(a):
                                  "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
                                  "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
                                  "requests": len(pkts)})
+    # the config's value-size mix (64 B - 4 KiB, uniform), 16 elements per bucket, 32 work-groups vs
+    # the CPU server with 4 threads
+    keys, vals = MC.dataset(64 * 16 * 3 // 4, vlen=(64, 4096))
+    table = dict(zip(keys, vals))
+    pkts = [MC.encode_get(i, k) for i, k in enumerate(MC.requests(keys, 20000))]
+    resp, lat, secs, _ = W.mc_serve_run(keys, vals, pkts, nwg=32, nbuckets=64, bucket_cap=32, client_threads=4,
+                                        window=8, send_gflags=G.WG | G.RELAXED | G.BLOCKING)
+    ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
+    lat_us = np.array(lat, dtype=np.float64) / 1e3
+    out["cases"].append({"server": "gpu", "sendto": "blocking", "elements_per_bucket": 16, "work_groups": 32,
+                         "value_bytes": "64-4096", "req_per_s": len(pkts) / secs,
+                         "lat_p50_us": float(np.median(lat_us)), "lat_p99_us": float(np.quantile(lat_us, 0.99)),
+                         "exact_replies": ok, "requests": len(pkts)})
+    kb, ko, kl, vb, vo, vl = MC.pack(keys, vals)
+    sock = MC.udp_server_socket()
+    stop = ctypes.c_int(0)
+    th = threading.Thread(target=lambda: oracle.lib().oracle_mc_serve(
+        sock.fileno(), 4, kb.ctypes.data, ko.ctypes.data, kl.ctypes.data, vb.ctypes.data, vo.ctypes.data,
+        vl.ctypes.data, len(keys), 64, ctypes.addressof(stop)))
+    th.start()
+    try:
+        resp, lat, secs = MC.run_client(sock.getsockname()[1], pkts, nthreads=4, window=8)
+    finally:
+        stop.value = 1
+        th.join()
+        sock.close()
+    ok = sum(1 for p, r in zip(pkts, resp) if r == OM.expected_response(p, table))
+    lat_us = np.array(lat, dtype=np.float64) / 1e3
+    out["cases"].append({"server": "cpu-oracle", "threads": 4, "elements_per_bucket": 16, "value_bytes": "64-4096",
+                         "req_per_s": len(pkts) / secs, "lat_p50_us": float(np.median(lat_us)),
+                         "lat_p99_us": float(np.quantile(lat_us, 0.99)), "exact_replies": ok,
+                         "requests": len(pkts)})
     # higher offered load (8 client sockets x 32 in flight): the GPU server with 128 work-groups
     # against the CPU server with 4 and 8 threads (profiles/r01_memcached_load_sweep.jsonl)
     keys, vals = MC.dataset(64 * 16 * 3 // 4, vlen=1024)
