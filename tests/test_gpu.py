@@ -93,6 +93,50 @@ def test_wordcount_ragged_corpus(ragged_corpus, scan_impl, chunk, blocks, thread
     assert res.req_ret.tolist() == want
 
 
+@pytest.mark.parametrize("trial", range(10))
+def test_wordcount_fuzz(tmpdir_shm, trial):
+    """Seeded random launch shapes through the public call: file count and sizes (incl. 0, 1 and
+    sizes next to chunk multiples), chunk, work-groups, threads per work-group, staging, ordering,
+    blocking or non-blocking prefetch, scan implementation.  Counts, per-file grep hits and (when
+    blocking) every per-chunk pread return equal the oracle's."""
+    rng = np.random.default_rng(1000 + trial)
+    chunk = int(rng.choice([4096, 8192, 4096 * 5 + 16 * 3, 65536, 256 << 10]))
+    nfiles = int(rng.integers(1, 7))
+    sizes = []
+    for _ in range(nfiles):
+        kind = int(rng.integers(4))
+        if kind == 0:
+            sizes.append(int(rng.choice([0, 1, 16, 17])))
+        elif kind == 1:
+            sizes.append(chunk * int(rng.integers(1, 5)) + int(rng.integers(-17, 18)))
+        else:
+            sizes.append(int(rng.integers(1, 3 << 20)))
+    sizes = [max(s, 0) for s in sizes]
+    c = inputs.make_corpus(nfiles, sizes, seed=inputs.SEED_CORPUS + trial, root=tmpdir_shm, tag=f"fuzz{trial}")
+    blocks = int(rng.choice([0, 1, 3, 37, 148, 300]))
+    threads = int(rng.choice([32, 64, 96, 128, 256]))
+    staging = [G.STAGE_DEVICE, G.STAGE_HOST, G.STAGE_MIXED(int(rng.integers(1, 16)))][int(rng.integers(3))]
+    order = G.STRONG if rng.integers(2) else G.RELAXED
+    blk = G.BLOCKING if rng.integers(3) else G.NONBLOCKING
+    prev = G.gsys_set_scan([G.SCAN_DFA, G.SCAN_TOKEN][int(rng.integers(2))])
+    try:
+        res = W.wordcount_files(c.paths, WORDS, PATS, chunk=chunk, blocks=blocks, threads=threads,
+                                gflags=G.WG | blk | order, staging=staging)
+    finally:
+        G.gsys_set_scan(prev)
+    shape = (chunk, sizes, blocks, threads, staging, order, blk)
+    h, hits = oracle_hist_hits(c.paths)
+    assert res.wait_rc == 0, shape
+    assert np.array_equal(as_u64(res.hist), h), shape
+    assert np.array_equal(h, c.census), shape
+    assert res.file_hits.tolist() == hits.tolist(), shape
+    if blk == G.BLOCKING:
+        want = []
+        for sz in sizes:
+            want += [plan.expected_pread_ret(sz, r[3], r[4]) for r in plan.wordcount_chunk_requests(sz, chunk)]
+        assert res.req_ret.tolist()[:len(want)] == want, shape
+
+
 @pytest.mark.parametrize("words,pats", [([], []), ([b"the"], []), ([], [b"the "])], ids=["none", "no-pats", "no-words"])
 def test_wordcount_degenerate_dictionaries(ragged_corpus, scan_impl, words, pats):
     """The GPU-issued pread path with an empty dictionary and / or no grep patterns: counts and
