@@ -93,7 +93,7 @@ def test_wordcount_ragged_corpus(ragged_corpus, scan_impl, chunk, blocks, thread
     assert res.req_ret.tolist() == want
 
 
-@pytest.mark.parametrize("trial", range(10))
+@pytest.mark.parametrize("trial", range(20))
 def test_wordcount_fuzz(tmpdir_shm, trial):
     """Seeded random launch shapes through the public call: file count and sizes (incl. 0, 1 and
     sizes next to chunk multiples), chunk, work-groups, threads per work-group, staging, ordering,
@@ -353,6 +353,49 @@ def test_concurrent_granularities_on_streams(file1m):
             off = ((c * iters + iters - 1) * length) % size
             want = data[off: off + length]
             assert bytes(host[c * length: c * length + len(want)]) == want, (gran, c)
+
+
+@pytest.mark.parametrize("trial", range(32))
+def test_bench_pread_fuzz(file1m, trial):
+    """Seeded random cells of the pread microbenchmark: granularity x blocking x ordering, read
+    length across the inline / pull-area / bounce / warp-copy / DMA limits, device or host
+    buffer, grid shape and calls per caller.  Blocking returns and byte sums equal the direct
+    read; after the drain every buffer holds its caller's last read."""
+    rng = np.random.default_rng(500 + trial)
+    gran, blk, order = VALID_CELLS[int(rng.integers(len(VALID_CELLS)))]
+    length = int(rng.choice([1, 255, 256, 257, 4095, 4096, 16384, 16385, 65536, 65537, 200_000]))
+    blocks = int(rng.integers(1, 9))
+    threads = int(rng.choice([32, 64, 96, 128]))
+    iters = int(rng.integers(1, 4))
+    hostbuf = bool(rng.integers(2))
+    size = os.path.getsize(file1m)
+    data = open(file1m, "rb").read()
+    callers = {G.WI: blocks * threads, G.WG: blocks, G.KERNEL: 1}[gran]
+    if gran == G.WI and length > 16384:
+        length = 16384 + int(rng.integers(0, 3))   # keep the work-item buffers small
+    nbytes = callers * length + 64
+    buf = (torch.zeros(nbytes, dtype=torch.uint8).pin_memory() if hostbuf
+           else torch.zeros(nbytes, dtype=torch.uint8, device="cuda"))
+    fd = os.open(file1m, os.O_RDONLY)
+    try:
+        ncall, ret, lat, sm, rc = W.bench_calls("pread", gran | blk | order | (G.HOSTBUF if hostbuf else 0), blocks,
+                                                threads, iters, fd, length, size, buf, want_sum=True)
+    finally:
+        os.close(fd)
+    shape = (gran, blk, order, length, blocks, threads, iters, hostbuf)
+    assert rc == 0 and ncall == callers, shape
+    reqs = plan.microbench_requests({G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}[gran], blocks, threads, iters,
+                                    length, size)
+    if blk == G.BLOCKING:
+        assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs], shape
+        assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs], shape
+    else:
+        assert ret.tolist() == [0] * len(reqs), shape
+    host = buf.cpu().numpy()
+    for c in range(callers):
+        off = ((c * iters + iters - 1) * length) % size
+        want = data[off: off + length]
+        assert bytes(host[c * length: c * length + len(want)]) == want, (shape, c)
 
 
 @pytest.mark.parametrize("gran,blk,order", VALID_CELLS)
