@@ -536,6 +536,46 @@ def test_pwrite_consumer_barrier(tmpdir_shm, gran, blk, order):
         assert got[c * length: (c + 1) * length] == want, c
 
 
+@pytest.mark.parametrize("trial", range(16))
+def test_bench_pwrite_fuzz(tmpdir_shm, trial):
+    """Seeded random pwrite cells (consumer calls): granularity x blocking x ordering, length
+    (1 B .. 64 KiB + 1), device or host buffer, grid shape, calls per caller (one where the scope
+    does not wait for the host before rewriting its buffer: non-blocking and kernel-scope calls).
+    Every call's bytes reach the file at its offset; every return is the length."""
+    rng = np.random.default_rng(900 + trial)
+    gran, blk, order = VALID_CELLS[int(rng.integers(len(VALID_CELLS)))]
+    length = int(rng.choice([1, 17, 256, 4096, 5000, 16385, 65537]))
+    blocks = int(rng.integers(1, 6))
+    threads = int(rng.choice([32, 64, 128]))
+    iters = 1 if (blk == G.NONBLOCKING or gran == G.KERNEL) else int(rng.integers(1, 4))
+    hostbuf = bool(rng.integers(2))
+    callers = {G.WI: blocks * threads, G.WG: blocks, G.KERNEL: 1}[gran]
+    if gran == G.WI:
+        length = min(length, 4096)
+    size = callers * iters * length
+    p = os.path.join(tmpdir_shm, f"pwf_{trial}.bin")
+    open(p, "wb").write(b"\0" * size)
+    buf = (torch.zeros(callers * length + 64, dtype=torch.uint8).pin_memory() if hostbuf
+           else torch.zeros(callers * length + 64, dtype=torch.uint8, device="cuda"))
+    fd = os.open(p, os.O_RDWR)
+    try:
+        _, ret, _, _, rc = W.bench_calls("pwrite", gran | blk | order | (G.HOSTBUF if hostbuf else 0), blocks,
+                                         threads, iters, fd, length, size, buf)
+    finally:
+        os.close(fd)
+    shape = (gran, blk, order, length, blocks, threads, iters, hostbuf)
+    assert rc == 0, shape
+    if blk == G.BLOCKING and gran != G.KERNEL:
+        assert ret.tolist() == [length] * (callers * iters), shape
+    elif blk == G.BLOCKING:   # kernel-scope consumer: the last block to arrive calls, nobody waits (A6)
+        assert set(ret.tolist()) <= {0, length}, shape
+    got = np.frombuffer(open(p, "rb").read(), dtype=np.uint8)
+    i = np.arange(length, dtype=np.uint64)
+    for idx in range(callers * iters):
+        want = ((idx * 131 + i * 7 + 13) & 0xFF).astype(np.uint8)
+        assert np.array_equal(got[idx * length: (idx + 1) * length], want), (shape, idx)
+
+
 # ---------------------------------------------------------------------------- protocol trace (rows a2-a5, a7)
 def _traced(run):
     """Run `run()` with protocol tracing on; return (records, eps): records are (req=(slot, seq),
