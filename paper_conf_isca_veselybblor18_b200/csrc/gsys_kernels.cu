@@ -760,8 +760,10 @@ __global__ void __launch_bounds__(1024, 1) bench_kernel(BenchArgs a) {   // <= 6
         if (a.kind == 2 && !wi && !(a.gflags & GSYS_NONBLOCKING) && !(a.gflags & GSYS_RELAXED)) {
             // strong consumer: Bar2 already separates the call from the next iteration's writes
         } else if (a.kind == 2) {
-            // relaxed / non-blocking consumer: the buffer may still be read by the host; the
-            // benchmark writes the next payload only after the scope's own call returned
+            // relaxed consumer: the block waits for its caller before writing the next payload.
+            // A non-blocking (or kernel-scope) call has returned before the host read the buffer,
+            // so with iters > 1 a later payload may reach the file in its place: those cells
+            // measure the call rate; the content checks run them with one call per caller
             __syncthreads();
         }
     }
