@@ -636,6 +636,42 @@ def test_protocol_trace_validates(file1m):
     assert sum(1 for r in htr if r[3] == protocol.FREE) == sum(1 for b in blocking.values() if not b)
 
 
+@pytest.mark.parametrize("trial", range(6))
+def test_protocol_trace_fuzz(file1m, trial):
+    """Seeded random mixes of three call cells (getrusage / pread into device or host buffers, any
+    valid granularity x blocking x ordering, lengths across the pull limits) traced together:
+    check_trace accepts the raw logs -- one live request per slot, every request's path in
+    timestamp order -- and the request count is the plan's."""
+    rng = np.random.default_rng(77 + trial)
+    size = os.path.getsize(file1m)
+    fd = os.open(file1m, os.O_RDONLY)
+    cells = []
+    for _ in range(3):
+        gran, blk, order = VALID_CELLS[int(rng.integers(len(VALID_CELLS)))]
+        kind = "getrusage" if rng.integers(3) == 0 else "pread"
+        blocks, threads, iters = int(rng.integers(1, 5)), int(rng.choice([32, 64])), int(rng.integers(1, 4))
+        length = int(rng.choice([100, 4096, 20000]))
+        hostbuf = kind == "pread" and bool(rng.integers(2))
+        cells.append((kind, gran | blk | order | (G.HOSTBUF if hostbuf else 0), blocks, threads, iters, length,
+                      hostbuf))
+    bufs = [(torch.zeros(8 * 64 * 20000, dtype=torch.uint8).pin_memory() if c[6]
+             else torch.zeros(8 * 64 * 20000, dtype=torch.uint8, device="cuda")) for c in cells]
+
+    def run():
+        for (kind, fl, blocks, threads, iters, length, _), b in zip(cells, bufs):
+            if kind == "pread":
+                W.bench_calls("pread", fl, blocks, threads, iters, fd, length, size, b)
+            else:
+                W.bench_calls("getrusage", fl, blocks, threads, iters)
+    try:
+        recs, blocking, eps, gtr, htr = _traced(run)
+    finally:
+        os.close(fd)
+    n_req = sum({G.WI: bl * th, G.WG: bl, G.KERNEL: 1}[fl & 7] * it for _, fl, bl, th, it, _, _ in cells)
+    assert len(blocking) == n_req, cells
+    assert protocol.check_trace(recs, blocking.__getitem__, eps=eps, seq_of=lambda r: r[1]) == n_req, cells
+
+
 def test_protocol_trace_catches_a_reordered_log(file1m):
     """The checker is not vacuous on real logs: moving one host pick-up before its GPU publish
     by more than the clock error fails."""
