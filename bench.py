@@ -616,7 +616,8 @@ def config1_latency(G, W, dev, words, pats, root):
 def wg_syscall_rate(G, W, dev, path):
     """The metric's other half, "GPU-issued syscalls/sec (WG granularity)": 592 work-groups
     (4/SM x 256 threads), each cell calibrated then run for >= 100 ms of calls.  getrusage blocking
-    and non-blocking; 4 KiB preads into device memory, blocking (the pull path, reading B12)."""
+    and non-blocking; 4 KiB preads into device memory, blocking (the pull path, reading B12) and
+    non-blocking (deferred pulls, reading B15)."""
     import torch
     blocks, threads = 592, 256
     size = os.path.getsize(path)
@@ -626,7 +627,8 @@ def wg_syscall_rate(G, W, dev, path):
     try:
         for name, kind, flags in (("getrusage_blocking", "getrusage", G.WG | G.BLOCKING | G.RELAXED),
                                   ("getrusage_nonblocking", "getrusage", G.WG | G.NONBLOCKING | G.RELAXED),
-                                  ("pread4k_device_blocking", "pread", G.WG | G.BLOCKING | G.RELAXED)):
+                                  ("pread4k_device_blocking", "pread", G.WG | G.BLOCKING | G.RELAXED),
+                                  ("pread4k_device_nonblocking", "pread", G.WG | G.NONBLOCKING | G.RELAXED)):
             kw = dict(fd=fd, length=4096, size=size, d_buf=dbuf) if kind == "pread" else {}
             iters = 20
             for _ in range(2):   # calibration pass, then the >= 100 ms pass
