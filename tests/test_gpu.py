@@ -299,6 +299,19 @@ def test_scan_device_trie_too_large_is_e2big(scan_impl):
         assert np.array_equal(hist, oracle.count_tokens(np.frombuffer(text, dtype=np.uint8), words)[:len(words)])
 
 
+def assert_call_sums(sm, reqs, data, gran, iters, ctx=None):
+    """Per-call byte sums read back by the calling scope.  A kernel-scope producer call has no
+    barrier before it (relaxed only, P20.33): a block done with call r may issue call r+1 into the
+    same buffer while a slower block still sums call r's bytes, so for that granularity only the
+    last call's sum is defined."""
+    got = sm.tolist()
+    assert len(got) == len(reqs), ctx
+    for i, r in enumerate(reqs):
+        if gran == G.KERNEL and r[1] != iters - 1:
+            continue
+        assert got[i] == sum(data[r[2]: r[2] + r[3]]), (ctx, i)
+
+
 # ---------------------------------------------------------------------------- microbenchmark matrix
 VALID_CELLS = [(G.WI, G.BLOCKING, G.STRONG), (G.WI, G.NONBLOCKING, G.STRONG),
                (G.WG, G.BLOCKING, G.STRONG), (G.WG, G.BLOCKING, G.RELAXED),
@@ -345,7 +358,7 @@ def test_concurrent_granularities_on_streams(file1m):
         reqs = plan.microbench_requests(gran, blocks, threads, iters, length, size)
         if not (fl & G.NONBLOCKING):
             assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs], gran
-            assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs], gran
+            assert_call_sums(sm, reqs, data, fl & 7, iters, gran)
         else:
             assert ret.tolist() == [0] * len(reqs), gran
         host = buf.cpu().numpy()
@@ -388,7 +401,7 @@ def test_bench_pread_fuzz(file1m, trial):
                                     length, size)
     if blk == G.BLOCKING:
         assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs], shape
-        assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs], shape
+        assert_call_sums(sm, reqs, data, gran, iters, shape)
     else:
         assert ret.tolist() == [0] * len(reqs), shape
     host = buf.cpu().numpy()
@@ -420,7 +433,7 @@ def test_bench_pread_matrix(file1m, gran, blk, order):
                                     length, size)
     if blk == G.BLOCKING:
         assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs]
-        assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs]
+        assert_call_sums(sm, reqs, data, gran, iters)
     else:
         assert ret.tolist() == [0] * len(reqs)
     # after the drain the buffers hold the last iteration's bytes
@@ -733,7 +746,7 @@ def test_pread_pull_sizes(file1m, gran, length, shift):
     reqs = plan.microbench_requests({G.WI: "wi", G.WG: "wg", G.KERNEL: "kernel"}[gran], blocks, threads, iters,
                                     length, size)
     assert ret.tolist() == [plan.expected_pread_ret(size, r[2], r[3]) for r in reqs]
-    assert sm.tolist() == [sum(data[r[2]: r[2] + r[3]]) for r in reqs]
+    assert_call_sums(sm, reqs, data, gran, iters)
     host = d_all.cpu().numpy()
     assert not host[:shift].any()
     for c in range(callers):
