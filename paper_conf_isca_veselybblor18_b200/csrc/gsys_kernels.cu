@@ -189,9 +189,12 @@ __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg
         W.w4 = *reinterpret_cast<const uint4*>(buf + (lane + 1u) * SLOT);
         const unsigned prevb = lane ? (unsigned)buf[(lane - 1u) * SLOT + 63u] : (unsigned)buf[33u * SLOT + 3u];
         const long long p0 = base + 64ll * lane;
+        // the block's "a pattern was seen" flag, read once per warp tile (an atomic read, set by
+        // atomic writes: the early exit is an optimisation, not a synchronisation)
+        const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
         if (p0 < own_end) {
             dfa_lane64(D, W, prevb, p0, own_end, valid_end, emit, emit2x);
-            if (grep && !*(volatile int*)S.hit && grep_lane64(T, W, p0, own_end, valid_end)) *S.hit = 1;
+            if (grep && !seen && grep_lane64(T, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
         }
         __syncwarp();                // every lane is done with this buffer before it is refilled
     }
@@ -266,9 +269,12 @@ __device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__
         unsigned pw = __shfl_up_sync(0xffffffffu, (unsigned)(M >> 63), 1);
         if (lane == 0u) pw = base > 0 ? gsys_tok::word4(*reinterpret_cast<const unsigned*>(buf + 32u * SLOT)) >> 31 : 0u;
         const long long p0 = base + 64ll * lane;
+        // the block's "a pattern was seen" flag, read once per warp tile (an atomic read, set by
+        // atomic writes: the early exit is an optimisation, not a synchronisation)
+        const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
         if (p0 < own_end) {
             gsys_tok::tok_lane64(T, R, span, M, la, pw != 0u, p0, own_end, valid_end, emit);
-            if (grep && !*(volatile int*)S.hit && grep_lane64(T.g, W, p0, own_end, valid_end)) *S.hit = 1;
+            if (grep && !seen && grep_lane64(T.g, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
         }
         __syncwarp();
     }
@@ -369,9 +375,12 @@ __device__ __forceinline__ void scan_range_tma(const unsigned char* __restrict__
         W.w4 = *reinterpret_cast<const uint4*>(buf + (lane + 1u) * SLOT);
         const unsigned prevb = lane ? (unsigned)buf[(lane - 1u) * SLOT + 63u] : (unsigned)buf[MPREV + 15u];
         const long long p0 = base + 64ll * lane;
+        // the block's "a pattern was seen" flag, read once per warp tile (an atomic read, set by
+        // atomic writes: the early exit is an optimisation, not a synchronisation)
+        const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
         if (p0 < own_end) {
             dfa_lane64(D, W, prevb, p0, own_end, valid_end, emit, emit2x);
-            if (grep && !*(volatile int*)S.hit && grep_lane64(T, W, p0, own_end, valid_end)) *S.hit = 1;
+            if (grep && !seen && grep_lane64(T, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
         }
         __syncwarp();                // every lane is done with this buffer before it is refilled
     }
