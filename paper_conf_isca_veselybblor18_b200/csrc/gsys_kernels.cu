@@ -79,19 +79,19 @@ __device__ __forceinline__ unsigned ld1(const unsigned char* p) {
 
 
 
-// Count a DFA entry e if it is an emission (e >= emit2: word (e - emit2) / 2) without a branch: an
-// unconditional shared increment at hb + 2 e (hb = histogram address - 2 emit2), or at the warp's
-// dummy word.  (A predicated RED is compiled into a branch around the atomic plus a reconvergence
-// barrier; an unconditional increment is one ATOMS.POPC.INC, which merges lanes on one address.)
-constexpr unsigned HSTRIDE = MAXD + 4;    // per-warp shared words: histogram + dummy (+ pad)
-__device__ __forceinline__ void red_emit(unsigned hb, unsigned dummy, unsigned e, unsigned emit2) {
-    asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(e >= emit2 ? hb + 2u * e : dummy) : "memory");
+// Count a DFA entry e if it is an emission (e >= emit2: word (e - emit2) / 2): a predicated shared
+// RED at hb + 2 e (hb = histogram address - 2 emit2).  The predicate is set inside the asm, so the
+// compiler emits @P RED (no branch, no reconvergence barrier) and lanes without a hit send nothing.
+constexpr unsigned HSTRIDE = MAXD + 4;    // per-warp shared words: histogram (+ pad)
+__device__ __forceinline__ void red_emit(unsigned hb, unsigned e, unsigned emit2) {
+    asm volatile("{ .reg .pred p; setp.ge.u32 p, %1, %2; @p red.shared.add.u32 [%0], 1; }"
+                 :: "r"(hb + 2u * e), "r"(e), "r"(emit2) : "memory");
 }
-// the larger of a 4-byte group's two pair maxima unconditionally, the smaller only when it is an
-// emission too (a branch taken when any lane saw two hits in 4 bytes)
-__device__ __forceinline__ void red_emit2(unsigned hb, unsigned dummy, unsigned hi, unsigned lo, unsigned emit2) {
-    red_emit(hb, dummy, hi, emit2);
-    if (lo >= emit2) asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hb + 2u * lo) : "memory");
+// the two pair maxima of a 4-byte group (at most one emission per pair)
+__device__ __forceinline__ void red_emit2(unsigned hb, unsigned hi, unsigned lo, unsigned emit2) {
+    asm volatile("{ .reg .pred p, q; setp.ge.u32 p, %2, %4; setp.ge.u32 q, %3, %4;\n\t"
+                 "@p red.shared.add.u32 [%0], 1; @q red.shared.add.u32 [%1], 1; }"
+                 :: "r"(hb + 2u * hi), "r"(hb + 2u * lo), "r"(hi), "r"(lo), "r"(emit2) : "memory");
 }
 
 // Scan positions [s, own_end) of a text whose valid bytes end at valid_end; seg0 points at the
@@ -160,13 +160,12 @@ template <int P, bool WIDE>
 __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                            long long valid_end, const ScanState& S) {
     const ScanTables& T = *S.T;
-    const Dfa<WIDE> D = dfa_view<WIDE>(T);
+    const Dfa<WIDE> D = dfa_view_shared<WIDE>(T);
     const bool grep = S.hit != nullptr && T.npat > 0;
     const unsigned emit2 = D.emit2;
     const unsigned hb = (unsigned)__cvta_generic_to_shared(S.whist) - 2u * emit2;
-    const unsigned dummy = (unsigned)__cvta_generic_to_shared(S.whist + MAXD);
-    auto emit = [hb, dummy, emit2](unsigned e) { red_emit(hb, dummy, e, emit2); };
-    auto emit2x = [hb, dummy, emit2](unsigned hi, unsigned lo) { red_emit2(hb, dummy, hi, lo, emit2); };
+    auto emit = [hb, emit2](unsigned e) { red_emit(hb, e, emit2); };
+    auto emit2x = [hb, emit2](unsigned hi, unsigned lo) { red_emit2(hb, hi, lo, emit2); };
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     unsigned char* stage = S.stage + warp * WARP_STAGE;
     const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
@@ -347,13 +346,12 @@ template <bool WIDE>
 __device__ __forceinline__ void scan_range_tma(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                                long long valid_end, const ScanState& S, unsigned& phase) {
     const ScanTables& T = *S.T;
-    const Dfa<WIDE> D = dfa_view<WIDE>(T);
+    const Dfa<WIDE> D = dfa_view_shared<WIDE>(T);
     const bool grep = S.hit != nullptr && T.npat > 0;
     const unsigned emit2 = D.emit2;
     const unsigned hb = (unsigned)__cvta_generic_to_shared(S.whist) - 2u * emit2;
-    const unsigned dummy = (unsigned)__cvta_generic_to_shared(S.whist + MAXD);
-    auto emit = [hb, dummy, emit2](unsigned e) { red_emit(hb, dummy, e, emit2); };
-    auto emit2x = [hb, dummy, emit2](unsigned hi, unsigned lo) { red_emit2(hb, dummy, hi, lo, emit2); };
+    auto emit = [hb, emit2](unsigned e) { red_emit(hb, e, emit2); };
+    auto emit2x = [hb, emit2](unsigned hi, unsigned lo) { red_emit2(hb, hi, lo, emit2); };
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     unsigned char* stage = S.stage + warp * MWARP_STAGE;
     const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
@@ -410,7 +408,16 @@ __device__ __forceinline__ unsigned* load_tables(unsigned char* smem, const Scan
     const size_t tb = (tables_bytes(gT->nsp, gT->ncol) + 15) & ~(size_t)15;
     const uint4* src = reinterpret_cast<const uint4*>(gT);
     uint4* dst = reinterpret_cast<uint4*>(smem);
-    for (unsigned i = threadIdx.x; i < tb / 16; i += blockDim.x) dst[i] = src[i];
+    // DFA entries are rebased to shared addresses (Dfa::org) as they are staged: org + 2 * nsp
+    // stays below 64 KiB (the table opens the dynamic window), so each u16 half adds without carry
+    static_assert(sizeof(ScanTables) % 16 == 0, "the DFA starts on a 16-byte boundary");
+    const unsigned org = (unsigned)__cvta_generic_to_shared(smem) + (unsigned)sizeof(ScanTables);
+    const unsigned add = org * 0x10001u;
+    for (unsigned i = threadIdx.x; i < tb / 16; i += blockDim.x) {
+        uint4 v = src[i];
+        if (i >= sizeof(ScanTables) / 16) { v.x += add; v.y += add; v.z += add; v.w += add; }
+        dst[i] = v;
+    }
     unsigned* shist = reinterpret_cast<unsigned*>(smem + tb);
     for (unsigned i = threadIdx.x; i < nwarps * HSTRIDE; i += blockDim.x) shist[i] = 0;
     S.stage = smem + tb + nwarps * HSTRIDE * 4;

@@ -145,33 +145,51 @@ GSYS_HD unsigned window_byte(const uint4& A, const uint4& B, unsigned i) {
     return (w >> (8 * (i & 3u))) & 0xffu;
 }
 
-// View of the transposed DFA (see header).  Entries are 2 * state; the DFA "state" carried by the
-// scan is the entry value itself.
+// View of the transposed DFA (see header).  Entries are org + 2 * state; the DFA "state" carried
+// by the scan is the entry value itself.  Host (emulation): org = 0 and entry(col, e) is read at
+// base + col * stride + e.  Device: the kernel adds org = the shared-window address of column 0 to
+// every entry when it stages the table (load_tables), so col * stride + e IS the shared address of
+// the next entry -- one IMAD and one LDS.U16 per byte, no base add.
 template <bool WIDE>
 struct Dfa {
-    const unsigned char* base;  // entry(col, e) at base + col * stride + e
+    const unsigned char* base;  // host: entry(col, e) at base + col * stride + e
     unsigned stride;            // 2 * nsp
-    unsigned emit2;             // first emission entry
+    unsigned emit2;             // first emission entry (org + 2 * nstates)
+    unsigned org;               // entry of state 0 (ROOT)
     GSYS_HD static unsigned col(unsigned b) { return WIDE ? col_wide(b) : col_narrow(b); }
     GSYS_HD unsigned at(unsigned c, unsigned e) const {
-        const unsigned v = *reinterpret_cast<const unsigned short*>(base + c * stride + e);
 #ifdef __CUDA_ARCH__
-        __builtin_assume(v < 65536u);   // lets max() of two entries skip a re-mask
-#endif
+        unsigned v;
+        asm volatile("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(c * stride + e));
         return v;
+#else
+        return *reinterpret_cast<const unsigned short*>(base + c * stride + e);
+#endif
     }
     GSYS_HD unsigned step(unsigned e, unsigned b) const { return at(col(b), e); }
+    GSYS_HD unsigned root() const { return org + 2u * ROOT; }
+    GSYS_HD unsigned dead() const { return org + 2u * DEAD; }
     // inside a token whose prefix is still a dictionary prefix (ROOT, DEAD, emissions are not)
-    GSYS_HD bool live(unsigned e) const { return e > 2u * DEAD && e < emit2; }
+    GSYS_HD bool live(unsigned e) const { return e > dead() && e < emit2; }
 };
+// Host view (org = 0) of a table in memory.
 template <bool WIDE>
 GSYS_HD Dfa<WIDE> dfa_view(const ScanTables& T) {
-    return Dfa<WIDE>{reinterpret_cast<const unsigned char*>(&T) + sizeof(ScanTables), 2u * T.nsp, T.emit2};
+    return Dfa<WIDE>{reinterpret_cast<const unsigned char*>(&T) + sizeof(ScanTables), 2u * T.nsp, T.emit2, 0u};
 }
+#ifdef __CUDACC__
+// Device view of a table staged in shared memory whose entries were rebased by org (see Dfa).
+template <bool WIDE>
+__device__ __forceinline__ Dfa<WIDE> dfa_view_shared(const ScanTables& T) {
+    const unsigned org = (unsigned)__cvta_generic_to_shared(&T) + (unsigned)sizeof(ScanTables);
+    return Dfa<WIDE>{nullptr, 2u * T.nsp, org + T.emit2, org};
+}
+#endif
 
 // Start entry of a span at p0: inside a token owned by the left neighbour -> DEAD.
-GSYS_HD unsigned start_entry(unsigned prevb, long long p0) {
-    return (p0 > 0 && is_word_byte(prevb)) ? 2u * DEAD : 2u * ROOT;
+template <bool WIDE>
+GSYS_HD unsigned start_entry(const Dfa<WIDE>& D, unsigned prevb, long long p0) {
+    return (p0 > 0 && is_word_byte(prevb)) ? D.dead() : D.root();
 }
 
 // One 16-byte step of the scan at text position p0 (the reference composition, host emulation):
@@ -187,7 +205,7 @@ GSYS_HD void dfa_segment(const Dfa<WIDE>& D, const uint4& A, const uint4& B, uns
     const unsigned nvalid = nvalid_ll >= 32 ? 32u : (unsigned)nvalid_ll;
     const long long nown_ll = own_end - p0;
     const unsigned nown = nown_ll >= 16 ? 16u : (unsigned)nown_ll;
-    unsigned e = start_entry(prevb, p0);
+    unsigned e = start_entry(D, prevb, p0);
     for (unsigned i = 0; i < nown && i < nvalid; i++) {
         e = D.step(e, window_byte(A, B, i));
         emit(e);
@@ -288,7 +306,7 @@ GSYS_HD void dfa_lane64(const Dfa<WIDE>& D, const Win& W, unsigned prevb, long l
     const unsigned nvalid = nvalid_ll >= 80 ? 80u : (unsigned)nvalid_ll;
     const long long nown_ll = own_end - p0;
     const unsigned nown = nown_ll >= 64 ? 64u : (unsigned)nown_ll;
-    unsigned e = start_entry(prevb, p0);
+    unsigned e = start_entry(D, prevb, p0);
     if (nown == 64u && nvalid >= 64u) {
         bool raw = false;
         if (WIDE) {
@@ -315,7 +333,7 @@ GSYS_UNROLL
                     lv = D.live(e);
                 }
             }
-            emit(lv0 ? e : 2u * ROOT);
+            emit(lv0 ? e : D.root());
             return;
         }
         const unsigned nla = nvalid - 64u;
