@@ -42,7 +42,7 @@ struct ScanState {
                                 // part of the token tables (token scan)
     const gsys_tok::TokTables* TT;   // shared memory: token tables (token scan) or nullptr
     unsigned* whist;            // this warp's shared histogram [64]
-    unsigned char* stage;       // shared memory, WARP_STAGE / TWARP_STAGE bytes per warp
+    unsigned char* stage;       // shared memory, WARP_STAGE / TWWARP_STAGE bytes per warp
     int* hit;                   // shared grep-hit flag of the current chunk (nullptr: no grep)
 };
 
@@ -204,8 +204,6 @@ __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg
 // Staging for the token scan: per 2 KiB warp tile, 32 lane slots of 80 B -- the lane's 64 bytes AND
 // the 16 bytes after them (a duplicate of the next slot's first 16 B, so a token window starting
 // anywhere in the span is contiguous in shared memory) -- then the 4 bytes before the tile.
-constexpr unsigned TSTAGE_BYTES = 32 * SLOT + 16;
-constexpr unsigned TWARP_STAGE = 2 * TSTAGE_BYTES;
 
 __device__ __forceinline__ void stage_tile_tok(unsigned buf, const unsigned char* seg0, long long s, long long base,
                                                long long valid_end, unsigned lane) {
@@ -229,20 +227,26 @@ __device__ __forceinline__ void stage_tile_tok(unsigned buf, const unsigned char
     if (lane == 0u) cp_async4(buf + 32u * SLOT, seg0 + (base > 0 ? base - 4 - s : 0), base > 0 ? 4u : 0u);
 }
 
-// Token-level scan of positions [s, own_end) (same contract as scan_range): warp tiles of 2 KiB
-// staged by cp.async (double-buffered); lane l takes the 64-byte span at base + 64 l, classifies it
-// (gsys_tok::mask64), gets the lookahead mask from lane l+1 and the previous byte's class from
-// lane l-1 by shuffles, and visits the tokens it owns (gsys_tok::tok_lane64).
-__device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__ seg0, long long s, long long own_end,
-                                               long long valid_end, const ScanState& S) {
+// Warp-cooperative token scan of positions [s, own_end) (gsys_tok::tokw_*; same contract as
+// scan_range; tiles staged by stage_tile_tok): per tile, phase A -- each lane classifies its span, the lanes'
+// start counts are prefix-summed with shuffles and every lane appends its entries to the warp's
+// list in shared memory; phase C -- lane j looks up entries j, j+32, ... of that list.
+constexpr unsigned TWWARP_STAGE = 2 * gsys_tok::TOKW_TILE + 2 * gsys_tok::TOKW_LIST;
+
+__device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict__ seg0, long long s, long long own_end,
+                                                long long valid_end, const ScanState& S) {
     const gsys_tok::TokTables& T = *S.TT;
     const bool grep = S.hit != nullptr && T.g.npat > 0;
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    unsigned char* stage = S.stage + warp * TWARP_STAGE;
+    unsigned char* stage = S.stage + warp * TWWARP_STAGE;
     const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
+    const unsigned list_s = stage_s + 2u * gsys_tok::TOKW_TILE;
     const unsigned hs = (unsigned)__cvta_generic_to_shared(S.whist);
-    auto emit = [hs](unsigned d) { asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hs + 4u * d)); };
-    const gsys_tok::TokRegs R = gsys_tok::tok_regs(T);
+    auto emit = [hs](unsigned d) { asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hs + 4u * d) : "memory"); };
+    gsys_tok::TokRegs R = gsys_tok::tok_regs(T);
+    // pin the shared-window addresses in registers (an opaque move: the compiler would otherwise
+    // rebuild them from SR_CgaCtaId inside the lookup loop)
+    asm volatile("mov.b32 %0, %0;" : "+r"(R.tabs));
     const unsigned one = T.one;
     const long long step = 2048ll * nwarps;
     long long base = s + 2048ll * warp;
@@ -250,32 +254,58 @@ __device__ __forceinline__ void scan_range_tok(const unsigned char* __restrict__
     cp_async_commit();
     for (unsigned it = 0; base < own_end; base += step, it ^= 1u) {
         const long long nxt = base + step;
-        if (nxt < own_end) stage_tile_tok(stage_s + (it ^ 1u) * TSTAGE_BYTES, seg0, s, nxt, valid_end, lane);
+        if (nxt < own_end) stage_tile_tok(stage_s + (it ^ 1u) * gsys_tok::TOKW_TILE, seg0, s, nxt, valid_end, lane);
         cp_async_commit();
         cp_async_wait<1>();
         __syncwarp();
-        const unsigned char* buf = stage + it * TSTAGE_BYTES;
-        const unsigned char* span = buf + lane * SLOT;
-        Win W;
-        W.w0 = *reinterpret_cast<const uint4*>(span);
-        W.w1 = *reinterpret_cast<const uint4*>(span + 16u);
-        W.w2 = *reinterpret_cast<const uint4*>(span + 32u);
-        W.w3 = *reinterpret_cast<const uint4*>(span + 48u);
-        W.w4 = *reinterpret_cast<const uint4*>(span + 64u);
-        const unsigned long long M = gsys_tok::mask64(W, one);
-        unsigned la = __shfl_down_sync(0xffffffffu, (unsigned)M & 0xffffu, 1);
-        if (lane == 31u) la = gsys_tok::mask16(W.w4);
-        unsigned pw = __shfl_up_sync(0xffffffffu, (unsigned)(M >> 63), 1);
-        if (lane == 0u) pw = base > 0 ? gsys_tok::word4(*reinterpret_cast<const unsigned*>(buf + 32u * SLOT)) >> 31 : 0u;
+        const unsigned char* buf = stage + it * gsys_tok::TOKW_TILE;
+        const unsigned buf_s = stage_s + it * gsys_tok::TOKW_TILE;
         const long long p0 = base + 64ll * lane;
-        // the block's "a pattern was seen" flag, read once per warp tile (an atomic read, set by
-        // atomic writes: the early exit is an optimisation, not a synchronisation)
-        const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
-        if (p0 < own_end) {
-            gsys_tok::tok_lane64(T, R, span, M, la, pw != 0u, p0, own_end, valid_end, emit);
-            if (grep && !seen && grep_lane64(T.g, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
+        unsigned n;
+        {   // phase A
+            const unsigned char* span = buf + lane * SLOT;
+            Win W;
+            W.w0 = *reinterpret_cast<const uint4*>(span);
+            W.w1 = *reinterpret_cast<const uint4*>(span + 16u);
+            W.w2 = *reinterpret_cast<const uint4*>(span + 32u);
+            W.w3 = *reinterpret_cast<const uint4*>(span + 48u);
+            W.w4 = *reinterpret_cast<const uint4*>(span + 64u);
+            const unsigned m0 = gsys_tok::mask16(W.w0, one) | (gsys_tok::mask16(W.w1, one) << 16);
+            const unsigned m1 = gsys_tok::mask16(W.w2, one) | (gsys_tok::mask16(W.w3, one) << 16);
+            unsigned m2 = __shfl_down_sync(0xffffffffu, m0, 1);
+            if (lane == 31u) m2 = gsys_tok::mask16(W.w4, one);
+            unsigned pw = __shfl_up_sync(0xffffffffu, m1 >> 31, 1);
+            if (lane == 0u) pw = base > 0 ? gsys_tok::word4(*reinterpret_cast<const unsigned*>(buf + 32u * SLOT)) >> 31 : 0u;
+            // the block's "a pattern was seen" flag, read once per warp tile (an atomic read, set by
+            // atomic writes: the early exit is an optimisation, not a synchronisation)
+            const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
+            if (grep && !seen && p0 < own_end && grep_lane64(T.g, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
+            const gsys_tok::TokwSpan sp = gsys_tok::tokw_span(m0, m1, m2, pw != 0u, p0, own_end, valid_end);
+            const unsigned cnt = (unsigned)__popc(sp.s0) + (unsigned)__popc(sp.s1);
+            unsigned incl = cnt;
+#pragma unroll
+            for (unsigned d = 1; d < 32u; d <<= 1) {
+                const unsigned v = __shfl_up_sync(0xffffffffu, incl, d);
+                if (lane >= d) incl += v;
+            }
+            n = __shfl_sync(0xffffffffu, incl, 31);
+            unsigned ptr = list_s + 2u * (incl - cnt);
+            gsys_tok::tokw_list(R, sp, lane * SLOT, [&ptr](unsigned e) {
+                asm volatile("st.shared.u16 [%0], %1;" :: "r"(ptr), "h"((unsigned short)e) : "memory");
+                ptr += 2u;
+            });
         }
         __syncwarp();
+        {   // phase C
+            const gsys_tok::TokwTile tile{buf, buf_s};
+#pragma unroll 2
+            for (unsigned j = lane; j < n; j += 32u) {
+                unsigned e;
+                asm volatile("ld.shared.u16 %0, [%1];" : "=r"(e) : "r"(list_s + 2u * j) : "memory");
+                gsys_tok::tokw_lookup(T, R, tile, e & 0xffffu, emit);
+            }
+        }
+        __syncwarp();                // every lane is done with this buffer and the list before reuse
     }
     cp_async_wait<0>();
 }
@@ -483,7 +513,7 @@ __device__ __forceinline__ bool wc_next_chunk(const WcArgs& a, unsigned* s_k, Wc
 template <bool TOK>
 __device__ __forceinline__ void scan_line(const unsigned char* seg0, long long s, long long own_end, long long valid_end,
                                           const ScanState& S) {
-    if (TOK) scan_range_tok(seg0, s, own_end, valid_end, S);
+    if (TOK) scan_range_tokw(seg0, s, own_end, valid_end, S);
     else scan_range<LD_CG, false>(seg0, s, own_end, valid_end, S);
 }
 
@@ -675,7 +705,7 @@ __global__ void __launch_bounds__(768, 1) scan_tma_kernel(ScanArgs a) {
 }
 
 // Token-level scan of HBM-resident text (gsys_tok): 1 block of up to 32 warps per SM.
-__global__ void __launch_bounds__(1024, 1) scan_tok_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(768, 1) scan_tok_kernel(ScanArgs a) {
     __shared__ int s_hit;
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
@@ -687,7 +717,7 @@ __global__ void __launch_bounds__(1024, 1) scan_tok_kernel(ScanArgs a) {
     for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         const long long s = (long long)k * a.chunk;
         const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
-        scan_range_tok(a.text + s, s, e, (long long)a.n, S);
+        scan_range_tokw(a.text + s, s, e, (long long)a.n, S);
     }
     __syncthreads();
     flush_hist(shist, nwarps, S.T->ndict, a.hist);
@@ -812,9 +842,9 @@ struct Workspace {
 };
 Workspace g_ws[64];
 std::mutex g_ws_mu;
-// scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.44 TB/s on the
-// 1 GiB HBM scan) or GSYS_SCAN_TOKEN (0.78 TB/s, profiles/r02_scan_ab2.jsonl); env GSYS_SCAN=dfa|token
-// at load, gsys_set_scan() at run time
+// scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.47 TB/s on the
+// 1 GiB HBM scan) or GSYS_SCAN_TOKEN (warp-cooperative token scan, 1.23 TB/s,
+// profiles/r02_tokw_ab.jsonl); env GSYS_SCAN=dfa|token at load, gsys_set_scan() at run time
 std::atomic<int> g_scan_impl{[] {
     const char* e = getenv("GSYS_SCAN");
     return (e && strcmp(e, "token") == 0) ? (int)GSYS_SCAN_TOKEN
@@ -1030,7 +1060,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
     if (nch == 0) return 0;
     void* args[] = {&a};
     const void* fn = tok ? (const void*)wc_kernel<true> : (const void*)wc_kernel<false>;
-    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + (tok ? TWARP_STAGE : WARP_STAGE));
+    size_t smem = align_up(tb, 16) + (threads / 32) * (HSTRIDE * 4 + (tok ? TWWARP_STAGE : WARP_STAGE));
     rc = ensure_smem_attr(fn, smem);
     if (rc) return rc;
     if (cudaMemsetAsync(W->next_chunk_d, 0, 4, s) != cudaSuccess) return -EIO;
@@ -1073,9 +1103,10 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if ((uintptr_t)d_text % 16) return -EINVAL;
     const int impl = g_scan_impl.load();
     const bool tok = impl == GSYS_SCAN_TOKEN;
-    // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 32 warps
-    if (threads == 0) threads = tok ? 1024 : 704;
-    if (threads % 32 || threads > (tok ? 1024u : 768u)) return -EINVAL;
+    // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 24
+    // warps (2 staging buffers + a 2 KiB start list per warp)
+    if (threads == 0) threads = tok ? 768 : 704;
+    if (threads % 32 || threads > 768u) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
@@ -1088,7 +1119,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     // (profiles/r02_scan_staging_ab.jsonl: 33 small bulk copies per 2 KiB tile cost more than the
     // LSU slots they free), so it is the opt-in GSYS_SCAN_DFA_TMA
     const bool tma = impl == GSYS_SCAN_DFA_TMA;
-    const size_t per_warp = HSTRIDE * 4 + (tok ? TWARP_STAGE : tma ? MWARP_STAGE : WARP_STAGE);
+    const size_t per_warp = HSTRIDE * 4 + (tok ? TWWARP_STAGE : tma ? MWARP_STAGE : WARP_STAGE);
     if (!tok && tc->blob.size() + (threads / 32) * per_warp > kSmemDynMax) {
         tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);
         if (!tc) return rc;

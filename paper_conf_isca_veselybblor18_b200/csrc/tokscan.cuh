@@ -7,14 +7,13 @@
 // owned by the chunk holding its first byte; a dictionary hit is a whole token byte-equal to one
 // of <= 64 words of <= 16 bytes ("search for occurrences of 64 strings", PAPER.md:32 P32.6).
 //
-// Instead of one DFA lookup per byte (scan_core.cuh: a shared-memory gather per byte, bound by
-// bank conflicts), a lane classifies its 64-byte span four bytes per SWAR step into a 64-bit
-// word-byte mask, derives the token starts with two shifts, and visits only the tokens: the
-// length comes from the mask (one count-trailing-zeros), tokens of a length no dictionary word
-// has are skipped, the first 8 (16) bytes are read from the staged span, hashed, and looked up in a
-// collision-free hash table of the dictionary (the builder picks multipliers until the words land
-// in distinct slots), then verified byte-exactly -- about four shared-memory accesses per token
-// (mean token 5.8 bytes plus separators) instead of one per byte.
+// Instead of one DFA lookup per byte (scan_core.cuh: a dependent shared-memory gather per byte), a
+// warp classifies each lane's 64-byte span four bytes per SWAR step into word-byte masks, lists the
+// token starts of the whole 2 KiB tile (offset + length from the masks), and then looks the listed
+// tokens up with every lane taking every 32nd entry: the token's first 16 bytes (aligned shared
+// loads + funnel shifts), masked to its length, hashed into a collision-free table of the dictionary
+// (the builder picks multipliers until the words land in distinct slots), verified byte-exactly
+// against the slot's key.  Measured against the DFA in DESIGN.md sec. 6.
 #pragma once
 #include <stddef.h>
 
@@ -32,6 +31,8 @@ constexpr unsigned MAXD = 64;
 
 struct TokTables {
     gsys_scan::ScanTables g;    // grep part (patterns, first-byte filter); its DFA fields are unused
+    uint4 nokey;                // all 0xff: the "key" of an empty slot (no masked token equals it);
+                                // it sits right before key[0], so slot value id reads key[id - 1]
     uint4 key[MAXD];            // word d's bytes 0..15, zero-padded
     unsigned ndict;
     unsigned lenmask;           // bit L: some matchable dictionary word has length L (1..16)
@@ -85,76 +86,6 @@ GSYS_HD unsigned mask16(const uint4& q, unsigned one = 1u) {
     return pack16(word4(q.x, one), word4(q.y, one), word4(q.z, one), word4(q.w, one));
 }
 
-// Word-byte mask of the lane's 64-byte span W.w0..w3 (bit i = byte p0 + i).
-GSYS_HD unsigned long long mask64(const Win& W, unsigned one = 1u) {
-    const unsigned a = mask16(W.w0, one) | (mask16(W.w1, one) << 16);
-    const unsigned b = mask16(W.w2, one) | (mask16(W.w3, one) << 16);
-    return (unsigned long long)a | ((unsigned long long)b << 32);
-}
-
-GSYS_HD unsigned ctz32(unsigned x) {
-#ifdef __CUDA_ARCH__
-    return (unsigned)__ffs((int)x) - 1u;
-#else
-    return (unsigned)__builtin_ctz(x);
-#endif
-}
-
-GSYS_HD unsigned ctz64(unsigned long long x) {
-#ifdef __CUDA_ARCH__
-    return (unsigned)__ffsll((long long)x) - 1u;
-#else
-    return (unsigned)__builtin_ctzll(x);
-#endif
-}
-
-// The 8 bytes at p (any alignment) as two little-endian u32: two aligned 8-byte loads + funnel
-// shifts.  On the device p is a shared-memory address (explicit ld.shared: no generic-address
-// resolution per load).
-GSYS_HD void load8(const unsigned char* p, unsigned& lo, unsigned& hi) {
-#ifdef __CUDA_ARCH__
-    const unsigned a = (unsigned)__cvta_generic_to_shared(p);
-    const unsigned q = a & ~7u;
-    unsigned w0, w1, w2, w3;
-    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(w0), "=r"(w1) : "r"(q));
-    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2+8];" : "=r"(w2), "=r"(w3) : "r"(q));
-    const unsigned o = a & 7u;
-#else
-    const uintptr_t a = (uintptr_t)p;
-    const unsigned* qq = reinterpret_cast<const unsigned*>(a & ~(uintptr_t)7);
-    const unsigned o = (unsigned)(a & 7u);
-    const unsigned w0 = qq[0], w1 = qq[1], w2 = qq[2], w3 = qq[3];
-#endif
-    const bool s4 = o & 4u;
-    const unsigned u0 = s4 ? w1 : w0, u1 = s4 ? w2 : w1, u2 = s4 ? w3 : w2;
-    const unsigned sh = (o & 3u) * 8u;
-    lo = GSYS_FSHR(u0, u1, sh);
-    hi = GSYS_FSHR(u1, u2, sh);
-}
-
-// 0xffffffff >> s with s clamped to [0, 32] (32 or more: 0)
-GSYS_HD unsigned shr_ones(int s) {
-    s = s < 0 ? 0 : s;
-#ifdef __CUDA_ARCH__
-    unsigned r;
-    asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(0xffffffffu), "r"((unsigned)s));   // PTX clamps shifts >= 32
-    return r;
-#else
-    return s >= 32 ? 0u : 0xffffffffu >> s;
-#endif
-}
-
-// Keep the first n (n >= 1) bytes of (lo, hi): bytes 0..3 in lo, 4..7 in hi.
-GSYS_HD void keep8(unsigned& lo, unsigned& hi, unsigned n) {
-    lo &= shr_ones(32 - 8 * (int)n);
-    hi &= shr_ones(64 - 8 * (int)n);
-}
-
-// The tokens owned by one lane span.  span: the span's bytes p0.. in memory (at least 96 readable
-// bytes; bytes at or past valid_end are never part of a token because the masks exclude them);
-// M: word-byte mask of the 64 span bytes; la: the mask of the 16 bytes after them; prev_word:
-// byte p0-1 exists and is a word byte.  Owned token starts are [p0, min(p0+64, own_end)); a token
-// may run up to 16 bytes into the lookahead (longer ones cannot match).  emit(d): one hit of word d.
 // Table fields a lane keeps in registers for the whole scan.
 struct TokRegs {
     unsigned lenmask, m0, m1, m4;
@@ -175,83 +106,174 @@ GSYS_HD unsigned tok_slot(const TokTables& T, const TokRegs& R, unsigned h) {
 #ifdef __CUDA_ARCH__
     unsigned v;
     asm("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(R.tabs + (unsigned)offsetof(TokTables, slot) + h));
-    return v & 0xffu;
+    return v;   // ld.u8 into a 32-bit register zero-extends
 #else
     (void)R;
     return T.slot[h];
 #endif
 }
-GSYS_HD void tok_key(const TokTables& T, const TokRegs& R, unsigned d, uint4& k, unsigned& klen) {
-#ifdef __CUDA_ARCH__
-    asm("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(k.x), "=r"(k.y), "=r"(k.z), "=r"(k.w)
-        : "r"(R.tabs + (unsigned)offsetof(TokTables, key) + 16u * d));
-    asm("ld.shared.u8 %0, [%1];" : "=r"(klen) : "r"(R.tabs + (unsigned)offsetof(TokTables, klen) + d));
-    klen &= 0xffu;
-#else
-    (void)R;
-    k = T.key[d];
-    klen = T.klen[d];
-#endif
-}
+// ------------------------------------------------------------------ warp-cooperative token scan
+// Round-2 form of the token path.  The first version ran each lane's tokens in a
+// lane-serial loop, so a warp spent as many rounds as its busiest lane had tokens (1.5-1.7x the
+// mean) on ~130-instruction iterations.  Here a warp tile is handled in two phases:
+//   A  every lane lists the token starts of its 64-byte span -- one u16 entry per start: the
+//      token's byte offset in the staged tile and its length (a few instructions per token);
+//   C  the warp's list is looked up with lane j taking entries j, j+32, ... (even work per lane):
+//      5 aligned shared loads + 4 funnel shifts give the first 16 bytes, a multiply hash of the
+//      first 8 and the length picks the dictionary slot, one 16-byte key load (predicated: only
+//      lanes whose slot is taken) verifies the whole token.
+// Entry: bits 0..11 = offset in the staged tile (lane * TOKW_SLOT + q), bits 12..15 = length - 1;
+// TOKW_SKIP for a start no dictionary word can match (length > 16 or not in lenmask).  TOKW_SKIP
+// decodes like an entry (offset 32 * TOKW_SLOT, the tile's tail area -- inside the staging buffer,
+// which holds TOKW_TILE bytes -- length 1), so phase C runs it through the same straight-line
+// lookup and only its final emit is gated off.
+constexpr unsigned TOKW_SLOT = 80;          // staged lane slot: the 64 span bytes + the 16 after them
+constexpr unsigned TOKW_SKIP = 32u * TOKW_SLOT;
+constexpr unsigned TOKW_TILE = 32u * TOKW_SLOT + 32u;   // a staged tile: slots, the 4 bytes before it, guard
+constexpr unsigned TOKW_LIST = 1024;        // entries per warp tile (at most one start per 2 bytes)
 
-// The tokens starting at the positions set in S (bit q = byte 32*half + q of the span): lo, hi are
-// the word-byte mask of that half and of the 32 bytes after it, so the run of word bytes from q is
-// one funnel shift away; a token of 32+ word bytes leaves no zero in the window (length > 16).
-template <class Emit>
-GSYS_HD void tok_visit(const TokTables& T, const TokRegs& R, const unsigned char* span, unsigned half, unsigned S,
-                       unsigned lo, unsigned hi, Emit&& emit) {
-    while (S) {
-        const unsigned q = ctz32(S);
-        S &= S - 1u;
-        const unsigned w = GSYS_FSHR(lo, hi, q);
-        const unsigned len = ~w ? ctz32(~w) : 32u;
-        if (!((R.lenmask >> (len & 31u)) & 1u) || len > 16u) continue;
-        const unsigned char* t = span + 32u * half + q;
-        unsigned a, b;
-        load8(t, a, b);
-        keep8(a, b, len);
-        const unsigned id = tok_slot(T, R, ((a * R.m0) ^ (b * R.m1) ^ (len * R.m4)) >> (32u - HBITS));
-        if (!id) continue;
-        uint4 k;
-        unsigned klen;
-        tok_key(T, R, id - 1u, k, klen);
-        if (klen != len || k.x != a || k.y != b) continue;
-        if (len > 8u) {   // bytes 8..15: only for the few long words
-            unsigned c, d;
-            load8(t + 8u, c, d);
-            keep8(c, d, len - 8u);
-            if (k.z != c || k.w != d) continue;
-        }
-        emit(id - 1u);
-    }
-}
-
-// The tokens owned by one lane span.  span: the span's bytes p0.. in memory (at least 80 readable
-// bytes; bytes at or past valid_end are never part of a token because the masks exclude them);
-// M: word-byte mask of the 64 span bytes; la: the mask of the 16 bytes after them; prev_word:
-// byte p0-1 exists and is a word byte.  Owned token starts are [p0, min(p0+64, own_end)); a token
-// may run up to 16 bytes into the lookahead (longer ones cannot match).  emit(d): one hit of word d.
-template <class Emit>
-GSYS_HD void tok_lane64(const TokTables& T, const TokRegs& R, const unsigned char* span, unsigned long long M,
-                        unsigned la, bool prev_word, long long p0, long long own_end, long long valid_end,
-                        Emit&& emit) {
+// The owned token starts of one lane span and its word-byte masks.  m0, m1: bytes 0..31, 32..63 of
+// the span; m2: the 32 bytes after it (at least the first 16 exact); prev_word: byte p0-1 exists
+// and is a word byte.  Bytes at or past valid_end never belong to a token; starts at or past
+// own_end are not owned.
+struct TokwSpan {
+    unsigned s0, s1;        // starts among bytes 0..31 / 32..63
+    unsigned m0, m1, m2;
+};
+GSYS_HD TokwSpan tokw_span(unsigned m0, unsigned m1, unsigned m2, bool prev_word, long long p0, long long own_end,
+                           long long valid_end) {
     const long long nvalid_ll = valid_end - p0;
-    if (nvalid_ll < 80) {   // end of data: bytes at or past valid_end terminate tokens
+    if (nvalid_ll < 96) {
         const unsigned nv = nvalid_ll <= 0 ? 0u : (unsigned)nvalid_ll;
-        if (nv < 64u) { M &= nv ? (~0ull >> (64u - nv)) : 0ull; la = 0u; }
-        else la &= (1u << (nv - 64u)) - 1u;
+        m0 &= nv >= 32u ? ~0u : ((1u << nv) - 1u);
+        m1 &= nv >= 64u ? ~0u : (nv <= 32u ? 0u : ((1u << (nv - 32u)) - 1u));
+        m2 &= nv <= 64u ? 0u : ((1u << (nv - 64u)) - 1u);
     }
-    const unsigned m0 = (unsigned)M, m1 = (unsigned)(M >> 32), m2 = la & 0xffffu;
-    unsigned s0 = m0 & ~((m0 << 1) | (prev_word ? 1u : 0u));
-    unsigned s1 = m1 & ~((m1 << 1) | (m0 >> 31));
+    TokwSpan r;
+    r.m0 = m0;
+    r.m1 = m1;
+    r.m2 = m2;
+    r.s0 = m0 & ~((m0 << 1) | (prev_word ? 1u : 0u));
+    r.s1 = m1 & ~((m1 << 1) | (m0 >> 31));
     const long long nown_ll = own_end - p0;
     if (nown_ll < 64) {
         const unsigned no = nown_ll <= 0 ? 0u : (unsigned)nown_ll;
-        s0 &= no >= 32u ? 0xffffffffu : ((1u << no) - 1u);
-        s1 &= no <= 32u ? 0u : ((1u << (no - 32u)) - 1u);
+        r.s0 &= no >= 32u ? ~0u : ((1u << no) - 1u);
+        r.s1 &= no <= 32u ? 0u : ((1u << (no - 32u)) - 1u);
     }
-    tok_visit(T, R, span, 0u, s0, m0, m1, emit);
-    tok_visit(T, R, span, 1u, s1, m1, m2, emit);
+    return r;
+}
+
+GSYS_HD unsigned tokw_brev(unsigned x) {
+#ifdef __CUDA_ARCH__
+    return __brev(x);
+#else
+    x = ((x >> 1) & 0x55555555u) | ((x & 0x55555555u) << 1);
+    x = ((x >> 2) & 0x33333333u) | ((x & 0x33333333u) << 2);
+    x = ((x >> 4) & 0x0f0f0f0fu) | ((x & 0x0f0f0f0fu) << 4);
+    x = ((x >> 8) & 0x00ff00ffu) | ((x & 0x00ff00ffu) << 8);
+    return (x >> 16) | (x << 16);
+#endif
+}
+GSYS_HD unsigned tokw_fshl(unsigned lo, unsigned hi, unsigned sh) {   // upper 32 bits of (hi:lo) << (sh & 31)
+#ifdef __CUDA_ARCH__
+    return __funnelshift_l(lo, hi, sh);
+#else
+    sh &= 31u;
+    return sh ? (hi << sh) | (lo >> (32u - sh)) : hi;
+#endif
+}
+
+// Position of the highest set bit (x != 0): one FLO (PTX bfind).
+GSYS_HD unsigned tokw_hibit(unsigned x) {
+#ifdef __CUDA_ARCH__
+    unsigned r;
+    asm("bfind.u32 %0, %1;" : "=r"(r) : "r"(x));
+    return r;
+#else
+    return 31u - (unsigned)__builtin_clz(x);
+#endif
+}
+
+// Phase A: one entry per start of the span; put(entry) appends it.  slot_off = the span's offset
+// in the staged tile.  Starts are taken highest first (one FLO each); the token length comes from
+// the bit-reversed 64-bit window of the mask as a count of leading ones: p = the highest 0 of the
+// shifted window (a guard bit at 14 caps the count at 17), len = 31 - p.  lenrev is lenmask
+// reversed (bit 31 - L for length L), so it is tested at p directly.
+template <class Put>
+GSYS_HD void tokw_list(const TokRegs& R, const TokwSpan& sp, unsigned slot_off, Put&& put) {
+    const unsigned lenrev = tokw_brev(R.lenmask);
+GSYS_UNROLL
+    for (int h = 0; h < 2; h++) {
+        unsigned S = h ? sp.s1 : sp.s0;
+        const unsigned lo = h ? sp.m1 : sp.m0, hi = h ? sp.m2 : sp.m1;
+        const unsigned ylo = tokw_brev(hi), yhi = tokw_brev(lo);   // the 64-bit window reversed
+        // entry = (slot_off + 32h + q) | ((len - 1) << 12) = base + q - (p << 12), len = 31 - p
+        const unsigned base = slot_off + 32u * (unsigned)h + (30u << 12);
+        while (S) {
+            const unsigned q = tokw_hibit(S);
+            S ^= 1u << q;
+            const unsigned z = tokw_fshl(ylo, yhi, q);        // bit 31 - k = mask bit q + k
+            const unsigned p = tokw_hibit(~z | 0x4000u);      // 31 - (run of word bytes from q), run <= 17
+            put(((lenrev >> p) & 1u) ? base + q - (p << 12) : TOKW_SKIP);
+        }
+    }
+}
+
+// The staged tile: a pointer (host emulation) and its shared-window address (device).
+struct TokwTile {
+    const unsigned char* p;
+    unsigned s;
+};
+GSYS_HD unsigned tokw_ld32(const TokwTile& t, unsigned off) {   // off: 4-byte aligned
+#ifdef __CUDA_ARCH__
+    unsigned v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(t.s + off));
+    return v;
+#else
+    unsigned v;
+    memcpy(&v, t.p + off, 4);
+    return v;
+#endif
+}
+// Phase C: look up one entry; emit(d) counts a hit of word d.  Straight-line: the 16 bytes at the
+// token start (5 aligned loads, 4 funnel shifts), masked to the token's length; the slot of
+// (first 8 bytes, length); the slot's key (an empty slot reads `nokey`, which equals no token);
+// a hit is all 16 bytes equal -- keys are zero-padded and word bytes are never 0, so equal masked
+// bytes mean equal lengths too.
+template <class Emit>
+GSYS_HD void tokw_lookup(const TokTables& T, const TokRegs& R, const TokwTile& tile, unsigned e, Emit&& emit) {
+    const unsigned off = e & 0xfffu, len = (e >> 12) + 1u;
+    const unsigned a4 = off & ~3u;
+    const unsigned sh = off * 8u;   // funnel shifts take the amount mod 32
+    const unsigned w0 = tokw_ld32(tile, a4), w1 = tokw_ld32(tile, a4 + 4u), w2 = tokw_ld32(tile, a4 + 8u);
+    const unsigned w3 = tokw_ld32(tile, a4 + 12u), w4 = tokw_ld32(tile, a4 + 16u);
+    // bytes 0..len-1 kept: two 64-bit shifts (PTX clamps shift amounts at the width); ALU work
+    // instead of a mask-table load -- the lookups are bound by the shared-memory pipe
+    const unsigned n8 = 8u * len, m8 = n8 > 64u ? n8 - 64u : 0u;
+    unsigned long long k0, k1;
+#ifdef __CUDA_ARCH__
+    asm("shl.b64 %0, %1, %2;" : "=l"(k0) : "l"(~0ull), "r"(n8));
+    asm("shl.b64 %0, %1, %2;" : "=l"(k1) : "l"(~0ull), "r"(m8));
+#else
+    k0 = n8 >= 64u ? 0ull : (~0ull << n8);
+    k1 = m8 >= 64u ? 0ull : (~0ull << m8);
+#endif
+    const unsigned a = GSYS_FSHR(w0, w1, sh) & ~(unsigned)k0, b = GSYS_FSHR(w1, w2, sh) & ~(unsigned)(k0 >> 32);
+    const unsigned c = GSYS_FSHR(w2, w3, sh) & ~(unsigned)k1, d = GSYS_FSHR(w3, w4, sh) & ~(unsigned)(k1 >> 32);
+    const unsigned id = tok_slot(T, R, ((a * R.m0) ^ (b * R.m1) ^ (len * R.m4)) >> (32u - HBITS));
+    // the slot's key, loaded only by lanes whose slot is taken (a predicated load: no branch, and
+    // lanes with an empty slot add no shared-memory wavefronts); an empty slot keeps `nokey`
+    uint4 k = make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu);
+#ifdef __CUDA_ARCH__
+    asm volatile("{ .reg .pred p; setp.ne.u32 p, %4, 0;\n\t"
+                 "@p ld.shared.v4.u32 {%0, %1, %2, %3}, [%5]; }"
+                 : "+r"(k.x), "+r"(k.y), "+r"(k.z), "+r"(k.w)
+                 : "r"(id), "r"(R.tabs + (unsigned)offsetof(TokTables, nokey) + 16u * id));
+#else
+    if (id) k = T.key[id - 1u];
+#endif
+    if (((a ^ k.x) | (b ^ k.y) | (c ^ k.z) | (d ^ k.w)) == 0u && e != TOKW_SKIP) emit(id - 1u);
 }
 
 // ------------------------------------------------------------------ host: table builder
@@ -267,6 +289,7 @@ inline int build_tok_tables(void* out, size_t cap, const char* dict, const uint8
     if (!out || cap < sizeof(TokTables)) return -ENOSPC;
     TokTables* T = (TokTables*)out;
     memset(T, 0, sizeof *T);
+    memset(&T->nokey, 0xff, sizeof T->nokey);
     T->ndict = ndict;
     T->one = 1u;
     bool match[MAXD] = {false};

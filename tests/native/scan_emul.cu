@@ -59,30 +59,43 @@ static int run(const uint8_t* text, uint64_t n, uint32_t chunk, const std::vecto
     return 0;
 }
 
-// Token-level scan (tokscan.cuh) over 64-byte lane spans exactly as the kernels run them: the span
-// mask, the lookahead mask (the kernels take it from the next lane), the previous byte's class.
-static int run_tok(const uint8_t* text, uint64_t n, uint32_t chunk, const gsys_tok::TokTables& T, uint64_t* hist,
-                   uint32_t npat, bool* any_out) {
-    std::vector<uint8_t> buf(n + 160, 'a');
-    if (n) memcpy(buf.data(), text, n);
+// Warp-cooperative token scan (tokscan.cuh tokw_*) exactly as scan_range_tokw runs it: per 2 KiB
+// warp tile from each chunk start, the 32 lane spans staged in 80-byte slots, every lane's word
+// masks, the next lane's first 32 mask bits as lookahead (lane 31: the 16 staged bytes after the
+// tile), phase A lists the starts of all lanes in lane order, phase C looks every entry up.
+static int run_tokw(const uint8_t* text, uint64_t n, uint32_t chunk, const gsys_tok::TokTables& T, uint64_t* hist,
+                    uint32_t npat, bool* any_out) {
     bool any = false;
     const long long N = (long long)n;
+    const gsys_tok::TokRegs R = gsys_tok::tok_regs(T);
+    std::vector<uint8_t> tile(gsys_tok::TOKW_TILE, 0);
+    auto byte_at = [&](long long q) -> uint8_t { return (q >= 0 && q < N) ? text[q] : 0; };
     for (uint64_t s = 0; s < n; s += chunk) {
-        const uint64_t e = s + chunk < n ? s + chunk : n;
-        for (uint64_t p0 = s; p0 < e; p0 += 64) {
-            uint4 V[5];
-            for (int k = 0; k < 5; k++) {
-                const uint64_t q = p0 + 16 * k;
-                if (q < n) memcpy(&V[k], &buf[q], 16);
-                else V[k] = make_uint4(0, 0, 0, 0);
+        const long long e = (long long)(s + chunk < n ? s + chunk : n);
+        for (long long base = (long long)s; base < e; base += 2048) {
+            Win W[32];
+            unsigned m0[32], m1[32], m2[32];
+            for (unsigned l = 0; l < 32; l++) {
+                const long long p0 = base + 64ll * l;
+                for (unsigned i = 0; i < gsys_tok::TOKW_SLOT; i++) tile[l * gsys_tok::TOKW_SLOT + i] = byte_at(p0 + i);
+                uint4 V[5];
+                for (int k = 0; k < 5; k++) memcpy(&V[k], &tile[l * gsys_tok::TOKW_SLOT + 16 * k], 16);
+                W[l] = Win{V[0], V[1], V[2], V[3], V[4]};
+                m0[l] = gsys_tok::mask16(V[0]) | (gsys_tok::mask16(V[1]) << 16);
+                m1[l] = gsys_tok::mask16(V[2]) | (gsys_tok::mask16(V[3]) << 16);
             }
-            Win W{V[0], V[1], V[2], V[3], V[4]};
-            const unsigned long long M = gsys_tok::mask64(W);
-            const unsigned la = gsys_tok::mask16(W.w4);
-            const bool prev_word = p0 > 0 && is_word_byte(buf[p0 - 1]);
-            gsys_tok::tok_lane64(T, gsys_tok::tok_regs(T), &buf[p0], M, la, prev_word, (long long)p0, (long long)e, N,
-                                 [hist](unsigned d) { hist[d]++; });
-            if (npat && !any && grep_lane64(T.g, W, (long long)p0, (long long)e, N)) any = true;
+            for (unsigned l = 0; l < 32; l++) m2[l] = l < 31 ? m0[l + 1] : gsys_tok::mask16(W[31].w4);
+            std::vector<unsigned> list;
+            for (unsigned l = 0; l < 32; l++) {
+                const long long p0 = base + 64ll * l;
+                const bool pw = l ? ((m1[l - 1] >> 31) & 1u) : (p0 > 0 && is_word_byte(byte_at(p0 - 1)));
+                const gsys_tok::TokwSpan sp = gsys_tok::tokw_span(m0[l], m1[l], m2[l], pw, p0, e, N);
+                gsys_tok::tokw_list(R, sp, l * gsys_tok::TOKW_SLOT, [&list](unsigned x) { list.push_back(x); });
+                if (npat && !any && p0 < e && grep_lane64(T.g, W[l], p0, e, N)) any = true;
+            }
+            if (list.size() > gsys_tok::TOKW_LIST) return -E2BIG;
+            const gsys_tok::TokwTile t{tile.data(), 0u};
+            for (unsigned x : list) gsys_tok::tokw_lookup(T, R, t, x, [hist](unsigned d) { hist[d]++; });
         }
     }
     *any_out = any;
@@ -91,7 +104,7 @@ static int run_tok(const uint8_t* text, uint64_t n, uint32_t chunk, const gsys_t
 
 // mode 0: 16-byte reference steps, narrow table; 1: 64-byte lane spans, narrow table (wc_kernel);
 // 2: 64-byte lane spans, wide table (scan_kernel); 3: 16-byte reference steps, wide table;
-// 4: token-level lane spans (tokscan.cuh).
+// 4: warp-cooperative token scan (tokscan.cuh tokw_*).
 extern "C" int scan_emul2(const uint8_t* text, uint64_t n, uint32_t chunk, const char* dict, const uint8_t* dlen,
                           uint32_t ndict, const char* pats, const uint8_t* plen, uint32_t npat, uint64_t* hist,
                           uint32_t* hit, int mode) {
@@ -101,7 +114,8 @@ extern "C" int scan_emul2(const uint8_t* text, uint64_t n, uint32_t chunk, const
         int rc = gsys_tok::build_tok_tables(tt.data(), tt.size() * 16, dict, dlen, ndict, pats, plen, npat, nullptr);
         if (rc) return rc;
         bool any = false;
-        rc = run_tok(text, n, chunk, *reinterpret_cast<const gsys_tok::TokTables*>(tt.data()), hist, npat, &any);
+        const auto& TT = *reinterpret_cast<const gsys_tok::TokTables*>(tt.data());
+        rc = run_tokw(text, n, chunk, TT, hist, npat, &any);
         if (hit) *hit = any ? 1u : 0u;
         return rc;
     }

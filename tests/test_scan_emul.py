@@ -38,7 +38,8 @@ def emul():
         for mode in (1, 2, 3, 4):
             # 1: wc_kernel's 64-byte lane spans (77-column table); 2: scan_kernel's lane spans (129
             # columns, raw-byte fast path); 3: 16-byte reference steps on the 129-column table;
-            # 4: the token-level lane spans (tokscan.cuh)
+            # 4: the warp-cooperative token scan (tokscan.cuh tokw_*: per-tile start lists, then
+            # lookups)
             h, g = run2(text, words, pats, chunk, mode)
             assert np.array_equal(h0, h) and g0 == g, mode
         return h0, g0

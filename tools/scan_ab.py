@@ -18,8 +18,10 @@ text = torch.cat([torch.from_file(p, dtype=torch.uint8, size=os.path.getsize(p))
 n = text.numel()
 words, pats = inputs.dictionary(), inputs.patterns()
 want_hit = int(any(c.pmasks[:64]))
-cells = [(G.SCAN_TOKEN, 1024, 256)] + [(G.SCAN_DFA_TMA, t, 256) for t in (704, 512, 768)] + \
-        [(G.SCAN_DFA, 704, 256)]
+IMPL = {"token": G.SCAN_TOKEN, "dfa_tma": G.SCAN_DFA_TMA, "dfa": G.SCAN_DFA}
+# SCAN_AB_CELLS="token:768:256,dfa:704:256" (impl:threads:chunk_kib) picks the cells
+cells = [(IMPL[i], int(t), int(k)) for i, t, k in (x.split(":") for x in os.environ.get(
+    "SCAN_AB_CELLS", "token:768:256,dfa_tma:704:256,dfa:704:256").split(","))]
 for impl, threads, ck in cells:
     G.gsys_set_scan(impl)
     chunk = ck << 10
