@@ -615,7 +615,7 @@ def config1_latency(G, W, dev, words, pats, root):
 
 def wg_syscall_rate(G, W, dev, path):
     """The metric's other half, "GPU-issued syscalls/sec (WG granularity)": 592 work-groups
-    (4/SM x 256 threads), each cell calibrated then run for >= 100 ms of calls.  getrusage blocking
+    (4/SM x 256 threads), each cell calibrated until one pass runs >= 150 ms of calls.  getrusage blocking
     and non-blocking; 4 KiB preads into device memory, blocking (the pull path, reading B12) and
     non-blocking (deferred pulls, reading B15)."""
     import torch
@@ -631,13 +631,16 @@ def wg_syscall_rate(G, W, dev, path):
                                   ("pread4k_device_nonblocking", "pread", G.WG | G.NONBLOCKING | G.RELAXED)):
             kw = dict(fd=fd, length=4096, size=size, d_buf=dbuf) if kind == "pread" else {}
             iters = 20
-            for _ in range(2):   # calibration pass, then the >= 100 ms pass
+            for _ in range(4):   # calibration passes until one pass lasts >= 150 ms (launch, ramp
+                # and the final drain are then a few per cent of it)
                 torch.cuda.synchronize()
                 t0 = time.perf_counter()
                 _, ret, lat, _, rc = W.bench_calls(kind, flags, blocks, threads, iters, **kw)
                 dt = time.perf_counter() - t0
                 rate = blocks * iters / dt
-                iters = int(min(max(20, rate * 0.1 / blocks), 4000))
+                if dt >= 0.15 or iters >= 4000:
+                    break
+                iters = int(min(max(20, rate * 0.25 / blocks), 4000))
             lat_us = (lat.double() / 1e3).cpu()
             blocking = not (flags & G.NONBLOCKING)
             ok = bool((ret == (4096 if kind == "pread" else 0)).all()) if blocking else bool((ret == 0).all())
