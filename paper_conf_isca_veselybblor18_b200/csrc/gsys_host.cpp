@@ -358,6 +358,8 @@ struct Worker {
     BounceRing<Tok, RingOps>* ring = nullptr;
     uint8_t* bounce_d = nullptr;     // device address of the (host-mapped) bounce
     DeferRing defer;                 // deferred pulls of non-blocking preads (B15)
+    DeferRing defer2;                // overflow store, allocated the first time `defer` is full
+    bool defer2_failed = false;      // its allocation failed: overflow takes the copy engine
     // destination -> ring position of the newest deferred pull this worker served into it
     // (overflow ordering).  Written by this worker only, so its lines stay in this core's cache;
     // the rare overflow reader takes every worker's lock and the newest pending entry
@@ -479,6 +481,8 @@ struct Instance {
     std::deque<std::shared_ptr<Split>> splits;
     std::atomic<int> nsplits{0};
     uint64_t split_min = 128u << 10;      // env GSYS_SPLIT_KB (0 = never split)
+    size_t defer_grow = 64u << 20;        // per-worker overflow store for deferred pulls, allocated
+                                          // on first overflow (env GSYS_DEFER_GROW_MB, 0 = none)
     Sharded st_split;                      // preads served in pieces
     Sharded st_deferred;                   // non-blocking preads served as deferred pulls (B15)
     Sharded st_flushed;                    // ... of which copied by gsys_wait's flush
@@ -817,8 +821,38 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
     uintptr_t dst = (uintptr_t)r.a[1];
     uint8_t* hp = nullptr;
     if (resolve(dst, n, &hp) != PK_DEVICE) return false;
-    const uint64_t want = std::min<uint64_t>(std::min<uint64_t>(n, GSYS_PREAD_CAP), defer.cap);
-    const size_t o = defer.alloc(want, r.pos);
+    uint64_t want = std::min<uint64_t>(std::min<uint64_t>(n, GSYS_PREAD_CAP), defer.cap);
+    DeferRing* st = &defer;
+    size_t o = defer.alloc(want, r.pos);
+    if (o == ~(size_t)0 && inst->defer_grow) {
+        // the store is full of pulls nobody has consumed yet (many callers, e.g. work-item
+        // granularity): a second, larger store takes the overflow -- allocated once, on demand,
+        // so callers that never fill the first keep its smaller, cache-friendlier footprint
+        if (!defer2.h && !defer2_failed) {
+            Timer tm(t_cuda);
+            uint8_t* hp = nullptr;
+            uint8_t* dp = nullptr;
+            if (cudaHostAlloc((void**)&hp, inst->defer_grow, cudaHostAllocMapped | cudaHostAllocPortable) ==
+                    cudaSuccess &&
+                cudaHostGetDevicePointer((void**)&dp, hp, 0) == cudaSuccess) {
+                std::lock_guard<std::mutex> g(defer2.mu);   // gsys_wait's flush reads the store under it
+                defer2.recs = defer.recs;
+                defer2.mask = defer.mask;
+                defer2.cap = inst->defer_grow;
+                defer2.d = dp;
+                defer2.h = hp;
+            } else {
+                cudaGetLastError();
+                if (hp) cudaFreeHost(hp);
+                defer2_failed = true;
+            }
+        }
+        if (defer2.h) {
+            want = std::min<uint64_t>(std::min<uint64_t>(n, GSYS_PREAD_CAP), defer2.cap);
+            o = defer2.alloc(want, r.pos);
+            st = &defer2;
+        }
+    }
     if (o == ~(size_t)0) {
         // the range store is full of pulls nobody has consumed yet: this request takes the
         // copy-engine path -- after any pending pull into the same buffer has landed (by copy
@@ -843,7 +877,7 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
         return false;
     }
     ssize_t z;
-    { Timer tm(t_sys); z = pread(fd, defer.h + o, want, off); }
+    { Timer tm(t_sys); z = pread(fd, st->h + o, want, off); }
     inst->st_host_preads.fetch_add(1, std::memory_order_relaxed);
     *ret = z < 0 ? -(int64_t)errno : (int64_t)z;
     if (z > 0) inst->st_bytes_read.fetch_add((uint64_t)z, std::memory_order_relaxed);
@@ -855,7 +889,7 @@ bool Worker::try_defer(Req& r, int fd, uint64_t n, int64_t off, int64_t* ret) {
         Timer tm(t_cuda);
         inst->flush_deferred(stream, false, r.pos - inst->ring_cap, false);
     }
-    __atomic_store_n(&rec.src, z > 0 ? (uint64_t)(uintptr_t)(defer.d + o) : 0ull, __ATOMIC_RELAXED);
+    __atomic_store_n(&rec.src, z > 0 ? (uint64_t)(uintptr_t)(st->d + o) : 0ull, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.dst, (uint64_t)dst, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.ret, (long long)*ret, __ATOMIC_RELAXED);
     __atomic_store_n(&rec.consumed, z > 0 ? 0u : 1u, __ATOMIC_RELAXED);   // nothing to copy: free at once
@@ -1624,6 +1658,8 @@ int make_instance(uint32_t slots, uint32_t window_us, Instance** out) {
     c.wd = I->wd_d;
     ev = getenv("GSYS_DEFER_MB");   // per worker; 0 = non-blocking device-buffer preads by DMA
     const size_t defer_mb = ev ? (size_t)atoll(ev) : 16;
+    ev = getenv("GSYS_DEFER_GROW_MB");
+    I->defer_grow = (size_t)(ev ? atoll(ev) : 64) << 20;
     c.nbrec = defer_mb ? (gsys_nbrec*)I->nbrec_d : nullptr;
     c.pull_big_bytes = I->pull_bytes;
     c.pull_big = I->pull_d;
@@ -1934,16 +1970,18 @@ int Instance::flush_deferred(cudaStream_t st, bool upto_all, uint32_t upto, bool
     std::lock_guard<std::mutex> fg(flush_mu);
     std::vector<std::pair<uint32_t, FlushRec>> all;   // (ring position, record)
     const uint32_t h = (uint32_t)head.load(std::memory_order_acquire);
+    (void)h;
     for (Worker* w : workers) {
-        if (!w->defer.h) continue;
-        std::lock_guard<std::mutex> g(w->defer.mu);
-        for (const DeferRing::Region& rg : w->defer.q) {
-            gsys_nbrec& r = nbrec_h[rg.pos & (ring_cap - 1)];
-            if (w->defer.consumed(rg) || !r.src || r.ret <= 0) continue;
-            if (!upto_all && (int32_t)(rg.pos - upto) > 0) continue;
-            if (only_dst && r.dst != only_dst) continue;
-            (void)h;
-            all.push_back({rg.pos, FlushRec{r.src, r.dst, r.ret, &nbrec_d[rg.pos & (ring_cap - 1)].consumed, rg.pos, 0u}});
+        for (DeferRing* dr : {&w->defer, &w->defer2}) {
+            std::lock_guard<std::mutex> g(dr->mu);
+            if (!dr->h) continue;
+            for (const DeferRing::Region& rg : dr->q) {
+                gsys_nbrec& r = nbrec_h[rg.pos & (ring_cap - 1)];
+                if (dr->consumed(rg) || !r.src || r.ret <= 0) continue;
+                if (!upto_all && (int32_t)(rg.pos - upto) > 0) continue;
+                if (only_dst && r.dst != only_dst) continue;
+                all.push_back({rg.pos, FlushRec{r.src, r.dst, r.ret, &nbrec_d[rg.pos & (ring_cap - 1)].consumed, rg.pos, 0u}});
+            }
         }
     }
     if (all.empty()) return 0;
@@ -2208,6 +2246,7 @@ int gsys_shutdown(void) {
         cudaStreamDestroy(w->stream);
         cudaFreeHost(w->bounce);
         if (w->defer.h) cudaFreeHost(w->defer.h);
+        if (w->defer2.h) cudaFreeHost(w->defer2.h);
         delete w;
     }
     cudaFreeHost(I->area_h);

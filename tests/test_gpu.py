@@ -1072,8 +1072,9 @@ def test_nonblocking_device_preads_are_deferred_and_land(file1m, side_stream):
 
 def test_deferred_pull_ring_overflow_falls_back(tmpdir_shm, file1m):
     """With a 1 MiB deferred range store per worker, 64 KiB non-blocking preads overflow it: the
-    rest take the copy-engine path, each after any pending pull into the same buffer has landed;
-    every buffer still ends with the caller's last read (a fresh process: the size is fixed at init)."""
+    rest take the overflow store (GSYS_DEFER_GROW_MB, allocated on the first overflow) and then the
+    copy-engine path, each after any pending pull into the same buffer has landed; every buffer
+    still ends with the caller's last read (fresh processes: the sizes are fixed at init)."""
     import subprocess
     import sys
     code = f"""
@@ -1099,6 +1100,16 @@ for c in range(blocks):
 assert rc == 0 and 0 < st['deferred'] < blocks * iters and st['flushed'] > 0, st
 print('ok', st['deferred'], st['flushed'])
 """
-    env = dict(os.environ, GSYS_DEFER_MB="1", GSYS_THREADS="4")
+    env = dict(os.environ, GSYS_DEFER_MB="1", GSYS_DEFER_GROW_MB="0", GSYS_THREADS="4")
     out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-3000:]
+    # with a 1 MiB overflow store allocated on the first overflow: deferred pulls land in both
+    # stores, the copy engine takes what neither holds, every buffer still ends with the last read
+    env = dict(os.environ, GSYS_DEFER_MB="1", GSYS_DEFER_GROW_MB="1", GSYS_THREADS="4")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-3000:]
+    # a store large enough for everything: no copy-engine overflow at all
+    code_all = code.replace("0 < st['deferred'] < blocks * iters", "st['deferred'] == blocks * iters")
+    env = dict(os.environ, GSYS_DEFER_MB="1", GSYS_DEFER_GROW_MB="16", GSYS_THREADS="4")
+    out = subprocess.run([sys.executable, "-c", code_all], env=env, capture_output=True, text=True, timeout=300)
     assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-3000:]
