@@ -269,6 +269,21 @@ def test_scan_device_degenerate(scan_impl, words, pats, size):
     assert hit == oracle.grep(arr, pats)
 
 
+@pytest.mark.parametrize("pattern", [b"a ", b" a", b"ab ", b"a b c d e f g h ", b"aaaaaaaaaaaaaaaaa ", b"9_"])
+def test_scan_device_dense_tokens(scan_impl, pattern):
+    """Token-dense text: one token per 2 bytes fills the warp-cooperative scan's start list to its
+    1024-entry maximum per 2 KiB tile; 1-byte words at every start, 17-byte tokens (too long to
+    match) at the other extreme; ragged sizes around the tile and the chunk."""
+    words = [b"a", b"b", b"ab", b"h", b"9_", b"aaaaaaaaaaaaaaaa"]
+    for size in (2048, 2049, 4095, (1 << 20) + 3):
+        text = (pattern * (size // len(pattern) + 1))[:size]
+        arr = np.frombuffer(text, dtype=np.uint8)
+        for chunk in (16, 2048, 256 << 10):
+            hist, hit = _scan_dev(text, words, [b"b c"], chunk)
+            assert np.array_equal(hist, oracle.count_tokens(arr, words)[:len(words)]), (pattern, size, chunk)
+            assert hit == oracle.grep(arr, [b"b c"])
+
+
 def test_scan_device_large_trie_uses_narrow_table(scan_impl):
     """A dictionary whose 129-column table no longer fits next to 16 warps' staging (482 trie
     states + 30 emission states) runs on the 77-column table: same counts."""

@@ -112,3 +112,17 @@ def test_scan_emul_duplicate_and_nonword_dictionary_entries(emul):
         hist, _ = emul(text, words, [], chunk)
         assert np.array_equal(hist, oracle.count_tokens(text, words))
         assert hist[1] == 0 and hist[2] == 0
+
+
+@pytest.mark.parametrize("pattern", [b"a ", b" a", b"ab ", b"a b c d e f g h ", b"aaaaaaaaaaaaaaaaa ", b"9_"])
+def test_scan_emul_dense_tokens(emul, pattern):
+    """One token per 2 bytes (the token scan's per-tile start list at its 1024-entry maximum),
+    1-byte and 16-byte words, 17-byte tokens; every scan form equals the oracle."""
+    words = [b"a", b"b", b"ab", b"h", b"9_", b"aaaaaaaaaaaaaaaa"]
+    for size in (2048, 2049, 4095, 70_001):
+        text = (pattern * (size // len(pattern) + 1))[:size]
+        arr = np.frombuffer(text, dtype=np.uint8)
+        for chunk in (16, 2048, 256 << 10):
+            h, g = emul(arr, words, [b"b c"], chunk)
+            assert np.array_equal(h, oracle.count_tokens(arr, words)[:len(words)]), (pattern, size, chunk)
+            assert g == oracle.grep(arr, [b"b c"])
