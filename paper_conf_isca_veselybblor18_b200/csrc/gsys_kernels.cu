@@ -232,8 +232,11 @@ __device__ __forceinline__ void stage_tile_tok(unsigned buf, const unsigned char
 // start counts are prefix-summed with shuffles and every lane appends its entries to the warp's
 // list in shared memory; phase C -- lane j looks up entries j, j+32, ... of that list.
 constexpr unsigned TWWARP_STAGE = 2 * gsys_tok::TOKW_TILE + 2 * gsys_tok::TOKW_LIST;
-static_assert(SLOT == gsys_tok::TOKW_SLOT && gsys_tok::TOKW_TILE >= 33 * SLOT,
-              "stage_tile_tok's lane slots and 'previous' word must fit the token scan's tile layout");
+// stage_tile_tok fills 32 lane slots and the 4-byte "previous" word at 32 * SLOT; a lookup reads 20
+// bytes from its (4-byte aligned) offset, TOKW_SKIP's included
+static_assert(SLOT == gsys_tok::TOKW_SLOT && gsys_tok::TOKW_SKIP == 32 * SLOT &&
+                  gsys_tok::TOKW_SKIP + 20 <= gsys_tok::TOKW_TILE,
+              "the token scan's tile layout must match stage_tile_tok's slots");
 
 __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                                 long long valid_end, const ScanState& S) {
