@@ -231,7 +231,11 @@ __device__ __forceinline__ void stage_tile_tok(unsigned buf, const unsigned char
 // scan_range; tiles staged by stage_tile_tok): per tile, phase A -- each lane classifies its span, the lanes'
 // start counts are prefix-summed with shuffles and every lane appends its entries to the warp's
 // list in shared memory; phase C -- lane j looks up entries j, j+32, ... of that list.
-constexpr unsigned TWWARP_STAGE = 2 * gsys_tok::TOKW_TILE + 2 * gsys_tok::TOKW_LIST;
+#ifndef GSYS_TOK_NBUF
+#define GSYS_TOK_NBUF 1     // staged tiles per warp: 1 lets 32 warps fit (their copies cover each
+                            // other's latency); 2 overlaps the next tile's copies within a warp
+#endif
+constexpr unsigned TWWARP_STAGE = GSYS_TOK_NBUF * gsys_tok::TOKW_TILE + 2 * gsys_tok::TOKW_LIST;
 // stage_tile_tok fills 32 lane slots and the 4-byte "previous" word at 32 * SLOT; a lookup reads 20
 // bytes from its (4-byte aligned) offset, TOKW_SKIP's included
 static_assert(SLOT == gsys_tok::TOKW_SLOT && gsys_tok::TOKW_SKIP == 32 * SLOT &&
@@ -245,7 +249,7 @@ __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict_
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     unsigned char* stage = S.stage + warp * TWWARP_STAGE;
     const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
-    const unsigned list_s = stage_s + 2u * gsys_tok::TOKW_TILE;
+    const unsigned list_s = stage_s + GSYS_TOK_NBUF * gsys_tok::TOKW_TILE;
     const unsigned hs = (unsigned)__cvta_generic_to_shared(S.whist);
     auto emit = [hs](unsigned d) { asm volatile("red.shared.add.u32 [%0], 1;" :: "r"(hs + 4u * d) : "memory"); };
     gsys_tok::TokRegs R = gsys_tok::tok_regs(T);
@@ -255,13 +259,21 @@ __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict_
     const unsigned one = T.one;
     const long long step = 2048ll * nwarps;
     long long base = s + 2048ll * warp;
+#if GSYS_TOK_NBUF == 2
     if (base < own_end) stage_tile_tok(stage_s, seg0, s, base, valid_end, lane);
     cp_async_commit();
-    for (unsigned it = 0; base < own_end; base += step, it ^= 1u) {
+#endif
+    for (unsigned it = 0; base < own_end; base += step, it ^= (GSYS_TOK_NBUF - 1u)) {
+#if GSYS_TOK_NBUF == 2
         const long long nxt = base + step;
         if (nxt < own_end) stage_tile_tok(stage_s + (it ^ 1u) * gsys_tok::TOKW_TILE, seg0, s, nxt, valid_end, lane);
         cp_async_commit();
         cp_async_wait<1>();
+#else   // one tile per warp: its copies are waited for at once (other warps cover the latency)
+        stage_tile_tok(stage_s, seg0, s, base, valid_end, lane);
+        cp_async_commit();
+        cp_async_wait<0>();
+#endif
         __syncwarp();
         const unsigned char* buf = stage + it * gsys_tok::TOKW_TILE;
         const unsigned buf_s = stage_s + it * gsys_tok::TOKW_TILE;
@@ -303,11 +315,14 @@ __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict_
         __syncwarp();
         {   // phase C
             const gsys_tok::TokwTile tile{buf, buf_s};
-#pragma unroll 2
-            for (unsigned j = lane; j < n; j += 32u) {
-                unsigned e;
-                asm volatile("ld.shared.u16 %0, [%1];" : "=r"(e) : "r"(list_s + 2u * j) : "memory");
-                gsys_tok::tokw_lookup(T, R, tile, e & 0xffffu, emit);
+            // two entries per round (j, j + 32): their loads are independent, so the lookups'
+            // shared-memory latencies overlap (four per round measured slower: registers)
+            for (unsigned j = lane; j < n; j += 64u) {
+                unsigned e0, e1 = gsys_tok::TOKW_SKIP;
+                asm volatile("ld.shared.u16 %0, [%1];" : "=r"(e0) : "r"(list_s + 2u * j) : "memory");
+                if (j + 32u < n) asm volatile("ld.shared.u16 %0, [%1];" : "=r"(e1) : "r"(list_s + 2u * j + 64u) : "memory");
+                gsys_tok::tokw_lookup(T, R, tile, e0 & 0xffffu, emit);
+                gsys_tok::tokw_lookup(T, R, tile, e1 & 0xffffu, emit);
             }
         }
         __syncwarp();                // every lane is done with this buffer and the list before reuse
@@ -710,7 +725,10 @@ __global__ void __launch_bounds__(768, 1) scan_tma_kernel(ScanArgs a) {
 }
 
 // Token-level scan of HBM-resident text (gsys_tok): 1 block of up to 32 warps per SM.
-__global__ void __launch_bounds__(768, 1) scan_tok_kernel(ScanArgs a) {
+#ifndef GSYS_TOK_MAXT
+#define GSYS_TOK_MAXT 1024  // token scan threads per block (register budget 65536 / GSYS_TOK_MAXT)
+#endif
+__global__ void __launch_bounds__(GSYS_TOK_MAXT, 1) scan_tok_kernel(ScanArgs a) {
     __shared__ int s_hit;
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
@@ -848,8 +866,8 @@ struct Workspace {
 Workspace g_ws[64];
 std::mutex g_ws_mu;
 // scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.47 TB/s on the
-// 1 GiB HBM scan) or GSYS_SCAN_TOKEN (warp-cooperative token scan, 1.23 TB/s,
-// profiles/r02_tokw_ab.jsonl); env GSYS_SCAN=dfa|token at load, gsys_set_scan() at run time
+// 1 GiB HBM scan) or GSYS_SCAN_TOKEN (warp-cooperative token scan, 1.38 TB/s,
+// profiles/r02_tokbuf2.jsonl); env GSYS_SCAN=dfa|token at load, gsys_set_scan() at run time
 std::atomic<int> g_scan_impl{[] {
     const char* e = getenv("GSYS_SCAN");
     return (e && strcmp(e, "token") == 0) ? (int)GSYS_SCAN_TOKEN
@@ -1108,10 +1126,10 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if ((uintptr_t)d_text % 16) return -EINVAL;
     const int impl = g_scan_impl.load();
     const bool tok = impl == GSYS_SCAN_TOKEN;
-    // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 24
-    // warps (2 staging buffers + a 2 KiB start list per warp)
-    if (threads == 0) threads = tok ? 768 : 704;
-    if (threads % 32 || threads > 768u) return -EINVAL;
+    // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 32
+    // warps (one staged tile + a 2 KiB start list per warp; profiles/r02_tokbuf2.jsonl)
+    if (threads == 0) threads = tok ? 1024 : 704;
+    if (threads % 32 || threads > (tok ? (unsigned)GSYS_TOK_MAXT : 768u)) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;

@@ -227,8 +227,10 @@ struct TokwTile {
 };
 GSYS_HD unsigned tokw_ld32(const TokwTile& t, unsigned off) {   // off: 4-byte aligned
 #ifdef __CUDA_ARCH__
+    // not volatile: the address depends on a list entry loaded after the warp's barrier, and the
+    // staged bytes do not change during the lookups, so the compiler may interleave two lookups
     unsigned v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(t.s + off));
+    asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(t.s + off));
     return v;
 #else
     unsigned v;
@@ -266,10 +268,10 @@ GSYS_HD void tokw_lookup(const TokTables& T, const TokRegs& R, const TokwTile& t
     // lanes with an empty slot add no shared-memory wavefronts); an empty slot keeps `nokey`
     uint4 k = make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu);
 #ifdef __CUDA_ARCH__
-    asm volatile("{ .reg .pred p; setp.ne.u32 p, %4, 0;\n\t"
-                 "@p ld.shared.v4.u32 {%0, %1, %2, %3}, [%5]; }"
-                 : "+r"(k.x), "+r"(k.y), "+r"(k.z), "+r"(k.w)
-                 : "r"(id), "r"(R.tabs + (unsigned)offsetof(TokTables, nokey) + 16u * id));
+    asm("{ .reg .pred p; setp.ne.u32 p, %4, 0;\n\t"
+        "@p ld.shared.v4.u32 {%0, %1, %2, %3}, [%5]; }"
+        : "+r"(k.x), "+r"(k.y), "+r"(k.z), "+r"(k.w)
+        : "r"(id), "r"(R.tabs + (unsigned)offsetof(TokTables, nokey) + 16u * id));
 #else
     if (id) k = T.key[id - 1u];
 #endif
