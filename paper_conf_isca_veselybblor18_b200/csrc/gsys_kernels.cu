@@ -257,6 +257,10 @@ __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict_
     // rebuild them from SR_CgaCtaId inside the lookup loop)
     asm volatile("mov.b32 %0, %0;" : "+r"(R.tabs));
     const unsigned one = T.one;
+    // grep's first-byte prefilter (grep_lane64): SWAR range constants; g_all -- no prefilter (a
+    // pattern starting with a byte >= 0x80)
+    const bool g_all = T.g.fb_hi >= 0x80u;
+    const unsigned g_add_lo = (0x80u - T.g.fb_lo) * 0x01010101u, g_add_hi = (0x7fu - T.g.fb_hi) * 0x01010101u;
     const long long step = 2048ll * nwarps;
     long long base = s + 2048ll * warp;
 #if GSYS_TOK_NBUF == 2
@@ -287,8 +291,12 @@ __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict_
             W.w2 = *reinterpret_cast<const uint4*>(span + 32u);
             W.w3 = *reinterpret_cast<const uint4*>(span + 48u);
             W.w4 = *reinterpret_cast<const uint4*>(span + 64u);
-            const unsigned m0 = gsys_tok::mask16(W.w0, one) | (gsys_tok::mask16(W.w1, one) << 16);
-            const unsigned m1 = gsys_tok::mask16(W.w2, one) | (gsys_tok::mask16(W.w3, one) << 16);
+            // word-byte masks, with grep's first-byte prefilter fused into the same pass
+            unsigned gacc = 0;
+            const unsigned m0 = gsys_tok::mask16g(W.w0, one, g_add_lo, g_add_hi, gacc) |
+                                (gsys_tok::mask16g(W.w1, one, g_add_lo, g_add_hi, gacc) << 16);
+            const unsigned m1 = gsys_tok::mask16g(W.w2, one, g_add_lo, g_add_hi, gacc) |
+                                (gsys_tok::mask16g(W.w3, one, g_add_lo, g_add_hi, gacc) << 16);
             unsigned m2 = __shfl_down_sync(0xffffffffu, m0, 1);
             if (lane == 31u) m2 = gsys_tok::mask16(W.w4, one);
             unsigned pw = __shfl_up_sync(0xffffffffu, m1 >> 31, 1);
@@ -296,7 +304,9 @@ __device__ __forceinline__ void scan_range_tokw(const unsigned char* __restrict_
             // the block's "a pattern was seen" flag, read once per warp tile (an atomic read, set by
             // atomic writes: the early exit is an optimisation, not a synchronisation)
             const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
-            if (grep && !seen && p0 < own_end && grep_lane64(T.g, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
+            if (grep && !seen && p0 < own_end && (g_all || (gacc & 0x80808080u)) &&
+                grep_lane64_steps(T.g, W, p0, own_end, valid_end))
+                atomicExch(S.hit, 1);
             const gsys_tok::TokwSpan sp = gsys_tok::tokw_span(m0, m1, m2, pw != 0u, p0, own_end, valid_end);
             const unsigned cnt = (unsigned)__popc(sp.s0) + (unsigned)__popc(sp.s1);
             unsigned incl = cnt;

@@ -356,7 +356,19 @@ GSYS_UNROLL
     }
 }
 
-// grep over a lane's span: the four 16-byte steps with their 32-byte windows.
+// grep's exact part over a lane's span: the four 16-byte steps with their 32-byte windows.
+GSYS_HD bool grep_lane64_steps(const ScanTables& T, const Win& W, long long p0, long long own_end,
+                               long long valid_end) {
+GSYS_UNROLL
+    for (int k = 0; k < 4; k++) {
+        const long long q = p0 + 16 * k;
+        if (q >= own_end) break;
+        if (grep_step(T, W.get((unsigned)k), W.get((unsigned)k + 1u), q, own_end, valid_end)) return true;
+    }
+    return false;
+}
+
+// grep over a lane's span: a SWAR first-byte prefilter, then the exact steps.
 GSYS_HD bool grep_lane64(const ScanTables& T, const Win& W, long long p0, long long own_end, long long valid_end) {
     if (T.npat == 0) return false;
     if (T.fb_hi < 0x80u) {
@@ -372,13 +384,7 @@ GSYS_HD bool grep_lane64(const ScanTables& T, const Win& W, long long p0, long l
                              r(W.w3.z) | r(W.w3.w);
         if (!(acc & 0x80808080u)) return false;
     }
-GSYS_UNROLL
-    for (int k = 0; k < 4; k++) {
-        const long long q = p0 + 16 * k;
-        if (q >= own_end) break;
-        if (grep_step(T, W.get((unsigned)k), W.get((unsigned)k + 1u), q, own_end, valid_end)) return true;
-    }
-    return false;
+    return grep_lane64_steps(T, W, p0, own_end, valid_end);
 }
 
 // Whole step (wordcount + grep) for one segment -- the reference composition used by the host

@@ -86,6 +86,26 @@ GSYS_HD unsigned mask16(const uint4& q, unsigned one = 1u) {
     return pack16(word4(q.x, one), word4(q.y, one), word4(q.z, one), word4(q.w, one));
 }
 
+// word4() plus grep's first-byte prefilter on the same 7-bit byte values (grep_lane64's SWAR
+// range test, fused: two IMADs and one LOP3 more per 4 bytes); gacc collects bit 7 of every byte
+// whose low 7 bits fall in the patterns' first-byte range.
+GSYS_HD unsigned word4g(unsigned w, unsigned one, unsigned add_lo, unsigned add_hi, unsigned& gacc) {
+    const unsigned a = w & 0x7f7f7f7fu;
+    gacc |= (a * one + add_lo) & ~(a * one + add_hi);
+    const unsigned x = a | 0x20202020u;
+    const unsigned g1 = x * one + 0x1f1f1f1fu;
+    const unsigned g2 = x * one + 0x05050505u;
+    const unsigned g3 = a * one + 0x50505050u;
+    const unsigned g4 = a * one + 0x46464646u;
+    const unsigned nu = (a ^ 0x5f5f5f5fu) * one + 0x7f7f7f7fu;
+    const unsigned v = (g1 & ~g2) | (g3 & ~g4);
+    return (v | ~nu) & ~w & 0x80808080u;
+}
+GSYS_HD unsigned mask16g(const uint4& q, unsigned one, unsigned add_lo, unsigned add_hi, unsigned& gacc) {
+    return pack16(word4g(q.x, one, add_lo, add_hi, gacc), word4g(q.y, one, add_lo, add_hi, gacc),
+                  word4g(q.z, one, add_lo, add_hi, gacc), word4g(q.w, one, add_lo, add_hi, gacc));
+}
+
 // Table fields a lane keeps in registers for the whole scan.
 struct TokRegs {
     unsigned lenmask, m0, m1, m4;
