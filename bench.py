@@ -534,6 +534,23 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
         e1.record(s)
         e1.synchronize()
     t = e0.elapsed_time(e1) / 1e3 / reps
+    # the selectable warp-cooperative token scan on the same text (GSYS_SCAN_TOKEN, 32 warps/SM)
+    tok = None
+    prev = G.gsys_set_scan(G.SCAN_TOKEN)
+    try:
+        with torch.cuda.stream(s):
+            for _ in range(3):
+                G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 1024, s)
+            t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            t0.record(s)
+            for _ in range(reps):
+                G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 1024, s)
+            t1.record(s)
+            t1.synchronize()
+        tok = {"kernel": "scan_tok_kernel (warp-cooperative token scan, 1 block/SM x 1024 threads)",
+               "achieved": n / (t0.elapsed_time(t1) / 1e3 / reps) / 1e9, "unit": "GB/s"}
+    finally:
+        G.gsys_set_scan(prev)
     peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
     ach = n / t / 1e9
@@ -565,6 +582,7 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
                            "peak_source": "profiles/r02_probes.jsonl (tools/probes/b200_probes.cu)"}
     return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "bytes": n,
             "traffic": traffic, "limiter": limiter, "ms": t * 1e3, "compute_roofline": compute,
+            "token_scan": dict(tok, frac=tok["achieved"] / peak) if tok else None,
             "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 704 threads (22 warps), 77-column transposed DFA in shared memory; 6 % above 512 threads with the 129-column table, profiles/r01_scan_threads_sweep.jsonl)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
 
