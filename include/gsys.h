@@ -346,7 +346,7 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
  * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n] (16-byte aligned); file
  * boundaries are not modelled (one file).  Adds into d_hist (NULL allowed when ndict == 0); d_hit (may be NULL) set to 1 if any
  * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 1024 (token scan)
- * or 704 (DFA scan), else a multiple of 32 up to 1024 (token) / 768 (DFA; its 129-column table is
+ * or 768 (DFA scan), else a multiple of 32 up to 1024 (token) / 768 (DFA; its 129-column table is
  * used when it fits beside the warps' staging, else the 77-column one).  -EINVAL on bad
  * sizes/alignment, -ENODEV before gsys_init. */
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,

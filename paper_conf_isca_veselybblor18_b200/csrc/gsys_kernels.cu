@@ -1136,9 +1136,9 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if ((uintptr_t)d_text % 16) return -EINVAL;
     const int impl = g_scan_impl.load();
     const bool tok = impl == GSYS_SCAN_TOKEN;
-    // DFA: 22 warps + the 77-column table (6 % above 16 warps + the 129-column one); token: 32
+    // DFA: 24 warps + the 77-column table (profiles/r02_dfa_threads.jsonl: 1 % above 22); token: 32
     // warps (one staged tile + a 2 KiB start list per warp; profiles/r02_tokbuf2.jsonl)
-    if (threads == 0) threads = tok ? 1024 : 704;
+    if (threads == 0) threads = tok ? 1024 : 768;
     if (threads % 32 || threads > (tok ? (unsigned)GSYS_TOK_MAXT : 768u)) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
