@@ -525,12 +525,12 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
     s = torch.cuda.Stream(device=dev)
     with torch.cuda.stream(s):
         for _ in range(3):
-            G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 768, s)
+            G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 1024, s)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         reps = 10
         e0.record(s)
         for _ in range(reps):
-            G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 768, s)
+            G.gsys_scan_device(text, n, chunk, words, pats, hist, hit, 0, 1024, s)
         e1.record(s)
         e1.synchronize()
     t = e0.elapsed_time(e1) / 1e3 / reps
@@ -583,7 +583,7 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
     return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "bytes": n,
             "traffic": traffic, "limiter": limiter, "ms": t * 1e3, "compute_roofline": compute,
             "token_scan": dict(tok, frac=tok["achieved"] / peak) if tok else None,
-            "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 768 threads (24 warps), 77-column transposed DFA in shared memory; 1 % above 704 threads, profiles/r02_dfa_threads.jsonl)",
+            "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 1024 threads (32 warps, one staged tile each), 129-column transposed DFA in shared memory; profiles/r02_dfa32.jsonl)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
 
 

@@ -345,9 +345,10 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
 /* Same scan over text already resident in device memory (no syscalls): the standalone scan
  * kernel measured against the HBM roofline.  d_text: DEVICE bytes [n] (16-byte aligned); file
  * boundaries are not modelled (one file).  Adds into d_hist (NULL allowed when ndict == 0); d_hit (may be NULL) set to 1 if any
- * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 1024 (token scan)
- * or 768 (DFA scan), else a multiple of 32 up to 1024 (token) / 768 (DFA; its 129-column table is
- * used when it fits beside the warps' staging, else the 77-column one).  -EINVAL on bad
+ * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 1024 (704 for
+ * GSYS_SCAN_DFA_TMA), else a
+ * multiple of 32 up to 1024 (768 for GSYS_SCAN_DFA_TMA); the DFA's 129-column table is used when it
+ * fits beside the warps' staging, else the 77-column one.  -EINVAL on bad
  * sizes/alignment, -ENODEV before gsys_init. */
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
                      const char* dict, const uint8_t* dlen, uint32_t ndict,

@@ -105,7 +105,15 @@ __device__ __forceinline__ void red_emit2(unsigned hb, unsigned hi, unsigned lo,
 // lookahead.  Every byte crosses the memory system once.
 constexpr unsigned SLOT = 80;
 constexpr unsigned STAGE_BYTES = 33 * SLOT + 16;       // slots + the 4-byte "previous" word (padded)
-constexpr unsigned WARP_STAGE = 2 * STAGE_BYTES;       // double buffer
+constexpr unsigned WARP_STAGE = 2 * STAGE_BYTES;       // double buffer (wc_kernel)
+#ifndef GSYS_DFA_NBUF
+#define GSYS_DFA_NBUF 1     // staged tiles per warp of the HBM DFA scan (scan_kernel): one tile lets
+                            // 32 warps and the 129-column table fit (profiles/r02_dfa32.jsonl)
+#endif
+#ifndef GSYS_DFA_MAXT
+#define GSYS_DFA_MAXT 1024  // scan_kernel threads per block
+#endif
+constexpr unsigned DWARP_STAGE = GSYS_DFA_NBUF * STAGE_BYTES;
 
 __device__ __forceinline__ void cp_async16(unsigned dst, const void* src, unsigned src_bytes) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(src), "r"(src_bytes) : "memory");
@@ -156,7 +164,9 @@ __device__ __forceinline__ void stage_tile(unsigned buf, const unsigned char* se
     }
 }
 
-template <int P, bool WIDE>
+// NBUF: staged tiles per warp -- 2 (wc_kernel: the next tile's copies, over PCIe in host staging,
+// overlap this tile's scan) or 1 (HBM scan: more warps fit, and they cover each other's latency)
+template <int P, bool WIDE, unsigned NBUF = 2>
 __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg0, long long s, long long own_end,
                                            long long valid_end, const ScanState& S) {
     const ScanTables& T = *S.T;
@@ -167,17 +177,25 @@ __device__ __forceinline__ void scan_range(const unsigned char* __restrict__ seg
     auto emit = [hb, emit2](unsigned e) { red_emit(hb, e, emit2); };
     auto emit2x = [hb, emit2](unsigned hi, unsigned lo) { red_emit2(hb, hi, lo, emit2); };
     const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    unsigned char* stage = S.stage + warp * WARP_STAGE;
+    unsigned char* stage = S.stage + warp * NBUF * STAGE_BYTES;
     const unsigned stage_s = (unsigned)__cvta_generic_to_shared(stage);
     const long long step = 2048ll * nwarps;
     long long base = s + 2048ll * warp;
-    if (base < own_end) stage_tile(stage_s, seg0, s, base, valid_end, lane);
-    cp_async_commit();
-    for (unsigned it = 0; base < own_end; base += step, it ^= 1u) {
-        const long long nxt = base + step;
-        if (nxt < own_end) stage_tile(stage_s + (it ^ 1u) * STAGE_BYTES, seg0, s, nxt, valid_end, lane);
+    if (NBUF == 2) {
+        if (base < own_end) stage_tile(stage_s, seg0, s, base, valid_end, lane);
         cp_async_commit();
-        cp_async_wait<1>();          // this tile's copies (issued one iteration earlier) have landed
+    }
+    for (unsigned it = 0; base < own_end; base += step, it ^= (NBUF - 1u)) {
+        if (NBUF == 2) {
+            const long long nxt = base + step;
+            if (nxt < own_end) stage_tile(stage_s + (it ^ 1u) * STAGE_BYTES, seg0, s, nxt, valid_end, lane);
+            cp_async_commit();
+            cp_async_wait<1>();      // this tile's copies (issued one iteration earlier) have landed
+        } else {
+            stage_tile(stage_s, seg0, s, base, valid_end, lane);
+            cp_async_commit();
+            cp_async_wait<0>();
+        }
         __syncwarp();
         const unsigned char* buf = stage + it * STAGE_BYTES;
         Win W;
@@ -683,7 +701,7 @@ struct ScanArgs {
     unsigned chunk, pad_;
 };
 
-__global__ void __launch_bounds__(768, 1) scan_kernel(ScanArgs a) {
+__global__ void __launch_bounds__(GSYS_DFA_MAXT, 1) scan_kernel(ScanArgs a) {
     __shared__ int s_hit;
     extern __shared__ __align__(16) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
@@ -696,8 +714,8 @@ __global__ void __launch_bounds__(768, 1) scan_kernel(ScanArgs a) {
     for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         const long long s = (long long)k * a.chunk;
         const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
-        if (sT.ncol == NCOL_WIDE) scan_range<LD_NC, true>(a.text + s, s, e, (long long)a.n, S);
-        else scan_range<LD_NC, false>(a.text + s, s, e, (long long)a.n, S);
+        if (sT.ncol == NCOL_WIDE) scan_range<LD_NC, true, GSYS_DFA_NBUF>(a.text + s, s, e, (long long)a.n, S);
+        else scan_range<LD_NC, false, GSYS_DFA_NBUF>(a.text + s, s, e, (long long)a.n, S);
     }
     __syncthreads();
     flush_hist(shist, nwarps, sT.ndict, a.hist);
@@ -1136,10 +1154,11 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     if ((uintptr_t)d_text % 16) return -EINVAL;
     const int impl = g_scan_impl.load();
     const bool tok = impl == GSYS_SCAN_TOKEN;
-    // DFA: 24 warps + the 77-column table (profiles/r02_dfa_threads.jsonl: 1 % above 22); token: 32
+    // DFA: 32 warps with one staged tile each + the 129-column table (profiles/r02_dfa32.jsonl:
+    // 1.67 TB/s against 1.48 for 24 double-buffered warps + the 77-column one); token: 32
     // warps (one staged tile + a 2 KiB start list per warp; profiles/r02_tokbuf2.jsonl)
-    if (threads == 0) threads = tok ? 1024 : 768;
-    if (threads % 32 || threads > (tok ? (unsigned)GSYS_TOK_MAXT : 768u)) return -EINVAL;
+    if (threads == 0) threads = impl == GSYS_SCAN_DFA_TMA ? 704 : 1024;
+    if (threads % 32 || threads > (tok ? (unsigned)GSYS_TOK_MAXT : impl == GSYS_SCAN_DFA_TMA ? 768u : (unsigned)GSYS_DFA_MAXT)) return -EINVAL;
     std::lock_guard<std::mutex> g(g_ws_mu);
     Workspace* W = workspace();
     if (!W) return -ENODEV;
@@ -1152,7 +1171,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     // (profiles/r02_scan_staging_ab.jsonl: 33 small bulk copies per 2 KiB tile cost more than the
     // LSU slots they free), so it is the opt-in GSYS_SCAN_DFA_TMA
     const bool tma = impl == GSYS_SCAN_DFA_TMA;
-    const size_t per_warp = HSTRIDE * 4 + (tok ? TWWARP_STAGE : tma ? MWARP_STAGE : WARP_STAGE);
+    const size_t per_warp = HSTRIDE * 4 + (tok ? TWWARP_STAGE : tma ? MWARP_STAGE : DWARP_STAGE);
     if (!tok && tc->blob.size() + (threads / 32) * per_warp > kSmemDynMax) {
         tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);
         if (!tc) return rc;

@@ -12,8 +12,8 @@ hit = torch.zeros(1, dtype=torch.int32, device="cuda")
 tok = len(sys.argv) > 1 and sys.argv[1] == "token"
 if tok:
     G.gsys_set_scan(G.SCAN_TOKEN)
-for _ in range(3):   # the bench's launch: 1 block/SM x 768 (DFA) / 1024 (token) threads, grep on
+for _ in range(3):   # the bench's launch: 1 block/SM x 1024 threads, grep on
     G.gsys_scan_device(text, text.numel(), 256 << 10, inputs.dictionary(), inputs.patterns(), hist, hit, 0,
-                       1024 if tok else 768)
+                       1024)
 torch.cuda.synchronize()
 print("ok")
