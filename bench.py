@@ -556,15 +556,15 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
     ach = n / t / 1e9
     del text
     traffic, limiter = None, None
-    summ = os.path.join(ROOT, "profiles", "r01_ncu_summary.json")
-    if os.path.exists(summ):   # the ncu --set full capture of the same 1 GiB scan
-        sk = json.load(open(summ)).get("scan_kernel_1GiB", {})
+    summ = os.path.join(ROOT, "profiles", "r02_scan_dfa32_ncu.json")
+    if os.path.exists(summ):   # ncu --set full of the same 1 GiB scan in this launch configuration (base units)
         try:
-            traffic = (float(sk["dram_read_bytes"]) + float(sk["dram_write_bytes"])) * n / (64 * (16 << 20))
-            limiter = (f"shared-memory pipe: l1tex {float(sk['l1tex__throughput.avg.pct_of_peak_sustained_active']):.0f}% "
-                       f"of peak (DFA lookups, bank conflicts), issue "
-                       f"{float(sk['smsp__issue_active.avg.pct_of_peak_sustained_active']):.0f}%")
-        except (KeyError, ValueError):
+            kv = json.load(open(summ))
+            traffic = (kv["dram__bytes_read.sum"]["value"] + kv["dram__bytes_write.sum"]["value"]) * n / kv["text_bytes"]
+            limiter = (f"shared-memory pipe: l1tex {kv['l1tex__throughput.avg.pct_of_peak_sustained_active']['value']:.0f}% "
+                       f"of peak (DFA gathers, 3.3 wavefronts per warp lookup), issue "
+                       f"{kv['smsp__issue_active.avg.pct_of_peak_sustained_active']['value']:.0f}%")
+        except (KeyError, ValueError, TypeError):
             pass
     # compute-side roofline: one random 16-bit shared-memory gather per byte (the DFA
     # lookup), against the measured random-gather rate of tools/probes/b200_probes.cu
