@@ -17,6 +17,7 @@
 // a predicated shared RED into the warp's histogram.  grep tests every owned position whose byte
 // is in the first-byte range of the patterns.  No tensor cores: nothing here is a contraction.
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <errno.h>
 #include <stdint.h>
@@ -692,29 +693,117 @@ __global__ void __launch_bounds__(256, 2) wc_kernel(WcArgs a) {
 
 // ------------------------------------------------------------------ scan of HBM-resident text
 struct ScanArgs {
+    CUtensorMap tmap;               // the text as rows of 64 bytes, 33-row boxes, 64B swizzle (tma_rows > 0)
     const ScanTables* tables;
     const unsigned char* text;
     unsigned long long n;
     unsigned long long* hist;
     unsigned* hit;
     unsigned long long nchunks;
-    unsigned chunk, pad_;
+    unsigned chunk;
+    unsigned tma_rows;              // full 64-byte rows in the tensor map (0: no tensor-map staging)
 };
 
-__global__ void __launch_bounds__(GSYS_DFA_MAXT, 1) scan_kernel(ScanArgs a) {
+// ------------------------------------------------------------------ DFA scan with swizzled TMA tiles
+// One 2 KiB warp tile (+ the 64-byte row after it) arrives as ONE tensor copy: 33 rows of 64 bytes
+// with the hardware 64B swizzle (16-byte chunk c of row r at chunk c ^ ((r >> 1) & 3)), so lane l
+// reads row l's chunks (and row l+1's first one) conflict-free with no padding and the staging uses
+// no LSU wavefronts.  Tiles that are not whole rows inside the tensor (chunk starts off a 64-byte
+// boundary, the text's last partial row) are copied by the lanes into the same swizzled layout,
+// zero-filled past valid_end.
+constexpr unsigned SW_ROWS = 33, SW_BYTES = SW_ROWS * 64;        // 2112
+constexpr unsigned SW_STRIDE = 2560;                               // per warp, keeps 512-B alignment
+__device__ __forceinline__ unsigned swz(unsigned row, unsigned chunk) {   // byte offset in a tile
+    return row * 64u + 16u * (chunk ^ ((row >> 1) & 3u));
+}
+__device__ __forceinline__ void stage_tile_swz_lanes(unsigned buf, const unsigned char* seg0, long long s, long long base,
+                                                     long long valid_end, unsigned lane) {
+    for (unsigned i = lane; i < SW_ROWS * 4u; i += 32u) {
+        const unsigned row = i >> 2, c = i & 3u;
+        const long long p = base + 64ll * row + 16ll * c;
+        const long long left = valid_end - p;
+        const unsigned nb = left >= 16 ? 16u : (left > 0 ? (unsigned)left : 0u);
+        cp_async16(buf + swz(row, c), seg0 + (nb ? p - s : 0), nb);
+    }
+}
+template <bool WIDE>
+__device__ __forceinline__ void scan_range_swz(const ScanArgs& a, const unsigned char* __restrict__ seg0, long long s,
+                                               long long own_end, long long valid_end, const ScanState& S,
+                                               unsigned char* tiles, unsigned mbar, unsigned& phase) {
+    const ScanTables& T = *S.T;
+    const Dfa<WIDE> D = dfa_view_shared<WIDE>(T);
+    const bool grep = S.hit != nullptr && T.npat > 0;
+    const unsigned emit2 = D.emit2;
+    const unsigned hb = (unsigned)__cvta_generic_to_shared(S.whist) - 2u * emit2;
+    auto emit = [hb, emit2](unsigned e) { red_emit(hb, e, emit2); };
+    auto emit2x = [hb, emit2](unsigned hi, unsigned lo) { red_emit2(hb, hi, lo, emit2); };
+    const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    unsigned char* buf = tiles + warp * SW_STRIDE;
+    const unsigned buf_s = (unsigned)__cvta_generic_to_shared(buf);
+    const long long step = 2048ll * nwarps;
+    for (long long base = s + 2048ll * warp; base < own_end; base += step) {
+        const bool tma = (base & 63) == 0 && base + 2048 + 64 <= 64ll * a.tma_rows;
+        if (tma) {
+            if (lane == 0u) {
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(mbar), "r"(SW_BYTES) : "memory");
+                asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                             :: "r"(buf_s), "l"(reinterpret_cast<unsigned long long>(&a.tmap)), "r"(0), "r"((int)(base >> 6)),
+                                "r"(mbar) : "memory");
+            }
+            mbar_wait(mbar, phase);
+            phase ^= 1u;
+        } else {
+            stage_tile_swz_lanes(buf_s, seg0, s, base, valid_end, lane);
+            cp_async_commit();
+            cp_async_wait<0>();
+        }
+        __syncwarp();
+        Win W;
+        W.w0 = *reinterpret_cast<const uint4*>(buf + swz(lane, 0));
+        W.w1 = *reinterpret_cast<const uint4*>(buf + swz(lane, 1));
+        W.w2 = *reinterpret_cast<const uint4*>(buf + swz(lane, 2));
+        W.w3 = *reinterpret_cast<const uint4*>(buf + swz(lane, 3));
+        W.w4 = *reinterpret_cast<const uint4*>(buf + swz(lane + 1u, 0));
+        const long long p0 = base + 64ll * lane;
+        unsigned prevb;
+        if (lane) prevb = buf[swz(lane - 1u, 3) + 15u];
+        else prevb = base > 0 ? (unsigned)__ldg(seg0 + (base - 1 - s)) : 0u;
+        const int seen = grep ? __shfl_sync(0xffffffffu, lane == 0u ? atomicOr(S.hit, 0) : 0, 0) : 0;
+        if (p0 < own_end) {
+            dfa_lane64(D, W, prevb, p0, own_end, valid_end, emit, emit2x);
+            if (grep && !seen && grep_lane64(T, W, p0, own_end, valid_end)) atomicExch(S.hit, 1);
+        }
+        __syncwarp();                // every lane is done with this tile before it is refilled
+    }
+}
+
+__global__ void __launch_bounds__(GSYS_DFA_MAXT, 1) scan_kernel(const __grid_constant__ ScanArgs a) {
     __shared__ int s_hit;
-    extern __shared__ __align__(16) unsigned char smem[];
+    __shared__ __align__(8) unsigned long long s_mbar[GSYS_DFA_MAXT / 32];
+    extern __shared__ __align__(1024) unsigned char smem[];
     const unsigned nwarps = blockDim.x / 32;
     ScanState S;
     unsigned* shist = load_tables(smem, a.tables, nwarps, S);
     const ScanTables& sT = *S.T;
+    const unsigned lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    // tensor-map tiles (a.tma_rows > 0): 1024-aligned per-warp tiles after the histograms
+    unsigned char* tiles = reinterpret_cast<unsigned char*>(((uintptr_t)S.stage + 1023) & ~(uintptr_t)1023);
+    const unsigned mbar = (unsigned)__cvta_generic_to_shared(&s_mbar[warp]);
+    if (a.tma_rows && lane == 0u) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(mbar) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
     if (threadIdx.x == 0) s_hit = 0;
     __syncthreads();
     S.hit = a.hit ? &s_hit : nullptr;
+    unsigned phase = 0;
     for (unsigned long long k = blockIdx.x; k < a.nchunks; k += gridDim.x) {
         const long long s = (long long)k * a.chunk;
         const long long e = s + a.chunk < (long long)a.n ? s + a.chunk : (long long)a.n;
-        if (sT.ncol == NCOL_WIDE) scan_range<LD_NC, true, GSYS_DFA_NBUF>(a.text + s, s, e, (long long)a.n, S);
+        if (a.tma_rows) {
+            if (sT.ncol == NCOL_WIDE) scan_range_swz<true>(a, a.text + s, s, e, (long long)a.n, S, tiles, mbar, phase);
+            else scan_range_swz<false>(a, a.text + s, s, e, (long long)a.n, S, tiles, mbar, phase);
+        } else if (sT.ncol == NCOL_WIDE) scan_range<LD_NC, true, GSYS_DFA_NBUF>(a.text + s, s, e, (long long)a.n, S);
         else scan_range<LD_NC, false, GSYS_DFA_NBUF>(a.text + s, s, e, (long long)a.n, S);
     }
     __syncthreads();
@@ -1141,6 +1230,31 @@ int gsys_read_profile(uint64_t* out3, int reset) {
     return 0;
 }
 
+}  // extern "C" (reopened below)
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link dependency)
+typedef CUresult (*PFN_tmap_t)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                               const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                               CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static PFN_tmap_t tmap_encoder() {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return (PFN_tmap_t)fn;
+}
+static bool swz_enabled() {
+    static const bool on = [] {
+        const char* e = getenv("GSYS_SCAN_SWZ");
+        return !(e && strcmp(e, "0") == 0);
+    }();
+    return on;
+}
+
+extern "C" {
+
 int gsys_set_scan(int impl) {
     if (impl != (int)GSYS_SCAN_TOKEN && impl != (int)GSYS_SCAN_DFA && impl != (int)GSYS_SCAN_DFA_TMA) return -EINVAL;
     return g_scan_impl.exchange(impl);
@@ -1171,8 +1285,24 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     // (profiles/r02_scan_staging_ab.jsonl: 33 small bulk copies per 2 KiB tile cost more than the
     // LSU slots they free), so it is the opt-in GSYS_SCAN_DFA_TMA
     const bool tma = impl == GSYS_SCAN_DFA_TMA;
-    const size_t per_warp = HSTRIDE * 4 + (tok ? TWWARP_STAGE : tma ? MWARP_STAGE : DWARP_STAGE);
-    if (!tok && tc->blob.size() + (threads / 32) * per_warp > kSmemDynMax) {
+    // the default DFA stages its tiles by one swizzled tensor copy each (scan_range_swz) when the
+    // text holds at least one tile of whole 64-byte rows (env GSYS_SCAN_SWZ=0: per-lane cp.async)
+    ScanArgs a;
+    memset(&a, 0, sizeof a);
+    if (!tok && !tma && n / 64 >= SW_ROWS && swz_enabled()) {
+        static PFN_tmap_t enc = tmap_encoder();
+        const cuuint64_t dims[2] = {64, n / 64};
+        const cuuint64_t strides[1] = {64};
+        const cuuint32_t box[2] = {64, SW_ROWS};
+        const cuuint32_t estr[2] = {1, 1};
+        if (enc && enc(&a.tmap, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(d_text), dims, strides, box,
+                       estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+                       CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS)
+            a.tma_rows = (unsigned)(n / 64);
+    }
+    const size_t per_warp = HSTRIDE * 4 + (tok ? TWWARP_STAGE : tma ? MWARP_STAGE : a.tma_rows ? SW_STRIDE : DWARP_STAGE);
+    const size_t slack = a.tma_rows ? 1024 : 0;   // the tiles start on a 1024-byte boundary
+    if (!tok && tc->blob.size() + (threads / 32) * per_warp + slack > kSmemDynMax) {
         tc = scan_tables(W, tok, NCOL_NARROW, dict, dlen, ndict, pats, plen, npat, &rc);
         if (!tc) return rc;
     }
@@ -1184,8 +1314,6 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     const bool blocks_auto = blocks == 0;
     if (blocks == 0) blocks = (uint32_t)W->sms;
     if (nch < blocks) blocks = (uint32_t)nch;
-    ScanArgs a;
-    memset(&a, 0, sizeof a);
     a.tables = reinterpret_cast<const ScanTables*>(tc->d);
     a.text = d_text;
     a.n = n;
@@ -1194,7 +1322,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk, const ch
     a.nchunks = nch;
     a.chunk = chunk;
     const void* fn = tok ? (const void*)scan_tok_kernel : tma ? (const void*)scan_tma_kernel : (const void*)scan_kernel;
-    size_t smem = align_up(tb, 16) + (threads / 32) * per_warp;
+    size_t smem = align_up(tb, 16) + (threads / 32) * per_warp + slack;
     rc = ensure_smem_attr(fn, smem);
     if (rc) return rc;
     if (blocks_auto) {   // one full wave: resident blocks per SM x SMs
