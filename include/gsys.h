@@ -360,7 +360,7 @@ int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
  * A9/A10): GSYS_SCAN_DFA (default) -- one transposed-DFA shared-memory lookup per byte
  * (csrc/scan_core.cuh); GSYS_SCAN_TOKEN -- SWAR word-byte masks, a per-tile list of token
  * starts, then per-token hash lookup and byte-exact verify spread over the warp
- * (csrc/tokscan.cuh; no 512-state trie limit, 0.84 of the DFA's rate on B200).  Env GSYS_SCAN=dfa|token|dfa_tma at load.  Returns the previous implementation, -EINVAL
+ * (csrc/tokscan.cuh; no 512-state trie limit, 0.78 of the DFA's rate on B200).  Env GSYS_SCAN=dfa|token|dfa_tma at load.  Returns the previous implementation, -EINVAL
  * for another value. */
 #define GSYS_SCAN_TOKEN 0
 #define GSYS_SCAN_DFA   1

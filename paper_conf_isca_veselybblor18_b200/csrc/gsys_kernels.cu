@@ -982,7 +982,7 @@ struct Workspace {
 };
 Workspace g_ws[64];
 std::mutex g_ws_mu;
-// scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.67 TB/s on the
+// scan implementation of wc_kernel / gsys_scan_device: GSYS_SCAN_DFA (default: 1.79 TB/s on the
 // 1 GiB HBM scan) or GSYS_SCAN_TOKEN (warp-cooperative token scan, 1.40 TB/s,
 // profiles/r02_tokg.jsonl); env GSYS_SCAN=dfa|token at load, gsys_set_scan() at run time
 std::atomic<int> g_scan_impl{[] {
