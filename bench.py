@@ -562,7 +562,7 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
             kv = json.load(open(summ))
             traffic = (kv["dram__bytes_read.sum"]["value"] + kv["dram__bytes_write.sum"]["value"]) * n / kv["text_bytes"]
             limiter = (f"shared-memory pipe: l1tex {kv['l1tex__throughput.avg.pct_of_peak_sustained_active']['value']:.0f}% "
-                       f"of peak (DFA gathers, 3.3 wavefronts per warp lookup), issue "
+                       f"of peak (DFA gathers, 3.3 wavefronts per warp lookup; tiles staged by swizzled tensor copies), issue "
                        f"{kv['smsp__issue_active.avg.pct_of_peak_sustained_active']['value']:.0f}%")
         except (KeyError, ValueError, TypeError):
             pass
@@ -583,7 +583,7 @@ def scan_roofline(G, dev, corpus, words, pats, chunk):
     return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak, "bytes": n,
             "traffic": traffic, "limiter": limiter, "ms": t * 1e3, "compute_roofline": compute,
             "token_scan": dict(tok, frac=tok["achieved"] / peak) if tok else None,
-            "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 1024 threads (32 warps, one staged tile each), 129-column transposed DFA in shared memory; profiles/r02_dfa32.jsonl)",
+            "kernel": "scan_kernel (HBM-resident text, 1 block/SM x 1024 threads (32 warps), each 2 KiB warp tile one swizzled tensor copy, 129-column transposed DFA in shared memory; profiles/r02_swz.jsonl)",
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)", "note": "input 1 GiB > L2; read-once"}
 
 
