@@ -780,7 +780,7 @@ __device__ __forceinline__ void scan_range_swz(const ScanArgs& a, const unsigned
 __global__ void __launch_bounds__(GSYS_DFA_MAXT, 1) scan_kernel(const __grid_constant__ ScanArgs a) {
     __shared__ int s_hit;
     __shared__ __align__(8) unsigned long long s_mbar[GSYS_DFA_MAXT / 32];
-    extern __shared__ __align__(1024) unsigned char smem[];
+    extern __shared__ __align__(16) unsigned char smem[];   // tiles aligned at run time (1024 B slack)
     const unsigned nwarps = blockDim.x / 32;
     ScanState S;
     unsigned* shist = load_tables(smem, a.tables, nwarps, S);
