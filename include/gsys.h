@@ -348,7 +348,9 @@ int gsys_wordcount(const int32_t* fds, const uint64_t* sizes, uint32_t nfiles, u
  * pattern occurs.  chunk: multiple of 16; blocks 0 = one full wave; threads 0 = 1024 (704 for
  * GSYS_SCAN_DFA_TMA), else a
  * multiple of 32 up to 1024 (768 for GSYS_SCAN_DFA_TMA); the DFA's 129-column table is used when it
- * fits beside the warps' staging, else the 77-column one.  -EINVAL on bad
+ * fits beside the warps' staging, else the 77-column one.  The DFA stages each warp tile of whole
+ * 64-byte rows by one swizzled tensor copy (a tensor map of d_text built per call; env
+ * GSYS_SCAN_SWZ=0 at load: per-lane copies).  -EINVAL on bad
  * sizes/alignment, -ENODEV before gsys_init. */
 int gsys_scan_device(const uint8_t* d_text, uint64_t n, uint32_t chunk,
                      const char* dict, const uint8_t* dlen, uint32_t ndict,
