@@ -284,6 +284,39 @@ def test_scan_device_dense_tokens(scan_impl, pattern):
             assert hit == oracle.grep(arr, [b"b c"])
 
 
+def test_scan_device_staging_paths_agree(tmp_path):
+    """The HBM DFA scan stages whole-row tiles by swizzled tensor copies and the rest by the lanes;
+    with GSYS_SCAN_SWZ=0 (a fresh process: read at load) every tile goes through the lanes.  Both
+    equal the oracle on a 3 MiB + 37 B text at 64-byte-aligned and unaligned chunk sizes."""
+    import subprocess
+    import sys
+    code = f"""
+import os, sys, numpy as np, torch
+sys.path.insert(0, {repr(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))})
+import inputs, oracle
+from paper_conf_isca_veselybblor18_b200 import gsys as G, workloads as W
+W.ensure_init()
+words, pats = inputs.dictionary(), inputs.patterns()
+size = (3 << 20) + 37
+buf, census, _ = inputs.gen_bytes(inputs.SEED_CORPUS, 5, size, grep_plants=True)
+t = torch.zeros(size + 64, dtype=torch.uint8, device='cuda')
+t[:size].copy_(torch.from_numpy(buf))
+want = oracle.count_tokens(buf, words)
+for chunk in (48, 4096, 1 << 20):
+    h = torch.zeros(64, dtype=torch.int64, device='cuda')
+    hit = torch.zeros(1, dtype=torch.int32, device='cuda')
+    G.gsys_scan_device(t, size, chunk, words, pats, h, hit)
+    torch.cuda.synchronize()
+    assert np.array_equal(h.cpu().numpy().astype(np.uint64), want), chunk
+    assert bool(hit.item()) == oracle.grep(buf, pats), chunk
+print('ok')
+"""
+    for swz in ("1", "0"):
+        env = dict(os.environ, GSYS_SCAN_SWZ=swz)
+        out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+        assert out.returncode == 0 and "ok" in out.stdout, (swz, out.stderr[-3000:])
+
+
 def test_scan_device_large_trie_uses_narrow_table(scan_impl):
     """A dictionary whose 129-column table no longer fits next to 16 warps' staging (482 trie
     states + 30 emission states) runs on the 77-column table: same counts."""
